@@ -1,0 +1,170 @@
+"""Seeded synthetic workload generators shared by the oracle tests, the GPU parity tests and bench.py.
+
+This module draws inputs only. It holds none of Multigrain's arithmetic: no mask
+union, no tile classification, no softmax. Both sides receive exactly the
+arrays produced here.
+
+* Q/K/V recipe: ``numpy.random.default_rng(seed + i)`` (PCG64)
+  draws Q (i=0), K (i=1), V (i=2) as float32 standard normals. They are rounded
+  to bf16 (or fp16) with round-to-nearest-even and returned as uint16 bit
+  patterns. The GPU receives these bits; the oracle upcasts them exactly to fp64.
+* Pattern recipe (BASELINE.json ``configs``):
+  - C1: B=1, H=1, L=512, w=64, G={0, 200}, E=∅;
+  - C2: Longformer-base, B=8, H=12, L=4096, w=512, G=[0,32), E=∅;
+  - C3: QDS, B=8, H=12, L=2048, w=256, G=[0,8) ∪ 56 sentence starts drawn by
+    ``default_rng(1).choice(arange(8, 2048), 56, replace=False)``, E=∅;
+  - C4: Longformer-large long doc, B=2, H=16, L=16384, w=512, G=∅,
+    E = 164 (=⌈0.01·L⌉) distinct uniform columns per row outside the band,
+    drawn row by row from ``default_rng(0)``;
+  - C5: C2's shape at B=64 (sharded over ranks in the scaling bench).
+  Paper context: local/global/selected/random atomic patterns, PAPER.md
+  lines 64-71 (§2.3); Longformer = L+S+G, QDS = L+S.
+"""
+from __future__ import annotations
+
+import math
+from dataclasses import dataclass, field
+
+import numpy as np
+
+__all__ = [
+    "Config", "CONFIGS", "get_config", "make_qkv", "to_bf16_bits", "to_fp16_bits",
+    "bits_to_f64", "random_residual", "qds_globals", "random_small_config",
+]
+
+
+def to_bf16_bits(x: np.ndarray) -> np.ndarray:
+    """float32 -> bf16 bit pattern (uint16), round-to-nearest-even; NaN kept quiet."""
+    x = np.ascontiguousarray(x, dtype=np.float32)
+    u = x.view(np.uint32).astype(np.uint64)
+    rounding = ((u >> 16) & 1) + 0x7FFF
+    r = ((u + rounding) >> 16).astype(np.uint16)
+    nan = np.isnan(x)
+    if nan.any():
+        r[nan] = 0x7FC0
+    return r
+
+
+def to_fp16_bits(x: np.ndarray) -> np.ndarray:
+    """float32 -> IEEE fp16 bit pattern (uint16), numpy's round-to-nearest-even."""
+    return np.ascontiguousarray(x, dtype=np.float32).astype(np.float16).view(np.uint16)
+
+
+def bits_to_f64(bits: np.ndarray, dtype: str = "bf16") -> np.ndarray:
+    """Exact upcast of 16-bit patterns to float64."""
+    bits = np.asarray(bits, dtype=np.uint16)
+    if dtype == "bf16":
+        return (bits.astype(np.uint32) << 16).view(np.float32).astype(np.float64)
+    if dtype == "fp16":
+        return bits.view(np.float16).astype(np.float64)
+    raise ValueError(dtype)
+
+
+@dataclass(frozen=True)
+class Config:
+    name: str
+    B: int
+    H: int
+    L: int
+    d: int
+    window: int
+    global_idx: np.ndarray = field(compare=False)
+    extra_idx: np.ndarray = field(compare=False)   # int32 [n, 2] COO (row, col)
+    seed: int = 0
+    note: str = ""
+
+    @property
+    def w1(self) -> int:
+        return self.window // 2
+
+
+def qds_globals(L: int = 2048, n_prefix: int = 8, n_sent: int = 56, seed: int = 1) -> np.ndarray:
+    """QDS-style sentence-level global tokens: [0, n_prefix) ∪ n_sent sorted irregular positions."""
+    rng = np.random.default_rng(seed)
+    sent = np.sort(rng.choice(np.arange(n_prefix, L), n_sent, replace=False))
+    return np.concatenate([np.arange(n_prefix), sent]).astype(np.int32)
+
+
+def random_residual(L: int, window: int, per_row: int, seed: int = 0) -> np.ndarray:
+    """Random fine-grained residual: per row r, `per_row` distinct uniform columns
+    with |r-c| > window/2, drawn in row order from default_rng(seed). Returns int32 [L*per_row, 2]."""
+    w1 = window // 2
+    rng = np.random.default_rng(seed)
+    cols = np.arange(L)
+    out = np.empty((L * per_row, 2), dtype=np.int32)
+    for r in range(L):
+        cand = cols[np.abs(cols - r) > w1]
+        k = min(per_row, cand.size)
+        pick = rng.choice(cand, k, replace=False) if k else np.empty(0, np.int64)
+        out[r * per_row:r * per_row + k, 0] = r
+        out[r * per_row:r * per_row + k, 1] = pick
+    return out
+
+
+_EMPTY_E = np.zeros((0, 2), dtype=np.int32)
+
+
+def _build_configs():
+    c = {}
+    c["C1"] = Config("C1", 1, 1, 512, 64, 64, np.array([0, 200], np.int32), _EMPTY_E, 0,
+                     "single head, L=512, window 64 + 2 global tokens")
+    c["C2"] = Config("C2", 8, 12, 4096, 64, 512, np.arange(32, dtype=np.int32), _EMPTY_E, 0,
+                     "Longformer-base L=4096, w=512, G=[0,32), B=8")
+    c["C3"] = Config("C3", 8, 12, 2048, 64, 256, qds_globals(), _EMPTY_E, 0,
+                     "QDS L=2048, w=256, 64 irregular global tokens, B=8")
+    c["C5"] = Config("C5", 64, 12, 4096, 64, 512, np.arange(32, dtype=np.int32), _EMPTY_E, 0,
+                     "C2 shape at B=64 (scaling sweep)")
+    return c
+
+
+CONFIGS = _build_configs()
+_C4_CACHE: dict = {}
+
+
+def get_config(name: str) -> Config:
+    """Return a BASELINE config by name (C1..C5). C4's residual is generated on first use (~1 s)."""
+    if name == "C4":
+        if "C4" not in _C4_CACHE:
+            L = 16384
+            _C4_CACHE["C4"] = Config("C4", 2, 16, L, 64, 512, np.zeros(0, np.int32),
+                                     random_residual(L, 512, math.ceil(0.01 * L), seed=0), 0,
+                                     "Longformer-large L=16384, w=512, 1% random residual, B=2")
+        return _C4_CACHE["C4"]
+    return CONFIGS[name]
+
+
+def make_qkv(B: int, H: int, L: int, d: int, seed: int = 0, dist: str = "normal",
+             global_idx: np.ndarray | None = None, dtype: str = "bf16"):
+    """Q, K, V as uint16 bit patterns of shape [B, H, L, d].
+
+    dist: "normal" (N(0,1)), "peaky" (Q x 4), "adversarial" (K rows at global positions x 8),
+    "zeros_q" (Q = 0), "ones_v" (V = 1).
+    """
+    shape = (B, H, L, d)
+    q = np.random.default_rng(seed + 0).standard_normal(shape, dtype=np.float32)
+    k = np.random.default_rng(seed + 1).standard_normal(shape, dtype=np.float32)
+    v = np.random.default_rng(seed + 2).standard_normal(shape, dtype=np.float32)
+    if dist == "peaky":
+        q *= 4.0
+    elif dist == "adversarial":
+        if global_idx is not None and len(global_idx):
+            k[:, :, np.asarray(global_idx), :] *= 8.0
+    elif dist == "zeros_q":
+        q[...] = 0.0
+    elif dist == "ones_v":
+        v[...] = 1.0
+    elif dist != "normal":
+        raise ValueError(dist)
+    conv = to_bf16_bits if dtype == "bf16" else to_fp16_bits
+    return conv(q), conv(k), conv(v)
+
+
+def random_small_config(rng: np.random.Generator, L_max: int = 64):
+    """A random tiny pattern for brute-force tests: (L, window, G, E)."""
+    L = int(rng.integers(1, L_max + 1))
+    window = 2 * int(rng.integers(0, L + 2))
+    nG = int(rng.integers(0, min(L, 4) + 1))
+    G = rng.choice(L, nG, replace=False).astype(np.int32) if nG else np.zeros(0, np.int32)
+    nE = int(rng.integers(0, 2 * L + 1))
+    E = rng.integers(0, L, size=(nE, 2)).astype(np.int32)
+    return L, window, G, E
