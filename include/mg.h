@@ -1,0 +1,213 @@
+/*
+ * mg.h — C ABI of the B200-native Multigrain compound sparse attention forward.
+ *
+ * Paper: H. Li, J. Choi, J. H. Ahn, "A Slice and Dice Approach to Accelerate Compound
+ * Sparse Attention on GPU" (IISWC 2022). "P:n" = line n of that paper's text
+ * (/root/reference/PAPER.md at build time; not needed at run time).
+ *
+ * What the library computes (§2.2): for every batch b and head h, with
+ * Q_h, K_h, V_h of shape L x D_h,
+ *     S = Q_h K_h^T * (1/sqrt(D_h))          (SDDMM + scaling; reading A1)
+ *     S[not M] = -inf                         (masking)
+ *     P = row-softmax(S) over the non-zeros   (SpSoftmax)
+ *     C_h = P V_h                              (SpMM)
+ * where M is the compound mask: sliding window |r-c| <= window/2, symmetric global
+ * tokens, and an arbitrary extra residual E.
+ *
+ * How (§3.1): a host plan splits M into three disjoint parts — coarse BSR tiles
+ * (tensor cores), a fine CSR residual (warp-per-row kernels), dense global rows — and
+ * the forward merges their softmax statistics so the result is exactly the masked
+ * softmax attention above (up to floating-point rounding).
+ *
+ * Conventions for every function:
+ *   - No exceptions cross the ABI. Every call returns an mg_status; on error a
+ *     thread-local message is available from mg_last_error().
+ *   - Validation happens before any device work; on error nothing is launched and
+ *     outputs are untouched.
+ *   - Index arrays are int32, tensors are 16-bit (bf16 or fp16) with element strides.
+ */
+#ifndef MG_H_
+#define MG_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define MG_ABI_VERSION 1
+
+#if defined(__GNUC__)
+#define MG_API __attribute__((visibility("default")))
+#else
+#define MG_API
+#endif
+
+typedef struct mg_plan_s* mg_plan_t;
+
+typedef enum {
+  MG_OK = 0,
+  MG_ERR_INVALID_ARG = 1,   /* bad sizes, indices out of range, null pointers, layout mismatch */
+  MG_ERR_UNSUPPORTED = 2,   /* valid but not implemented in v1 (d != 64, block != 128 on fwd, ...) */
+  MG_ERR_OUT_OF_MEMORY = 3, /* host or device allocation failed */
+  MG_ERR_CUDA = 4,          /* a CUDA runtime/driver error; message in mg_last_error() */
+  MG_ERR_INTERNAL = 5
+} mg_status;
+
+typedef enum { MG_BF16 = 0, MG_FP16 = 1 } mg_dtype;
+
+/* A [batch, heads, seq_len, head_dim] view of 16-bit data with element strides; the
+ * head_dim stride is 1. Both [B,H,L,d] (stride_l = d) and [B,L,H,d] (stride_h = d,
+ * stride_l = H*d) are accepted (per-head L x D_h slices of L x D_m hidden states).
+ * `data` is a device pointer for mg_sparse_attention_fwd and a host pointer for
+ * mg_sparse_attention_fwd_host. data must be 16-byte aligned and every stride a multiple
+ * of 8 elements (TMA requirement). */
+typedef struct {
+  void* data;
+  int32_t dtype;      /* mg_dtype */
+  int32_t reserved;
+  int64_t batch;
+  int64_t heads;
+  int64_t seq_len;
+  int64_t head_dim;
+  int64_t stride_b, stride_h, stride_l;
+} mg_tensor;
+
+/* ------------------------------------------------------------------------------------
+ * Plan (§3.1 steps 1-2: classification and metadata "before inferring the model").
+ *
+ * mg_plan_create(L, heads, d, window, global_idx, n_global, extra_idx, n_extra, &plan)
+ *   L          sequence length, > 0.
+ *   heads      number of heads, > 0 (the pattern is shared by all heads).
+ *   d          head dimension; v1 supports d == 64 only (else MG_ERR_UNSUPPORTED).
+ *   window     local window size, >= 0 and even: |r-c| <= window/2 is valid (reading A2).
+ *   global_idx host int32[n_global], positions of global tokens in [0, L); attend to and are
+ *              attended by every token (reading A3). Duplicates collapse.
+ *   extra_idx  host int32[n_extra][2], (row, col) pairs of extra valid elements in [0, L)^2
+ *              (random / selected / dilated residual). Duplicates collapse; pairs
+ *              already inside the band or a global row/column are absorbed.
+ *   plan       out: a new plan. The index arrays are copied; the caller may free them.
+ * The partition is the canonical one (DESIGN.md §3 O-3): tiles of b x b (b = 128) touched by
+ * the band of a non-global row are coarse; the coarse tile owns every union element it
+ * covers (overlap invalidation); the remaining non-global elements form the CSR
+ * residual; global rows are dense and owned by the dense-row part.
+ * If a CUDA device is present the metadata is uploaded synchronously to the current device;
+ * otherwise the upload is deferred to the first forward call.
+ * Errors: INVALID_ARG (L <= 0, heads <= 0, d <= 0, window < 0 or odd, index out of range,
+ * null array with a non-zero count, null plan), UNSUPPORTED (d != 64, CSR nnz >= 2^31),
+ * OUT_OF_MEMORY, CUDA.
+ * ---------------------------------------------------------------------------------- */
+MG_API mg_status mg_plan_create(int64_t L, int32_t heads, int32_t d, int32_t window,
+                         const int32_t* global_idx, int64_t n_global,
+                         const int32_t* extra_idx, int64_t n_extra,
+                         mg_plan_t* plan_out);
+
+/* Test/ablation options. Zero-initialised means "default". */
+typedef struct {
+  int32_t block;          /* tile size b; 0 -> 128. Any b <= 64 or multiple of 64 builds a plan
+                             (for export tests); the forward requires b == 128. */
+  int32_t force_all_fine; /* 1: no coarse tiles; every non-global element goes to the CSR part */
+  int32_t strip_max_cols; /* max gathered columns per row block for the tensor-core strip path of
+                             the CSR residual; 0 -> default (128); -1 disables the strip path */
+  int32_t num_sms;        /* persistent grid size override; 0 -> device SM count */
+  int32_t reserved[4];
+} mg_plan_opts;
+
+MG_API mg_status mg_plan_create_ex(int64_t L, int32_t heads, int32_t d, int32_t window,
+                            const int32_t* global_idx, int64_t n_global,
+                            const int32_t* extra_idx, int64_t n_extra,
+                            const mg_plan_opts* opts, mg_plan_t* plan_out);
+
+/* Frees host and device memory of the plan. Must not race with in-flight forwards that use
+ * it (synchronize their streams first). Null is accepted (no-op). */
+MG_API mg_status mg_plan_destroy(mg_plan_t plan);
+
+/* Thread-local message of the last failing call on this thread ("" if none). */
+MG_API const char* mg_last_error(void);
+
+typedef struct {
+  int64_t L;
+  int32_t heads, d, window, block;
+  int64_t n_row_blocks;     /* nb = ceil(L / b) */
+  int64_t n_tiles;          /* |T|, coarse BSR tiles */
+  int64_t n_full_tiles;     /* tiles whose b*b bits are all set */
+  int64_t nnz_coarse;       /* popcount of all tile masks */
+  int64_t nnz_fine;         /* CSR residual nnz */
+  int64_t n_global;         /* |G| */
+  int64_t nnz_total;        /* |M| = nnz_coarse + nnz_fine + n_global * L */
+  int64_t n_fine_rows;      /* rows run by the CUDA-core fine kernel */
+  int64_t nnz_fine_strip;   /* CSR nnz executed by the tensor-core strip path */
+  int64_t nnz_fine_cuda;    /* CSR nnz executed by the warp-per-row CUDA-core kernel */
+  int64_t n_items;          /* coarse-kernel work items per (batch, head) */
+  int64_t n_strip_tiles;    /* gathered strip tiles per (batch, head) */
+  int64_t computed_scores;  /* tensor-core scores per (batch, head) incl. masked waste */
+  int32_t kernels_per_fwd;  /* kernel launches per mg_sparse_attention_fwd call */
+  int32_t reserved;
+} mg_plan_info;
+
+MG_API mg_status mg_plan_info_get(mg_plan_t plan, mg_plan_info* info);
+
+/* Copies the canonical partition into host buffers sized from mg_plan_info:
+ *   bsr_row_ptr int32[n_row_blocks+1], bsr_col int32[n_tiles],
+ *   tile_masks uint64[n_tiles * block * ceil(block/64)] (row-major, LSB = lowest column),
+ *   csr_row_ptr int32[L+1], csr_col int32[nnz_fine], global_rows int32[n_global].
+ * Any pointer may be null to skip that array. */
+MG_API mg_status mg_plan_export(mg_plan_t plan, int32_t* bsr_row_ptr, int32_t* bsr_col, uint64_t* tile_masks,
+                         int32_t* csr_row_ptr, int32_t* csr_col, int32_t* global_rows);
+
+/* ------------------------------------------------------------------------------------
+ * Forward (P:96 step 3).
+ * mg_sparse_attention_fwd(plan, Q, K, V, O, stream)
+ *   Q, K, V  device tensors [batch, heads, L, d] (mg_tensor strides), read only.
+ *   O        device tensor, same shape; written for every (b, h, row).
+ *   stream   a cudaStream_t (passed as void*); 0 = legacy default stream.
+ * Asynchronous: returns after enqueueing; no host synchronisation on the steady-state path.
+ * Q/K/V/O must stay alive until the stream work completes. The plan's fwd workspace (fp32
+ * partial statistics of the CSR part) is plan-owned and grown stream-ordered on `stream`,
+ * so one plan must not be used by two concurrent forwards on different streams.
+ * Errors: INVALID_ARG (null, shape/dtype mismatch with the plan or between tensors,
+ * head_dim stride != 1, misaligned data or strides), UNSUPPORTED (block != 128,
+ * dtypes that differ), CUDA.
+ * ---------------------------------------------------------------------------------- */
+MG_API mg_status mg_sparse_attention_fwd(mg_plan_t plan, const mg_tensor* Q, const mg_tensor* K,
+                                  const mg_tensor* V, mg_tensor* O, void* stream);
+
+/* Same computation with HOST tensors: copies Q/K/V host->device into plan-owned staging
+ * buffers on `stream`, runs the forward, copies O device->host, all stream-ordered and
+ * asynchronous (host buffers should be pinned for the copies to overlap; the caller
+ * synchronises `stream` before reading O). Same errors as mg_sparse_attention_fwd. */
+MG_API mg_status mg_sparse_attention_fwd_host(mg_plan_t plan, const mg_tensor* Q, const mg_tensor* K,
+                                       const mg_tensor* V, mg_tensor* O, void* stream);
+
+/* ------------------------------------------------------------------------------------
+ * Profiling (tracing subsystem). When enabled, every forward records CUDA events on its
+ * stream around each kernel it launches; mg_plan_get_profile() synchronises on the recorded
+ * events, returns the summed device durations since the last enable/reset, and resets.
+ * Durations are per kernel class: fine = CUDA-core CSR kernel, coarse = tensor-core kernel
+ * (band + strip + dense-row items), total = from the first to the last launch of each call.
+ * ---------------------------------------------------------------------------------- */
+typedef struct {
+  int64_t calls;
+  double fine_ms, coarse_ms, total_ms;
+} mg_profile;
+
+MG_API mg_status mg_plan_set_profiling(mg_plan_t plan, int32_t enable);
+MG_API mg_status mg_plan_get_profile(mg_plan_t plan, mg_profile* out);
+
+/* ------------------------------------------------------------------------------------
+ * Diagnostics (used by the GPU tests; not part of the attention path).
+ * mg_selftest_umma(mode, A, B, D, stream): one 128 x N x K tcgen05 MMA on device buffers.
+ *   mode 0: D[128x128] fp32 = A[128x64] bf16 (K-major, SMEM) * B[128x64]^T bf16 (K-major)
+ *   mode 1: D[128x64]  fp32 = A[128x128] bf16 (staged SMEM->TMEM, TS form) * B[128x64] bf16
+ *           (B row-major over K: MN-major operand)
+ * All buffers are row-major device arrays. Returns CUDA on launch failure.
+ * ---------------------------------------------------------------------------------- */
+MG_API mg_status mg_selftest_umma(int32_t mode, const void* A, const void* B, float* D, void* stream);
+
+MG_API int32_t mg_abi_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* MG_H_ */

@@ -1,0 +1,142 @@
+"""Python-side names of the C ABI (include/mg.h): marshalling only, no arithmetic."""
+from __future__ import annotations
+
+import ctypes as C
+
+import numpy as np
+
+from . import _lib
+from ._lib import check, load, mg_plan_info, mg_plan_opts, mg_profile, mg_tensor
+
+
+def _i32(a) -> np.ndarray:
+    return np.ascontiguousarray(np.asarray(a, dtype=np.int32))
+
+
+def _ptr_i32(a: np.ndarray):
+    return a.ctypes.data_as(C.POINTER(C.c_int32)) if a.size else None
+
+
+class Plan:
+    """mg_plan_create / mg_plan_create_ex (metadata built once before inference).
+
+    Args follow include/mg.h: L, heads, d, window, global_idx (int array), extra_idx (int [n, 2]).
+    Options (test/ablation): block, force_all_fine, strip_max_cols, num_sms.
+    """
+
+    def __init__(self, L: int, heads: int, d: int, window: int, global_idx=(), extra_idx=None, *,
+                 block: int = 0, force_all_fine: bool = False, strip_max_cols: int = 0, num_sms: int = 0):
+        lib = load()
+        g = _i32(list(global_idx) if not isinstance(global_idx, np.ndarray) else global_idx).reshape(-1)
+        e = _i32(np.zeros((0, 2)) if extra_idx is None else extra_idx).reshape(-1, 2)
+        self._handle = C.c_void_p()
+        self._lib = lib
+        opts = mg_plan_opts(block, int(force_all_fine), strip_max_cols, num_sms)
+        if block or force_all_fine or strip_max_cols or num_sms:
+            st = lib.mg_plan_create_ex(L, heads, d, window, _ptr_i32(g), g.size, _ptr_i32(e), e.shape[0],
+                                       C.byref(opts), C.byref(self._handle))
+        else:
+            st = lib.mg_plan_create(L, heads, d, window, _ptr_i32(g), g.size, _ptr_i32(e), e.shape[0],
+                                    C.byref(self._handle))
+        check(st)
+        self.L, self.heads, self.d, self.window = L, heads, d, window
+
+    @property
+    def handle(self):
+        return self._handle
+
+    def info(self) -> dict:
+        inf = mg_plan_info()
+        check(self._lib.mg_plan_info_get(self._handle, C.byref(inf)))
+        return {name: getattr(inf, name) for name, _ in mg_plan_info._fields_ if name != "reserved"}
+
+    def export(self) -> dict:
+        inf = self.info()
+        b = inf["block"]
+        wpr = -(-b // 64)
+        out = {
+            "bsr_row_ptr": np.zeros(inf["n_row_blocks"] + 1, np.int32),
+            "bsr_col": np.zeros(inf["n_tiles"], np.int32),
+            "tile_masks": np.zeros((inf["n_tiles"], b, wpr), np.uint64),
+            "csr_row_ptr": np.zeros(inf["L"] + 1, np.int32),
+            "csr_col": np.zeros(inf["nnz_fine"], np.int32),
+            "global_rows": np.zeros(inf["n_global"], np.int32),
+        }
+        i32 = lambda a: a.ctypes.data_as(C.POINTER(C.c_int32))
+        check(self._lib.mg_plan_export(self._handle, i32(out["bsr_row_ptr"]), i32(out["bsr_col"]),
+                                       out["tile_masks"].ctypes.data_as(C.POINTER(C.c_uint64)),
+                                       i32(out["csr_row_ptr"]), i32(out["csr_col"]), i32(out["global_rows"])))
+        return out
+
+    def set_profiling(self, enable: bool = True) -> None:
+        """mg_plan_set_profiling: record CUDA events around each kernel of every forward."""
+        check(self._lib.mg_plan_set_profiling(self._handle, int(enable)))
+
+    def get_profile(self) -> dict:
+        """mg_plan_get_profile: summed per-kernel-class device ms since the last reset (then resets)."""
+        pr = mg_profile()
+        check(self._lib.mg_plan_get_profile(self._handle, C.byref(pr)))
+        return {"calls": pr.calls, "fine_ms": pr.fine_ms, "coarse_ms": pr.coarse_ms, "total_ms": pr.total_ms}
+
+    def close(self):
+        if getattr(self, "_handle", None) is not None and self._handle.value:
+            self._lib.mg_plan_destroy(self._handle)
+            self._handle = C.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def tensor_desc(t) -> mg_tensor:
+    """mg_tensor for a torch tensor viewed as [B, H, L, d] (any strides with a unit d-stride)."""
+    import torch
+    if t.dim() != 4:
+        raise ValueError("expected a 4-D [B, H, L, d] tensor")
+    if t.dtype == torch.bfloat16:
+        dt = _lib.MG_BF16
+    elif t.dtype == torch.float16:
+        dt = _lib.MG_FP16
+    else:
+        raise TypeError(f"unsupported dtype {t.dtype}")
+    if t.stride(3) != 1:
+        raise ValueError("head_dim stride must be 1")
+    B, H, L, d = t.shape
+    sb, sh, sl, _ = t.stride()
+    return mg_tensor(t.data_ptr(), dt, 0, B, H, L, d, sb, sh, sl)
+
+
+def _stream_ptr(stream):
+    import torch
+    if stream is None:
+        stream = torch.cuda.current_stream()
+    return C.c_void_p(stream.cuda_stream)
+
+
+def sparse_attention_fwd(plan: Plan, Q, K, V, O=None, stream=None):
+    """mg_sparse_attention_fwd on device tensors [B, H, L, d]; returns O (allocated if None)."""
+    import torch
+    if O is None:
+        O = torch.empty(Q.shape, dtype=Q.dtype, device=Q.device)
+    dq, dk, dv, do = tensor_desc(Q), tensor_desc(K), tensor_desc(V), tensor_desc(O)
+    check(plan._lib.mg_sparse_attention_fwd(plan.handle, C.byref(dq), C.byref(dk), C.byref(dv), C.byref(do),
+                                            _stream_ptr(stream)))
+    return O
+
+
+def sparse_attention_fwd_host(plan: Plan, Q, K, V, O, stream=None):
+    """mg_sparse_attention_fwd_host on dense HOST tensors (pinned for async copies). Asynchronous:
+    synchronise `stream` before reading O."""
+    dq, dk, dv, do = tensor_desc(Q), tensor_desc(K), tensor_desc(V), tensor_desc(O)
+    check(plan._lib.mg_sparse_attention_fwd_host(plan.handle, C.byref(dq), C.byref(dk), C.byref(dv),
+                                                 C.byref(do), _stream_ptr(stream)))
+    return O
+
+
+def selftest_umma(mode: int, A, B, D, stream=None):
+    """mg_selftest_umma: one tcgen05 MMA on device buffers (diagnostics)."""
+    check(load().mg_selftest_umma(mode, C.c_void_p(A.data_ptr()), C.c_void_p(B.data_ptr()),
+                                  C.c_void_p(D.data_ptr()), _stream_ptr(stream)))
+    return D

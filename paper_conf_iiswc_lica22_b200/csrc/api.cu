@@ -1,0 +1,481 @@
+// C ABI of the Multigrain forward (include/mg.h). Host-side: validation, plan lifetime,
+// device upload, TMA descriptors, workspace, launches. Every step of the attention runs in the
+// kernels of coarse_sm100.cu and fine_rows.cu; there is no CPU fallback.
+#include <cudaTypedefs.h>
+
+#include <algorithm>
+#include <cstring>
+#include <mutex>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "kernels.cuh"
+#include "mg.h"
+#include "plan.hpp"
+
+namespace {
+
+thread_local std::string g_err;
+
+mg_status fail(mg_status s, const std::string& msg) {
+  g_err = msg;
+  return s;
+}
+mg_status cuda_fail(cudaError_t e, const char* where) {
+  return fail(MG_ERR_CUDA, std::string(where) + ": " + cudaGetErrorName(e) + " (" + cudaGetErrorString(e) + ")");
+}
+
+PFN_cuTensorMapEncodeTiled_v12000 tensor_map_encoder() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void* ptr = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &ptr, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(ptr);
+  });
+  return fn;
+}
+
+}  // namespace
+
+struct mg_plan_s {
+  mg::HostPlan hp;
+  int device = -1;
+  bool uploaded = false;
+  int num_sms = 0;
+  int num_sms_override = 0;
+  std::vector<void*> allocs;
+  mg::Item* d_items = nullptr;
+  mg::TileRef* d_trefs = nullptr;
+  uint64_t* d_masks = nullptr;
+  int32_t* d_strip_cols = nullptr;
+  int32_t* d_global_rows = nullptr;
+  int32_t* d_fine_slot = nullptr;
+  int32_t* d_fine_rows = nullptr;
+  int32_t* d_fine_row_ptr = nullptr;
+  int32_t* d_fine_col = nullptr;
+  int32_t* d_counter = nullptr;
+  // stream-ordered workspaces
+  float* d_part = nullptr;
+  size_t part_cap = 0;      // in (row, bh) partial slots
+  uint8_t* d_stage = nullptr;
+  size_t stage_cap = 0;     // bytes
+  // profiling: 4 events per recorded call (start, after fine, after coarse, end)
+  bool profiling = false;
+  std::vector<cudaEvent_t> prof_events;
+  size_t prof_used = 0;
+  std::vector<uint8_t> prof_has_fine, prof_has_coarse;
+
+  cudaEvent_t prof_event() {
+    if (prof_used == prof_events.size()) {
+      cudaEvent_t e = nullptr;
+      if (cudaEventCreate(&e) != cudaSuccess) return nullptr;
+      prof_events.push_back(e);
+    }
+    return prof_events[prof_used++];
+  }
+
+  ~mg_plan_s() {
+    for (cudaEvent_t e : prof_events) cudaEventDestroy(e);
+    for (void* p : allocs) cudaFree(p);
+    if (d_part) cudaFree(d_part);
+    if (d_stage) cudaFree(d_stage);
+  }
+};
+
+namespace {
+
+template <class T>
+cudaError_t upload_vec(mg_plan_s* p, T** dst, const std::vector<T>& v) {
+  const size_t bytes = std::max<size_t>(v.size() * sizeof(T), 16);
+  cudaError_t e = cudaMalloc(reinterpret_cast<void**>(dst), bytes);
+  if (e != cudaSuccess) return e;
+  p->allocs.push_back(*dst);
+  if (!v.empty()) e = cudaMemcpy(*dst, v.data(), v.size() * sizeof(T), cudaMemcpyHostToDevice);
+  return e;
+}
+
+mg_status upload(mg_plan_s* p) {
+  if (p->uploaded) return MG_OK;
+  if (!p->hp.kernel_ready) return fail(MG_ERR_UNSUPPORTED, "the forward requires block == 128");
+  cudaError_t e = cudaGetDevice(&p->device);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaGetDevice");
+  e = cudaDeviceGetAttribute(&p->num_sms, cudaDevAttrMultiProcessorCount, p->device);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaDeviceGetAttribute");
+  int major = 0;
+  cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, p->device);
+  if (major != 10) return fail(MG_ERR_UNSUPPORTED, "this library is built for sm_100a (B200) only");
+  const mg::HostPlan& h = p->hp;
+  if ((e = upload_vec(p, &p->d_items, h.items)) != cudaSuccess ||
+      (e = upload_vec(p, &p->d_trefs, h.trefs)) != cudaSuccess ||
+      (e = upload_vec(p, &p->d_masks, h.dev_masks)) != cudaSuccess ||
+      (e = upload_vec(p, &p->d_strip_cols, h.strip_cols)) != cudaSuccess ||
+      (e = upload_vec(p, &p->d_global_rows, h.global_rows)) != cudaSuccess ||
+      (e = upload_vec(p, &p->d_fine_slot, h.fine_slot)) != cudaSuccess ||
+      (e = upload_vec(p, &p->d_fine_rows, h.fine_rows)) != cudaSuccess ||
+      (e = upload_vec(p, &p->d_fine_row_ptr, h.fine_row_ptr)) != cudaSuccess ||
+      (e = upload_vec(p, &p->d_fine_col, h.fine_col)) != cudaSuccess ||
+      (e = upload_vec(p, &p->d_counter, std::vector<int32_t>(4, 0))) != cudaSuccess)
+    return e == cudaErrorMemoryAllocation ? fail(MG_ERR_OUT_OF_MEMORY, "device allocation failed")
+                                          : cuda_fail(e, "plan upload");
+  p->uploaded = true;
+  return MG_OK;
+}
+
+mg_status create_impl(int64_t L, int32_t heads, int32_t d, int32_t window, const int32_t* global_idx,
+                      int64_t n_global, const int32_t* extra_idx, int64_t n_extra, const mg_plan_opts* opts,
+                      mg_plan_t* plan_out) {
+  if (!plan_out) return fail(MG_ERR_INVALID_ARG, "plan_out is null");
+  *plan_out = nullptr;
+  mg::PlanOptions po;
+  int sms_override = 0;
+  if (opts) {
+    if (opts->block != 0) po.block = opts->block;
+    po.force_all_fine = opts->force_all_fine != 0;
+    if (opts->strip_max_cols != 0) po.strip_max_cols = opts->strip_max_cols < 0 ? 0 : opts->strip_max_cols;
+    if (po.strip_max_cols > 128) return fail(MG_ERR_INVALID_ARG, "strip_max_cols must be <= 128");
+    if (opts->num_sms < 0) return fail(MG_ERR_INVALID_ARG, "num_sms must be >= 0");
+    sms_override = opts->num_sms;
+  }
+  mg_plan_s* p = new (std::nothrow) mg_plan_s();
+  if (!p) return fail(MG_ERR_OUT_OF_MEMORY, "host allocation failed");
+  bool unsupported = false;
+  std::string err;
+  try {
+    err = mg::build_plan(p->hp, L, heads, d, window, global_idx, n_global, extra_idx, n_extra, po, &unsupported);
+  } catch (const std::bad_alloc&) {
+    delete p;
+    return fail(MG_ERR_OUT_OF_MEMORY, "host allocation failed while building the plan");
+  } catch (...) {
+    delete p;
+    return fail(MG_ERR_INTERNAL, "exception while building the plan");
+  }
+  if (!err.empty()) {
+    delete p;
+    return fail(unsupported ? MG_ERR_UNSUPPORTED : MG_ERR_INVALID_ARG, err);
+  }
+  p->num_sms_override = sms_override;
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess) {
+    ndev = 0;
+    cudaGetLastError();
+  }
+  if (ndev > 0 && p->hp.kernel_ready) {
+    const mg_status s = upload(p);
+    if (s != MG_OK) {
+      delete p;
+      return s;
+    }
+  }
+  *plan_out = p;
+  return MG_OK;
+}
+
+mg_status check_tensor(const mg_tensor* t, const char* name, const mg_plan_s* p, bool host) {
+  const std::string n(name);
+  if (!t) return fail(MG_ERR_INVALID_ARG, n + " is null");
+  if (!t->data) return fail(MG_ERR_INVALID_ARG, n + ".data is null");
+  if (t->dtype != MG_BF16 && t->dtype != MG_FP16) return fail(MG_ERR_INVALID_ARG, n + ".dtype is not bf16/fp16");
+  if (t->batch <= 0) return fail(MG_ERR_INVALID_ARG, n + ".batch must be > 0");
+  if (t->heads != p->hp.heads) return fail(MG_ERR_INVALID_ARG, n + ".heads does not match the plan");
+  if (t->seq_len != p->hp.L) return fail(MG_ERR_INVALID_ARG, n + ".seq_len does not match the plan");
+  if (t->head_dim != p->hp.d) return fail(MG_ERR_INVALID_ARG, n + ".head_dim does not match the plan");
+  if (t->stride_b < 0 || t->stride_h < 0 || t->stride_l < 0) return fail(MG_ERR_INVALID_ARG, n + ": negative stride");
+  if ((t->stride_b % 8) || (t->stride_h % 8) || (t->stride_l % 8))
+    return fail(MG_ERR_INVALID_ARG, n + ": strides must be multiples of 8 elements");
+  if (reinterpret_cast<uintptr_t>(t->data) % 16) return fail(MG_ERR_INVALID_ARG, n + ".data must be 16-byte aligned");
+  if (host) {
+    // host tensors must be dense (either [B,H,L,d] or [B,L,H,d]) so they move as one span
+    const int64_t total = t->batch * t->heads * t->seq_len * t->head_dim;
+    const int64_t span = (t->batch - 1) * t->stride_b + (t->heads - 1) * t->stride_h +
+                         (t->seq_len - 1) * t->stride_l + t->head_dim;
+    if (span != total) return fail(MG_ERR_INVALID_ARG, n + ": host tensors must be dense");
+  }
+  return MG_OK;
+}
+
+mg_status check_all(const mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const mg_tensor* V,
+                    const mg_tensor* O, bool host) {
+  mg_status s;
+  if ((s = check_tensor(Q, "Q", p, host)) != MG_OK || (s = check_tensor(K, "K", p, host)) != MG_OK ||
+      (s = check_tensor(V, "V", p, host)) != MG_OK || (s = check_tensor(O, "O", p, host)) != MG_OK)
+    return s;
+  if (K->batch != Q->batch || V->batch != Q->batch || O->batch != Q->batch)
+    return fail(MG_ERR_INVALID_ARG, "Q/K/V/O batch sizes differ");
+  if (K->dtype != Q->dtype || V->dtype != Q->dtype || O->dtype != Q->dtype)
+    return fail(MG_ERR_UNSUPPORTED, "Q/K/V/O dtypes differ");
+  if (!p->hp.kernel_ready) return fail(MG_ERR_UNSUPPORTED, "the forward requires block == 128");
+  if ((int64_t)Q->batch * p->hp.heads >= (int64_t(1) << 31) / std::max<int64_t>(1, (int64_t)p->hp.items.size()))
+    return fail(MG_ERR_UNSUPPORTED, "batch * heads * work items exceeds int32");
+  return MG_OK;
+}
+
+bool encode_map(CUtensorMap* m, const mg_tensor* t) {
+  auto fn = tensor_map_encoder();
+  if (!fn) return false;
+  const int64_t s16 = 64;  // a harmless stride for extent-1 dimensions
+  cuuint64_t dims[4] = {(cuuint64_t)t->head_dim, (cuuint64_t)t->seq_len, (cuuint64_t)t->heads, (cuuint64_t)t->batch};
+  cuuint64_t strides[3] = {(cuuint64_t)std::max<int64_t>(t->stride_l, s16) * 2,
+                           (cuuint64_t)std::max<int64_t>(t->stride_h, s16) * 2,
+                           (cuuint64_t)std::max<int64_t>(t->stride_b, s16) * 2};
+  cuuint32_t box[4] = {64, 128, 1, 1};
+  cuuint32_t es[4] = {1, 1, 1, 1};
+  const CUtensorMapDataType dt =
+      t->dtype == MG_BF16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16;
+  const CUresult r = fn(m, dt, 4, t->data, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                        CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                        CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  return r == CUDA_SUCCESS;
+}
+
+mg::TensorView view(const mg_tensor* t) {
+  return mg::TensorView{static_cast<uint16_t*>(t->data), t->stride_b, t->stride_h, t->stride_l};
+}
+
+mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const mg_tensor* V, mg_tensor* O,
+                   cudaStream_t stream) {
+  mg_status s = upload(p);
+  if (s != MG_OK) return s;
+  int dev = -1;
+  cudaGetDevice(&dev);
+  if (dev != p->device) return fail(MG_ERR_INVALID_ARG, "the plan was uploaded to another device");
+  const mg::HostPlan& h = p->hp;
+  const bool bf16 = Q->dtype == MG_BF16;
+  const int BH = (int)(Q->batch * h.heads);
+  const int nf = (int)h.fine_rows.size();
+  const float scale_log2 = (float)(1.4426950408889634 / std::sqrt((double)h.d));
+  cudaError_t e;
+  // fp32 partials of the CUDA-core CSR rows that are merged by the coarse epilogue
+  const size_t need = (size_t)BH * nf;
+  if (need > p->part_cap) {
+    if (p->d_part) {
+      if ((e = cudaFreeAsync(p->d_part, stream)) != cudaSuccess) return cuda_fail(e, "cudaFreeAsync");
+      p->d_part = nullptr;
+    }
+    if ((e = cudaMallocAsync(reinterpret_cast<void**>(&p->d_part), need * 66 * sizeof(float), stream)) != cudaSuccess)
+      return e == cudaErrorMemoryAllocation ? fail(MG_ERR_OUT_OF_MEMORY, "workspace allocation failed")
+                                            : cuda_fail(e, "cudaMallocAsync");
+    p->part_cap = need;
+  }
+  float* part_acc = p->d_part;
+  float2* part_ml = reinterpret_cast<float2*>(p->d_part + need * 64);
+
+  cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
+  if (p->profiling) {
+    for (int i = 0; i < 4; ++i)
+      if (!(ev[i] = p->prof_event())) return fail(MG_ERR_CUDA, "cudaEventCreate failed");
+    p->prof_has_fine.push_back(nf > 0);
+    p->prof_has_coarse.push_back(!h.items.empty());
+    cudaEventRecord(ev[0], stream);
+  }
+  if (nf > 0) {
+    mg::FineParams fp{};
+    fp.fine_rows = p->d_fine_rows;
+    fp.row_ptr = p->d_fine_row_ptr;
+    fp.cols = p->d_fine_col;
+    fp.part_acc = part_acc;
+    fp.part_ml = part_ml;
+    fp.q = view(Q); fp.k = view(K); fp.v = view(V); fp.o = view(O);
+    fp.H = h.heads; fp.BH = BH; fp.n_fine_rows = nf;
+    fp.scale_log2 = scale_log2;
+    if ((e = mg::launch_fine(fp, bf16, stream)) != cudaSuccess) return cuda_fail(e, "fine kernel launch");
+  }
+  if (p->profiling) cudaEventRecord(ev[1], stream);
+  if (!h.items.empty()) {
+    CUtensorMap tq, tk, tv;
+    if (!encode_map(&tq, Q) || !encode_map(&tk, K) || !encode_map(&tv, V))
+      return fail(MG_ERR_CUDA, "cuTensorMapEncodeTiled failed (driver entry point unavailable or bad layout)");
+    mg::CoarseParams cp{};
+    cp.items = p->d_items;
+    cp.trefs = p->d_trefs;
+    cp.masks = p->d_masks;
+    cp.strip_cols = p->d_strip_cols;
+    cp.global_rows = p->d_global_rows;
+    cp.fine_slot = p->d_fine_slot;
+    cp.part_acc = part_acc;
+    cp.part_ml = part_ml;
+    cp.counter = p->d_counter;
+    cp.q = view(Q); cp.k = view(K); cp.v = view(V); cp.o = view(O);
+    cp.L = h.L;
+    cp.H = h.heads;
+    cp.BH = BH;
+    cp.n_items = (int)h.items.size();
+    cp.n_dense_items = h.n_dense_items;
+    cp.n_global = (int)h.global_rows.size();
+    cp.n_fine_rows = nf;
+    cp.total_units = cp.n_items * BH;
+    cp.scale_log2 = scale_log2;
+    if ((e = cudaMemsetAsync(p->d_counter, 0, sizeof(int32_t), stream)) != cudaSuccess)
+      return cuda_fail(e, "cudaMemsetAsync");
+    const int sms = p->num_sms_override > 0 ? p->num_sms_override : p->num_sms;
+    const int grid = std::min(sms, cp.total_units);
+    if (p->profiling) cudaEventRecord(ev[2], stream);  // after the counter reset
+    if ((e = mg::launch_coarse(cp, tq, tk, tv, bf16, grid, stream)) != cudaSuccess)
+      return cuda_fail(e, "coarse kernel launch");
+  } else if (p->profiling) {
+    cudaEventRecord(ev[2], stream);
+  }
+  if (p->profiling) cudaEventRecord(ev[3], stream);
+  return MG_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+int32_t mg_abi_version(void) { return MG_ABI_VERSION; }
+
+const char* mg_last_error(void) { return g_err.c_str(); }
+
+mg_status mg_plan_create(int64_t L, int32_t heads, int32_t d, int32_t window, const int32_t* global_idx,
+                         int64_t n_global, const int32_t* extra_idx, int64_t n_extra, mg_plan_t* plan_out) {
+  g_err.clear();
+  return create_impl(L, heads, d, window, global_idx, n_global, extra_idx, n_extra, nullptr, plan_out);
+}
+
+mg_status mg_plan_create_ex(int64_t L, int32_t heads, int32_t d, int32_t window, const int32_t* global_idx,
+                            int64_t n_global, const int32_t* extra_idx, int64_t n_extra, const mg_plan_opts* opts,
+                            mg_plan_t* plan_out) {
+  g_err.clear();
+  return create_impl(L, heads, d, window, global_idx, n_global, extra_idx, n_extra, opts, plan_out);
+}
+
+mg_status mg_plan_destroy(mg_plan_t plan) {
+  g_err.clear();
+  delete plan;
+  return MG_OK;
+}
+
+mg_status mg_plan_info_get(mg_plan_t plan, mg_plan_info* info) {
+  g_err.clear();
+  if (!plan || !info) return fail(MG_ERR_INVALID_ARG, "null argument");
+  const mg::HostPlan& h = plan->hp;
+  std::memset(info, 0, sizeof(*info));
+  info->L = h.L;
+  info->heads = h.heads;
+  info->d = h.d;
+  info->window = h.window;
+  info->block = h.block;
+  info->n_row_blocks = h.nb();
+  info->n_tiles = (int64_t)h.bsr_col.size();
+  info->n_full_tiles = h.n_full_tiles;
+  info->nnz_coarse = h.nnz_coarse;
+  info->nnz_fine = (int64_t)h.csr_col.size();
+  info->n_global = (int64_t)h.global_rows.size();
+  info->nnz_total = h.nnz_coarse + info->nnz_fine + info->n_global * h.L;
+  info->n_fine_rows = (int64_t)h.fine_rows.size();
+  info->nnz_fine_strip = h.nnz_fine_strip;
+  info->nnz_fine_cuda = (int64_t)h.fine_col.size();
+  info->n_items = (int64_t)h.items.size();
+  info->n_strip_tiles = h.n_strip_tiles;
+  info->computed_scores = h.computed_scores;
+  info->kernels_per_fwd = (h.fine_rows.empty() ? 0 : 1) + (h.items.empty() ? 0 : 1);
+  return MG_OK;
+}
+
+mg_status mg_plan_export(mg_plan_t plan, int32_t* bsr_row_ptr, int32_t* bsr_col, uint64_t* tile_masks,
+                         int32_t* csr_row_ptr, int32_t* csr_col, int32_t* global_rows) {
+  g_err.clear();
+  if (!plan) return fail(MG_ERR_INVALID_ARG, "plan is null");
+  const mg::HostPlan& h = plan->hp;
+  auto cp = [](auto* dst, const auto& v) {
+    if (dst && !v.empty()) std::memcpy(dst, v.data(), v.size() * sizeof(v[0]));
+  };
+  cp(bsr_row_ptr, h.bsr_row_ptr);
+  cp(bsr_col, h.bsr_col);
+  cp(tile_masks, h.tile_masks);
+  cp(csr_row_ptr, h.csr_row_ptr);
+  cp(csr_col, h.csr_col);
+  cp(global_rows, h.global_rows);
+  return MG_OK;
+}
+
+mg_status mg_sparse_attention_fwd(mg_plan_t plan, const mg_tensor* Q, const mg_tensor* K, const mg_tensor* V,
+                                  mg_tensor* O, void* stream) {
+  g_err.clear();
+  if (!plan) return fail(MG_ERR_INVALID_ARG, "plan is null");
+  mg_status s = check_all(plan, Q, K, V, O, false);
+  if (s != MG_OK) return s;
+  return fwd_impl(plan, Q, K, V, O, static_cast<cudaStream_t>(stream));
+}
+
+mg_status mg_sparse_attention_fwd_host(mg_plan_t plan, const mg_tensor* Q, const mg_tensor* K, const mg_tensor* V,
+                                       mg_tensor* O, void* stream_) {
+  g_err.clear();
+  if (!plan) return fail(MG_ERR_INVALID_ARG, "plan is null");
+  mg_status s = check_all(plan, Q, K, V, O, true);
+  if (s != MG_OK) return s;
+  if ((s = upload(plan)) != MG_OK) return s;
+  cudaStream_t stream = static_cast<cudaStream_t>(stream_);
+  const size_t bytes = (size_t)Q->batch * Q->heads * Q->seq_len * Q->head_dim * 2;
+  cudaError_t e;
+  if (4 * bytes > plan->stage_cap) {
+    if (plan->d_stage) {
+      if ((e = cudaFreeAsync(plan->d_stage, stream)) != cudaSuccess) return cuda_fail(e, "cudaFreeAsync");
+      plan->d_stage = nullptr;
+    }
+    if ((e = cudaMallocAsync(reinterpret_cast<void**>(&plan->d_stage), 4 * bytes, stream)) != cudaSuccess)
+      return e == cudaErrorMemoryAllocation ? fail(MG_ERR_OUT_OF_MEMORY, "staging allocation failed")
+                                            : cuda_fail(e, "cudaMallocAsync");
+    plan->stage_cap = 4 * bytes;
+  }
+  mg_tensor dq = *Q, dk = *K, dv = *V, dO = *O;
+  dq.data = plan->d_stage;
+  dk.data = plan->d_stage + bytes;
+  dv.data = plan->d_stage + 2 * bytes;
+  dO.data = plan->d_stage + 3 * bytes;
+  if ((e = cudaMemcpyAsync(dq.data, Q->data, bytes, cudaMemcpyHostToDevice, stream)) != cudaSuccess ||
+      (e = cudaMemcpyAsync(dk.data, K->data, bytes, cudaMemcpyHostToDevice, stream)) != cudaSuccess ||
+      (e = cudaMemcpyAsync(dv.data, V->data, bytes, cudaMemcpyHostToDevice, stream)) != cudaSuccess)
+    return cuda_fail(e, "H2D copy");
+  if ((s = fwd_impl(plan, &dq, &dk, &dv, &dO, stream)) != MG_OK) return s;
+  if ((e = cudaMemcpyAsync(O->data, dO.data, bytes, cudaMemcpyDeviceToHost, stream)) != cudaSuccess)
+    return cuda_fail(e, "D2H copy");
+  return MG_OK;
+}
+
+mg_status mg_plan_set_profiling(mg_plan_t plan, int32_t enable) {
+  g_err.clear();
+  if (!plan) return fail(MG_ERR_INVALID_ARG, "plan is null");
+  plan->profiling = enable != 0;
+  plan->prof_used = 0;
+  plan->prof_has_fine.clear();
+  plan->prof_has_coarse.clear();
+  return MG_OK;
+}
+
+mg_status mg_plan_get_profile(mg_plan_t plan, mg_profile* out) {
+  g_err.clear();
+  if (!plan || !out) return fail(MG_ERR_INVALID_ARG, "null argument");
+  std::memset(out, 0, sizeof(*out));
+  const size_t calls = plan->prof_used / 4;
+  for (size_t c = 0; c < calls; ++c) {
+    cudaEvent_t* ev = plan->prof_events.data() + 4 * c;
+    cudaError_t e = cudaEventSynchronize(ev[3]);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaEventSynchronize");
+    float a = 0.f, b = 0.f, t = 0.f;
+    cudaEventElapsedTime(&a, ev[0], ev[1]);
+    cudaEventElapsedTime(&b, ev[2], ev[3]);
+    cudaEventElapsedTime(&t, ev[0], ev[3]);
+    if (plan->prof_has_fine[c]) out->fine_ms += a;
+    if (plan->prof_has_coarse[c]) out->coarse_ms += b;
+    out->total_ms += t;
+  }
+  out->calls = (int64_t)calls;
+  plan->prof_used = 0;
+  plan->prof_has_fine.clear();
+  plan->prof_has_coarse.clear();
+  return MG_OK;
+}
+
+mg_status mg_selftest_umma(int32_t mode, const void* A, const void* B, float* D, void* stream) {
+  g_err.clear();
+  if (!A || !B || !D || (mode != 0 && mode != 1)) return fail(MG_ERR_INVALID_ARG, "bad selftest arguments");
+  const cudaError_t e = mg::launch_selftest_umma(mode, A, B, D, static_cast<cudaStream_t>(stream));
+  return e == cudaSuccess ? MG_OK : cuda_fail(e, "selftest launch");
+}
+
+}  // extern "C"

@@ -1,0 +1,56 @@
+// Device-side parameter blocks and launchers of the Multigrain forward kernels (sm_100a).
+#pragma once
+
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <cstdint>
+
+#include "plan.hpp"
+
+namespace mg {
+
+// Strided [B, H, L, 64] 16-bit tensor view (element strides).
+struct TensorView {
+  uint16_t* data;
+  int64_t sb, sh, sl;
+};
+
+// Coarse / dense-row / strip kernel: tcgen05 SDDMM -> online SpSoftmax -> tcgen05 SpMM,
+// persistent over (item, batch*head) units. See coarse_sm100.cu.
+struct CoarseParams {
+  const Item* items;
+  const TileRef* trefs;
+  const uint64_t* masks;
+  const int32_t* strip_cols;
+  const int32_t* global_rows;
+  const int32_t* fine_slot;   // [L]; >= 0: merge fine partial of that slot
+  const float* part_acc;      // [BH * n_fine_rows * 64]
+  const float2* part_ml;      // [BH * n_fine_rows]  (max in raw score units, sum)
+  int32_t* counter;           // work counter (zeroed before launch)
+  TensorView q, k, v, o;
+  int64_t L;
+  int32_t H, BH;
+  int32_t n_items, n_dense_items;
+  int32_t n_global, n_fine_rows;
+  int32_t total_units;
+  float scale_log2;           // (1/sqrt(d)) * log2(e)
+};
+
+// Fine CSR kernel: warp per (row, batch*head); SDDMM -> online softmax -> SpMM on CUDA cores.
+struct FineParams {
+  const int32_t* fine_rows;    // row | (final << 31)
+  const int32_t* row_ptr;      // [n_fine_rows + 1]
+  const int32_t* cols;
+  float* part_acc;
+  float2* part_ml;
+  TensorView q, k, v, o;
+  int32_t H, BH, n_fine_rows;
+  float scale_log2;
+};
+
+cudaError_t launch_coarse(const CoarseParams& p, const CUtensorMap& tmq, const CUtensorMap& tmk,
+                          const CUtensorMap& tmv, bool bf16, int grid, cudaStream_t stream);
+cudaError_t launch_fine(const FineParams& p, bool bf16, cudaStream_t stream);
+cudaError_t launch_selftest_umma(int mode, const void* A, const void* B, float* D, cudaStream_t stream);
+
+}  // namespace mg

@@ -1,0 +1,235 @@
+// Host plan builder. See plan.hpp and DESIGN.md §3-§5.
+//
+// Canonical partition (must be bit-identical to oracle/plan.py; readings A2-A7):
+//   M(r,c) = |r-c| <= w/2 or G[r] or G[c] or (r,c) in E
+//   T = {(I,J): some non-global r in row block I has band columns in column block J}
+//       ("local pattern -> coarse BSR"; tau = 0)
+//   tile bits = M restricted to the tile, global rows cleared
+//   CSR = non-global union elements outside T ("selected -> fine CSR")
+#include "plan.hpp"
+
+#include <algorithm>
+#include <cstring>
+
+namespace mg {
+
+namespace {
+
+inline int popcount64(uint64_t x) { return __builtin_popcountll(x); }
+
+}  // namespace
+
+std::string build_plan(HostPlan& p, int64_t L, int32_t heads, int32_t d, int32_t window,
+                       const int32_t* global_idx, int64_t n_global, const int32_t* extra_idx,
+                       int64_t n_extra, const PlanOptions& opts, bool* unsupported) {
+  *unsupported = false;
+  if (L <= 0) return "L must be > 0";
+  if (heads <= 0) return "heads must be > 0";
+  if (d <= 0) return "d must be > 0";
+  if (window < 0 || (window & 1)) return "window must be >= 0 and even";
+  if (n_global < 0 || n_extra < 0) return "negative index count";
+  if (n_global > 0 && !global_idx) return "global_idx is null";
+  if (n_extra > 0 && !extra_idx) return "extra_idx is null";
+  const int b = opts.block;
+  if (b < 1 || (b > 64 && b % 64) || b > 1024) return "block must be <= 64 or a multiple of 64 (<= 1024)";
+  if (d != 64) { *unsupported = true; return "v1 supports head_dim == 64 only"; }
+  for (int64_t i = 0; i < n_global; ++i)
+    if (global_idx[i] < 0 || global_idx[i] >= L) return "global index out of range";
+  for (int64_t i = 0; i < 2 * n_extra; ++i)
+    if (extra_idx[i] < 0 || extra_idx[i] >= L) return "extra index out of range";
+
+  p = HostPlan();
+  p.L = L; p.heads = heads; p.d = d; p.window = window; p.block = b; p.opts = opts;
+  const int64_t w1 = window / 2;
+  const int64_t nb = p.nb();
+  const int wpr = p.wpr();
+
+  // ---- global rows: sorted unique
+  std::vector<uint8_t> isG(L, 0);
+  for (int64_t i = 0; i < n_global; ++i) isG[global_idx[i]] = 1;
+  for (int64_t r = 0; r < L; ++r) if (isG[r]) p.global_rows.push_back((int32_t)r);
+  const std::vector<int32_t>& gcols = p.global_rows;
+
+  // ---- extras: set semantics, grouped by row
+  std::vector<int64_t> keys(n_extra);
+  for (int64_t i = 0; i < n_extra; ++i) keys[i] = (int64_t)extra_idx[2 * i] * L + extra_idx[2 * i + 1];
+  std::sort(keys.begin(), keys.end());
+  keys.erase(std::unique(keys.begin(), keys.end()), keys.end());
+  std::vector<int64_t> ext_ptr(L + 1, 0);
+  for (int64_t k : keys) ext_ptr[k / L + 1]++;
+  for (int64_t r = 0; r < L; ++r) ext_ptr[r + 1] += ext_ptr[r];
+
+  // ---- per row block: tiles, bits, CSR
+  std::vector<int32_t> tile_of_J(nb, -1);
+  std::vector<int64_t> csr_ptr(L + 1, 0);
+  p.bsr_row_ptr.push_back(0);
+  std::vector<int32_t> outside;  // scratch: sorted off-band columns of one row
+  for (int64_t I = 0; I < nb; ++I) {
+    const int64_t r0 = I * b, r1 = std::min<int64_t>(L, r0 + b);
+    std::vector<uint8_t> inT(nb, 0);
+    if (!opts.force_all_fine) {
+      for (int64_t r = r0; r < r1; ++r) {
+        if (isG[r]) continue;
+        const int64_t jlo = std::max<int64_t>(0, r - w1) / b;
+        const int64_t jhi = std::min<int64_t>(L - 1, r + w1) / b;
+        for (int64_t J = jlo; J <= jhi; ++J) inT[J] = 1;
+      }
+    }
+    const int64_t tbase = (int64_t)p.bsr_col.size();
+    for (int64_t J = 0; J < nb; ++J) {
+      tile_of_J[J] = -1;
+      if (inT[J]) { tile_of_J[J] = (int32_t)p.bsr_col.size(); p.bsr_col.push_back((int32_t)J); }
+    }
+    p.bsr_row_ptr.push_back((int32_t)p.bsr_col.size());
+    p.tile_masks.resize(p.bsr_col.size() * (size_t)b * wpr, 0ull);
+    (void)tbase;
+
+    for (int64_t r = r0; r < r1; ++r) {
+      if (isG[r]) continue;  // global rows: owned by the dense-row part
+      const int64_t a = r - r0;
+      auto take = [&](int64_t c) {  // c is a union column of row r
+        const int64_t J = c / b;
+        const int32_t t = tile_of_J[J];
+        if (t >= 0) {
+          const int64_t beta = c - J * b;
+          p.tile_masks[((size_t)t * b + a) * wpr + beta / 64] |= 1ull << (beta % 64);
+        } else {
+          p.csr_col.push_back((int32_t)c);
+          csr_ptr[r + 1]++;
+        }
+      };
+      const int64_t lo = std::max<int64_t>(0, r - w1), hi = std::min<int64_t>(L - 1, r + w1);
+      // off-band columns from globals and extras, merged ascending, unique
+      outside.clear();
+      size_t gi = 0;
+      int64_t ei = ext_ptr[r], ee = ext_ptr[r + 1];
+      while (gi < gcols.size() || ei < ee) {
+        int64_t c;
+        if (ei >= ee || (gi < gcols.size() && gcols[gi] <= keys[ei] % L)) {
+          c = gcols[gi++];
+          if (ei < ee && keys[ei] % L == c) ++ei;
+        } else {
+          c = keys[ei++] % L;
+        }
+        if (c < lo || c > hi) outside.push_back((int32_t)c);
+      }
+      // emit in ascending column order: outside-left, band, outside-right
+      size_t oi = 0;
+      while (oi < outside.size() && outside[oi] < lo) take(outside[oi++]);
+      for (int64_t c = lo; c <= hi; ++c) take(c);
+      while (oi < outside.size()) take(outside[oi++]);
+    }
+  }
+  for (int64_t r = 0; r < L; ++r) csr_ptr[r + 1] += csr_ptr[r];
+  if (csr_ptr[L] >= (int64_t(1) << 31)) { *unsupported = true; return "CSR nnz >= 2^31"; }
+  p.csr_row_ptr.assign(csr_ptr.begin(), csr_ptr.end());
+
+  const int64_t nt = (int64_t)p.bsr_col.size();
+  for (int64_t t = 0; t < nt; ++t) {
+    int64_t pc = 0;
+    for (int64_t w = 0; w < (int64_t)b * wpr; ++w) pc += popcount64(p.tile_masks[t * b * wpr + w]);
+    p.nnz_coarse += pc;
+    if (pc == (int64_t)b * b) p.n_full_tiles++;
+  }
+
+  // ---- kernel-side structures (tcgen05 path needs b == 128)
+  if (b != 128) return "";
+  p.kernel_ready = true;
+  const int64_t B = 128;
+  p.dev_masks.assign(p.tile_masks.begin(), p.tile_masks.end());  // 256 words per tile
+  std::vector<uint8_t> tile_full(nt, 0);
+  for (int64_t t = 0; t < nt; ++t) {
+    bool full = true;
+    for (int w = 0; w < 256 && full; ++w) full = p.tile_masks[t * 256 + w] == ~0ull;
+    tile_full[t] = full;
+  }
+  auto new_mask = [&]() -> int32_t {
+    const int32_t id = (int32_t)(p.dev_masks.size() / 256);
+    p.dev_masks.resize(p.dev_masks.size() + 256, 0ull);
+    return id;
+  };
+
+  // dense items (global rows), 128 gathered rows each, every column tile
+  int32_t ragged_mask = -1;
+  if (L % B) {
+    ragged_mask = new_mask();
+    const int64_t valid = L - (nb - 1) * B;
+    for (int a = 0; a < 128; ++a)
+      for (int64_t c = 0; c < valid; ++c) p.dev_masks[(size_t)ragged_mask * 256 + a * 2 + c / 64] |= 1ull << (c % 64);
+  }
+  const int64_t G = (int64_t)p.global_rows.size();
+  for (int64_t k = 0; k < G; k += 128) {
+    Item it{1, (int32_t)k, (int32_t)nb, (int32_t)p.trefs.size()};
+    for (int64_t J = 0; J < nb; ++J)
+      p.trefs.push_back(TileRef{(int32_t)(J * B), (J == nb - 1) ? ragged_mask : -1, 128, 0});
+    p.items.push_back(it);
+    p.computed_scores += nb * B * B;
+  }
+  p.n_dense_items = (int32_t)p.items.size();
+
+  // band items and the CSR residual split (tensor-core strip vs CUDA-core rows)
+  p.fine_slot.assign(L, -1);
+  std::vector<int32_t> cuda_rows;      // rows run by the fine kernel
+  std::vector<uint8_t> cuda_final;     // 1 = the fine kernel writes O (no coarse part in the row block)
+  const int strip_max = opts.strip_max_cols;
+  for (int64_t I = 0; I < nb; ++I) {
+    const int64_t r0 = I * B, r1 = std::min<int64_t>(L, r0 + B);
+    const int32_t tb = p.bsr_row_ptr[I], te = p.bsr_row_ptr[I + 1];
+    const bool has_tiles = te > tb;
+    // distinct CSR columns of this row block
+    std::vector<int32_t> cols;
+    for (int64_t r = r0; r < r1; ++r)
+      cols.insert(cols.end(), p.csr_col.begin() + p.csr_row_ptr[r], p.csr_col.begin() + p.csr_row_ptr[r + 1]);
+    std::sort(cols.begin(), cols.end());
+    cols.erase(std::unique(cols.begin(), cols.end()), cols.end());
+    const bool use_strip = has_tiles && !cols.empty() && strip_max > 0 && (int)cols.size() <= strip_max;
+    if (has_tiles) {
+      Item it{0, (int32_t)r0, te - tb + (use_strip ? 1 : 0), (int32_t)p.trefs.size()};
+      for (int32_t t = tb; t < te; ++t) {
+        p.trefs.push_back(TileRef{p.bsr_col[t] * (int32_t)B, tile_full[t] ? -1 : t, 128, 0});
+        p.computed_scores += B * B;
+      }
+      if (use_strip) {
+        const int ncols = (int)((cols.size() + 31) / 32 * 32);
+        const int32_t off = (int32_t)p.strip_cols.size();
+        for (int i = 0; i < ncols; ++i) p.strip_cols.push_back(i < (int)cols.size() ? cols[i] : -1);
+        const int32_t m = new_mask();
+        bool full = true;
+        for (int64_t r = r0; r < r0 + B; ++r) {
+          const int64_t a = r - r0;
+          if (r >= r1) { full = false; continue; }
+          const int32_t* cb = p.csr_col.data() + p.csr_row_ptr[r];
+          const int32_t* ce = p.csr_col.data() + p.csr_row_ptr[r + 1];
+          if (ce - cb != ncols) full = false;
+          for (const int32_t* c = cb; c != ce; ++c) {
+            const int64_t beta = std::lower_bound(cols.begin(), cols.end(), *c) - cols.begin();
+            p.dev_masks[(size_t)m * 256 + a * 2 + beta / 64] |= 1ull << (beta % 64);
+          }
+          p.nnz_fine_strip += ce - cb;
+        }
+        p.trefs.push_back(TileRef{off, full ? -1 : m, ncols, 1});
+        p.n_strip_tiles++;
+        p.computed_scores += B * ncols;
+      }
+      p.items.push_back(it);
+    }
+    if (!use_strip) {
+      for (int64_t r = r0; r < r1; ++r) {
+        if (p.csr_row_ptr[r + 1] == p.csr_row_ptr[r]) continue;
+        if (has_tiles) p.fine_slot[r] = (int32_t)cuda_rows.size();
+        cuda_rows.push_back((int32_t)r);
+        cuda_final.push_back(has_tiles ? 0 : 1);
+      }
+    }
+  }
+  p.fine_row_ptr.push_back(0);
+  for (size_t i = 0; i < cuda_rows.size(); ++i) {
+    const int32_t r = cuda_rows[i];
+    p.fine_col.insert(p.fine_col.end(), p.csr_col.begin() + p.csr_row_ptr[r], p.csr_col.begin() + p.csr_row_ptr[r + 1]);
+    p.fine_row_ptr.push_back((int32_t)p.fine_col.size());
+    p.fine_rows.push_back(r | (cuda_final[i] ? (int32_t)0x80000000 : 0));
+  }
+  return "";
+}
+
+}  // namespace mg

@@ -1,0 +1,59 @@
+// Host-side Multigrain plan: canonical coarse/fine/dense-row partition + kernel work lists.
+// Paper: P:94-96 (§3.1 steps 1-2, metadata generated before inference), P:101 (local ->
+// coarse BSR, selected -> fine CSR), P:103/P:133 (global rows dense and independent),
+// P:126 (overlap invalidated). Rules: DESIGN.md §3 (O-3).
+#pragma once
+
+#include <cstdint>
+#include <string>
+#include <vector>
+
+namespace mg {
+
+struct PlanOptions {
+  int block = 128;
+  bool force_all_fine = false;
+  int strip_max_cols = 128;  // <= 0 disables the tensor-core strip path for the CSR residual
+};
+
+// Device work-list encodings.
+//   Item  {kind, row0, ntiles, tref_begin}: kind 0 = band row block starting at row0;
+//         kind 1 = gathered dense global rows global_rows[row0 .. row0+128) (ntiles = nb).
+//   TileRef {arg, mask, ncols, kind}: kind 0 = contiguous column tile at column `arg`;
+//         kind 1 = gathered strip whose column list starts at strip_cols[arg];
+//         mask = index of a 128 x 2-word bitmask or -1 for "all valid".
+struct Item { int32_t kind, row0, ntiles, tref_begin; };
+struct TileRef { int32_t arg, mask, ncols, kind; };
+
+struct HostPlan {
+  // inputs
+  int64_t L = 0;
+  int32_t heads = 0, d = 0, window = 0, block = 128;
+  PlanOptions opts;
+  // canonical partition (exported, bit-exact vs oracle)
+  std::vector<int32_t> global_rows, bsr_row_ptr, bsr_col, csr_row_ptr, csr_col;
+  std::vector<uint64_t> tile_masks;  // n_tiles * block * wpr
+  int64_t nnz_coarse = 0, n_full_tiles = 0;
+  // kernel-side structures (built only when block == 128)
+  bool kernel_ready = false;
+  std::vector<uint64_t> dev_masks;   // 128 x 2 words per entry: tiles, then strip/ragged masks
+  std::vector<Item> items;           // dense items first, then band items in row-block order
+  int32_t n_dense_items = 0;
+  std::vector<TileRef> trefs;
+  std::vector<int32_t> strip_cols;   // gathered column lists (padded with -1)
+  std::vector<int32_t> fine_rows;    // rows executed by the CUDA-core fine kernel; bit 31 = write final O
+  std::vector<int32_t> fine_slot;    // per row: index into fine_rows for partial merge, or -1
+  std::vector<int32_t> fine_row_ptr; // compacted CSR (cuda part only) [n_fine_rows + 1]
+  std::vector<int32_t> fine_col;
+  int64_t nnz_fine_strip = 0, n_strip_tiles = 0, computed_scores = 0;
+
+  int64_t nb() const { return (L + block - 1) / block; }
+  int wpr() const { return (block + 63) / 64; }
+};
+
+// Returns "" on success, else an error message; *unsupported is set for UNSUPPORTED errors.
+std::string build_plan(HostPlan& p, int64_t L, int32_t heads, int32_t d, int32_t window,
+                       const int32_t* global_idx, int64_t n_global, const int32_t* extra_idx,
+                       int64_t n_extra, const PlanOptions& opts, bool* unsupported);
+
+}  // namespace mg

@@ -1,0 +1,162 @@
+"""C-ABI library tests that need no GPU.
+
+* libmg.so loads and exports every symbol include/mg.h declares;
+* mg_plan_export is bit-identical to the oracle's canonical plan (O-3) on every BASELINE config
+  at b = 64 and 128, on random tiny patterns at small b, and on ragged L;
+* every validation branch of mg_plan_create returns its documented status;
+* mg_plan_info counts match the closed forms / oracle.
+"""
+import os
+import re
+
+import numpy as np
+import pytest
+
+import paper_conf_iiswc_lica22_b200 as mg
+from paper_conf_iiswc_lica22_b200 import _lib
+from oracle import canonical_plan, union_mask_dense
+from workloads import get_config, random_small_config
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def header_symbols():
+    src = open(os.path.join(ROOT, "include", "mg.h")).read()
+    return sorted(set(re.findall(r"^MG_API\s+[\w\s\*]+?\b(mg_\w+)\s*\(", src, flags=re.M)))
+
+
+def test_library_loads_and_exports_header_symbols():
+    lib = mg.load_library()
+    names = header_symbols()
+    assert len(names) >= 10
+    assert sorted(_lib.EXPORTED) == names
+    for n in names:
+        assert hasattr(lib, n), n
+    assert lib.mg_abi_version() == 1
+
+
+def compare(plan: "mg.Plan", L, window, G, E, b):
+    ref = canonical_plan(L, window, G, E, b)
+    got = plan.export()
+    assert np.array_equal(got["bsr_row_ptr"], ref.bsr_row_ptr)
+    assert np.array_equal(got["bsr_col"], ref.bsr_col)
+    assert np.array_equal(got["tile_masks"], ref.tile_masks)
+    assert np.array_equal(got["csr_row_ptr"], ref.csr_row_ptr)
+    assert np.array_equal(got["csr_col"], ref.csr_col)
+    assert np.array_equal(got["global_rows"], ref.global_rows)
+    inf = plan.info()
+    assert inf["n_tiles"] == ref.n_tiles
+    assert inf["n_full_tiles"] == ref.n_full_tiles()
+    assert inf["nnz_coarse"] == int(ref.tile_popcount().sum())
+    assert inf["nnz_fine"] == ref.csr_col.size
+    return inf
+
+
+@pytest.mark.parametrize("cfg", ["C1", "C2", "C3"])
+@pytest.mark.parametrize("b", [64, 128])
+def test_plan_export_matches_oracle_configs(cfg, b):
+    c = get_config(cfg)
+    p = mg.Plan(c.L, c.H, c.d, c.window, c.global_idx, c.extra_idx, block=b)
+    inf = compare(p, c.L, c.window, c.global_idx, c.extra_idx, b)
+    M_count = {"C1": 34_074, "C2": 2_280_160, "C3": 738_658}[cfg]
+    assert inf["nnz_total"] == M_count
+
+
+@pytest.mark.slow
+def test_plan_export_matches_oracle_c4():
+    c = get_config("C4")
+    p = mg.Plan(c.L, c.H, c.d, c.window, c.global_idx, c.extra_idx)
+    inf = compare(p, c.L, c.window, c.global_idx, c.extra_idx, 128)
+    assert inf["nnz_total"] == 11_026_176
+
+
+@pytest.mark.parametrize("seed", range(30))
+def test_plan_export_matches_oracle_random(seed):
+    rng = np.random.default_rng(500 + seed)
+    L, window, G, E = random_small_config(rng, 70)
+    b = int(rng.choice([1, 2, 4, 8, 16, 64]))
+    p = mg.Plan(L, 2, 64, window, G, E, block=b)
+    compare(p, L, window, G, E, b)
+
+
+@pytest.mark.parametrize("L,window,G", [(300, 40, [0, 5, 299]), (129, 0, []), (1000, 200, [17]), (128, 254, [0])])
+def test_plan_export_ragged_and_edges(L, window, G):
+    rng = np.random.default_rng(L)
+    E = rng.integers(0, L, size=(50, 2))
+    p = mg.Plan(L, 1, 64, window, G, E)
+    compare(p, L, window, G, E, 128)
+
+
+def test_force_all_fine_partition():
+    c = get_config("C1")
+    p = mg.Plan(c.L, 1, 64, c.window, c.global_idx, c.extra_idx, force_all_fine=True)
+    inf = p.info()
+    assert inf["n_tiles"] == 0
+    M = union_mask_dense(c.L, c.window, c.global_idx, c.extra_idx)
+    assert inf["nnz_fine"] + len(c.global_idx) * c.L == M.sum()
+    exp = p.export()
+    for r in range(c.L):
+        cols = exp["csr_col"][exp["csr_row_ptr"][r]:exp["csr_row_ptr"][r + 1]]
+        if r in set(c.global_idx.tolist()):
+            assert cols.size == 0
+        else:
+            assert np.array_equal(cols, np.nonzero(M[r])[0])
+
+
+def test_strip_partition_counts():
+    c = get_config("C2")
+    p = mg.Plan(c.L, c.H, c.d, c.window, c.global_idx, c.extra_idx)
+    inf = p.info()
+    # C2's CSR residual is the 32 global columns outside band tiles: every row block carries it as a strip
+    assert inf["nnz_fine_strip"] == inf["nnz_fine"] == 118_784
+    assert inf["nnz_fine_cuda"] == 0 and inf["kernels_per_fwd"] == 1
+    p2 = mg.Plan(c.L, c.H, c.d, c.window, c.global_idx, c.extra_idx, strip_max_cols=-1)
+    inf2 = p2.info()
+    assert inf2["nnz_fine_strip"] == 0 and inf2["nnz_fine_cuda"] == 118_784 and inf2["kernels_per_fwd"] == 2
+
+
+def status_of(fn):
+    with pytest.raises(mg.MGError) as ei:
+        fn()
+    return ei.value.status
+
+
+@pytest.mark.parametrize("kwargs,status", [
+    (dict(L=0, heads=1, d=64, window=2), _lib.MG_ERR_INVALID_ARG),
+    (dict(L=64, heads=0, d=64, window=2), _lib.MG_ERR_INVALID_ARG),
+    (dict(L=64, heads=1, d=0, window=2), _lib.MG_ERR_INVALID_ARG),
+    (dict(L=64, heads=1, d=64, window=3), _lib.MG_ERR_INVALID_ARG),
+    (dict(L=64, heads=1, d=64, window=-2), _lib.MG_ERR_INVALID_ARG),
+    (dict(L=64, heads=1, d=64, window=2, global_idx=[64]), _lib.MG_ERR_INVALID_ARG),
+    (dict(L=64, heads=1, d=64, window=2, global_idx=[-1]), _lib.MG_ERR_INVALID_ARG),
+    (dict(L=64, heads=1, d=64, window=2, extra_idx=[[0, 64]]), _lib.MG_ERR_INVALID_ARG),
+    (dict(L=64, heads=1, d=64, window=2, extra_idx=[[-3, 1]]), _lib.MG_ERR_INVALID_ARG),
+    (dict(L=64, heads=1, d=128, window=2), _lib.MG_ERR_UNSUPPORTED),
+    (dict(L=64, heads=1, d=64, window=2, block=96), _lib.MG_ERR_INVALID_ARG),
+    (dict(L=64, heads=1, d=64, window=2, strip_max_cols=256), _lib.MG_ERR_INVALID_ARG),
+])
+def test_plan_create_validation(kwargs, status):
+    assert status_of(lambda: mg.Plan(**kwargs)) == status
+
+
+def test_null_arguments_via_ctypes():
+    import ctypes as C
+    lib = mg.load_library()
+    assert lib.mg_plan_create(16, 1, 64, 2, None, 3, None, 0, None) == _lib.MG_ERR_INVALID_ARG
+    h = C.c_void_p()
+    assert lib.mg_plan_create(16, 1, 64, 2, None, 3, None, 0, C.byref(h)) == _lib.MG_ERR_INVALID_ARG
+    assert b"null" in lib.mg_last_error()
+    assert lib.mg_plan_create(16, 1, 64, 2, None, 0, None, 2, C.byref(h)) == _lib.MG_ERR_INVALID_ARG
+    assert lib.mg_plan_info_get(None, None) == _lib.MG_ERR_INVALID_ARG
+    assert lib.mg_plan_destroy(None) == _lib.MG_OK
+    assert lib.mg_sparse_attention_fwd(None, None, None, None, None, None) == _lib.MG_ERR_INVALID_ARG
+
+
+def test_duplicates_collapse():
+    G = [3, 3, 9]
+    E = [[1, 40], [1, 40], [40, 1]]
+    p1 = mg.Plan(64, 1, 64, 4, G, E, block=8)
+    p2 = mg.Plan(64, 1, 64, 4, [9, 3], [[40, 1], [1, 40]], block=8)
+    a, b = p1.export(), p2.export()
+    for k in a:
+        assert np.array_equal(a[k], b[k]), k

@@ -1,0 +1,201 @@
+"""GPU parity: the CUDA path (through the C ABI) vs the fp64 oracle on the same seeded inputs.
+
+Bar (BASELINE.json north_star): outputs in bf16/fp16 with fp32 accumulation within max-abs 2e-2
+and mean-abs 2e-3 of the fp64 oracle. Element-by-element at sizes the oracle finishes in seconds
+(several 128-row tiles and ragged tails); sampled rows at the BASELINE full sizes in the same
+launch configuration bench.py times.
+"""
+import numpy as np
+import pytest
+import torch
+
+import paper_conf_iiswc_lica22_b200 as mg
+from oracle import (ExtraIndex, attention_rows, dense_masked_attention, global_flags, head_inputs_f64)
+from workloads import bits_to_f64, get_config, make_qkv, random_residual
+from gpu_util import TOL_MAX, TOL_MEAN, err_stats, from_device, to_device
+
+pytestmark = pytest.mark.gpu
+
+
+def run_gpu(plan, q, k, v, dtype="bf16", layout="bhld"):
+    Q, K, V = (to_device(x, dtype) for x in (q, k, v))
+    if layout == "blhd":
+        # physical [B, L, H, d], passed as a [B, H, L, d] strided view (L x D_m hidden states)
+        Q, K, V = (x.transpose(1, 2).contiguous().transpose(1, 2) for x in (Q, K, V))
+        O = torch.empty_like(Q.transpose(1, 2)).transpose(1, 2)
+    else:
+        O = torch.empty_like(Q)
+    out = mg.sparse_attention_fwd(plan, Q, K, V, O)
+    torch.cuda.synchronize()
+    return from_device(out)
+
+
+def oracle_full(q, k, v, window, G, E, dtype="bf16"):
+    B, H, L, d = q.shape
+    ref = np.zeros((B, H, L, d))
+    for b in range(B):
+        for h in range(H):
+            Q, K, V = head_inputs_f64(q, k, v, b, h, dtype)
+            ref[b, h] = dense_masked_attention(Q, K, V, window, G, E)
+    return ref
+
+
+def check(got, ref, tol_max=TOL_MAX, tol_mean=TOL_MEAN):
+    mx, mean = err_stats(got, ref)
+    assert np.isfinite(got).all()
+    assert mx <= tol_max and mean <= tol_mean, (mx, mean)
+    return mx, mean
+
+
+@pytest.mark.parametrize("dist", ["normal", "peaky", "adversarial"])
+def test_c1_full(dist):
+    c = get_config("C1")
+    q, k, v = make_qkv(c.B, c.H, c.L, c.d, seed=c.seed, dist=dist, global_idx=c.global_idx)
+    plan = mg.Plan(c.L, c.H, c.d, c.window, c.global_idx, c.extra_idx)
+    got = run_gpu(plan, q, k, v)
+    ref = oracle_full(q, k, v, c.window, c.global_idx, c.extra_idx)
+    if dist == "peaky":
+        check(got, ref, tol_max=2e-2 * max(1.0, np.abs(ref).max() / 4))
+    else:
+        check(got, ref)
+
+
+MIXED = dict(B=2, H=3, L=1024, window=128, G=np.array([0, 1, 2, 130, 777], np.int32))
+
+
+def mixed_extra(L, seed=3, per_row=6):
+    return random_residual(L, 128, per_row, seed=seed)
+
+
+@pytest.mark.parametrize("strip", [0, -1])
+@pytest.mark.parametrize("all_fine", [False, True])
+def test_mixed_pattern_all_parts(strip, all_fine):
+    """Band tiles + strip tiles or CUDA-core CSR rows + dense global rows, several heads."""
+    m = MIXED
+    E = mixed_extra(m["L"])
+    q, k, v = make_qkv(m["B"], m["H"], m["L"], 64, seed=5, dist="adversarial", global_idx=m["G"])
+    plan = mg.Plan(m["L"], m["H"], 64, m["window"], m["G"], E, strip_max_cols=strip, force_all_fine=all_fine)
+    inf = plan.info()
+    if all_fine:
+        assert inf["n_tiles"] == 0 and inf["nnz_fine_cuda"] == inf["nnz_fine"]
+    got = run_gpu(plan, q, k, v)
+    ref = oracle_full(q, k, v, m["window"], m["G"], E)
+    check(got, ref)
+
+
+def test_strip_path_c2_pattern_small():
+    """C2-like globals [0, 32) with fewer blocks: the CSR residual runs as tensor-core strips."""
+    L, G = 1024, np.arange(32, dtype=np.int32)
+    plan = mg.Plan(L, 2, 64, 256, G, None)
+    inf = plan.info()
+    assert inf["nnz_fine_strip"] == inf["nnz_fine"] > 0 and inf["n_strip_tiles"] > 0
+    q, k, v = make_qkv(1, 2, L, 64, seed=9, dist="adversarial", global_idx=G)
+    check(run_gpu(plan, q, k, v), oracle_full(q, k, v, 256, G, np.zeros((0, 2))))
+
+
+@pytest.mark.parametrize("L,window,G", [(1000, 64, [0, 999]), (300, 40, [5]), (129, 0, []), (64, 16, [3]),
+                                        (200, 512, [])])
+def test_ragged_lengths(L, window, G):
+    E = np.random.default_rng(L).integers(0, L, size=(3 * L, 2)).astype(np.int32)
+    q, k, v = make_qkv(2, 2, L, 64, seed=L)
+    plan = mg.Plan(L, 2, 64, window, G, E)
+    check(run_gpu(plan, q, k, v), oracle_full(q, k, v, window, G, E))
+
+
+def test_blhd_layout():
+    m = MIXED
+    E = mixed_extra(m["L"], seed=8)
+    q, k, v = make_qkv(m["B"], m["H"], m["L"], 64, seed=2)
+    plan = mg.Plan(m["L"], m["H"], 64, m["window"], m["G"], E)
+    check(run_gpu(plan, q, k, v, layout="blhd"), oracle_full(q, k, v, m["window"], m["G"], E))
+
+
+def test_fp16():
+    c = get_config("C1")
+    q, k, v = make_qkv(1, 2, c.L, 64, seed=4, dtype="fp16")
+    plan = mg.Plan(c.L, 2, 64, c.window, c.global_idx, c.extra_idx)
+    got = run_gpu(plan, q, k, v, dtype="fp16")
+    check(got, oracle_full(q, k, v, c.window, c.global_idx, c.extra_idx, dtype="fp16"))
+
+
+def test_diagonal_only_is_identity():
+    L = 512
+    q, k, v = make_qkv(1, 2, L, 64, seed=1)
+    plan = mg.Plan(L, 2, 64, 0, [], None)
+    got = run_gpu(plan, q, k, v)
+    assert np.array_equal(got, bits_to_f64(v))          # P = 1 on the diagonal: exact
+
+
+def test_ones_v_and_zero_q():
+    c = get_config("C1")
+    q, k, v = make_qkv(1, 1, c.L, 64, seed=1, dist="ones_v")
+    plan = mg.Plan(c.L, 1, 64, c.window, c.global_idx, c.extra_idx)
+    got = run_gpu(plan, q, k, v)
+    assert np.abs(got - 1.0).max() <= 2 ** -7
+    q, k, v = make_qkv(1, 1, c.L, 64, seed=1, dist="zeros_q")
+    check(run_gpu(plan, q, k, v), oracle_full(q, k, v, c.window, c.global_idx, c.extra_idx))
+
+
+def test_repeat_calls_deterministic_and_batch_growth():
+    c = get_config("C1")
+    plan = mg.Plan(c.L, 1, 64, c.window, c.global_idx, c.extra_idx)
+    q, k, v = make_qkv(1, 1, c.L, 64, seed=3)
+    a = run_gpu(plan, q, k, v)
+    b = run_gpu(plan, q, k, v)
+    assert np.array_equal(a, b)
+    q4, k4, v4 = make_qkv(4, 1, c.L, 64, seed=3)     # workspace grows with the batch
+    check(run_gpu(plan, q4, k4, v4), oracle_full(q4, k4, v4, c.window, c.global_idx, c.extra_idx))
+
+
+def test_invalid_tensor_args():
+    c = get_config("C1")
+    plan = mg.Plan(c.L, 1, 64, c.window, c.global_idx, c.extra_idx)
+    Q = torch.zeros(1, 1, c.L, 64, dtype=torch.bfloat16, device="cuda")
+    with pytest.raises(mg.MGError):                     # heads mismatch
+        mg.sparse_attention_fwd(plan, Q.expand(1, 2, c.L, 64), Q, Q)
+    with pytest.raises(mg.MGError):                     # dtype mismatch
+        mg.sparse_attention_fwd(plan, Q, Q.half(), Q)
+    with pytest.raises(mg.MGError):                     # seq_len mismatch
+        Z = torch.zeros(1, 1, c.L - 8, 64, dtype=torch.bfloat16, device="cuda")
+        mg.sparse_attention_fwd(plan, Z, Z, Z)
+
+
+def test_host_entry_point_matches_device():
+    m = MIXED
+    E = mixed_extra(m["L"], seed=4)
+    q, k, v = make_qkv(m["B"], m["H"], m["L"], 64, seed=6)
+    plan = mg.Plan(m["L"], m["H"], 64, m["window"], m["G"], E)
+    dev = run_gpu(plan, q, k, v)
+    h = [torch.from_numpy(x.view(np.int16)).view(torch.bfloat16).pin_memory() for x in (q, k, v)]
+    O = torch.empty_like(h[0]).pin_memory()
+    mg.sparse_attention_fwd_host(plan, h[0], h[1], h[2], O)
+    torch.cuda.synchronize()
+    assert np.array_equal(from_device(O), dev)
+
+
+# ------------------------------------------------------------------ full BASELINE sizes (sampled)
+def sample_rows(L, G, rng, n=48):
+    rows = set(rng.choice(L, n, replace=False).tolist())
+    rows |= {0, 1, 127, 128, L - 1, L - 128}
+    rows |= set(np.asarray(G)[:4].tolist())
+    return sorted(r for r in rows if 0 <= r < L)
+
+
+@pytest.mark.parametrize("cfg", ["C2", "C3", "C4"])
+def test_full_size_sampled(cfg):
+    c = get_config(cfg)
+    q, k, v = make_qkv(c.B, c.H, c.L, c.d, seed=c.seed)
+    plan = mg.Plan(c.L, c.H, c.d, c.window, c.global_idx, c.extra_idx)
+    got = run_gpu(plan, q, k, v)
+    assert np.isfinite(got).all()
+    rng = np.random.default_rng(17)
+    g = global_flags(c.L, c.global_idx)
+    ex = ExtraIndex(c.L, c.extra_idx)
+    errs = []
+    for (b, h) in [(0, 0), (c.B - 1, c.H - 1), (c.B // 2, 1)]:
+        rows = sample_rows(c.L, c.global_idx, rng)
+        Q, K, V = head_inputs_f64(q, k, v, b, h)
+        ref = attention_rows(Q, K, V, rows, c.window, g, ex)
+        errs.append(np.abs(got[b, h, rows] - ref))
+    e = np.concatenate(errs)
+    assert e.max() <= TOL_MAX and e.mean() <= TOL_MEAN, (e.max(), e.mean())
