@@ -1,0 +1,385 @@
+"""Benchmark of the Multigrain compound sparse attention forward on B200 (BASELINE.json metric).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload C2] [--impl mine|reference]
+
+One "step" = one mg_sparse_attention_fwd over one batch of the workload (every hot-path step:
+plan already built, SDDMM -> merged SpSoftmax -> SpMM over the coarse, fine and dense-row parts).
+N=1 workload: C2 (Longformer-base L=4096, H=12, B=8, w=512, 32 global tokens) — BASELINE.json
+configs[1], the config its metric is quoted on. N>1 (torchrun, one process per GPU): every rank
+runs its own C2 batch (weak scaling over batch x heads; no data-path collective — the parts are
+independent), then an NCCL all_gather of O is timed separately (north_star: gather outputs only).
+
+Timing: W untimed warm-up steps; the K timed steps are bracketed by barrier + synchronize; each
+step is preceded by a 256 MB L2 flush (outside its CUDA-event pair) and timed with CUDA events on
+the launching stream; max over ranks. value = useful TFLOP/s of the whole job,
+useful flops = 4 * nnz(M) * d * B * H.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "sparse-attn fwd ms and useful TFLOP/s per B200 (Longformer L=4096), 1/2/4/8 GPU"
+UNIT = "TFLOP/s"
+FALLBACK_PEAKS = {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0}
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=1000)
+    ap.add_argument("--warmup", type=int, default=20)
+    ap.add_argument("--workload", default="C2", choices=["C1", "C2", "C3", "C4"])
+    ap.add_argument("--impl", default="mine", choices=["mine", "reference"])
+    ap.add_argument("--e2e-steps", type=int, default=30)
+    ap.add_argument("--cpu-seconds", type=float, default=12.0, help="CPU oracle sample budget")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-flush", action="store_true")
+    ap.add_argument("--strip-max-cols", type=int, default=0)
+    return ap.parse_args()
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return d, "measured (MEASURED_PEAKS.json)"
+    return dict(FALLBACK_PEAKS), "fallback (B200_PROFILING.md)"
+
+
+def workload_config(cfg, n_gpus):
+    return {
+        "workload": f"{cfg.name}: {cfg.note}",
+        "B_per_gpu": cfg.B, "H": cfg.H, "L": cfg.L, "d": cfg.d, "window": cfg.window,
+        "n_global": int(len(cfg.global_idx)), "n_extra": int(len(cfg.extra_idx)),
+        "global_batch": cfg.B * n_gpus,
+        "parallelism": f"{n_gpus} rank(s), batch x heads sharded, no data-path collective",
+        "l2": "256 MB L2 flush written before every timed step (outside the event pair)",
+        "inputs": "Q,K,V ~ N(0,1) -> bf16 (workloads.make_qkv, seed 0 + 1000*rank)",
+    }
+
+
+# ------------------------------------------------------------------ clocks (NVML, during the region)
+class ClockSampler:
+    REASONS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap", 0x8: "hw_slowdown",
+               0x10: "sync_boost", 0x20: "sw_thermal_slowdown", 0x40: "hw_thermal_slowdown",
+               0x80: "hw_power_brake_slowdown", 0x100: "display_clock_setting"}
+
+    def __init__(self, device_index: int, period_s: float = 0.002):
+        self.ok = False
+        self.samples, self.reasons = [], 0
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(device_index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.ok = True
+        except Exception as e:  # noqa: BLE001
+            self.err = str(e)
+        self.period = period_s
+        self._stop = threading.Event()
+
+    def _run(self):
+        nv = self.nv
+        while not self._stop.is_set():
+            try:
+                self.samples.append(nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM))
+                try:
+                    r = nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                except AttributeError:
+                    r = nv.nvmlDeviceGetCurrentClocksThrottleReasons(self.h)
+                self.reasons |= int(r)
+            except Exception:  # noqa: BLE001
+                pass
+            time.sleep(self.period)
+
+    def start(self):
+        if self.ok:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+
+    def stop(self):
+        if self.ok:
+            self._stop.set()
+            self.t.join()
+
+    def summary(self):
+        if not self.ok:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": [], "error": getattr(self, "err", "")}
+        reasons = [n for bit, n in self.REASONS.items() if self.reasons & bit and bit != 0x1]
+        return {"sm_mhz": statistics.median(self.samples) if self.samples else None,
+                "sm_max_mhz": self.max_mhz, "reasons": reasons, "samples": len(self.samples)}
+
+
+def nvml_index(local: int) -> int:
+    """NVML (physical) index of the local CUDA device, honouring CUDA_VISIBLE_DEVICES."""
+    vis = os.environ.get("CUDA_VISIBLE_DEVICES")
+    if vis:
+        ids = [x.strip() for x in vis.split(",") if x.strip()]
+        if local < len(ids) and ids[local].isdigit():
+            return int(ids[local])
+    return local
+
+
+# ------------------------------------------------------------------ CPU oracle baseline
+def blas_threads():
+    try:
+        from threadpoolctl import threadpool_info
+        n = [i.get("num_threads", 1) for i in threadpool_info() if i.get("user_api") == "blas"]
+        return max(n) if n else 1
+    except Exception:  # noqa: BLE001
+        return 1
+
+
+def cpu_oracle_heads(cfg, budget_s: float):
+    """Time the oracle's dense masked attention (O-4, fp64) head by head until the budget is spent."""
+    from oracle import ExtraIndex, dense_masked_attention, global_flags, head_inputs_f64
+    from oracle.mask import mask_row_cols
+    from workloads import make_qkv
+    g, ex = global_flags(cfg.L, cfg.global_idx), ExtraIndex(cfg.L, cfg.extra_idx)
+    nnz = sum(mask_row_cols(r, cfg.L, cfg.window, g, ex).size for r in range(cfg.L))
+    q, k, v = make_qkv(1, min(cfg.H, 12), cfg.L, cfg.d, seed=cfg.seed)
+    done, t0 = 0, time.perf_counter()
+    while done < q.shape[1]:
+        Q, K, V = head_inputs_f64(q, k, v, 0, done)
+        dense_masked_attention(Q, K, V, cfg.window, cfg.global_idx, cfg.extra_idx)
+        done += 1
+        if time.perf_counter() - t0 > budget_s:
+            break
+    dt = time.perf_counter() - t0
+    return {"value": 4.0 * nnz * cfg.d * done / dt / 1e12, "unit": UNIT, "cores": blas_threads(),
+            "kind": "oracle",
+            "sample": f"oracle.dense_masked_attention (fp64 numpy) on {done} of {cfg.B * cfg.H} (b,h) heads of "
+                      f"{cfg.name}, {dt:.1f} s wall; useful flops counted as for the GPU"}
+
+
+def run_reference(args):
+    """--impl reference: the oracle (as it stands) on the host cores, one bounded sample per step."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    import numpy as np
+    from oracle import ExtraIndex, attention_rows, global_flags, head_inputs_f64
+    from oracle.mask import mask_row_cols
+    from workloads import get_config, make_qkv
+    cfg = get_config(args.workload)
+    q, k, v = make_qkv(1, 1, cfg.L, cfg.d, seed=cfg.seed)
+    Q, K, V = head_inputs_f64(q, k, v, 0, 0)
+    g = global_flags(cfg.L, cfg.global_idx)
+    ex = ExtraIndex(cfg.L, cfg.extra_idx)
+    R = 32
+    rng = np.random.default_rng(0)
+
+    def step():
+        rows = rng.choice(cfg.L, R, replace=False)
+        nnz = sum(mask_row_cols(int(r), cfg.L, cfg.window, g, ex).size for r in rows)
+        t0 = time.perf_counter()
+        attention_rows(Q, K, V, rows, cfg.window, g, ex)
+        return time.perf_counter() - t0, nnz
+
+    for _ in range(args.warmup):
+        step()
+    tot_t, tot_nnz = 0.0, 0
+    for _ in range(args.steps):
+        t, n = step()
+        tot_t += t
+        tot_nnz += n
+    value = 4.0 * tot_nnz * cfg.d / tot_t / 1e12
+    cores = 1  # attention_rows: per-row numpy on one thread (vectors of <= L elements)
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * tot_t / args.steps,
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": workload_config(cfg, args.gpus),
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle",
+                         "sample": f"oracle.attention_rows (fp64) on {R} random rows of one (b,h) head of "
+                                   f"{cfg.name} per step"},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# ------------------------------------------------------------------ GPU arm
+def main():
+    args = parse()
+    if args.impl == "reference":
+        return run_reference(args)
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_iiswc_lica22_b200 as mg
+    from workloads import get_config, make_qkv
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        if world == 1 and args.gpus > 1:
+            raise SystemExit("--gpus N > 1 must be launched with torchrun (one process per GPU)")
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    dev = torch.device("cuda", local)
+
+    cfg = get_config(args.workload)
+    plan = mg.Plan(cfg.L, cfg.H, cfg.d, cfg.window, cfg.global_idx, cfg.extra_idx,
+                   strip_max_cols=args.strip_max_cols)
+    info = plan.info()
+    BH = cfg.B * cfg.H
+    useful = 4.0 * info["nnz_total"] * cfg.d * BH
+
+    q, k, v = make_qkv(cfg.B, cfg.H, cfg.L, cfg.d, seed=cfg.seed + 1000 * rank)
+    host = [torch.from_numpy(x.view(np.int16)).view(torch.bfloat16) for x in (q, k, v)]
+    Q, K, V = (h.to(dev) for h in host)
+    O = torch.empty_like(Q)
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    stream = torch.cuda.current_stream()
+
+    def fwd():
+        mg.sparse_attention_fwd(plan, Q, K, V, O, stream)
+
+    for _ in range(args.warmup):
+        if not args.no_flush:
+            flush.zero_()
+        fwd()
+    torch.cuda.synchronize()
+
+    starts = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    ends = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    sampler = ClockSampler(nvml_index(local))
+    plan.set_profiling(True)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    sampler.start()
+    for i in range(args.steps):
+        if not args.no_flush:
+            flush.zero_()
+        starts[i].record(stream)
+        fwd()
+        ends[i].record(stream)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    sampler.stop()
+    prof = plan.get_profile()
+    plan.set_profiling(False)
+    step_ms = [s.elapsed_time(e) for s, e in zip(starts, ends)]
+    t_ms = torch.tensor([sum(step_ms)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t_ms, op=dist.ReduceOp.MAX)
+    total_ms = float(t_ms.item())
+    ms_per_step = total_ms / args.steps
+    value = world * useful / (ms_per_step * 1e-3) / 1e12
+
+    # ---------------- e2e: host buffers through the C ABI (H2D + fwd + D2H every step)
+    hq, hk, hv = (h.pin_memory() for h in host)
+    hO = torch.empty_like(hq).pin_memory()
+    n_e2e = max(1, min(args.e2e_steps, args.steps))
+    for _ in range(2):
+        mg.sparse_attention_fwd_host(plan, hq, hk, hv, hO, stream)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for _ in range(n_e2e):
+        mg.sparse_attention_fwd_host(plan, hq, hk, hv, hO, stream)
+    e1.record(stream)
+    torch.cuda.synchronize()
+    e2e_ms = torch.tensor([e0.elapsed_time(e1) / n_e2e], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(e2e_ms, op=dist.ReduceOp.MAX)
+    e2e_value = world * useful / (float(e2e_ms.item()) * 1e-3) / 1e12
+    nbytes = Q.numel() * 2
+
+    # ---------------- N>1: NCCL all_gather of O, timed separately (not part of the fwd)
+    gather_ms = None
+    if world > 1:
+        out = torch.empty((world,) + tuple(O.shape), dtype=O.dtype, device=dev)
+        dist.all_gather_into_tensor(out, O)
+        torch.cuda.synchronize()
+        dist.barrier()
+        g0, g1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        g0.record(stream)
+        for _ in range(5):
+            dist.all_gather_into_tensor(out, O)
+        g1.record(stream)
+        torch.cuda.synchronize()
+        gt = torch.tensor([g0.elapsed_time(g1) / 5], dtype=torch.float64, device=dev)
+        dist.all_reduce(gt, op=dist.ReduceOp.MAX)
+        gather_ms = float(gt.item())
+
+    # ---------------- roofline of the dominant kernel (live, from the library's own events)
+    peaks, peak_src = load_peaks()
+    coarse_avg = prof["coarse_ms"] / max(1, prof["calls"])
+    fine_avg = prof["fine_ms"] / max(1, prof["calls"])
+    if coarse_avg >= fine_avg:
+        coarse_nnz = info["nnz_coarse"] + info["nnz_fine_strip"] + info["n_global"] * cfg.L
+        flops = 4.0 * coarse_nnz * cfg.d * BH
+        achieved = flops / (coarse_avg * 1e-3) / 1e12
+        peak = peaks["bf16_tflops"]
+        roof = {"kernel": "coarse_kernel (tcgen05 SDDMM + online SpSoftmax + SpMM)", "bound": "tensor",
+                "achieved": achieved, "peak": peak, "unit": "TFLOP/s", "frac": achieved / peak,
+                "avg_launch_ms": coarse_avg, "algorithmic_per_launch": flops,
+                "algorithmic_rule": "4*d flops per valid element it owns (coarse + strip + dense-row)",
+                "peak_source": peak_src + " bf16 burst", "traffic": None}
+    else:
+        nbytes_f = info["nnz_fine_cuda"] * BH * (2 * cfg.d * 2 + 4) + info["n_fine_rows"] * BH * (2 * cfg.d + 264)
+        achieved = nbytes_f / (fine_avg * 1e-3) / 1e9
+        peak = peaks["hbm_gbs"]
+        roof = {"kernel": "fine_rows_kernel (CUDA-core CSR)", "bound": "hbm", "achieved": achieved, "peak": peak,
+                "unit": "GB/s", "frac": achieved / peak, "avg_launch_ms": fine_avg,
+                "algorithmic_per_launch": nbytes_f,
+                "algorithmic_rule": "per nnz: K row + V row (2*d*2 B) + 4 B index; per row: Q read + partial write",
+                "peak_source": peak_src, "traffic": None}
+    tr_path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(tr_path):
+        tr = json.load(open(tr_path)).get(cfg.name, {})
+        key = "coarse" if roof["bound"] == "tensor" else "fine"
+        if key in tr:
+            roof["traffic"] = tr[key].get("dram_bytes_per_launch")
+            roof["traffic_source"] = tr[key].get("source")
+
+    line = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "bf16", "data": "synthetic", "config": workload_config(cfg, world),
+        "fwd_ms": {"mean": ms_per_step, "median": statistics.median(step_ms), "min": min(step_ms)},
+        "useful_gflop_per_gpu": useful / 1e9,
+        "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": 3 * nbytes, "d2h_bytes_per_step": nbytes,
+                "ms_per_step": float(e2e_ms.item()),
+                "path": "mg_sparse_attention_fwd_host (pinned host Q/K/V/O, copies inside the timed region)"},
+        "gpu_launches": int(args.steps * info["kernels_per_fwd"]),
+        "kernels_per_fwd": info["kernels_per_fwd"],
+        "roofline": roof,
+        "clocks": sampler.summary(),
+        "plan": {k_: info[k_] for k_ in ("n_tiles", "n_full_tiles", "nnz_total", "nnz_fine", "nnz_fine_strip",
+                                          "nnz_fine_cuda", "n_items", "computed_scores")},
+        "paper_context": "Multigrain reports 2.07x (Longformer) / 1.55x (QDS) end-to-end over Triton, FP16, "
+                         "A100/RTX 3090 (PAPER.md P:12); no absolute numbers are published",
+    }
+    if gather_ms is not None:
+        line["allgather_O_ms"] = gather_ms
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        line["cpu_baseline"] = cpu_oracle_heads(cfg, args.cpu_seconds)
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -47,7 +47,7 @@ __device__ __forceinline__ uint32_t pack2(float lo, float hi) {
 }  // namespace
 
 template <bool kBF16>
-__global__ void __launch_bounds__(256) fine_rows_kernel(const FineParams p) {
+__global__ void __launch_bounds__(256, 2) fine_rows_kernel(const FineParams p) {
   const int lane = threadIdx.x & 31;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   if (gw >= (int64_t)p.BH * p.n_fine_rows) return;
