@@ -204,6 +204,12 @@ MG_API mg_status mg_plan_get_profile(mg_plan_t plan, mg_profile* out);
  * ---------------------------------------------------------------------------------- */
 MG_API mg_status mg_selftest_umma(int32_t mode, const void* A, const void* B, float* D, void* stream);
 
+/* mg_plan_set_trace(plan, buf, cap): diagnostics. While set, CTA 0 of the tensor-core kernel
+ * appends (clock64, role<<56 | event<<48 | arg) pairs of uint64 to the device buffer `buf`
+ * (capacity `cap` pairs; pair 0 holds the running count, the caller zeroes it). (null, 0)
+ * turns tracing off. Used to read the warp-role pipeline timeline. */
+MG_API mg_status mg_plan_set_trace(mg_plan_t plan, void* device_buffer, int64_t capacity_events);
+
 MG_API int32_t mg_abi_version(void);
 
 #ifdef __cplusplus

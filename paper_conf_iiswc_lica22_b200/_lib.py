@@ -15,7 +15,7 @@ STATUS_NAMES = {0: "OK", 1: "INVALID_ARG", 2: "UNSUPPORTED", 3: "OUT_OF_MEMORY",
 EXPORTED = [
     "mg_plan_create", "mg_plan_create_ex", "mg_plan_destroy", "mg_last_error", "mg_plan_info_get",
     "mg_plan_export", "mg_sparse_attention_fwd", "mg_sparse_attention_fwd_host", "mg_selftest_umma",
-    "mg_abi_version", "mg_plan_set_profiling", "mg_plan_get_profile",
+    "mg_abi_version", "mg_plan_set_profiling", "mg_plan_get_profile", "mg_plan_set_trace",
 ]
 
 
@@ -73,6 +73,7 @@ def load() -> C.CDLL:
     lib.mg_selftest_umma.argtypes = [C.c_int32, P, P, P, P]
     lib.mg_plan_set_profiling.argtypes = [P, C.c_int32]
     lib.mg_plan_get_profile.argtypes = [P, C.POINTER(mg_profile)]
+    lib.mg_plan_set_trace.argtypes = [P, P, C.c_int64]
     lib.mg_abi_version.restype = C.c_int32
     lib.mg_abi_version.argtypes = []
     for name in EXPORTED:

@@ -63,6 +63,9 @@ struct mg_plan_s {
   size_t part_cap = 0;      // in (row, bh) partial slots
   uint8_t* d_stage = nullptr;
   size_t stage_cap = 0;     // bytes
+  // diagnostics: device event-trace buffer of the coarse kernel (CTA 0)
+  unsigned long long* trace = nullptr;
+  int32_t trace_cap = 0;
   // profiling: 4 events per recorded call (start, after fine, after coarse, end)
   bool profiling = false;
   std::vector<cudaEvent_t> prof_events;
@@ -308,6 +311,8 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
     cp.n_fine_rows = nf;
     cp.total_units = cp.n_items * BH;
     cp.scale_log2 = scale_log2;
+    cp.trace = p->trace;
+    cp.trace_cap = p->trace_cap;
     if ((e = cudaMemsetAsync(p->d_counter, 0, sizeof(int32_t), stream)) != cudaSuccess)
       return cuda_fail(e, "cudaMemsetAsync");
     const int sms = p->num_sms_override > 0 ? p->num_sms_override : p->num_sms;
@@ -468,6 +473,16 @@ mg_status mg_plan_get_profile(mg_plan_t plan, mg_profile* out) {
   plan->prof_used = 0;
   plan->prof_has_fine.clear();
   plan->prof_has_coarse.clear();
+  return MG_OK;
+}
+
+mg_status mg_plan_set_trace(mg_plan_t plan, void* device_buffer, int64_t capacity_events) {
+  g_err.clear();
+  if (!plan || (device_buffer == nullptr) != (capacity_events == 0) || capacity_events < 0 ||
+      capacity_events > (int64_t(1) << 30))
+    return fail(MG_ERR_INVALID_ARG, "bad trace buffer");
+  plan->trace = static_cast<unsigned long long*>(device_buffer);
+  plan->trace_cap = (int32_t)capacity_events;
   return MG_OK;
 }
 

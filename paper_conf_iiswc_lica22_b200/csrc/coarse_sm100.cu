@@ -104,6 +104,28 @@ __device__ __forceinline__ uint64_t mask_window(uint64_t w0, uint64_t w1, int of
   return off >= 64 ? w1 : (w0 >> off);
 }
 
+// Diagnostics: CTA 0 appends (clock64, role<<56 | event<<48 | arg) to its role's private segment
+// of p.trace (4 segments of trace_cap/4 pairs; pair 0 of a segment holds the count). Plain
+// stores only, so the timeline is not perturbed by atomics. Roles: 0 producer, 1 MMA, 2 softmax
+// warp 4, 3 softmax warp 8.
+struct Tracer {
+  unsigned long long* seg = nullptr;
+  uint32_t n = 0, cap = 0;
+  __device__ __forceinline__ Tracer(const CoarseParams& p, uint32_t role) {
+    if (p.trace != nullptr && blockIdx.x == 0) {
+      cap = (uint32_t)(p.trace_cap / 4);
+      seg = p.trace + 2ull * role * cap;
+    }
+  }
+  __device__ __forceinline__ void operator()(uint32_t role, uint32_t ev, uint32_t arg) {
+    if (seg == nullptr || n + 2 >= cap) return;
+    ++n;
+    seg[2 * n] = clock64();
+    seg[2 * n + 1] = ((unsigned long long)role << 56) | ((unsigned long long)ev << 48) | arg;
+    seg[0] = n;
+  }
+};
+
 }  // namespace
 
 template <bool kBF16>
@@ -176,6 +198,7 @@ __global__ void __launch_bounds__(kThreads, 1)
   asm volatile("setmaxnreg.dec.sync.aligned.u32 88;" ::: "memory");
   if (warp == 0) {
     // ============================================================ producer
+    Tracer trace(p, 0);
     const uint64_t pol_kv = policy_evict_last();   // K/V tiles are re-read by neighbouring row blocks
     const uint64_t pol_q = policy_evict_first();   // Q tile is read once
     uint32_t it = 0, g = 0, qi = 0;
@@ -204,7 +227,9 @@ __global__ void __launch_bounds__(kThreads, 1)
       const int bb = bh / p.H, hh = bh % p.H;
       const uint32_t qb = qi & 1;
       uint8_t* dQ = sQ + qb * kTileBytes;
+      if (lane == 0) trace(0, 1, u);                       // item fetched
       mbar_wait(q_empty(qb), ((qi >> 1) & 1) ^ 1);
+      if (lane == 0) trace(0, 2, qi);                      // Q buffer free
       if (item.kind == 0) {
         if (lane == 0) {
           mbar_arrive_expect_tx(q_full(qb), kTileBytes);
@@ -222,6 +247,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         const TileRef tr = p.trefs[item.tref_begin + j];
         const uint32_t st = g % kStages, sph = (g / kStages) & 1;
         mbar_wait(kv_empty(st), sph ^ 1);
+        if (lane == 0) trace(0, 3, g);                     // stage free, loads issued
         uint8_t* dK = sK + st * kTileBytes;
         uint8_t* dV = sV + st * kTileBytes;
         const uint32_t dM = smem_u32(sM + st * kMaskBytes);
@@ -261,11 +287,14 @@ __global__ void __launch_bounds__(kThreads, 1)
     // Within an item S_{j+1} is issued before P_j V_j; the last P.V of an item is issued at once
     // and the next item's S_0 follows it (its Q is already in the other Q buffer).
     const bool leader = lane == 0;
+    Tracer trace(p, 1);
     uint32_t it = 0, g = 0, qi = 0;
     auto issue_pv = [&](uint32_t x, int ncols, uint32_t st) {
       const uint32_t buf = x & 1, xs = x % 3;
       mbar_wait(p_full(buf), (x >> 1) & 1);
+      if (leader) trace(1, 4, x);                          // P ready
       mbar_wait(v_full(st), (x / kStages) & 1);
+      if (leader) trace(1, 5, x);                          // V ready, PV issued
       tc_fence_after();
       if (leader) {
         const int h = ncols >> 1, nk = h >> 4;
@@ -296,6 +325,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       const uint32_t qb = qi & 1;
       const uint32_t sQa = smem_u32(sQ + qb * kTileBytes);
       mbar_wait(q_full(qb), (qi >> 1) & 1);
+      if (leader) trace(1, 0, qi);                         // Q ready
       ++qi;
       tc_fence_after();
       int prev_n = 0;
@@ -304,8 +334,10 @@ __global__ void __launch_bounds__(kThreads, 1)
         const uint32_t gg = g + j, xs = gg % 3;
         const uint32_t st = gg % kStages;
         mbar_wait(k_full(st), (gg / kStages) & 1);
+        if (leader) trace(1, 1, gg);                       // K ready
         const int ncols = ctl->tref[st].ncols;
         if (gg >= 3) mbar_wait(o_empty(xs), ((gg / 3) - 1) & 1);
+        if (leader) trace(1, 2, gg);                       // S buffer free, S issued
         tc_fence_after();
         if (leader) {
           const uint32_t idesc_s = idesc_f16(kBF16, 128, ncols, false, false);
@@ -336,6 +368,8 @@ __global__ void __launch_bounds__(kThreads, 1)
     const uint32_t lane_base = (uint32_t)(q4 * 32) << 16;
     const float c = p.scale_log2;
     const float2 c2 = make_float2(c, c);
+    Tracer trace(p, 2 + (warp >> 3));
+    const bool tr_on_item = (warp == 4 || warp == 8) && lane == 0;
     uint32_t it = 0, g = 0;
     float oacc[64];
     while (true) {
@@ -392,7 +426,10 @@ __global__ void __launch_bounds__(kThreads, 1)
           const ulonglong2 mw = *reinterpret_cast<const ulonglong2*>(sM + st * kMaskBytes + t * 16);
           bits = mask_window(mw.x, mw.y, wg * h);
         }
+        const bool tr_on = (warp == 4 || warp == 8) && lane == 0;
+        if (tr_on) trace(2 + (warp >> 3), 1, gg);                         // tile start
         mbar_wait(s_full(xs), (gg / 3) & 1);
+        if (tr_on) trace(2 + (warp >> 3), 2, gg);                         // S ready
         tc_fence_after();
         float alpha = 1.f;
         if (active) {
@@ -460,10 +497,13 @@ __global__ void __launch_bounds__(kThreads, 1)
         tc_fence_before();
         __syncwarp();
         if (lane == 0) mbar_arrive(p_full(buf));
+        if (tr_on) trace(2 + (warp >> 3), 3, gg);                         // P stored
         if (j >= 1) consume(gg - 1, alpha_prev);
+        if (tr_on) trace(2 + (warp >> 3), 4, gg);                         // O_{j-1} consumed
         alpha_prev = alpha;
       }
       consume(g + item.ntiles - 1, alpha_prev);
+      if (tr_on_item) trace(2 + (warp >> 3), 5, g + item.ntiles - 1);   // item O complete
       g += item.ntiles;
 
       // ---- epilogue: merge the two column halves (+ the fine partial), normalise, store O
@@ -483,6 +523,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         *reinterpret_cast<float2*>(mine + 32) = make_float2(m, l);
       }
       named_bar_sync(1, 256);
+      if (tr_on_item) trace(2 + (warp >> 3), 6, 0);           // halves exchanged
       const float* other = xch + ((1 - wg) * 128 + t) * kXchStride;
       int r = -1;
       if (item.kind == 0) {

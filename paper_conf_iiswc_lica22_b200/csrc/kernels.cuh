@@ -34,6 +34,8 @@ struct CoarseParams {
   int32_t n_global, n_fine_rows;
   int32_t total_units;
   float scale_log2;           // (1/sqrt(d)) * log2(e)
+  unsigned long long* trace;  // diagnostics: event trace of CTA 0 (null = off)
+  int32_t trace_cap;
 };
 
 // Fine CSR kernel: warp per (row, batch*head); SDDMM -> online softmax -> SpMM on CUDA cores.
