@@ -10,6 +10,7 @@
 
 #include <algorithm>
 #include <cstring>
+#include <iterator>
 
 namespace mg {
 
@@ -148,9 +149,14 @@ std::string build_plan(HostPlan& p, int64_t L, int32_t heads, int32_t d, int32_t
     p.dev_masks.resize(p.dev_masks.size() + 256, 0ull);
     return id;
   };
+  auto count = [&](int32_t mask, int ncols, int nrows) {
+    if (mask == kMaskSkip || nrows == 0) return;
+    p.computed_scores += B * ncols;
+    p.softmax_tiles += 1;
+  };
 
-  // dense items (global rows), 128 gathered rows each, every column tile
-  int32_t ragged_mask = -1;
+  // dense items (global rows): two streams of up to 128 gathered rows, every column tile
+  int32_t ragged_mask = kMaskFull;
   if (L % B) {
     ragged_mask = new_mask();
     const int64_t valid = L - (nb - 1) * B;
@@ -158,76 +164,156 @@ std::string build_plan(HostPlan& p, int64_t L, int32_t heads, int32_t d, int32_t
       for (int64_t c = 0; c < valid; ++c) p.dev_masks[(size_t)ragged_mask * 256 + a * 2 + c / 64] |= 1ull << (c % 64);
   }
   const int64_t G = (int64_t)p.global_rows.size();
-  for (int64_t k = 0; k < G; k += 128) {
-    Item it{1, (int32_t)k, (int32_t)nb, (int32_t)p.trefs.size()};
-    for (int64_t J = 0; J < nb; ++J)
-      p.trefs.push_back(TileRef{(int32_t)(J * B), (J == nb - 1) ? ragged_mask : -1, 128, 0});
+  for (int64_t k = 0; k < G; k += 256) {
+    const int32_t na = (int32_t)std::min<int64_t>(128, G - k);
+    const int32_t nbr = (int32_t)std::max<int64_t>(0, std::min<int64_t>(128, G - k - 128));
+    Item it{1, (int32_t)k, (int32_t)(k + 128), (int32_t)nb, (int32_t)p.trefs.size(), na, nbr, 0, ~0ull,
+            nbr ? ~0ull : 0ull};
+    for (int64_t J = 0; J < nb; ++J) {
+      const int32_t m = (J == nb - 1) ? ragged_mask : kMaskFull;
+      p.trefs.push_back(TileRef{(int32_t)(J * B), 0, 128, m, nbr ? m : kMaskSkip, 0, 0, 0});
+      count(m, 128, na);
+      count(nbr ? m : kMaskSkip, 128, nbr);
+    }
     p.items.push_back(it);
-    p.computed_scores += nb * B * B;
   }
   p.n_dense_items = (int32_t)p.items.size();
 
-  // band items and the CSR residual split (tensor-core strip vs CUDA-core rows)
-  p.fine_slot.assign(L, -1);
-  std::vector<int32_t> cuda_rows;      // rows run by the fine kernel
-  std::vector<uint8_t> cuda_final;     // 1 = the fine kernel writes O (no coarse part in the row block)
-  const int strip_max = opts.strip_max_cols;
+  // distinct CSR columns of each row block
+  std::vector<std::vector<int32_t>> blk_cols(nb);
   for (int64_t I = 0; I < nb; ++I) {
     const int64_t r0 = I * B, r1 = std::min<int64_t>(L, r0 + B);
-    const int32_t tb = p.bsr_row_ptr[I], te = p.bsr_row_ptr[I + 1];
-    const bool has_tiles = te > tb;
-    // distinct CSR columns of this row block
-    std::vector<int32_t> cols;
+    auto& cols = blk_cols[I];
     for (int64_t r = r0; r < r1; ++r)
       cols.insert(cols.end(), p.csr_col.begin() + p.csr_row_ptr[r], p.csr_col.begin() + p.csr_row_ptr[r + 1]);
     std::sort(cols.begin(), cols.end());
     cols.erase(std::unique(cols.begin(), cols.end()), cols.end());
-    const bool use_strip = has_tiles && !cols.empty() && strip_max > 0 && (int)cols.size() <= strip_max;
-    if (has_tiles) {
-      Item it{0, (int32_t)r0, te - tb + (use_strip ? 1 : 0), (int32_t)p.trefs.size()};
-      for (int32_t t = tb; t < te; ++t) {
-        p.trefs.push_back(TileRef{p.bsr_col[t] * (int32_t)B, tile_full[t] ? -1 : t, 128, 0});
-        p.computed_scores += B * B;
+  }
+  const int strip_max = opts.strip_max_cols;
+  std::vector<uint8_t> blk_strip(nb, 0);  // CSR residual of the block carried by a strip tile
+  // strip tile over `cols` with the bitmask of row block I (kMaskSkip if I < 0)
+  auto strip_mask = [&](int64_t I, const std::vector<int32_t>& cols, int ncols) -> int32_t {
+    if (I < 0) return kMaskSkip;
+    const int64_t r0 = I * B, r1 = std::min<int64_t>(L, r0 + B);
+    const int32_t m = new_mask();
+    bool full = r1 - r0 == B;
+    for (int64_t r = r0; r < r0 + B; ++r) {
+      const int64_t a = r - r0;
+      if (r >= r1) continue;
+      const int32_t* cb = p.csr_col.data() + p.csr_row_ptr[r];
+      const int32_t* ce = p.csr_col.data() + p.csr_row_ptr[r + 1];
+      if (ce - cb != ncols) full = false;
+      for (const int32_t* c = cb; c != ce; ++c) {
+        const int64_t beta = std::lower_bound(cols.begin(), cols.end(), *c) - cols.begin();
+        p.dev_masks[(size_t)m * 256 + a * 2 + beta / 64] |= 1ull << (beta % 64);
       }
-      if (use_strip) {
-        const int ncols = (int)((cols.size() + 31) / 32 * 32);
-        const int32_t off = (int32_t)p.strip_cols.size();
-        for (int i = 0; i < ncols; ++i) p.strip_cols.push_back(i < (int)cols.size() ? cols[i] : -1);
-        const int32_t m = new_mask();
-        bool full = true;
-        for (int64_t r = r0; r < r0 + B; ++r) {
-          const int64_t a = r - r0;
-          if (r >= r1) { full = false; continue; }
-          const int32_t* cb = p.csr_col.data() + p.csr_row_ptr[r];
-          const int32_t* ce = p.csr_col.data() + p.csr_row_ptr[r + 1];
-          if (ce - cb != ncols) full = false;
-          for (const int32_t* c = cb; c != ce; ++c) {
-            const int64_t beta = std::lower_bound(cols.begin(), cols.end(), *c) - cols.begin();
-            p.dev_masks[(size_t)m * 256 + a * 2 + beta / 64] |= 1ull << (beta % 64);
-          }
-          p.nnz_fine_strip += ce - cb;
-        }
-        p.trefs.push_back(TileRef{off, full ? -1 : m, ncols, 1});
-        p.n_strip_tiles++;
-        p.computed_scores += B * ncols;
-      }
-      p.items.push_back(it);
+      p.nnz_fine_strip += ce - cb;
     }
-    if (!use_strip) {
-      for (int64_t r = r0; r < r1; ++r) {
-        if (p.csr_row_ptr[r + 1] == p.csr_row_ptr[r]) continue;
-        if (has_tiles) p.fine_slot[r] = (int32_t)cuda_rows.size();
-        cuda_rows.push_back((int32_t)r);
-        cuda_final.push_back(has_tiles ? 0 : 1);
+    if (full) {  // drop the unused mask again (it is the last one allocated)
+      p.dev_masks.resize(p.dev_masks.size() - 256);
+      return kMaskFull;
+    }
+    return m;
+  };
+  auto push_strip = [&](int64_t IA, int64_t IB, const std::vector<int32_t>& cols) {
+    const int ncols = (int)((cols.size() + 31) / 32 * 32);
+    const int32_t off = (int32_t)p.strip_cols.size();
+    for (int i = 0; i < ncols; ++i) p.strip_cols.push_back(i < (int)cols.size() ? cols[i] : -1);
+    const int32_t ma = strip_mask(IA, cols, ncols);
+    const int32_t mb = strip_mask(IB, cols, ncols);
+    p.trefs.push_back(TileRef{off, 1, ncols, ma, mb, 0, 0, 0});
+    count(ma, ncols, 1);
+    count(mb, ncols, 1);
+    p.n_strip_tiles++;
+  };
+
+  // band items: consecutive row blocks that have coarse tiles, paired (A, B)
+  std::vector<int64_t> tiled;
+  for (int64_t I = 0; I < nb; ++I)
+    if (p.bsr_row_ptr[I + 1] > p.bsr_row_ptr[I]) tiled.push_back(I);
+  for (size_t k = 0; k < tiled.size();) {
+    const int64_t IA = tiled[k];
+    int64_t IB = k + 1 < tiled.size() ? tiled[k + 1] : -1;
+    if (IB >= 0) {  // pair only while the union stays within a 64-tile use bitmap (+ strips)
+      int64_t lo = std::min(p.bsr_col[p.bsr_row_ptr[IA]], p.bsr_col[p.bsr_row_ptr[IB]]);
+      int64_t hi = std::max(p.bsr_col[p.bsr_row_ptr[IA + 1] - 1], p.bsr_col[p.bsr_row_ptr[IB + 1] - 1]);
+      if (hi - lo + 1 > 62) IB = -1;
+    }
+    k += IB >= 0 ? 2 : 1;
+    auto nrows_of = [&](int64_t I) -> int32_t { return I < 0 ? 0 : (int32_t)std::min<int64_t>(B, L - I * B); };
+    Item it{0, (int32_t)(IA * B), (int32_t)(IB < 0 ? 0 : IB * B), 0, (int32_t)p.trefs.size(), nrows_of(IA),
+            nrows_of(IB), 0, 0ull, 0ull};
+    // union of the two blocks' column tiles, ascending
+    std::vector<std::pair<int32_t, std::pair<int32_t, int32_t>>> u;  // J -> (maskA, maskB)
+    auto add_block = [&](int64_t I, bool isA) {
+      if (I < 0) return;
+      for (int32_t t = p.bsr_row_ptr[I]; t < p.bsr_row_ptr[I + 1]; ++t) {
+        const int32_t J = p.bsr_col[t];
+        const int32_t m = tile_full[t] ? kMaskFull : t;
+        auto itr = std::find_if(u.begin(), u.end(), [&](const auto& e) { return e.first == J; });
+        if (itr == u.end()) {
+          u.push_back({J, {kMaskSkip, kMaskSkip}});
+          itr = u.end() - 1;
+        }
+        (isA ? itr->second.first : itr->second.second) = m;
       }
+    };
+    add_block(IA, true);
+    add_block(IB, false);
+    std::sort(u.begin(), u.end());
+    for (const auto& e : u) {
+      p.trefs.push_back(TileRef{e.first * (int32_t)B, 0, 128, e.second.first, e.second.second, 0, 0, 0});
+      count(e.second.first, 128, it.nrowsA);
+      count(e.second.second, 128, it.nrowsB);
+    }
+    // CSR residual as tensor-core strips where the blocks' distinct columns are few
+    const std::vector<int32_t>& ca = blk_cols[IA];
+    const std::vector<int32_t> empty;
+    const std::vector<int32_t>& cb = IB < 0 ? empty : blk_cols[IB];
+    const bool sa = strip_max > 0 && !ca.empty() && (int)ca.size() <= strip_max;
+    const bool sb = strip_max > 0 && !cb.empty() && (int)cb.size() <= strip_max;
+    if (sa && sb) {
+      std::vector<int32_t> un;
+      std::set_union(ca.begin(), ca.end(), cb.begin(), cb.end(), std::back_inserter(un));
+      if ((int)un.size() <= strip_max) {
+        push_strip(IA, IB, un);
+      } else {
+        push_strip(IA, -1, ca);
+        push_strip(-1, IB, cb);
+      }
+    } else if (sa) {
+      push_strip(IA, -1, ca);
+    } else if (sb) {
+      push_strip(-1, IB, cb);
+    }
+    if (sa) blk_strip[IA] = 1;
+    if (sb) blk_strip[IB] = 1;
+    it.ntiles = (int32_t)p.trefs.size() - it.tref_begin;
+    for (int32_t j = 0; j < it.ntiles && j < 64; ++j) {
+      const TileRef& r = p.trefs[it.tref_begin + j];
+      if (r.maskA != kMaskSkip && it.nrowsA) it.useA |= 1ull << j;
+      if (r.maskB != kMaskSkip && it.nrowsB) it.useB |= 1ull << j;
+    }
+    p.items.push_back(it);
+  }
+
+  // CSR rows left to the CUDA-core fine kernel
+  p.fine_slot.assign(L, -1);
+  for (int64_t I = 0; I < nb; ++I) {
+    if (blk_strip[I]) continue;
+    const bool has_tiles = p.bsr_row_ptr[I + 1] > p.bsr_row_ptr[I];
+    const int64_t r0 = I * B, r1 = std::min<int64_t>(L, r0 + B);
+    for (int64_t r = r0; r < r1; ++r) {
+      if (p.csr_row_ptr[r + 1] == p.csr_row_ptr[r]) continue;
+      if (has_tiles) p.fine_slot[r] = (int32_t)p.fine_rows.size();
+      p.fine_rows.push_back((int32_t)r | (has_tiles ? 0 : (int32_t)0x80000000));
     }
   }
-  p.fine_row_ptr.push_back(0);
-  for (size_t i = 0; i < cuda_rows.size(); ++i) {
-    const int32_t r = cuda_rows[i];
+  p.fine_row_ptr.assign(1, 0);
+  for (int32_t enc : p.fine_rows) {
+    const int32_t r = enc & 0x7fffffff;
     p.fine_col.insert(p.fine_col.end(), p.csr_col.begin() + p.csr_row_ptr[r], p.csr_col.begin() + p.csr_row_ptr[r + 1]);
     p.fine_row_ptr.push_back((int32_t)p.fine_col.size());
-    p.fine_rows.push_back(r | (cuda_final[i] ? (int32_t)0x80000000 : 0));
   }
   return "";
 }

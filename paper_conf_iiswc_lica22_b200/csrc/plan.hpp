@@ -16,14 +16,23 @@ struct PlanOptions {
   int strip_max_cols = 128;  // <= 0 disables the tensor-core strip path for the CSR residual
 };
 
-// Device work-list encodings.
-//   Item  {kind, row0, ntiles, tref_begin}: kind 0 = band row block starting at row0;
-//         kind 1 = gathered dense global rows global_rows[row0 .. row0+128) (ntiles = nb).
-//   TileRef {arg, mask, ncols, kind}: kind 0 = contiguous column tile at column `arg`;
-//         kind 1 = gathered strip whose column list starts at strip_cols[arg];
-//         mask = index of a 128 x 2-word bitmask or -1 for "all valid".
-struct Item { int32_t kind, row0, ntiles, tref_begin; };
-struct TileRef { int32_t arg, mask, ncols, kind; };
+// Device work-list encodings. The tensor-core kernel runs two softmax
+// streams (A and B) on two 128-row Q tiles that share the K/V tiles of one work item.
+//   Item {kind, rowA, rowB, ntiles, tref_begin, nrowsA, nrowsB}:
+//     kind 0: band row blocks starting at rows rowA and rowB (adjacent blocks with coarse tiles);
+//     kind 1: gathered global rows global_rows[rowA ..) and global_rows[rowB ..) (dense part);
+//     nrowsX = valid rows of stream X (0 = stream unused); useX = bit j set if stream X uses tile j
+//     (items with more than 64 tiles are dense items whose active streams use every tile).
+//   TileRef {arg, kind, ncols, maskA, maskB}: one K/V tile of the item, loaded once:
+//     kind 0 = contiguous column tile at column `arg`; kind 1 = gathered strip whose column list
+//     starts at strip_cols[arg]; maskX = index of a 128 x 2-word bitmask for stream X,
+//     -1 = all valid, -2 = stream X does not use this tile.
+struct Item {
+  int32_t kind, rowA, rowB, ntiles, tref_begin, nrowsA, nrowsB, pad;
+  uint64_t useA, useB;
+};
+struct TileRef { int32_t arg, kind, ncols, maskA, maskB, pad0, pad1, pad2; };
+constexpr int32_t kMaskFull = -1, kMaskSkip = -2;
 
 struct HostPlan {
   // inputs
@@ -45,7 +54,7 @@ struct HostPlan {
   std::vector<int32_t> fine_slot;    // per row: index into fine_rows for partial merge, or -1
   std::vector<int32_t> fine_row_ptr; // compacted CSR (cuda part only) [n_fine_rows + 1]
   std::vector<int32_t> fine_col;
-  int64_t nnz_fine_strip = 0, n_strip_tiles = 0, computed_scores = 0;
+  int64_t nnz_fine_strip = 0, n_strip_tiles = 0, computed_scores = 0, softmax_tiles = 0;
 
   int64_t nb() const { return (L + block - 1) / block; }
   int wpr() const { return (block + 63) / 64; }
