@@ -4,6 +4,7 @@
 #include <cudaTypedefs.h>
 
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 #include <new>
@@ -311,6 +312,11 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
     cp.n_fine_rows = nf;
     cp.total_units = cp.n_items * BH;
     cp.scale_log2 = scale_log2;
+    static const int dbg = [] {
+      const char* e = std::getenv("MG_DEBUG_FLAGS");
+      return e ? std::atoi(e) : 0;
+    }();
+    cp.debug_flags = dbg;
     cp.trace = p->trace;
     cp.trace_cap = p->trace_cap;
     if ((e = cudaMemsetAsync(p->d_counter, 0, sizeof(int32_t), stream)) != cudaSuccess)

@@ -13,13 +13,14 @@
 // Warp roles (one 384-thread CTA per SM, persistent, dynamic work counter):
 //   warp 0      producer: work fetch, TMA of Q/K/V tiles (SWIZZLE_128B), bulk copies of tile
 //               bitmasks, row gathers (global rows, strip columns)
-//   warp 1      MMA issuer (lane 0): per K/V tile S_A, S_B, then P_A V, P_B V of the previous tile
-//   warp 2      TMEM allocator
+//   warps 1, 3  MMA issuers for streams A and B (lane 0): S half tiles two ahead, P.V behind
+//   warp 2      TMEM allocator, then scheduler: publishes work items, L2-prefetches their tiles
 //   warps 4..7  softmax WG A, warps 8..11 softmax WG B: two independent streams, so one WG's
 //               waits overlap the other's exp work (MUFU is the bound)
-// TMEM (512 columns): S_A [0,128) S_B [128,256) P_A [256,320) P_B [320,384) O_A [384,448)
-// O_B [448,512). S is released as soon as it is in registers; O accumulates in TMEM across the
-// item's tiles (P.V with accumulate) with lazy rescaling by the softmax warps (FA4-style).
+// TMEM (512 columns): per stream, three 64-column half-tile buffers (S_h, then P_h over it as
+// 16-bit pairs) and a 64-column O accumulator. The pipeline unit is a half tile (64 keys): the MMA
+// runs S two halves ahead; O accumulates in TMEM across the item (P.V with accumulate) with lazy
+// rescaling by the softmax warps (FA4-style).
 #include <cuda_bf16.h>
 #include <cuda_fp16.h>
 
@@ -36,7 +37,8 @@ constexpr int kStages = 4;
 constexpr int kThreads = 384;
 constexpr uint32_t kTileBytes = 128 * 128;  // 128 rows x 64 x 16-bit
 constexpr uint32_t kMaskBytes = 128 * 16;   // 128 rows x 2 x u64
-constexpr uint32_t kTmemS = 0, kTmemP = 256, kTmemO = 384;
+// TMEM per stream w (256 columns at w*256): three 64-column S/P half-tile buffers, then O.
+constexpr uint32_t kTmemOOff = 192;
 
 struct __align__(16) ItemSlot {
   Item item;
@@ -55,7 +57,7 @@ struct __align__(16) SmemCtl {
   ItemSlot slot[2];
   uint64_t q_full[2], q_empty[2];
   uint64_t k_full[kStages], v_full[kStages], kv_empty[kStages];
-  uint64_t s_full[2], s_empty[2], p_full[2], o_full[2];  // per stream
+  uint64_t s_full[2][3], p_full[2][3], pv_done[2][3];   // per stream, per half-tile buffer
   uint64_t item_full[2], item_empty[2];
   uint32_t tmem_base;
 };
@@ -205,12 +207,13 @@ __global__ void __launch_bounds__(kThreads, 1)
     for (int b = 0; b < 2; ++b) {
       mbar_init(bar(ctl->q_full[b]), 1);
       mbar_init(bar(ctl->q_empty[b]), 2);           // one commit per MMA warp
-      mbar_init(bar(ctl->s_full[b]), 1);
-      mbar_init(bar(ctl->s_empty[b]), 4);
-      mbar_init(bar(ctl->p_full[b]), 4);
-      mbar_init(bar(ctl->o_full[b]), 1);
+      for (int x = 0; x < 3; ++x) {
+        mbar_init(bar(ctl->s_full[b][x]), 1);
+        mbar_init(bar(ctl->p_full[b][x]), 4);
+        mbar_init(bar(ctl->pv_done[b][x]), 1);
+      }
       mbar_init(bar(ctl->item_full[b]), 1);
-      mbar_init(bar(ctl->item_empty[b]), 10);       // 2 MMA warps + 8 softmax warps
+      mbar_init(bar(ctl->item_empty[b]), 11);       // producer + 2 MMA warps + 8 softmax warps
     }
     for (int s = 0; s < kStages; ++s) {
       mbar_init(bar(ctl->k_full[s]), 1);
@@ -219,7 +222,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     }
     fence_barrier_init();
   }
-  if (warp == 0 && lane == 0) {
+  if (warp == 2 && lane == 0) {
     prefetch_tmap(&tmq);
     prefetch_tmap(&tmk);
     prefetch_tmap(&tmv);
@@ -243,30 +246,18 @@ __global__ void __launch_bounds__(kThreads, 1)
       uint32_t it = 0, g = 0, qi = 0;
       while (true) {
         const uint32_t slot = it & 1, ph = (it >> 1) & 1;
-        int u = 0;
-        if (lane == 0) {
-          mbar_wait(bar(ctl->item_empty[slot]), ph ^ 1);
-          u = atomicAdd(p.counter, 1);
-          ItemSlot is;
-          is.u = u;
-          if (u < p.total_units) {
-            const UnitInfo ui = decode_unit(p, u);
-            is.item = p.items[ui.item];
-            is.bh = ui.bh;
-          }
-          ctl->slot[slot] = is;
-          mbar_arrive(bar(ctl->item_full[slot]));
-        }
-        u = __shfl_sync(0xffffffffu, u, 0);
-        ++it;
-        if (u >= p.total_units) break;
-        __syncwarp();
+        mbar_wait(bar(ctl->item_full[slot]), ph);
+        const int u = ctl->slot[slot].u;
         const Item item = ctl->slot[slot].item;
         const int bh = ctl->slot[slot].bh;
+        __syncwarp();
+        if (lane == 0) mbar_arrive(bar(ctl->item_empty[slot]));
+        ++it;
+        if (u >= p.total_units) break;
         const int bb = bh / p.H, hh = bh % p.H;
+        if (lane == 0) trace(0, 1, u);
         const uint32_t qs = qi & 1;
         const uint32_t dQ = sQ + qs * 2 * kTileBytes;
-        if (lane == 0) trace(0, 1, u);
         mbar_wait(bar(ctl->q_empty[qs]), ((qi >> 1) & 1) ^ 1);
         if (item.kind == 0) {
           if (lane == 0) {
@@ -321,19 +312,63 @@ __global__ void __launch_bounds__(kThreads, 1)
           }
         }
       }
+    } else if (warp == 2) {
+      // ========================================================== scheduler
+      // Publishes work items in a 2-deep ring (dynamic counter) as soon as a slot frees, i.e. up
+      // to two items ahead of the slowest consumer, and warms L2 with each item's Q and K/V tiles
+      // (TMA prefetch, one lane per tile) so the producer's later TMA loads hit L2.
+      Tracer trace(p, 0);
+      uint32_t it = 0;
+      while (true) {
+        const uint32_t slot = it & 1, ph = (it >> 1) & 1;
+        int u = 0;
+        if (lane == 0) {
+          trace(0, 4, it);
+          mbar_wait(bar(ctl->item_empty[slot]), ph ^ 1);
+          trace(0, 5, it);
+          u = atomicAdd(p.counter, 1);
+          ItemSlot is;
+          is.u = u;
+          if (u < p.total_units) {
+            const UnitInfo ui = decode_unit(p, u);
+            is.item = p.items[ui.item];
+            is.bh = ui.bh;
+          }
+          ctl->slot[slot] = is;
+          mbar_arrive(bar(ctl->item_full[slot]));
+        }
+        ++it;
+        u = __shfl_sync(0xffffffffu, u, 0);
+        if (u >= p.total_units) break;
+        __syncwarp();
+        const Item item = ctl->slot[slot].item;
+        const int bh = ctl->slot[slot].bh;
+        const int bb = bh / p.H, hh = bh % p.H;
+        if (lane == 0 && item.kind == 0) {
+          tma_prefetch_4d(&tmq, 0, item.rowA, hh, bb);
+          if (item.nrowsB) tma_prefetch_4d(&tmq, 0, item.rowB, hh, bb);
+        }
+        for (int j = lane; j < item.ntiles; j += 32) {
+          const TileRef tr = p.trefs[item.tref_begin + j];
+          if (tr.kind == 0) {
+            tma_prefetch_4d(&tmk, 0, tr.arg, hh, bb);
+            tma_prefetch_4d(&tmv, 0, tr.arg, hh, bb);
+          }
+        }
+      }
     } else if (warp == 1 || warp == 3) {
       // ========================================================== MMA issuers (one warp per stream)
-      // Stream w = (warp == 3): per K/V tile j, S_w(j) then P_w(j-1) V(j-1). The streams never
-      // wait on each other; each releases a K/V stage after its own P.V (kv_empty counts 2).
-      // The whole warp walks the schedule; lane 0 issues tcgen05.mma / commit.
+      // The pipeline unit is a half tile (64 keys): S_h = Q K_h^T (N = 64) into one of three TMEM
+      // buffers of the stream, P_h written by the softmax over the same buffer (16-bit pairs), then
+      // O += P_h V_h. S runs two halves ahead of P.V; a buffer is reused once its P.V completed.
+      // Streams never wait on each other; each releases a K/V stage after its own last P.V of the
+      // tile (kv_empty counts 2). The whole warp walks the schedule; lane 0 issues.
       const int w = warp == 3 ? 1 : 0;
       const bool leader = lane == 0;
       Tracer trace(p, 1);
-      uint32_t it = 0, g = 0, qi = 0, nS = 0, nP = 0;
-      const uint32_t idesc_pv = idesc_f16(kBF16, 128, 64, false, true);
-      const uint32_t dS = tmem + kTmemS + w * 128;
-      const uint32_t dO = tmem + kTmemO + w * 64;
-      const uint32_t aP = tmem + kTmemP + w * 64;
+      uint32_t it = 0, g = 0, qi = 0, hS = 0, hP = 0;   // halves with S / P.V issued (CTA lifetime)
+      const uint32_t tbase = tmem + w * 256;
+      const uint32_t dO = tbase + kTmemOOff;
       while (true) {
         const uint32_t slot = it & 1, ph = (it >> 1) & 1;
         mbar_wait(bar(ctl->item_full[slot]), ph);
@@ -343,67 +378,103 @@ __global__ void __launch_bounds__(kThreads, 1)
         if (leader) mbar_arrive(bar(ctl->item_empty[slot]));
         ++it;
         if (u >= p.total_units) break;
-        const int nrows = w == 0 ? item.nrowsA : item.nrowsB;
         const uint32_t qs = qi & 1;
         const uint32_t qa = sQ + qs * 2 * kTileBytes + w * kTileBytes;
         mbar_wait(bar(ctl->q_full[qs]), (qi >> 1) & 1);
         ++qi;
-        bool first = true, prev_use = false;
-        int prev_n = 0;
-        uint32_t prev_st = 0, prev_g = 0;
-        auto release_prev = [&]() {   // P.V of the previous tile (if used), then free its stage
-          if (prev_use) {
-            mbar_wait(bar(ctl->v_full[prev_st]), (prev_g / kStages) & 1);
-            mbar_wait(bar(ctl->p_full[w]), nP & 1);
-            tc_fence_after();
-            if (leader) {
-              const uint32_t vA = sV + prev_st * kTileBytes;
-              for (int kk = 0; kk < (prev_n >> 4); ++kk)
-                mma_ts(dO, aP + kk * 8, smem_desc_sw128(vA + kk * 2048, 8192, 1024), idesc_pv,
-                       (first && kk == 0) ? 0u : 1u);
-              mma_commit(bar(ctl->o_full[w]));
-              mma_commit(bar(ctl->kv_empty[prev_st]));
+        const int nt = item.ntiles;
+        // S cursor (tile sj, half sh of nsh) and P.V cursor (tile pj, half phh)
+        int sj = 0, sh = 0, nsh = 0;
+        int pj = 0, phh = 0;
+        bool first_pv = true, s_done = false;
+        // advance the S cursor to the next half this stream uses (waits k_full of used tiles only:
+        // skipped tiles are released by the P.V cursor, which may be far behind)
+        auto s_advance = [&]() -> bool {
+          while (true) {
+            if (sh < nsh) return true;
+            if (sj >= nt) return false;
+            if (item_uses(item, w, sj)) {
+              const uint32_t gg = g + sj, st = gg % kStages;
+              mbar_wait(bar(ctl->k_full[st]), (gg / kStages) & 1);
+              nsh = ctl->tref[st].ncols > 64 ? 2 : 1;
+              sh = 0;
+              ++sj;
+              return true;
             }
-            first = false;
-            ++nP;
-          } else if (leader) {
-            mbar_arrive(bar(ctl->kv_empty[prev_st]));
+            ++sj;
+            nsh = 0;
+            sh = 0;
           }
-          __syncwarp();
         };
-        for (int j = 0; j < item.ntiles; ++j) {
-          const uint32_t gg = g + j, st = gg % kStages;
-          mbar_wait(bar(ctl->k_full[st]), (gg / kStages) & 1);
-          const TileRef tr = ctl->tref[st];
-          const bool use = item_uses(item, w, j);
-          if (use) {
-            if (nS > 0) mbar_wait(bar(ctl->s_empty[w]), (nS - 1) & 1);
-            tc_fence_after();
-            if (leader) {
-              const uint32_t idesc_s = idesc_f16(kBF16, 128, tr.ncols, false, false);
-              const uint32_t kA = sK + st * kTileBytes;
-#pragma unroll
-              for (int kk = 0; kk < 4; ++kk)
-                mma_ss(dS, smem_desc_sw128(qa + kk * 32, 16, 1024), smem_desc_sw128(kA + kk * 32, 16, 1024),
-                       idesc_s, kk > 0);
-              mma_commit(bar(ctl->s_full[w]));
-            }
-            __syncwarp();
-            ++nS;
-          }
-          if (j == item.ntiles - 1) {
+        auto issue_s = [&]() {
+          if (s_done) return;
+          if (!s_advance()) {
+            s_done = true;
             if (leader) mma_commit(bar(ctl->q_empty[qs]));
             __syncwarp();
+            return;
           }
-          if (j >= 1) release_prev();
-          prev_use = use;
-          prev_n = tr.ncols;
-          prev_st = st;
-          prev_g = gg;
-        }
-        release_prev();
-        if (leader && w == 0) trace(1, 2, g + item.ntiles - 1);
-        g += item.ntiles;
+          const uint32_t gg = g + sj - 1, st = gg % kStages;
+          const int ncols = ctl->tref[st].ncols;
+          const int n = ncols - sh * 64 > 64 ? 64 : ncols - sh * 64;   // keys in this half
+          const uint32_t b = hS % 3;
+          if (hS >= 3) mbar_wait(bar(ctl->pv_done[w][b]), ((hS - 3) / 3) & 1);
+          tc_fence_after();
+          if (leader) {
+            const uint32_t idesc_s = idesc_f16(kBF16, 128, n, false, false);
+            const uint32_t kA = sK + st * kTileBytes + sh * 8192;
+#pragma unroll
+            for (int kk = 0; kk < 4; ++kk)
+              mma_ss(tbase + b * 64, smem_desc_sw128(qa + kk * 32, 16, 1024), smem_desc_sw128(kA + kk * 32, 16, 1024),
+                     idesc_s, kk > 0);
+            mma_commit(bar(ctl->s_full[w][b]));
+          }
+          __syncwarp();
+          ++sh;
+          ++hS;
+        };
+        // next P.V: releases the stages of tiles it passes (skipped tiles, finished tiles)
+        auto issue_pv = [&]() -> bool {
+          while (pj < nt && !item_uses(item, w, pj)) {     // tiles this stream skips
+            const uint32_t gs = g + pj;
+            mbar_wait(bar(ctl->k_full[gs % kStages]), (gs / kStages) & 1);   // stage holds this tile
+            if (leader) mbar_arrive(bar(ctl->kv_empty[gs % kStages]));
+            __syncwarp();
+            ++pj;
+          }
+          if (pj >= nt) return false;
+          const uint32_t gg = g + pj, st = gg % kStages;
+          const int ncols = ctl->tref[st].ncols;
+          const int nh = ncols > 64 ? 2 : 1;
+          const int n = ncols - phh * 64 > 64 ? 64 : ncols - phh * 64;
+          const uint32_t b = hP % 3;
+          if (phh == 0) mbar_wait(bar(ctl->v_full[st]), (gg / kStages) & 1);
+          mbar_wait(bar(ctl->p_full[w][b]), (hP / 3) & 1);
+          tc_fence_after();
+          if (leader) {
+            const uint32_t idesc_pv = idesc_f16(kBF16, 128, 64, false, true);
+            const uint32_t vA = sV + st * kTileBytes + phh * 8192;
+            for (int kk = 0; kk < (n >> 4); ++kk)
+              mma_ts(dO, tbase + b * 64 + kk * 8, smem_desc_sw128(vA + kk * 2048, 8192, 1024), idesc_pv,
+                     (first_pv && kk == 0) ? 0u : 1u);
+            mma_commit(bar(ctl->pv_done[w][b]));
+            if (phh == nh - 1) mma_commit(bar(ctl->kv_empty[st]));
+          }
+          __syncwarp();
+          first_pv = false;
+          ++hP;
+          if (++phh == nh) {
+            phh = 0;
+            ++pj;
+          }
+          return true;
+        };
+        issue_s();
+        issue_s();
+        while (issue_pv()) issue_s();
+        if (!s_done) issue_s();                            // commits q_empty when nothing is left
+        if (leader) trace(1, 2, g + nt - 1);
+        g += nt;
       }
     }
   } else {
@@ -413,17 +484,28 @@ __global__ void __launch_bounds__(kThreads, 1)
     const int q4 = warp & 3;                               // TMEM lane quarter
     const int t = q4 * 32 + lane;                          // row of the stream's Q tile = TMEM lane
     const uint32_t lane_base = (uint32_t)(q4 * 32) << 16;
-    const uint32_t tS = tmem + lane_base + kTmemS + w * 128;
-    const uint32_t tP = tmem + lane_base + kTmemP + w * 64;
-    const uint32_t tO = tmem + lane_base + kTmemO + w * 64;
+    const uint32_t tbase = tmem + lane_base + w * 256;
+    const uint32_t tO = tbase + kTmemOOff;
     const float c = p.scale_log2;
     const float2 c2 = make_float2(c, c);
     Tracer trace(p, 2 + w);
     const bool tr_on = (warp == 4 || warp == 8) && lane == 0;
-    // lazy rescaling (O accumulates in TMEM): the exponent uses a stale row max m until a tile's
-    // max exceeds it by more than 2^8 in probability, so p <= 256 and O/l rarely need a rescale
+    const bool dry = (p.debug_flags & 1) != 0;
+    // Exp ping-pong between the two softmax warps sharing an SMSP (stream A warp q, stream B
+    // warp q): they alternate their exp half-tiles (A first) through two named barriers, so each
+    // overlaps its loads/max/waits with the other's MUFU work.
+    const uint32_t bar_a_go = 1 + q4, bar_b_go = 5 + q4;
+    auto turn_begin = [&](bool on) {
+      if (on) named_bar_sync(w == 0 ? bar_a_go : bar_b_go, 64);
+    };
+    auto turn_end = [&](bool on) {
+      if (on) asm volatile("bar.arrive %0, %1;" ::"r"(w == 0 ? bar_b_go : bar_a_go), "r"(64) : "memory");
+    };
+    if (w == 1) turn_end(true);                            // A takes the first turn
+    // lazy rescaling (O accumulates in TMEM): the exponent uses a stale row max m until a half
+    // tile's max exceeds it by more than 2^8 in probability, so p <= 256 and O rarely needs a rescale
     const float thresh = 8.f / c;
-    uint32_t it = 0, g = 0, n = 0;                         // n: tiles processed by this stream
+    uint32_t it = 0, g = 0, hs = 0;                        // hs: halves processed by this stream
     while (true) {
       const uint32_t slot = it & 1, ph = (it >> 1) & 1;
       mbar_wait(bar(ctl->item_full[slot]), ph);
@@ -436,57 +518,56 @@ __global__ void __launch_bounds__(kThreads, 1)
       if (u >= p.total_units) break;
       const int nrows = w == 0 ? item.nrowsA : item.nrowsB;
       const bool active = q4 * 32 < nrows;                 // this warp has real rows
+      // epilogue metadata, loaded now so its latency hides behind the item's tiles
+      int r_out = -1, slot_f = -1;
+      if (t < nrows) {
+        const int rbase = w == 0 ? item.rowA : item.rowB;
+        r_out = item.kind == 0 ? rbase + t : __ldg(p.global_rows + rbase + t);
+        if (item.kind == 0) slot_f = __ldg(p.fine_slot + rbase + t);
+      }
       float m = -INFINITY, l = 0.f;
-      uint32_t n_item = 0;
+      uint32_t h_item = 0;
+      const bool pp = item.turns > 0;                      // both streams active: ping-pong
+      int turns_done = 0;
       for (int j = 0; j < item.ntiles && nrows > 0; ++j) {
-        const uint32_t gg = g + j, st = gg % kStages;
         // a skipped tile's stage may already be recycled: decide from the item's use bitmap
         if (!item_uses(item, w, j)) continue;
-        // tile descriptor + bitmask landed with the stage's K tile
-        mbar_wait(bar(ctl->k_full[st]), (gg / kStages) & 1);
+        const uint32_t gg = g + j, st = gg % kStages;
+        mbar_wait(bar(ctl->k_full[st]), (gg / kStages) & 1);   // tile descriptor + bitmask
         const TileRef tr = ctl->tref[st];
-        const int32_t mk = w == 0 ? tr.maskA : tr.maskB;
-        const int nch = tr.ncols >> 4;                     // 16-column chunks (2..8)
-        const bool partial = mk >= 0;
+        const bool partial = (w == 0 ? tr.maskA : tr.maskB) >= 0;
         uint64_t w0 = ~0ull, w1 = ~0ull;
         if (partial && active) {
           const int4 mw = ld_shared_v4(sM + st * 2 * kMaskBytes + w * kMaskBytes + t * 16);
           w0 = ((uint64_t)(uint32_t)mw.y << 32) | (uint32_t)mw.x;
           w1 = ((uint64_t)(uint32_t)mw.w << 32) | (uint32_t)mw.z;
         }
-        if (tr_on) trace(2 + w, 1, gg);
-        mbar_wait(bar(ctl->s_full[w]), n & 1);
-        if (tr_on) trace(2 + w, 2, gg);
-        tc_fence_after();
-        // S is read once, as two 64-column halves (four x16 loads in flight, one wait each). Each
-        // half runs max -> lazy rescale -> exp -> P store; if the second half raises the row max
-        // beyond the threshold, the first half's P (already in TMEM) is rescaled with O and l.
-        const int nhalf = nch > 4 ? 2 : 1;
-        for (int hf = 0; hf < nhalf; ++hf) {
-          const int nc = hf == 0 ? (nch > 4 ? 4 : nch) : nch - 4;   // 16-column chunks in this half
+        const int nh = tr.ncols > 64 ? 2 : 1;
+        for (int hh = 0; hh < nh; ++hh, ++hs, ++h_item) {
+          const int nc = (tr.ncols - hh * 64 > 64 ? 64 : tr.ncols - hh * 64) >> 4;   // 16-col chunks
+          const uint32_t b = hs % 3;
+          const uint32_t tS = tbase + b * 64;
+          const uint64_t wd = hh ? w1 : w0;
+          if (tr_on) trace(2 + w, 1, gg);
+          mbar_wait(bar(ctl->s_full[w][b]), (hs / 3) & 1);
+          tc_fence_after();
           uint32_t r0[16], r1[16], r2[16], r3[16];
           if (active) {
-            const uint32_t a = tS + hf * 64;
-            tmem_ld16(a, r0);
-            if (nc > 1) tmem_ld16(a + 16, r1);
-            if (nc > 2) tmem_ld16(a + 32, r2);
-            if (nc > 3) tmem_ld16(a + 48, r3);
+            tmem_ld16(tS, r0);
+            if (nc > 1) tmem_ld16(tS + 16, r1);
+            if (nc > 2) tmem_ld16(tS + 32, r2);
+            if (nc > 3) tmem_ld16(tS + 48, r3);
             tmem_wait_ld();
           }
-          if (hf == nhalf - 1) {                           // S buffer free for the next tile
-            tc_fence_before();
-            __syncwarp();
-            if (lane == 0) mbar_arrive(bar(ctl->s_empty[w]));
-          }
+          if (tr_on) trace(2 + w, 2, gg);
           float tmax = -INFINITY;
-          if (active) {
+          if (active && !dry) {
             float mx0 = -INFINITY, mx1 = -INFINITY;
-            const int cb = hf * 4;
             if (partial) {
-              chunk_max<true>(r0, chunk_bits16(w0, w1, cb), mx0, mx1);
-              if (nc > 1) chunk_max<true>(r1, chunk_bits16(w0, w1, cb + 1), mx0, mx1);
-              if (nc > 2) chunk_max<true>(r2, chunk_bits16(w0, w1, cb + 2), mx0, mx1);
-              if (nc > 3) chunk_max<true>(r3, chunk_bits16(w0, w1, cb + 3), mx0, mx1);
+              chunk_max<true>(r0, (uint32_t)wd & 0xffffu, mx0, mx1);
+              if (nc > 1) chunk_max<true>(r1, (uint32_t)(wd >> 16) & 0xffffu, mx0, mx1);
+              if (nc > 2) chunk_max<true>(r2, (uint32_t)(wd >> 32) & 0xffffu, mx0, mx1);
+              if (nc > 3) chunk_max<true>(r3, (uint32_t)(wd >> 48) & 0xffffu, mx0, mx1);
             } else {
               chunk_max<false>(r0, 0xffffu, mx0, mx1);
               if (nc > 1) chunk_max<false>(r1, 0xffffu, mx0, mx1);
@@ -495,7 +576,7 @@ __global__ void __launch_bounds__(kThreads, 1)
             }
             tmax = fmaxf(mx0, mx1);
           }
-          // lazy rescale decision (warp-uniform for the TMEM accesses)
+          // lazy rescale decision (warp-uniform for the TMEM access)
           const bool need = tmax > m + thresh || (m == -INFINITY && tmax != -INFINITY);
           float alpha = 1.f;
           if (need) {
@@ -503,14 +584,11 @@ __global__ void __launch_bounds__(kThreads, 1)
             m = tmax;
           }
           l *= alpha;
-          const bool any_rescale = __any_sync(0xffffffffu, need && alpha != 0.f);
-          if (hf == 0 && n_item > 0) {
-            // previous P.V done: the P buffer may be overwritten and O may be rescaled
-            mbar_wait(bar(ctl->o_full[w]), (n - 1) & 1);
+          if (__any_sync(0xffffffffu, need && alpha != 0.f) && h_item > 0) {
+            // O holds earlier halves of this item: wait for the last issued P.V, then rescale
+            mbar_wait(bar(ctl->pv_done[w][(hs - 1) % 3]), ((hs - 1) / 3) & 1);
             tc_fence_after();
-          }
-          if (any_rescale && active) {
-            if (n_item > 0) {
+            if (active) {
 #pragma unroll
               for (int h2 = 0; h2 < 4; ++h2) {
                 uint32_t r[16];
@@ -521,78 +599,64 @@ __global__ void __launch_bounds__(kThreads, 1)
                 tmem_st16(tO + h2 * 16, r);
               }
             }
-            if (hf == 1) {                                 // first half's P, 32 packed columns
-              tmem_wait_st();
-#pragma unroll
-              for (int h2 = 0; h2 < 2; ++h2) {
-                uint32_t r[16];
-                tmem_ld16(tP + h2 * 16, r);
-                tmem_wait_ld();
-#pragma unroll
-                for (int i = 0; i < 16; ++i) {
-                  float lo, hi;
-                  unpack2<kBF16>(r[i], lo, hi);
-                  r[i] = pack2<kBF16>(lo * alpha, hi * alpha);
-                }
-                tmem_st16(tP + h2 * 16, r);
-              }
-            }
           }
-          if (active) {
+          // p = 2^(s*c - m*c) (masked -> 0), packed to 16-bit pairs over this half's own S buffer
+          turn_begin(pp);
+          if (active && !dry) {
             const float mu = (m == -INFINITY) ? 0.f : m;
             const float2 nb2 = make_float2(-mu * c, -mu * c);
             float2 rs0 = make_float2(0.f, 0.f), rs1 = make_float2(0.f, 0.f);
-            const uint32_t pb = tP + hf * 32;
-            const int cb = hf * 4;
             if (partial) {
-              chunk_exp<true, kBF16>(r0, chunk_bits16(w0, w1, cb), c2, nb2, rs0, rs1, pb);
-              if (nc > 1) chunk_exp<true, kBF16>(r1, chunk_bits16(w0, w1, cb + 1), c2, nb2, rs0, rs1, pb + 8);
-              if (nc > 2) chunk_exp<true, kBF16>(r2, chunk_bits16(w0, w1, cb + 2), c2, nb2, rs0, rs1, pb + 16);
-              if (nc > 3) chunk_exp<true, kBF16>(r3, chunk_bits16(w0, w1, cb + 3), c2, nb2, rs0, rs1, pb + 24);
+              chunk_exp<true, kBF16>(r0, (uint32_t)wd & 0xffffu, c2, nb2, rs0, rs1, tS);
+              if (nc > 1) chunk_exp<true, kBF16>(r1, (uint32_t)(wd >> 16) & 0xffffu, c2, nb2, rs0, rs1, tS + 8);
+              if (nc > 2) chunk_exp<true, kBF16>(r2, (uint32_t)(wd >> 32) & 0xffffu, c2, nb2, rs0, rs1, tS + 16);
+              if (nc > 3) chunk_exp<true, kBF16>(r3, (uint32_t)(wd >> 48) & 0xffffu, c2, nb2, rs0, rs1, tS + 24);
             } else {
-              chunk_exp<false, kBF16>(r0, 0xffffu, c2, nb2, rs0, rs1, pb);
-              if (nc > 1) chunk_exp<false, kBF16>(r1, 0xffffu, c2, nb2, rs0, rs1, pb + 8);
-              if (nc > 2) chunk_exp<false, kBF16>(r2, 0xffffu, c2, nb2, rs0, rs1, pb + 16);
-              if (nc > 3) chunk_exp<false, kBF16>(r3, 0xffffu, c2, nb2, rs0, rs1, pb + 24);
+              chunk_exp<false, kBF16>(r0, 0xffffu, c2, nb2, rs0, rs1, tS);
+              if (nc > 1) chunk_exp<false, kBF16>(r1, 0xffffu, c2, nb2, rs0, rs1, tS + 8);
+              if (nc > 2) chunk_exp<false, kBF16>(r2, 0xffffu, c2, nb2, rs0, rs1, tS + 16);
+              if (nc > 3) chunk_exp<false, kBF16>(r3, 0xffffu, c2, nb2, rs0, rs1, tS + 24);
             }
             l += (rs0.x + rs0.y) + (rs1.x + rs1.y);
           }
+          turn_end(pp);
+          ++turns_done;
+          if (active) tmem_wait_st();
+          tc_fence_before();
+          __syncwarp();
+          if (lane == 0) mbar_arrive(bar(ctl->p_full[w][b]));
+          if (tr_on) trace(2 + w, 3, gg);
         }
-        if (active) tmem_wait_st();
-        tc_fence_before();
-        __syncwarp();
-        if (lane == 0) mbar_arrive(bar(ctl->p_full[w]));
-        if (tr_on) trace(2 + w, 3, gg);
-        ++n;
-        ++n_item;
       }
       g += item.ntiles;
-      if (n_item == 0) continue;                           // stream unused in this item
+      for (; pp && turns_done < item.turns; ++turns_done) {  // keep the turn sequences aligned
+        turn_begin(true);
+        turn_end(true);
+      }
+      if (h_item == 0) continue;                           // stream unused in this item
       // the item's last P.V: O is complete in TMEM
-      mbar_wait(bar(ctl->o_full[w]), (n - 1) & 1);
+      mbar_wait(bar(ctl->pv_done[w][(hs - 1) % 3]), ((hs - 1) / 3) & 1);
       tc_fence_after();
       float oacc[64];
       if (active) {
 #pragma unroll
-        for (int h2 = 0; h2 < 2; ++h2) {
-          uint32_t r[32];
-          tmem_ld32(tO + h2 * 32, r);
-          tmem_wait_ld();
+        for (int h2 = 0; h2 < 4; ++h2) {
+          uint32_t r[16];
+          tmem_ld16(tO + h2 * 16, r);
 #pragma unroll
-          for (int i = 0; i < 32; ++i) oacc[h2 * 32 + i] = __uint_as_float(r[i]);
+          for (int i = 0; i < 16; ++i) oacc[h2 * 16 + i] = __uint_as_float(r[i]);
         }
+        tmem_wait_ld();
       }
       tc_fence_before();
       if (tr_on) trace(2 + w, 5, g - 1);
 
       // ---- epilogue: merge the fine partial (if any), normalise, store the row's 64 outputs
-      if (t < nrows) {
-        const int rbase = w == 0 ? item.rowA : item.rowB;
-        const int r = item.kind == 0 ? rbase + t : __ldg(p.global_rows + rbase + t);
+      if (r_out >= 0) {
+        const int r = r_out;
         float mf = -INFINITY, lf = 0.f;
         const float* accf = nullptr;
-        if (item.kind == 0) {
-          const int slot_f = __ldg(p.fine_slot + r);
+        {
           if (slot_f >= 0) {
             const size_t idx = (size_t)ubh * p.n_fine_rows + slot_f;
             const float2 ml = p.part_ml[idx];
@@ -632,6 +696,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     }
   }
 
+  if (warp >= 4 && warp < 8) named_bar_sync(1 + (warp & 3), 64);  // match stream B's last turn hand-off
   tc_fence_before();
   __syncthreads();
   if (warp == 2) tmem_dealloc(tmem, 512);

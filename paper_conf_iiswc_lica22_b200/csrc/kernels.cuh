@@ -36,6 +36,7 @@ struct CoarseParams {
   float scale_log2;           // (1/sqrt(d)) * log2(e)
   unsigned long long* trace;  // diagnostics: event trace of CTA 0 (null = off)
   int32_t trace_cap;
+  int32_t debug_flags;        // diagnostics (env MG_DEBUG_FLAGS): 1 = softmax skips its arithmetic
 };
 
 // Fine CSR kernel: warp per (row, batch*head); SDDMM -> online softmax -> SpMM on CUDA cores.

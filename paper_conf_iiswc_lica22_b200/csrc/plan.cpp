@@ -167,8 +167,8 @@ std::string build_plan(HostPlan& p, int64_t L, int32_t heads, int32_t d, int32_t
   for (int64_t k = 0; k < G; k += 256) {
     const int32_t na = (int32_t)std::min<int64_t>(128, G - k);
     const int32_t nbr = (int32_t)std::max<int64_t>(0, std::min<int64_t>(128, G - k - 128));
-    Item it{1, (int32_t)k, (int32_t)(k + 128), (int32_t)nb, (int32_t)p.trefs.size(), na, nbr, 0, ~0ull,
-            nbr ? ~0ull : 0ull};
+    Item it{1, (int32_t)k, (int32_t)(k + 128), (int32_t)nb, (int32_t)p.trefs.size(), na, nbr,
+            nbr ? (int32_t)(2 * nb) : 0, ~0ull, nbr ? ~0ull : 0ull};
     for (int64_t J = 0; J < nb; ++J) {
       const int32_t m = (J == nb - 1) ? ragged_mask : kMaskFull;
       p.trefs.push_back(TileRef{(int32_t)(J * B), 0, 128, m, nbr ? m : kMaskSkip, 0, 0, 0});
@@ -289,11 +289,13 @@ std::string build_plan(HostPlan& p, int64_t L, int32_t heads, int32_t d, int32_t
     if (sa) blk_strip[IA] = 1;
     if (sb) blk_strip[IB] = 1;
     it.ntiles = (int32_t)p.trefs.size() - it.tref_begin;
+    int32_t ha = 0, hb = 0;
     for (int32_t j = 0; j < it.ntiles && j < 64; ++j) {
       const TileRef& r = p.trefs[it.tref_begin + j];
-      if (r.maskA != kMaskSkip && it.nrowsA) it.useA |= 1ull << j;
-      if (r.maskB != kMaskSkip && it.nrowsB) it.useB |= 1ull << j;
+      if (r.maskA != kMaskSkip && it.nrowsA) { it.useA |= 1ull << j; ha += (r.ncols + 63) / 64; }
+      if (r.maskB != kMaskSkip && it.nrowsB) { it.useB |= 1ull << j; hb += (r.ncols + 63) / 64; }
     }
+    it.turns = (it.nrowsA && it.nrowsB) ? std::max(ha, hb) : 0;
     p.items.push_back(it);
   }
 

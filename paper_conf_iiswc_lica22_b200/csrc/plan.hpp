@@ -28,7 +28,8 @@ struct PlanOptions {
 //     starts at strip_cols[arg]; maskX = index of a 128 x 2-word bitmask for stream X,
 //     -1 = all valid, -2 = stream X does not use this tile.
 struct Item {
-  int32_t kind, rowA, rowB, ntiles, tref_begin, nrowsA, nrowsB, pad;
+  int32_t kind, rowA, rowB, ntiles, tref_begin, nrowsA, nrowsB;
+  int32_t turns;  // exp half-tiles per softmax stream (max over A, B) when both are active, else 0
   uint64_t useA, useB;
 };
 struct TileRef { int32_t arg, kind, ncols, maskA, maskB, pad0, pad1, pad2; };

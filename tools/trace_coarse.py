@@ -17,11 +17,14 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import paper_conf_iiswc_lica22_b200 as mg  # noqa: E402
 from workloads import get_config, make_qkv  # noqa: E402
 
-NAMES = {(0, 1): "P:item", (0, 2): "P:qfree", (0, 3): "P:kvfree",
+NAMES = {(0, 1): "P:item", (0, 2): "P:qfree", (0, 3): "P:kvfree", (0, 4): "P:slotwait", (0, 5): "P:slotfree",
          (1, 0): "M:qready", (1, 1): "M:kready", (1, 2): "M:Sissue", (1, 4): "M:Pready", (1, 5): "M:PVissue",
          (2, 1): "S:tile", (2, 2): "S:Sready", (2, 3): "S:Pstored", (2, 4): "S:Oconsumed", (2, 5): "S:itemO",
-         (2, 6): "S:xch", (3, 1): "T:tile", (3, 2): "T:Sready", (3, 3): "T:Pstored", (3, 4): "T:Oconsumed",
-         (3, 5): "T:itemO", (3, 6): "T:xch"}
+         (2, 6): "S:xch", (2, 7): "S:ld0", (2, 8): "S:max0", (2, 9): "S:pvwait0", (2, 10): "S:exp0",
+         (2, 11): "S:ld1", (2, 12): "S:max1", (2, 13): "S:pvwait1", (2, 14): "S:exp1", (3, 1): "T:tile", (3, 2): "T:Sready", (3, 3): "T:Pstored", (3, 4): "T:Oconsumed",
+         (3, 5): "T:itemO", (3, 6): "T:xch",
+         (3, 7): "T:ld0", (3, 8): "T:max0", (3, 9): "T:pvwait0", (3, 10): "T:exp0",
+         (3, 11): "T:ld1", (3, 12): "T:max1", (3, 13): "T:pvwait1", (3, 14): "T:exp1"}
 
 
 def main():
@@ -63,7 +66,7 @@ def main():
     print(f"\n{n} events, span {int(ev[-1, 0] - t0)} cycles")
     print("mean cycles between consecutive events of the same role:")
     for (a, b), v_ in sorted(gaps.items(), key=lambda x: -sum(x[1])):
-        print(f"  {a:<12} -> {b:<12} n={len(v_):>5} mean={np.mean(v_):>8.1f} total={sum(v_):>10}")
+        print(f"  {str(a):<12} -> {str(b):<12} n={len(v_):>5} mean={np.mean(v_):>8.1f} total={sum(v_):>10}")
 
 
 if __name__ == "__main__":
