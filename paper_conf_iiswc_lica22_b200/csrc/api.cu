@@ -59,6 +59,7 @@ struct mg_plan_s {
   int32_t* d_fine_row_ptr = nullptr;
   int32_t* d_fine_col = nullptr;
   int32_t* d_counter = nullptr;
+  float* d_dense_xch = nullptr;   // per-CTA scratch of the tensor-core kernel (kind-2 merge)
   // stream-ordered workspaces
   float* d_part = nullptr;
   size_t part_cap = 0;      // in (row, bh) partial slots
@@ -122,7 +123,8 @@ mg_status upload(mg_plan_s* p) {
       (e = upload_vec(p, &p->d_fine_rows, h.fine_rows)) != cudaSuccess ||
       (e = upload_vec(p, &p->d_fine_row_ptr, h.fine_row_ptr)) != cudaSuccess ||
       (e = upload_vec(p, &p->d_fine_col, h.fine_col)) != cudaSuccess ||
-      (e = upload_vec(p, &p->d_counter, std::vector<int32_t>(4, 0))) != cudaSuccess)
+      (e = upload_vec(p, &p->d_counter, std::vector<int32_t>(4, 0))) != cudaSuccess ||
+      (e = upload_vec(p, &p->d_dense_xch, std::vector<float>((size_t)p->num_sms * 128 * 68, 0.f))) != cudaSuccess)
     return e == cudaErrorMemoryAllocation ? fail(MG_ERR_OUT_OF_MEMORY, "device allocation failed")
                                           : cuda_fail(e, "plan upload");
   p->uploaded = true;
@@ -302,6 +304,7 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
     cp.part_acc = part_acc;
     cp.part_ml = part_ml;
     cp.counter = p->d_counter;
+    cp.dense_xch = p->d_dense_xch;
     cp.q = view(Q); cp.k = view(K); cp.v = view(V); cp.o = view(O);
     cp.L = h.L;
     cp.H = h.heads;
@@ -321,7 +324,7 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
     cp.trace_cap = p->trace_cap;
     if ((e = cudaMemsetAsync(p->d_counter, 0, sizeof(int32_t), stream)) != cudaSuccess)
       return cuda_fail(e, "cudaMemsetAsync");
-    const int sms = p->num_sms_override > 0 ? p->num_sms_override : p->num_sms;
+    const int sms = p->num_sms_override > 0 ? std::min(p->num_sms_override, p->num_sms) : p->num_sms;
     const int grid = std::min(sms, cp.total_units);
     if (p->profiling) cudaEventRecord(ev[2], stream);  // after the counter reset
     if ((e = mg::launch_coarse(cp, tq, tk, tv, bf16, grid, stream)) != cudaSuccess)

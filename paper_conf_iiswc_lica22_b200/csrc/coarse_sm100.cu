@@ -37,8 +37,8 @@ constexpr int kStages = 4;
 constexpr int kThreads = 384;
 constexpr uint32_t kTileBytes = 128 * 128;  // 128 rows x 64 x 16-bit
 constexpr uint32_t kMaskBytes = 128 * 16;   // 128 rows x 2 x u64
-// TMEM per stream w (256 columns at w*256): three 64-column S/P half-tile buffers, then O.
-constexpr uint32_t kTmemOOff = 192;
+// TMEM per stream w (256 columns at w*256): S [0,128), P (16-bit pairs) [128,192), O [192,256).
+constexpr uint32_t kTmemPOff = 128, kTmemOOff = 192;
 
 struct __align__(16) ItemSlot {
   Item item;
@@ -48,6 +48,7 @@ struct __align__(16) ItemSlot {
 // does stream w use tile j of the item (without touching the stage)
 __device__ __forceinline__ bool item_uses(const Item& it, int w, int j) {
   if ((w == 0 ? it.nrowsA : it.nrowsB) == 0) return false;
+  if (it.kind == 2) return (j & 1) == w;
   if (j >= 64) return true;
   return (((w == 0 ? it.useA : it.useB) >> j) & 1ull) != 0;
 }
@@ -57,7 +58,7 @@ struct __align__(16) SmemCtl {
   ItemSlot slot[2];
   uint64_t q_full[2], q_empty[2];
   uint64_t k_full[kStages], v_full[kStages], kv_empty[kStages];
-  uint64_t s_full[2][3], p_full[2][3], pv_done[2][3];   // per stream, per half-tile buffer
+  uint64_t s_full[2], s_free[2], p_full[2], pv_done[2];  // per stream
   uint64_t item_full[2], item_empty[2];
   uint32_t tmem_base;
 };
@@ -207,11 +208,10 @@ __global__ void __launch_bounds__(kThreads, 1)
     for (int b = 0; b < 2; ++b) {
       mbar_init(bar(ctl->q_full[b]), 1);
       mbar_init(bar(ctl->q_empty[b]), 2);           // one commit per MMA warp
-      for (int x = 0; x < 3; ++x) {
-        mbar_init(bar(ctl->s_full[b][x]), 1);
-        mbar_init(bar(ctl->p_full[b][x]), 4);
-        mbar_init(bar(ctl->pv_done[b][x]), 1);
-      }
+      mbar_init(bar(ctl->s_full[b]), 1);
+      mbar_init(bar(ctl->s_free[b]), 4);
+      mbar_init(bar(ctl->p_full[b]), 4);
+      mbar_init(bar(ctl->pv_done[b]), 1);
       mbar_init(bar(ctl->item_full[b]), 1);
       mbar_init(bar(ctl->item_empty[b]), 11);       // producer + 2 MMA warps + 8 softmax warps
     }
@@ -268,7 +268,8 @@ __global__ void __launch_bounds__(kThreads, 1)
         } else {
           const uint16_t* qsrc = p.q.data + bb * p.q.sb + hh * p.q.sh;
           gather_rows(dQ, qsrc, p.q.sl, p.global_rows + item.rowA, item.nrowsA, 128, lane);
-          if (item.nrowsB) gather_rows(dQ + kTileBytes, qsrc, p.q.sl, p.global_rows + item.rowB, item.nrowsB, 128, lane);
+          if (item.nrowsB && item.kind == 1)
+            gather_rows(dQ + kTileBytes, qsrc, p.q.sl, p.global_rows + item.rowB, item.nrowsB, 128, lane);
           fence_proxy_async_smem();
           __syncwarp();
           if (lane == 0) mbar_arrive(bar(ctl->q_full[qs]));
@@ -288,7 +289,12 @@ __global__ void __launch_bounds__(kThreads, 1)
             if (tr.maskB >= 0)
               bulk_load(dM + kMaskBytes, p.masks + (size_t)tr.maskB * 256, kMaskBytes, bar(ctl->k_full[st]));
           };
-          if (tr.kind == 0) {
+          if (p.debug_flags & 4) {
+            if (lane == 0) {
+              mbar_arrive(bar(ctl->k_full[st]));
+              mbar_arrive(bar(ctl->v_full[st]));
+            }
+          } else if (tr.kind == 0) {
             if (lane == 0) {
               mbar_arrive_expect_tx(bar(ctl->k_full[st]), kTileBytes + mbytes);
               tma_load_4d(dK, &tmk, bar(ctl->k_full[st]), 0, tr.arg, hh, bb, pol_kv);
@@ -358,17 +364,15 @@ __global__ void __launch_bounds__(kThreads, 1)
       }
     } else if (warp == 1 || warp == 3) {
       // ========================================================== MMA issuers (one warp per stream)
-      // The pipeline unit is a half tile (64 keys): S_h = Q K_h^T (N = 64) into one of three TMEM
-      // buffers of the stream, P_h written by the softmax over the same buffer (16-bit pairs), then
-      // O += P_h V_h. S runs two halves ahead of P.V; a buffer is reused once its P.V completed.
-      // Streams never wait on each other; each releases a K/V stage after its own last P.V of the
-      // tile (kv_empty counts 2). The whole warp walks the schedule; lane 0 issues.
+      // Per used tile j of the stream: S_{next} = Q K_{next}^T (N = tile width) as soon as the
+      // softmax has read S_j into registers, then O += P_j V_j once P_j is stored. Streams never
+      // wait on each other; each releases a K/V stage after its own P.V of the tile (kv_empty
+      // counts 2); tiles a stream skips are released once loaded. Lane 0 issues.
       const int w = warp == 3 ? 1 : 0;
       const bool leader = lane == 0;
       Tracer trace(p, 1);
-      uint32_t it = 0, g = 0, qi = 0, hS = 0, hP = 0;   // halves with S / P.V issued (CTA lifetime)
+      uint32_t it = 0, g = 0, qi = 0, nS = 0, nP = 0;   // S / P.V issued (CTA lifetime)
       const uint32_t tbase = tmem + w * 256;
-      const uint32_t dO = tbase + kTmemOOff;
       while (true) {
         const uint32_t slot = it & 1, ph = (it >> 1) & 1;
         mbar_wait(bar(ctl->item_full[slot]), ph);
@@ -379,100 +383,85 @@ __global__ void __launch_bounds__(kThreads, 1)
         ++it;
         if (u >= p.total_units) break;
         const uint32_t qs = qi & 1;
-        const uint32_t qa = sQ + qs * 2 * kTileBytes + w * kTileBytes;
+        const uint32_t qa = sQ + qs * 2 * kTileBytes + (item.kind == 2 ? 0 : w * kTileBytes);
         mbar_wait(bar(ctl->q_full[qs]), (qi >> 1) & 1);
         ++qi;
         const int nt = item.ntiles;
-        // S cursor (tile sj, half sh of nsh) and P.V cursor (tile pj, half phh)
-        int sj = 0, sh = 0, nsh = 0;
-        int pj = 0, phh = 0;
-        bool first_pv = true, s_done = false;
-        // advance the S cursor to the next half this stream uses (waits k_full of used tiles only:
-        // skipped tiles are released by the P.V cursor, which may be far behind)
-        auto s_advance = [&]() -> bool {
-          while (true) {
-            if (sh < nsh) return true;
-            if (sj >= nt) return false;
-            if (item_uses(item, w, sj)) {
-              const uint32_t gg = g + sj, st = gg % kStages;
-              mbar_wait(bar(ctl->k_full[st]), (gg / kStages) & 1);
-              nsh = ctl->tref[st].ncols > 64 ? 2 : 1;
-              sh = 0;
-              ++sj;
-              return true;
-            }
-            ++sj;
-            nsh = 0;
-            sh = 0;
-          }
-        };
-        auto issue_s = [&]() {
-          if (s_done) return;
-          if (!s_advance()) {
-            s_done = true;
-            if (leader) mma_commit(bar(ctl->q_empty[qs]));
-            __syncwarp();
-            return;
-          }
-          const uint32_t gg = g + sj - 1, st = gg % kStages;
-          const int ncols = ctl->tref[st].ncols;
-          const int n = ncols - sh * 64 > 64 ? 64 : ncols - sh * 64;   // keys in this half
-          const uint32_t b = hS % 3;
-          if (hS >= 3) mbar_wait(bar(ctl->pv_done[w][b]), ((hS - 3) / 3) & 1);
-          tc_fence_after();
-          if (leader) {
-            const uint32_t idesc_s = idesc_f16(kBF16, 128, n, false, false);
-            const uint32_t kA = sK + st * kTileBytes + sh * 8192;
-#pragma unroll
-            for (int kk = 0; kk < 4; ++kk)
-              mma_ss(tbase + b * 64, smem_desc_sw128(qa + kk * 32, 16, 1024), smem_desc_sw128(kA + kk * 32, 16, 1024),
-                     idesc_s, kk > 0);
-            mma_commit(bar(ctl->s_full[w][b]));
-          }
-          __syncwarp();
-          ++sh;
-          ++hS;
-        };
-        // next P.V: releases the stages of tiles it passes (skipped tiles, finished tiles)
-        auto issue_pv = [&]() -> bool {
-          while (pj < nt && !item_uses(item, w, pj)) {     // tiles this stream skips
-            const uint32_t gs = g + pj;
-            mbar_wait(bar(ctl->k_full[gs % kStages]), (gs / kStages) & 1);   // stage holds this tile
+        int rel = 0;                                       // next tile whose stage is not yet released
+        auto release_skipped = [&](int upto) {             // skipped tiles in [rel, upto)
+          for (; rel < upto; ++rel) {
+            if (item_uses(item, w, rel)) break;
+            const uint32_t gs = g + rel;
+            mbar_wait(bar(ctl->k_full[gs % kStages]), (gs / kStages) & 1);
             if (leader) mbar_arrive(bar(ctl->kv_empty[gs % kStages]));
             __syncwarp();
-            ++pj;
           }
-          if (pj >= nt) return false;
-          const uint32_t gg = g + pj, st = gg % kStages;
+        };
+        auto next_used = [&](int from) {
+          while (from < nt && !item_uses(item, w, from)) ++from;
+          return from;
+        };
+        auto issue_s = [&](int j) {
+          const uint32_t gg = g + j, st = gg % kStages;
+          mbar_wait(bar(ctl->k_full[st]), (gg / kStages) & 1);
           const int ncols = ctl->tref[st].ncols;
-          const int nh = ncols > 64 ? 2 : 1;
-          const int n = ncols - phh * 64 > 64 ? 64 : ncols - phh * 64;
-          const uint32_t b = hP % 3;
-          if (phh == 0) mbar_wait(bar(ctl->v_full[st]), (gg / kStages) & 1);
-          mbar_wait(bar(ctl->p_full[w][b]), (hP / 3) & 1);
+          if (nS > 0) mbar_wait(bar(ctl->s_free[w]), (nS - 1) & 1);
+          tc_fence_after();
+          if (leader) {
+            const uint32_t idesc_s = idesc_f16(kBF16, 128, ncols, false, false);
+            const uint32_t kA = sK + st * kTileBytes;
+#pragma unroll
+            for (int kk = 0; kk < ((p.debug_flags & 2) ? 0 : 4); ++kk)
+              mma_ss(tbase, smem_desc_sw128(qa + kk * 32, 16, 1024), smem_desc_sw128(kA + kk * 32, 16, 1024),
+                     idesc_s, kk > 0);
+            mma_commit(bar(ctl->s_full[w]));
+          }
+          __syncwarp();
+          ++nS;
+        };
+        bool first_pv = true;
+        auto issue_pv = [&](int j) {
+          const uint32_t gg = g + j, st = gg % kStages;
+          const int ncols = ctl->tref[st].ncols;
+          mbar_wait(bar(ctl->v_full[st]), (gg / kStages) & 1);
+          mbar_wait(bar(ctl->p_full[w]), nP & 1);
           tc_fence_after();
           if (leader) {
             const uint32_t idesc_pv = idesc_f16(kBF16, 128, 64, false, true);
-            const uint32_t vA = sV + st * kTileBytes + phh * 8192;
-            for (int kk = 0; kk < (n >> 4); ++kk)
-              mma_ts(dO, tbase + b * 64 + kk * 8, smem_desc_sw128(vA + kk * 2048, 8192, 1024), idesc_pv,
-                     (first_pv && kk == 0) ? 0u : 1u);
-            mma_commit(bar(ctl->pv_done[w][b]));
-            if (phh == nh - 1) mma_commit(bar(ctl->kv_empty[st]));
+            const uint32_t vA = sV + st * kTileBytes;
+            for (int kk = 0; kk < ((p.debug_flags & 2) ? 0 : (ncols >> 4)); ++kk)
+              mma_ts(tbase + kTmemOOff, tbase + kTmemPOff + kk * 8, smem_desc_sw128(vA + kk * 2048, 8192, 1024),
+                     idesc_pv, (first_pv && kk == 0) ? 0u : 1u);
+            mma_commit(bar(ctl->pv_done[w]));
+            mma_commit(bar(ctl->kv_empty[st]));
           }
           __syncwarp();
           first_pv = false;
-          ++hP;
-          if (++phh == nh) {
-            phh = 0;
-            ++pj;
-          }
-          return true;
+          ++nP;
         };
-        issue_s();
-        issue_s();
-        while (issue_pv()) issue_s();
-        if (!s_done) issue_s();                            // commits q_empty when nothing is left
+        int j = next_used(0);
+        if (j < nt) {
+          release_skipped(j);
+          issue_s(j);
+        }
+        while (j < nt) {
+          const int jn = next_used(j + 1);
+          rel = j + 1;
+          release_skipped(jn);                             // tiles this stream skips before jn
+          if (jn < nt) {
+            issue_s(jn);
+          } else if (leader) {
+            mma_commit(bar(ctl->q_empty[qs]));             // last S of the item issued
+          }
+          __syncwarp();
+          issue_pv(j);
+          j = jn;
+        }
+        if (next_used(0) >= nt) {                          // the stream has no tile in this item
+          release_skipped(nt);
+          if (leader) mma_commit(bar(ctl->q_empty[qs]));
+          __syncwarp();
+        }
         if (leader) trace(1, 2, g + nt - 1);
         g += nt;
       }
@@ -485,6 +474,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     const int t = q4 * 32 + lane;                          // row of the stream's Q tile = TMEM lane
     const uint32_t lane_base = (uint32_t)(q4 * 32) << 16;
     const uint32_t tbase = tmem + lane_base + w * 256;
+    const uint32_t tP = tbase + kTmemPOff;
     const uint32_t tO = tbase + kTmemOOff;
     const float c = p.scale_log2;
     const float2 c2 = make_float2(c, c);
@@ -505,7 +495,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     // lazy rescaling (O accumulates in TMEM): the exponent uses a stale row max m until a half
     // tile's max exceeds it by more than 2^8 in probability, so p <= 256 and O rarely needs a rescale
     const float thresh = 8.f / c;
-    uint32_t it = 0, g = 0, hs = 0;                        // hs: halves processed by this stream
+    uint32_t it = 0, g = 0, n = 0;                         // n: tiles processed by this stream
     while (true) {
       const uint32_t slot = it & 1, ph = (it >> 1) & 1;
       mbar_wait(bar(ctl->item_full[slot]), ph);
@@ -523,11 +513,12 @@ __global__ void __launch_bounds__(kThreads, 1)
       if (t < nrows) {
         const int rbase = w == 0 ? item.rowA : item.rowB;
         r_out = item.kind == 0 ? rbase + t : __ldg(p.global_rows + rbase + t);
+        if (item.kind == 2 && w == 1) r_out = -1;          // stream B hands its partial to A
         if (item.kind == 0) slot_f = __ldg(p.fine_slot + rbase + t);
       }
       float m = -INFINITY, l = 0.f;
-      uint32_t h_item = 0;
-      const bool pp = item.turns > 0;                      // both streams active: ping-pong
+      uint32_t n_item = 0;
+      const bool pp = item.turns > 0 && !(p.debug_flags & 8);   // both streams active: ping-pong
       int turns_done = 0;
       for (int j = 0; j < item.ntiles && nrows > 0; ++j) {
         // a skipped tile's stage may already be recycled: decide from the item's use bitmap
@@ -543,23 +534,30 @@ __global__ void __launch_bounds__(kThreads, 1)
           w1 = ((uint64_t)(uint32_t)mw.w << 32) | (uint32_t)mw.z;
         }
         const int nh = tr.ncols > 64 ? 2 : 1;
-        for (int hh = 0; hh < nh; ++hh, ++hs, ++h_item) {
+        if (tr_on) trace(2 + w, 1, gg);
+        mbar_wait(bar(ctl->s_full[w]), n & 1);
+        if (tr_on) trace(2 + w, 2, gg);
+        tc_fence_after();
+        // S_j is read in two 64-column halves (four x16 loads in flight, one wait each); each half
+        // runs max -> lazy rescale -> exp -> P store. The S buffer is released after the second
+        // half's load so the MMA computes the next tile's S during this tile's exps.
+        for (int hh = 0; hh < nh; ++hh) {
           const int nc = (tr.ncols - hh * 64 > 64 ? 64 : tr.ncols - hh * 64) >> 4;   // 16-col chunks
-          const uint32_t b = hs % 3;
-          const uint32_t tS = tbase + b * 64;
+          const uint32_t tS = tbase + hh * 64;
           const uint64_t wd = hh ? w1 : w0;
-          if (tr_on) trace(2 + w, 1, gg);
-          mbar_wait(bar(ctl->s_full[w][b]), (hs / 3) & 1);
-          tc_fence_after();
           uint32_t r0[16], r1[16], r2[16], r3[16];
-          if (active) {
+          if (active && !(p.debug_flags & 16)) {
             tmem_ld16(tS, r0);
             if (nc > 1) tmem_ld16(tS + 16, r1);
             if (nc > 2) tmem_ld16(tS + 32, r2);
             if (nc > 3) tmem_ld16(tS + 48, r3);
             tmem_wait_ld();
           }
-          if (tr_on) trace(2 + w, 2, gg);
+          if (hh == nh - 1) {                              // S buffer free for the next tile
+            tc_fence_before();
+            __syncwarp();
+            if (lane == 0) mbar_arrive(bar(ctl->s_free[w]));
+          }
           float tmax = -INFINITY;
           if (active && !dry) {
             float mx0 = -INFINITY, mx1 = -INFINITY;
@@ -576,7 +574,7 @@ __global__ void __launch_bounds__(kThreads, 1)
             }
             tmax = fmaxf(mx0, mx1);
           }
-          // lazy rescale decision (warp-uniform for the TMEM access)
+          // lazy rescale decision (warp-uniform for the TMEM accesses)
           const bool need = tmax > m + thresh || (m == -INFINITY && tmax != -INFINITY);
           float alpha = 1.f;
           if (need) {
@@ -584,11 +582,14 @@ __global__ void __launch_bounds__(kThreads, 1)
             m = tmax;
           }
           l *= alpha;
-          if (__any_sync(0xffffffffu, need && alpha != 0.f) && h_item > 0) {
-            // O holds earlier halves of this item: wait for the last issued P.V, then rescale
-            mbar_wait(bar(ctl->pv_done[w][(hs - 1) % 3]), ((hs - 1) / 3) & 1);
+          const bool any_rescale = __any_sync(0xffffffffu, need && alpha != 0.f);
+          if (hh == 0 && n_item > 0 && !(p.debug_flags & 32)) {
+            // previous P.V done: P may be overwritten, O holds the earlier tiles
+            mbar_wait(bar(ctl->pv_done[w]), (n - 1) & 1);
             tc_fence_after();
-            if (active) {
+          }
+          if (any_rescale && active) {
+            if (n_item > 0) {
 #pragma unroll
               for (int h2 = 0; h2 < 4; ++h2) {
                 uint32_t r[16];
@@ -599,43 +600,62 @@ __global__ void __launch_bounds__(kThreads, 1)
                 tmem_st16(tO + h2 * 16, r);
               }
             }
+            if (hh == 1) {                                 // first half's P (32 packed columns)
+              tmem_wait_st();
+#pragma unroll
+              for (int h2 = 0; h2 < 2; ++h2) {
+                uint32_t r[16];
+                tmem_ld16(tP + h2 * 16, r);
+                tmem_wait_ld();
+#pragma unroll
+                for (int i = 0; i < 16; ++i) {
+                  float lo, hi;
+                  unpack2<kBF16>(r[i], lo, hi);
+                  r[i] = pack2<kBF16>(lo * alpha, hi * alpha);
+                }
+                tmem_st16(tP + h2 * 16, r);
+              }
+            }
           }
-          // p = 2^(s*c - m*c) (masked -> 0), packed to 16-bit pairs over this half's own S buffer
+          // p = 2^(s*c - m*c) (masked -> 0), packed to 16-bit pairs (A operand of P.V)
           turn_begin(pp);
           if (active && !dry) {
             const float mu = (m == -INFINITY) ? 0.f : m;
             const float2 nb2 = make_float2(-mu * c, -mu * c);
             float2 rs0 = make_float2(0.f, 0.f), rs1 = make_float2(0.f, 0.f);
+            const uint32_t pb = tP + hh * 32;
             if (partial) {
-              chunk_exp<true, kBF16>(r0, (uint32_t)wd & 0xffffu, c2, nb2, rs0, rs1, tS);
-              if (nc > 1) chunk_exp<true, kBF16>(r1, (uint32_t)(wd >> 16) & 0xffffu, c2, nb2, rs0, rs1, tS + 8);
-              if (nc > 2) chunk_exp<true, kBF16>(r2, (uint32_t)(wd >> 32) & 0xffffu, c2, nb2, rs0, rs1, tS + 16);
-              if (nc > 3) chunk_exp<true, kBF16>(r3, (uint32_t)(wd >> 48) & 0xffffu, c2, nb2, rs0, rs1, tS + 24);
+              chunk_exp<true, kBF16>(r0, (uint32_t)wd & 0xffffu, c2, nb2, rs0, rs1, pb);
+              if (nc > 1) chunk_exp<true, kBF16>(r1, (uint32_t)(wd >> 16) & 0xffffu, c2, nb2, rs0, rs1, pb + 8);
+              if (nc > 2) chunk_exp<true, kBF16>(r2, (uint32_t)(wd >> 32) & 0xffffu, c2, nb2, rs0, rs1, pb + 16);
+              if (nc > 3) chunk_exp<true, kBF16>(r3, (uint32_t)(wd >> 48) & 0xffffu, c2, nb2, rs0, rs1, pb + 24);
             } else {
-              chunk_exp<false, kBF16>(r0, 0xffffu, c2, nb2, rs0, rs1, tS);
-              if (nc > 1) chunk_exp<false, kBF16>(r1, 0xffffu, c2, nb2, rs0, rs1, tS + 8);
-              if (nc > 2) chunk_exp<false, kBF16>(r2, 0xffffu, c2, nb2, rs0, rs1, tS + 16);
-              if (nc > 3) chunk_exp<false, kBF16>(r3, 0xffffu, c2, nb2, rs0, rs1, tS + 24);
+              chunk_exp<false, kBF16>(r0, 0xffffu, c2, nb2, rs0, rs1, pb);
+              if (nc > 1) chunk_exp<false, kBF16>(r1, 0xffffu, c2, nb2, rs0, rs1, pb + 8);
+              if (nc > 2) chunk_exp<false, kBF16>(r2, 0xffffu, c2, nb2, rs0, rs1, pb + 16);
+              if (nc > 3) chunk_exp<false, kBF16>(r3, 0xffffu, c2, nb2, rs0, rs1, pb + 24);
             }
             l += (rs0.x + rs0.y) + (rs1.x + rs1.y);
           }
           turn_end(pp);
           ++turns_done;
-          if (active) tmem_wait_st();
-          tc_fence_before();
-          __syncwarp();
-          if (lane == 0) mbar_arrive(bar(ctl->p_full[w][b]));
-          if (tr_on) trace(2 + w, 3, gg);
         }
+        if (active) tmem_wait_st();
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(bar(ctl->p_full[w]));
+        if (tr_on) trace(2 + w, 3, gg);
+        ++n;
+        ++n_item;
       }
       g += item.ntiles;
       for (; pp && turns_done < item.turns; ++turns_done) {  // keep the turn sequences aligned
         turn_begin(true);
         turn_end(true);
       }
-      if (h_item == 0) continue;                           // stream unused in this item
+      if (n_item == 0) continue;                           // stream unused in this item
       // the item's last P.V: O is complete in TMEM
-      mbar_wait(bar(ctl->pv_done[w][(hs - 1) % 3]), ((hs - 1) / 3) & 1);
+      mbar_wait(bar(ctl->pv_done[w]), (n - 1) & 1);
       tc_fence_after();
       float oacc[64];
       if (active) {
@@ -650,6 +670,38 @@ __global__ void __launch_bounds__(kThreads, 1)
       }
       tc_fence_before();
       if (tr_on) trace(2 + w, 5, g - 1);
+      if (item.kind == 2) {
+        // split dense item: B's partial (m, l, O) rows -> per-CTA scratch -> A merges (LSE)
+        float* xr = p.dense_xch + ((size_t)blockIdx.x * 128 + t) * 68;
+        if (w == 1) {
+          if (active) {
+            *reinterpret_cast<float2*>(xr) = make_float2(m, l);
+#pragma unroll
+            for (int i = 0; i < 64; i += 4)
+              *reinterpret_cast<float4*>(xr + 4 + i) = make_float4(oacc[i], oacc[i + 1], oacc[i + 2], oacc[i + 3]);
+          }
+          __threadfence_block();
+          asm volatile("bar.arrive 9, 256;" ::: "memory");
+        } else {
+          named_bar_sync(9, 256);
+          if (active) {
+            const float2 mlb = *reinterpret_cast<const float2*>(xr);
+            const float mt = fmaxf(m, mlb.x);
+            const float mu2 = mt == -INFINITY ? 0.f : mt;
+            const float aa = ex2((m - mu2) * c), ab = ex2((mlb.x - mu2) * c);
+            l = l * aa + mlb.y * ab;
+#pragma unroll
+            for (int i = 0; i < 64; i += 4) {
+              const float4 ob = *reinterpret_cast<const float4*>(xr + 4 + i);
+              oacc[i] = oacc[i] * aa + ob.x * ab;
+              oacc[i + 1] = oacc[i + 1] * aa + ob.y * ab;
+              oacc[i + 2] = oacc[i + 2] * aa + ob.z * ab;
+              oacc[i + 3] = oacc[i + 3] * aa + ob.w * ab;
+            }
+            m = mt;
+          }
+        }
+      }
 
       // ---- epilogue: merge the fine partial (if any), normalise, store the row's 64 outputs
       if (r_out >= 0) {

@@ -27,6 +27,7 @@ struct CoarseParams {
   const float* part_acc;      // [BH * n_fine_rows * 64]
   const float2* part_ml;      // [BH * n_fine_rows]  (max in raw score units, sum)
   int32_t* counter;           // work counter (zeroed before launch)
+  float* dense_xch;           // [grid][128][68] per-CTA scratch: stream B's partial rows of kind-2 items
   TensorView q, k, v, o;
   int64_t L;
   int32_t H, BH;
@@ -36,7 +37,7 @@ struct CoarseParams {
   float scale_log2;           // (1/sqrt(d)) * log2(e)
   unsigned long long* trace;  // diagnostics: event trace of CTA 0 (null = off)
   int32_t trace_cap;
-  int32_t debug_flags;        // diagnostics (env MG_DEBUG_FLAGS): 1 = softmax skips its arithmetic
+  int32_t debug_flags;        // diagnostics (env MG_DEBUG_FLAGS): 1 = no softmax arithmetic, 2 = no MMA, 4 = no loads
 };
 
 // Fine CSR kernel: warp per (row, batch*head); SDDMM -> online softmax -> SpMM on CUDA cores.

@@ -163,17 +163,20 @@ std::string build_plan(HostPlan& p, int64_t L, int32_t heads, int32_t d, int32_t
     for (int a = 0; a < 128; ++a)
       for (int64_t c = 0; c < valid; ++c) p.dev_masks[(size_t)ragged_mask * 256 + a * 2 + c / 64] |= 1ull << (c % 64);
   }
+  // dense items (global rows): 128 gathered rows; the two softmax streams take alternate column
+  // tiles of the same rows (split-KV inside the CTA) and merge their partial rows at the end
   const int64_t G = (int64_t)p.global_rows.size();
-  for (int64_t k = 0; k < G; k += 256) {
-    const int32_t na = (int32_t)std::min<int64_t>(128, G - k);
-    const int32_t nbr = (int32_t)std::max<int64_t>(0, std::min<int64_t>(128, G - k - 128));
-    Item it{1, (int32_t)k, (int32_t)(k + 128), (int32_t)nb, (int32_t)p.trefs.size(), na, nbr,
-            nbr ? (int32_t)(2 * nb) : 0, ~0ull, nbr ? ~0ull : 0ull};
+  for (int64_t k = 0; k < G; k += 128) {
+    const int32_t nr = (int32_t)std::min<int64_t>(128, G - k);
+    const bool two = nb > 1;
+    Item it{two ? 2 : 1, (int32_t)k, (int32_t)k, (int32_t)nb, (int32_t)p.trefs.size(), nr, two ? nr : 0,
+            two ? (int32_t)(2 * ((nb + 1) / 2)) : 0, 0ull, 0ull};
     for (int64_t J = 0; J < nb; ++J) {
       const int32_t m = (J == nb - 1) ? ragged_mask : kMaskFull;
-      p.trefs.push_back(TileRef{(int32_t)(J * B), 0, 128, m, nbr ? m : kMaskSkip, 0, 0, 0});
-      count(m, 128, na);
-      count(nbr ? m : kMaskSkip, 128, nbr);
+      const bool a_uses = !two || (J % 2 == 0);
+      p.trefs.push_back(TileRef{(int32_t)(J * B), 0, 128, a_uses ? m : kMaskSkip, a_uses ? kMaskSkip : m, 0, 0, 0});
+      count(m, 128, nr);
+      if (J < 64) (a_uses ? it.useA : it.useB) |= 1ull << J;
     }
     p.items.push_back(it);
   }

@@ -20,9 +20,11 @@ struct PlanOptions {
 // streams (A and B) on two 128-row Q tiles that share the K/V tiles of one work item.
 //   Item {kind, rowA, rowB, ntiles, tref_begin, nrowsA, nrowsB}:
 //     kind 0: band row blocks starting at rows rowA and rowB (adjacent blocks with coarse tiles);
-//     kind 1: gathered global rows global_rows[rowA ..) and global_rows[rowB ..) (dense part);
+//     kind 1: gathered global rows global_rows[rowA ..) against every column tile (dense part);
+//     kind 2: like kind 1, but both streams work on the same rows (rowA == rowB) and take
+//             alternate column tiles (A even, B odd); their partial rows are merged at the end;
 //     nrowsX = valid rows of stream X (0 = stream unused); useX = bit j set if stream X uses tile j
-//     (items with more than 64 tiles are dense items whose active streams use every tile).
+//     (items with more than 64 tiles are dense items: kind 1 uses every tile, kind 2 alternates).
 //   TileRef {arg, kind, ncols, maskA, maskB}: one K/V tile of the item, loaded once:
 //     kind 0 = contiguous column tile at column `arg`; kind 1 = gathered strip whose column list
 //     starts at strip_cols[arg]; maskX = index of a 128 x 2-word bitmask for stream X,
