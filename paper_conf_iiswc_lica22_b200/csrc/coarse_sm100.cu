@@ -481,17 +481,6 @@ __global__ void __launch_bounds__(kThreads, 1)
     Tracer trace(p, 2 + w);
     const bool tr_on = (warp == 4 || warp == 8) && lane == 0;
     const bool dry = (p.debug_flags & 1) != 0;
-    // Exp ping-pong between the two softmax warps sharing an SMSP (stream A warp q, stream B
-    // warp q): they alternate their exp half-tiles (A first) through two named barriers, so each
-    // overlaps its loads/max/waits with the other's MUFU work.
-    const uint32_t bar_a_go = 1 + q4, bar_b_go = 5 + q4;
-    auto turn_begin = [&](bool on) {
-      if (on) named_bar_sync(w == 0 ? bar_a_go : bar_b_go, 64);
-    };
-    auto turn_end = [&](bool on) {
-      if (on) asm volatile("bar.arrive %0, %1;" ::"r"(w == 0 ? bar_b_go : bar_a_go), "r"(64) : "memory");
-    };
-    if (w == 1) turn_end(true);                            // A takes the first turn
     // lazy rescaling (O accumulates in TMEM): the exponent uses a stale row max m until a half
     // tile's max exceeds it by more than 2^8 in probability, so p <= 256 and O rarely needs a rescale
     const float thresh = 8.f / c;
@@ -518,8 +507,6 @@ __global__ void __launch_bounds__(kThreads, 1)
       }
       float m = -INFINITY, l = 0.f;
       uint32_t n_item = 0;
-      const bool pp = item.turns > 0 && !(p.debug_flags & 8);   // both streams active: ping-pong
-      int turns_done = 0;
       for (int j = 0; j < item.ntiles && nrows > 0; ++j) {
         // a skipped tile's stage may already be recycled: decide from the item's use bitmap
         if (!item_uses(item, w, j)) continue;
@@ -618,7 +605,6 @@ __global__ void __launch_bounds__(kThreads, 1)
             }
           }
           // p = 2^(s*c - m*c) (masked -> 0), packed to 16-bit pairs (A operand of P.V)
-          turn_begin(pp);
           if (active && !dry) {
             const float mu = (m == -INFINITY) ? 0.f : m;
             const float2 nb2 = make_float2(-mu * c, -mu * c);
@@ -637,8 +623,6 @@ __global__ void __launch_bounds__(kThreads, 1)
             }
             l += (rs0.x + rs0.y) + (rs1.x + rs1.y);
           }
-          turn_end(pp);
-          ++turns_done;
         }
         if (active) tmem_wait_st();
         tc_fence_before();
@@ -649,10 +633,6 @@ __global__ void __launch_bounds__(kThreads, 1)
         ++n_item;
       }
       g += item.ntiles;
-      for (; pp && turns_done < item.turns; ++turns_done) {  // keep the turn sequences aligned
-        turn_begin(true);
-        turn_end(true);
-      }
       if (n_item == 0) continue;                           // stream unused in this item
       // the item's last P.V: O is complete in TMEM
       mbar_wait(bar(ctl->pv_done[w]), (n - 1) & 1);
@@ -748,7 +728,6 @@ __global__ void __launch_bounds__(kThreads, 1)
     }
   }
 
-  if (warp >= 4 && warp < 8) named_bar_sync(1 + (warp & 3), 64);  // match stream B's last turn hand-off
   tc_fence_before();
   __syncthreads();
   if (warp == 2) tmem_dealloc(tmem, 512);
