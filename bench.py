@@ -239,7 +239,8 @@ def main():
     BH = cfg.B * cfg.H
     useful = 4.0 * info["nnz_total"] * cfg.d * BH
 
-    q, k, v = make_qkv(cfg.B, cfg.H, cfg.L, cfg.d, seed=cfg.seed + 1000 * rank)
+    from paper_conf_iiswc_lica22_b200.dist import rank_seed
+    q, k, v = make_qkv(cfg.B, cfg.H, cfg.L, cfg.d, seed=rank_seed(cfg.seed, rank))
     host = [torch.from_numpy(x.view(np.int16)).view(torch.bfloat16) for x in (q, k, v)]
     Q, K, V = (h.to(dev) for h in host)
     O = torch.empty_like(Q)
@@ -307,14 +308,14 @@ def main():
     # ---------------- N>1: NCCL all_gather of O, timed separately (not part of the fwd)
     gather_ms = None
     if world > 1:
-        out = torch.empty((world,) + tuple(O.shape), dtype=O.dtype, device=dev)
-        dist.all_gather_into_tensor(out, O)
+        from paper_conf_iiswc_lica22_b200.dist import gather_outputs
+        gather_outputs(O)
         torch.cuda.synchronize()
         dist.barrier()
         g0, g1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         g0.record(stream)
         for _ in range(5):
-            dist.all_gather_into_tensor(out, O)
+            gather_outputs(O)
         g1.record(stream)
         torch.cuda.synchronize()
         gt = torch.tensor([g0.elapsed_time(g1) / 5], dtype=torch.float64, device=dev)
