@@ -204,10 +204,12 @@ MG_API mg_status mg_plan_get_profile(mg_plan_t plan, mg_profile* out);
  * ---------------------------------------------------------------------------------- */
 MG_API mg_status mg_selftest_umma(int32_t mode, const void* A, const void* B, float* D, void* stream);
 
-/* mg_plan_set_trace(plan, buf, cap): diagnostics. While set, CTA 0 of the tensor-core kernel
- * appends (clock64, role<<56 | event<<48 | arg) pairs of uint64 to the device buffer `buf`
- * (capacity `cap` pairs; pair 0 holds the running count, the caller zeroes it). (null, 0)
- * turns tracing off. Used to read the warp-role pipeline timeline. */
+/* mg_plan_set_trace(plan, buf, cap): diagnostics. While set, a library built with MG_TRACE adds
+ * per-role, per-phase cycle counters of the tensor-core kernel (uint64, summed over CTAs) to the
+ * zeroed device buffer `buf` of `cap` >= 128 uint64 elements: element role*16 + k is phase k of
+ * role (0 producer, 1 MMA issuer, 2/3 softmax column halves), element role*16 + 15 the number of
+ * CTAs that reported. Normal builds ignore the buffer. (null, 0) turns it off. Errors:
+ * INVALID_ARG for a null plan or a buffer with cap < 128. */
 MG_API mg_status mg_plan_set_trace(mg_plan_t plan, void* device_buffer, int64_t capacity_events);
 
 MG_API int32_t mg_abi_version(void);

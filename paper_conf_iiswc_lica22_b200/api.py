@@ -79,11 +79,12 @@ class Plan:
         return {"calls": pr.calls, "fine_ms": pr.fine_ms, "coarse_ms": pr.coarse_ms, "total_ms": pr.total_ms}
 
     def set_trace(self, buf=None) -> None:
-        """mg_plan_set_trace: device int64 tensor [cap, 2] (row 0 = count, zeroed) or None to stop."""
+        """mg_plan_set_trace: zeroed device int64 tensor of >= 128 elements (MG_TRACE builds add their
+        per-role phase counters to it, see tools/trace_coarse.py) or None to stop."""
         if buf is None:
             check(self._lib.mg_plan_set_trace(self._handle, None, 0))
         else:
-            check(self._lib.mg_plan_set_trace(self._handle, C.c_void_p(buf.data_ptr()), buf.shape[0]))
+            check(self._lib.mg_plan_set_trace(self._handle, C.c_void_p(buf.data_ptr()), buf.numel()))
 
     def close(self):
         if getattr(self, "_handle", None) is not None and self._handle.value:

@@ -59,7 +59,6 @@ struct mg_plan_s {
   int32_t* d_fine_row_ptr = nullptr;
   int32_t* d_fine_col = nullptr;
   int32_t* d_counter = nullptr;
-  float* d_dense_xch = nullptr;   // per-CTA scratch of the tensor-core kernel (kind-2 merge)
   // stream-ordered workspaces
   float* d_part = nullptr;
   size_t part_cap = 0;      // in (row, bh) partial slots
@@ -123,8 +122,7 @@ mg_status upload(mg_plan_s* p) {
       (e = upload_vec(p, &p->d_fine_rows, h.fine_rows)) != cudaSuccess ||
       (e = upload_vec(p, &p->d_fine_row_ptr, h.fine_row_ptr)) != cudaSuccess ||
       (e = upload_vec(p, &p->d_fine_col, h.fine_col)) != cudaSuccess ||
-      (e = upload_vec(p, &p->d_counter, std::vector<int32_t>(4, 0))) != cudaSuccess ||
-      (e = upload_vec(p, &p->d_dense_xch, std::vector<float>((size_t)p->num_sms * 128 * 68, 0.f))) != cudaSuccess)
+      (e = upload_vec(p, &p->d_counter, std::vector<int32_t>(4, 0))) != cudaSuccess)
     return e == cudaErrorMemoryAllocation ? fail(MG_ERR_OUT_OF_MEMORY, "device allocation failed")
                                           : cuda_fail(e, "plan upload");
   p->uploaded = true;
@@ -304,7 +302,6 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
     cp.part_acc = part_acc;
     cp.part_ml = part_ml;
     cp.counter = p->d_counter;
-    cp.dense_xch = p->d_dense_xch;
     cp.q = view(Q); cp.k = view(K); cp.v = view(V); cp.o = view(O);
     cp.L = h.L;
     cp.H = h.heads;
@@ -487,8 +484,8 @@ mg_status mg_plan_get_profile(mg_plan_t plan, mg_profile* out) {
 
 mg_status mg_plan_set_trace(mg_plan_t plan, void* device_buffer, int64_t capacity_events) {
   g_err.clear();
-  if (!plan || (device_buffer == nullptr) != (capacity_events == 0) || capacity_events < 0 ||
-      capacity_events > (int64_t(1) << 30))
+  if (!plan || (device_buffer == nullptr) != (capacity_events == 0) ||
+      (device_buffer != nullptr && capacity_events < 128) || capacity_events > (int64_t(1) << 30))
     return fail(MG_ERR_INVALID_ARG, "bad trace buffer");
   plan->trace = static_cast<unsigned long long*>(device_buffer);
   plan->trace_cap = (int32_t)capacity_events;

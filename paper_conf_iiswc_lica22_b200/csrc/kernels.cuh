@@ -27,7 +27,6 @@ struct CoarseParams {
   const float* part_acc;      // [BH * n_fine_rows * 64]
   const float2* part_ml;      // [BH * n_fine_rows]  (max in raw score units, sum)
   int32_t* counter;           // work counter (zeroed before launch)
-  float* dense_xch;           // [grid][128][68] per-CTA scratch: stream B's partial rows of kind-2 items
   TensorView q, k, v, o;
   int64_t L;
   int32_t H, BH;

@@ -163,20 +163,15 @@ std::string build_plan(HostPlan& p, int64_t L, int32_t heads, int32_t d, int32_t
     for (int a = 0; a < 128; ++a)
       for (int64_t c = 0; c < valid; ++c) p.dev_masks[(size_t)ragged_mask * 256 + a * 2 + c / 64] |= 1ull << (c % 64);
   }
-  // dense items (global rows): 128 gathered rows; the two softmax streams take alternate column
-  // tiles of the same rows (split-KV inside the CTA) and merge their partial rows at the end
+  // dense items (global rows): up to 128 gathered rows against every column tile
   const int64_t G = (int64_t)p.global_rows.size();
   for (int64_t k = 0; k < G; k += 128) {
     const int32_t nr = (int32_t)std::min<int64_t>(128, G - k);
-    const bool two = nb > 1;
-    Item it{two ? 2 : 1, (int32_t)k, (int32_t)k, (int32_t)nb, (int32_t)p.trefs.size(), nr, two ? nr : 0,
-            two ? (int32_t)(2 * ((nb + 1) / 2)) : 0, 0ull, 0ull};
+    Item it{1, (int32_t)k, 0, (int32_t)nb, (int32_t)p.trefs.size(), nr, 0, 0, 0ull, 0ull};
     for (int64_t J = 0; J < nb; ++J) {
       const int32_t m = (J == nb - 1) ? ragged_mask : kMaskFull;
-      const bool a_uses = !two || (J % 2 == 0);
-      p.trefs.push_back(TileRef{(int32_t)(J * B), 0, 128, a_uses ? m : kMaskSkip, a_uses ? kMaskSkip : m, 0, 0, 0});
+      p.trefs.push_back(TileRef{(int32_t)(J * B), 0, 128, m, kMaskSkip, 0, 0, 0});
       count(m, 128, nr);
-      if (J < 64) (a_uses ? it.useA : it.useB) |= 1ull << J;
     }
     p.items.push_back(it);
   }
@@ -218,87 +213,33 @@ std::string build_plan(HostPlan& p, int64_t L, int32_t heads, int32_t d, int32_t
     }
     return m;
   };
-  auto push_strip = [&](int64_t IA, int64_t IB, const std::vector<int32_t>& cols) {
+  auto push_strip = [&](int64_t I, const std::vector<int32_t>& cols) {
     const int ncols = (int)((cols.size() + 31) / 32 * 32);
     const int32_t off = (int32_t)p.strip_cols.size();
     for (int i = 0; i < ncols; ++i) p.strip_cols.push_back(i < (int)cols.size() ? cols[i] : -1);
-    const int32_t ma = strip_mask(IA, cols, ncols);
-    const int32_t mb = strip_mask(IB, cols, ncols);
-    p.trefs.push_back(TileRef{off, 1, ncols, ma, mb, 0, 0, 0});
-    count(ma, ncols, 1);
-    count(mb, ncols, 1);
+    const int32_t m = strip_mask(I, cols, ncols);
+    p.trefs.push_back(TileRef{off, 1, ncols, m, kMaskSkip, 0, 0, 0});
+    count(m, ncols, 1);
     p.n_strip_tiles++;
   };
 
-  // band items: consecutive row blocks that have coarse tiles, paired (A, B)
-  std::vector<int64_t> tiled;
-  for (int64_t I = 0; I < nb; ++I)
-    if (p.bsr_row_ptr[I + 1] > p.bsr_row_ptr[I]) tiled.push_back(I);
-  for (size_t k = 0; k < tiled.size();) {
-    const int64_t IA = tiled[k];
-    int64_t IB = k + 1 < tiled.size() ? tiled[k + 1] : -1;
-    if (IB >= 0) {  // pair only while the union stays within a 64-tile use bitmap (+ strips)
-      int64_t lo = std::min(p.bsr_col[p.bsr_row_ptr[IA]], p.bsr_col[p.bsr_row_ptr[IB]]);
-      int64_t hi = std::max(p.bsr_col[p.bsr_row_ptr[IA + 1] - 1], p.bsr_col[p.bsr_row_ptr[IB + 1] - 1]);
-      if (hi - lo + 1 > 62) IB = -1;
+  // band items: one per row block with coarse tiles (its BSR tiles, then its strip if any)
+  for (int64_t I = 0; I < nb; ++I) {
+    if (p.bsr_row_ptr[I + 1] == p.bsr_row_ptr[I]) continue;
+    const int32_t nr = (int32_t)std::min<int64_t>(B, L - I * B);
+    Item it{0, (int32_t)(I * B), 0, 0, (int32_t)p.trefs.size(), nr, 0, 0, 0ull, 0ull};
+    for (int32_t t = p.bsr_row_ptr[I]; t < p.bsr_row_ptr[I + 1]; ++t) {
+      const int32_t m = tile_full[t] ? kMaskFull : t;
+      p.trefs.push_back(TileRef{p.bsr_col[t] * (int32_t)B, 0, 128, m, kMaskSkip, 0, 0, 0});
+      count(m, 128, nr);
     }
-    k += IB >= 0 ? 2 : 1;
-    auto nrows_of = [&](int64_t I) -> int32_t { return I < 0 ? 0 : (int32_t)std::min<int64_t>(B, L - I * B); };
-    Item it{0, (int32_t)(IA * B), (int32_t)(IB < 0 ? 0 : IB * B), 0, (int32_t)p.trefs.size(), nrows_of(IA),
-            nrows_of(IB), 0, 0ull, 0ull};
-    // union of the two blocks' column tiles, ascending
-    std::vector<std::pair<int32_t, std::pair<int32_t, int32_t>>> u;  // J -> (maskA, maskB)
-    auto add_block = [&](int64_t I, bool isA) {
-      if (I < 0) return;
-      for (int32_t t = p.bsr_row_ptr[I]; t < p.bsr_row_ptr[I + 1]; ++t) {
-        const int32_t J = p.bsr_col[t];
-        const int32_t m = tile_full[t] ? kMaskFull : t;
-        auto itr = std::find_if(u.begin(), u.end(), [&](const auto& e) { return e.first == J; });
-        if (itr == u.end()) {
-          u.push_back({J, {kMaskSkip, kMaskSkip}});
-          itr = u.end() - 1;
-        }
-        (isA ? itr->second.first : itr->second.second) = m;
-      }
-    };
-    add_block(IA, true);
-    add_block(IB, false);
-    std::sort(u.begin(), u.end());
-    for (const auto& e : u) {
-      p.trefs.push_back(TileRef{e.first * (int32_t)B, 0, 128, e.second.first, e.second.second, 0, 0, 0});
-      count(e.second.first, 128, it.nrowsA);
-      count(e.second.second, 128, it.nrowsB);
+    // CSR residual as a tensor-core strip where the block's distinct columns are few
+    const std::vector<int32_t>& cols = blk_cols[I];
+    if (strip_max > 0 && !cols.empty() && (int)cols.size() <= strip_max) {
+      push_strip(I, cols);
+      blk_strip[I] = 1;
     }
-    // CSR residual as tensor-core strips where the blocks' distinct columns are few
-    const std::vector<int32_t>& ca = blk_cols[IA];
-    const std::vector<int32_t> empty;
-    const std::vector<int32_t>& cb = IB < 0 ? empty : blk_cols[IB];
-    const bool sa = strip_max > 0 && !ca.empty() && (int)ca.size() <= strip_max;
-    const bool sb = strip_max > 0 && !cb.empty() && (int)cb.size() <= strip_max;
-    if (sa && sb) {
-      std::vector<int32_t> un;
-      std::set_union(ca.begin(), ca.end(), cb.begin(), cb.end(), std::back_inserter(un));
-      if ((int)un.size() <= strip_max) {
-        push_strip(IA, IB, un);
-      } else {
-        push_strip(IA, -1, ca);
-        push_strip(-1, IB, cb);
-      }
-    } else if (sa) {
-      push_strip(IA, -1, ca);
-    } else if (sb) {
-      push_strip(-1, IB, cb);
-    }
-    if (sa) blk_strip[IA] = 1;
-    if (sb) blk_strip[IB] = 1;
     it.ntiles = (int32_t)p.trefs.size() - it.tref_begin;
-    int32_t ha = 0, hb = 0;
-    for (int32_t j = 0; j < it.ntiles && j < 64; ++j) {
-      const TileRef& r = p.trefs[it.tref_begin + j];
-      if (r.maskA != kMaskSkip && it.nrowsA) { it.useA |= 1ull << j; ha += (r.ncols + 63) / 64; }
-      if (r.maskB != kMaskSkip && it.nrowsB) { it.useB |= 1ull << j; hb += (r.ncols + 63) / 64; }
-    }
-    it.turns = (it.nrowsA && it.nrowsB) ? std::max(ha, hb) : 0;
     p.items.push_back(it);
   }
 

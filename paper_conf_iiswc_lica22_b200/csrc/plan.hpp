@@ -16,22 +16,19 @@ struct PlanOptions {
   int strip_max_cols = 128;  // <= 0 disables the tensor-core strip path for the CSR residual
 };
 
-// Device work-list encodings. The tensor-core kernel runs two softmax
-// streams (A and B) on two 128-row Q tiles that share the K/V tiles of one work item.
-//   Item {kind, rowA, rowB, ntiles, tref_begin, nrowsA, nrowsB}:
-//     kind 0: band row blocks starting at rows rowA and rowB (adjacent blocks with coarse tiles);
+// Device work-list encodings. The tensor-core kernel processes one 128-row
+// Q tile per work item against the item's list of K/V tiles.
+//   Item {kind, rowA, -, ntiles, tref_begin, nrowsA, ...}:
+//     kind 0: band row block starting at row rowA (a block with coarse tiles);
 //     kind 1: gathered global rows global_rows[rowA ..) against every column tile (dense part);
-//     kind 2: like kind 1, but both streams work on the same rows (rowA == rowB) and take
-//             alternate column tiles (A even, B odd); their partial rows are merged at the end;
-//     nrowsX = valid rows of stream X (0 = stream unused); useX = bit j set if stream X uses tile j
-//     (items with more than 64 tiles are dense items: kind 1 uses every tile, kind 2 alternates).
-//   TileRef {arg, kind, ncols, maskA, maskB}: one K/V tile of the item, loaded once:
+//     nrowsA = valid rows of the Q tile. rowB, nrowsB, turns, useA, useB are reserved (0).
+//   TileRef {arg, kind, ncols, maskA, -}: one K/V tile of the item:
 //     kind 0 = contiguous column tile at column `arg`; kind 1 = gathered strip whose column list
-//     starts at strip_cols[arg]; maskX = index of a 128 x 2-word bitmask for stream X,
-//     -1 = all valid, -2 = stream X does not use this tile.
+//     starts at strip_cols[arg] (ncols a multiple of 32); maskA = index of a 128 x 2-word bitmask,
+//     -1 = all valid. maskB is reserved (-2).
 struct Item {
   int32_t kind, rowA, rowB, ntiles, tref_begin, nrowsA, nrowsB;
-  int32_t turns;  // exp half-tiles per softmax stream (max over A, B) when both are active, else 0
+  int32_t turns;
   uint64_t useA, useB;
 };
 struct TileRef { int32_t arg, kind, ncols, maskA, maskB, pad0, pad1, pad2; };
