@@ -9,22 +9,23 @@
 //     block's CSR residual on the tensor cores); the epilogue merges the fp32 partial statistics
 //     written by the CUDA-core fine kernel for any remaining CSR rows (compound SpSoftmax);
 //   kind 1 items: gathered global rows against every column tile (dense-row part).
-// Column-split softmax: the key columns of every tile are split into two halves (h = 0, 1); the
-// 8 softmax warps form two groups, one per half, each running an independent online softmax over
-// its half of every tile with its own O accumulator in TMEM (O_h = sum_j P_j,h V_j,h). The two
-// partial rows (m_h, l_h, O_h) are merged once per item in the epilogue. Everything the softmax
-// warps touch is double-buffered (S, P), so in steady state they never wait on an MMA: MUFU ex2
+// Column-group softmax: the 16-column chunks of every tile are dealt round-robin to four column
+// groups (group cg owns chunks cg and cg + 4). 16 softmax warps = 4 groups x 4 TMEM lane quarters;
+// each warp runs an independent online softmax over its group's columns for its 32 rows, with its
+// own O accumulator in TMEM (O_cg = sum_j P_j,cg V_j,cg). The four partial rows (m, l, O_cg) are
+// merged once per item in the epilogue. Four warps per SMSP hide each other's latencies; MUFU ex2
 // throughput is the bound.
-// Warp roles (one 384-thread CTA per SM, persistent, dynamic work counter):
+// P aliasing: a warp writes its packed P (16-bit pairs) over the S columns it has just read, and
+// P.V(n) reads it from there. tcgen05.mma ops issued by one thread execute in order, so S(n+2),
+// issued after P.V(n), cannot overwrite the buffer before P.V(n) has read it: no "S free" barrier.
+// Warp roles (one 640-thread CTA per SM, persistent, dynamic work counter):
 //   warp 0      producer: TMA of Q/K/V tiles (SWIZZLE_128B), bulk copies of tile bitmasks,
 //               row gathers (global rows, strip columns)
-//   warp 1      MMA issuer (lane 0): S one tile ahead, P.V of both halves behind
+//   warp 1      MMA issuer (lane 0): S(n), then P.V(n-1) of all groups
 //   warp 2      TMEM allocator, then scheduler: publishes work items, L2-prefetches their tiles
 //   warp 3      idle after setup
-//   warps 4..7  softmax, column half 0 (TMEM lane quarter = warp % 4)
-//   warps 8..11 softmax, column half 1
-// TMEM (512 columns): S[b] at b*128 (b = tile parity), P[b][h] at 256 + b*64 + h*32 (16-bit
-// pairs), O_h at 384 + h*64.
+//   warps 4..19 softmax: column group cg = (warp - 4) / 4, TMEM lane quarter = warp % 4
+// TMEM (512 columns): S/P[b] at b*128 (b = tile parity), O_cg at 256 + cg*64.
 #include <cuda_bf16.h>
 #include <cuda_fp16.h>
 
@@ -38,10 +39,10 @@ using namespace ptx;
 namespace {
 
 constexpr int kStages = 5;
-constexpr int kThreads = 384;
+constexpr int kThreads = 640;
 constexpr uint32_t kTileBytes = 128 * 128;  // 128 rows x 64 x 16-bit
 constexpr uint32_t kMaskBytes = 128 * 16;   // 128 rows x 2 x u64
-constexpr uint32_t kTmemP = 256, kTmemO = 384;
+constexpr uint32_t kTmemO = 256;
 
 struct __align__(16) ItemSlot {
   Item item;
@@ -51,11 +52,10 @@ struct __align__(16) ItemSlot {
 struct __align__(16) SmemCtl {
   TileRef tref[kStages];
   ItemSlot slot[2];
-  float2 xch[2][2][128];                     // [item parity][half][row] (m, l) for the merge
+  float2 xch[2][4][128];                     // [item parity][group][row] (m, l) for the merge
   uint64_t q_full[2], q_empty[2];
   uint64_t kv_full[kStages], kv_empty[kStages];
-  uint64_t s_full[2], s_free[2];             // per S buffer
-  uint64_t p_full[2], pv_done[2][2];         // [P buffer], [half][P buffer]
+  uint64_t s_full[2], p_full[2], pv_done[2];  // per S/P buffer
   uint64_t o_free;
   uint64_t item_full[2], item_empty[2];
   uint32_t tmem_base;
@@ -63,10 +63,10 @@ struct __align__(16) SmemCtl {
 
 constexpr size_t kSmemBytes = 1024 + kTileBytes * (2 + 2 * kStages) + kMaskBytes * kStages + sizeof(SmemCtl);
 static_assert(kSmemBytes <= 227 * 1024, "shared memory budget");
-// setmaxnreg.inc draws from the CTA's pool (168 x 384 = 64512 registers at launch):
-// 128 x kRegsCtl + 256 x kRegsSoftmax must not exceed it, or the inc blocks forever.
-constexpr int kRegsCtl = 48, kRegsSoftmax = 224;
-static_assert(128 * kRegsCtl + 256 * kRegsSoftmax <= 168 * 384, "register pool");
+// setmaxnreg.inc draws from the CTA's pool (96 x 640 = 61440 registers at launch):
+// 128 x kRegsCtl + 512 x kRegsSoftmax must not exceed it, or the inc blocks forever.
+constexpr int kRegsCtl = 56, kRegsSoftmax = 104;
+static_assert(128 * kRegsCtl + 512 * kRegsSoftmax <= 96 * 640, "register pool");
 
 struct UnitInfo {
   int item, bh;
@@ -214,13 +214,12 @@ __global__ void __launch_bounds__(kThreads, 1)
       mbar_init(bar(ctl->q_full[b]), 1);
       mbar_init(bar(ctl->q_empty[b]), 1);
       mbar_init(bar(ctl->s_full[b]), 1);
-      mbar_init(bar(ctl->s_free[b]), 8);            // all 8 softmax warps read their half of S
-      mbar_init(bar(ctl->p_full[b]), 8);            // both halves' P stored
-      for (int h = 0; h < 2; ++h) mbar_init(bar(ctl->pv_done[h][b]), 1);
+      mbar_init(bar(ctl->p_full[b]), 16);           // all 16 softmax warps stored their P
+      mbar_init(bar(ctl->pv_done[b]), 1);
       mbar_init(bar(ctl->item_full[b]), 1);
-      mbar_init(bar(ctl->item_empty[b]), 10);       // producer + MMA + 8 softmax warps
+      mbar_init(bar(ctl->item_empty[b]), 18);       // producer + MMA + 16 softmax warps
     }
-    mbar_init(bar(ctl->o_free), 8);
+    mbar_init(bar(ctl->o_free), 16);
     for (int s = 0; s < kStages; ++s) {
       mbar_init(bar(ctl->kv_full[s]), 1);
       mbar_init(bar(ctl->kv_empty[s]), 1);
@@ -353,50 +352,55 @@ __global__ void __launch_bounds__(kThreads, 1)
   } else if (warp == 1) {
     // ============================================================ MMA issuer (lane 0)
     asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(kRegsCtl) : "memory");
-    // Tile sequence over the CTA's lifetime: n = 0, 1, 2, ...; S(n) -> S[n&1], P(n, h) ->
-    // P[n&1][h]. Order: S(n+1) is issued before P.V(n), so the next tile's scores are ready
-    // when the softmax finishes tile n. S(n) needs S[n&1] released by tile n-2's readers;
-    // P.V(n, h) needs P(n, h) stored; the first P.V of an item (accumulate = 0) needs the
-    // previous item's epilogue to have read O.
+    // Tile sequence over the CTA's lifetime: n = 0, 1, 2, ...; S(n) -> S/P[n&1]. Iteration n
+    // issues S(n), then P.V(n-1) once every softmax warp stored P(n-1). S(n) reuses the buffer of
+    // tile n-2, whose P.V was issued earlier by this thread (in-order execution). The first P.V of
+    // an item's column group (accumulate = 0) also waits until the previous item's epilogue has
+    // read O (o_free).
     const bool leader = lane == 0;
     Prof prof(leader && blockIdx.x < 148);
     uint32_t it = 0, g = 0, n = 0, items_done = 0;
     // pending P.V: the tile issued last (stage, width, tile index, first-of-item)
     bool pend = false, pend_first = false;
-    uint32_t pend_st = 0, pend_g = 0, pend_n = 0;
+    uint32_t pend_st = 0, pend_n = 0;
     int pend_ncols = 0;
+    uint32_t started = 0;                              // column groups with an accumulator this item
     auto issue_pv = [&]() {
       if (!pend) return;
       const uint32_t b = pend_n & 1, st = pend_st;
-      if (pend_first && items_done > 0) mbar_wait(bar(ctl->o_free), (items_done - 1) & 1);
+      if (pend_first) {
+        if (items_done > 0) mbar_wait(bar(ctl->o_free), (items_done - 1) & 1);
+        ++items_done;
+        started = 0;
+      }
       prof.mark(5);
-      const int hc = pend_ncols >> 1;
-      const uint32_t vA = sV + st * kTileBytes;
-      const uint32_t idesc_pv = idesc_f16(kBF16, 128, 64, false, true);
       mbar_wait(bar(ctl->p_full[b]), (pend_n >> 1) & 1);
       prof.mark(6);
       tc_fence_after();
-      for (int h = 0; h < 2; ++h) {
-        if (leader) {
-          const uint32_t tPh = tmem + kTmemP + b * 64 + h * 32;
-          const uint32_t vh = vA + (uint32_t)(h * hc / 16) * 2048;
-          for (int kk = 0; kk < ((p.debug_flags & 2) ? 0 : (hc >> 4)); ++kk)
-            mma_ts(tmem + kTmemO + h * 64, tPh + kk * 8, smem_desc_sw128(vh + kk * 2048, 8192, 1024), idesc_pv,
-                   (pend_first && kk == 0) ? 0u : 1u);
-          mma_commit(bar(ctl->pv_done[h][b]));
-          if (h == 1) mma_commit(bar(ctl->kv_empty[st]));
+      if (leader && !(p.debug_flags & 2)) {
+        const uint32_t vA = sV + st * kTileBytes;
+        const uint32_t idesc_pv = idesc_f16(kBF16, 128, 64, false, true);
+        // chunk c (16 keys): P at S/P[b] columns [16c, 16c + 8) (packed), V rows [16c, 16c + 16)
+        for (int c = 0; c < (pend_ncols >> 4); ++c) {
+          const int cg = c & 3;
+          mma_ts(tmem + kTmemO + cg * 64, tmem + b * 128 + c * 16, smem_desc_sw128(vA + c * 2048, 8192, 1024),
+                 idesc_pv, (started >> cg) & 1u);
+          started |= 1u << cg;
         }
-        __syncwarp();
-        prof.mark(7 + 2 * h);
       }
-      if (pend_first) ++items_done;
+      if (leader) {
+        mma_commit(bar(ctl->pv_done[b]));
+        mma_commit(bar(ctl->kv_empty[st]));
+      }
+      __syncwarp();
+      prof.mark(7);
       pend = false;
     };
     while (true) {
       const uint32_t slot = it & 1, ph = (it >> 1) & 1;
       mbar_wait(bar(ctl->item_full[slot]), ph);
       const int u = ctl->slot[slot].u;
-      const Item item = ctl->slot[slot].item;
+      const int ntiles = ctl->slot[slot].item.ntiles;
       __syncwarp();
       if (leader) mbar_arrive(bar(ctl->item_empty[slot]));
       if (u >= p.total_units) break;
@@ -406,13 +410,11 @@ __global__ void __launch_bounds__(kThreads, 1)
       mbar_wait(bar(ctl->q_full[qs]), ph);
       prof.mark(1);
       ++it;
-      for (int j = 0; j < item.ntiles; ++j, ++g, ++n) {
+      for (int j = 0; j < ntiles; ++j, ++g, ++n) {
         const uint32_t st = g % kStages, b = n & 1;
         mbar_wait(bar(ctl->kv_full[st]), (g / kStages) & 1);
         prof.mark(2);
         const int ncols = ctl->tref[st].ncols;
-        if (n >= 2) mbar_wait(bar(ctl->s_free[b]), ((n - 2) >> 1) & 1);
-        prof.mark(3);
         tc_fence_after();
         if (leader) {
           const uint32_t idesc_s = idesc_f16(kBF16, 128, ncols, false, false);
@@ -422,7 +424,7 @@ __global__ void __launch_bounds__(kThreads, 1)
             mma_ss(tmem + b * 128, smem_desc_sw128(qa + kk * 32, 16, 1024), smem_desc_sw128(kA + kk * 32, 16, 1024),
                    idesc_s, kk > 0);
           mma_commit(bar(ctl->s_full[b]));
-          if (j == item.ntiles - 1) mma_commit(bar(ctl->q_empty[qs]));   // last S of the item
+          if (j == ntiles - 1) mma_commit(bar(ctl->q_empty[qs]));   // last S of the item
         }
         __syncwarp();
         prof.mark(4);
@@ -430,7 +432,6 @@ __global__ void __launch_bounds__(kThreads, 1)
         pend = true;
         pend_first = j == 0;
         pend_st = st;
-        pend_g = g;
         pend_n = n;
         pend_ncols = ncols;
       }
@@ -442,11 +443,10 @@ __global__ void __launch_bounds__(kThreads, 1)
   } else {
     // ============================================================ softmax + epilogue
     asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(kRegsSoftmax) : "memory");
-    const int h = (warp - 4) >> 2;                         // column half
+    const int cg = (warp - 4) >> 2;                        // column group: chunks cg, cg + 4
     const int q4 = warp & 3;                               // TMEM lane quarter
     const int t = q4 * 32 + lane;                          // row of the Q tile = TMEM lane
-    const uint32_t lane_base = (uint32_t)(q4 * 32) << 16;
-    const uint32_t tl = tmem + lane_base;
+    const uint32_t tl = tmem + ((uint32_t)(q4 * 32) << 16);
     const float c = p.scale_log2;
     const float2 c2 = make_float2(c, c);
     Prof prof((warp == 4 || warp == 8) && lane == 0 && blockIdx.x < 148);
@@ -466,67 +466,82 @@ __global__ void __launch_bounds__(kThreads, 1)
     };
     Epi pend{0.f, 0.f, -1, -1, 0, 0, 0, false, false};
     auto epilogue = [&](const Epi& e) {
-      // both halves' partial rows are merged; half h writes output columns [32h, 32h + 32) from
-      // O_0 and O_1 (same TMEM lane), plus the fine partial if any
-      mbar_wait(bar(ctl->pv_done[h][e.n_last & 1]), (e.n_last >> 1) & 1);   // the item's last P.V
-      ctl->xch[e.ipar][h][t] = make_float2(e.m, e.l);
-      named_bar_sync(1, 256);                              // both halves' P.V done, (m, l) visible
-      tc_fence_after();
+      // the four groups' partial rows are merged; warp (cg, q4) writes output columns
+      // [16cg, 16cg + 16) of its rows from O_0..O_3 (same TMEM lane), plus the fine partial if any.
+      // (m, l) are final after the item's last tile: exchange them first, so that the only wait
+      // between the item's last P.V and o_free is the O read itself.
+      ctl->xch[e.ipar][cg][t] = make_float2(e.m, e.l);
+      named_bar_sync(1, 512);                              // (m, l) of all groups visible
+      float mg[4], lg[4];
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        const float2 v = ctl->xch[e.ipar][k][t];
+        mg[k] = v.x;
+        lg[k] = v.y;
+      }
+      float mf = -INFINITY, lf = 0.f;
+      const float* accf = nullptr;
+      if (e.slot_f >= 0) {
+        const size_t idx = (size_t)e.ubh * p.n_fine_rows + e.slot_f;
+        const float2 ml = p.part_ml[idx];
+        mf = ml.x;
+        lf = ml.y;
+        accf = p.part_acc + idx * 64 + cg * 16;
+      }
+      const float mt = fmaxf(fmaxf(fmaxf(mg[0], mg[1]), fmaxf(mg[2], mg[3])), mf);
+      const float mu = mt == -INFINITY ? 0.f : mt;
+      float a[4], den = 0.f;
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        a[k] = ex2((mg[k] - mu) * c);                      // 0 for a group with no valid column
+        den += lg[k] * a[k];
+      }
+      const float af = ex2((mf - mu) * c);
+      den += lf * af;
       prof.mark(9);
-      const float2 mlo = ctl->xch[e.ipar][h ^ 1][t];
-      uint32_t oa[2][16], ob[2][16];
+      mbar_wait(bar(ctl->pv_done[e.n_last & 1]), (e.n_last >> 1) & 1);   // the item's last P.V
+      tc_fence_after();
+      float acc[16];
+#pragma unroll
+      for (int i = 0; i < 16; ++i) acc[i] = 0.f;
       if (e.active) {
-        tmem_ld16(tl + kTmemO + h * 32, oa[0]);
-        tmem_ld16(tl + kTmemO + h * 32 + 16, oa[1]);
-        tmem_ld16(tl + kTmemO + 64 + h * 32, ob[0]);
-        tmem_ld16(tl + kTmemO + 64 + h * 32 + 16, ob[1]);
-        tmem_wait_ld();
+#pragma unroll
+        for (int k = 0; k < 4; k += 2) {
+          uint32_t o0[16], o1[16];
+          tmem_ld16(tl + kTmemO + k * 64 + cg * 16, o0);
+          tmem_ld16(tl + kTmemO + (k + 1) * 64 + cg * 16, o1);
+          tmem_wait_ld();
+#pragma unroll
+          for (int i = 0; i < 16; ++i)
+            acc[i] += __uint_as_float(o0[i]) * a[k] + __uint_as_float(o1[i]) * a[k + 1];
+        }
       }
       tc_fence_before();
       __syncwarp();
       if (lane == 0) mbar_arrive(bar(ctl->o_free));        // O may be overwritten by the next item
       prof.mark(10);
-      if (e.r_out >= 0) {
-        const float m0 = h == 0 ? e.m : mlo.x, l0 = h == 0 ? e.l : mlo.y;
-        const float m1 = h == 0 ? mlo.x : e.m, l1 = h == 0 ? mlo.y : e.l;
-        float mf = -INFINITY, lf = 0.f;
-        const float* accf = nullptr;
-        if (e.slot_f >= 0) {
-          const size_t idx = (size_t)e.ubh * p.n_fine_rows + e.slot_f;
-          const float2 ml = p.part_ml[idx];
-          mf = ml.x;
-          lf = ml.y;
-          accf = p.part_acc + idx * 64 + h * 32;
-        }
-        const float mt = fmaxf(fmaxf(m0, m1), mf);
-        if (mt != -INFINITY) {
-          const float a0 = ex2((m0 - mt) * c), a1 = ex2((m1 - mt) * c), af = ex2((mf - mt) * c);
-          const float inv = 1.f / (l0 * a0 + l1 * a1 + lf * af);
-          const int bb = e.ubh / p.H, hh = e.ubh % p.H;
-          uint16_t* orow = p.o.data + bb * p.o.sb + hh * p.o.sh + (int64_t)e.r_out * p.o.sl + h * 32;
+      if (e.r_out >= 0 && mt != -INFINITY) {
+        if (accf) {
 #pragma unroll
-          for (int q8 = 0; q8 < 4; ++q8) {
-            float v[8];
-#pragma unroll
-            for (int k = 0; k < 8; ++k) {
-              const int i = q8 * 8 + k;
-              v[k] = __uint_as_float(oa[i >> 4][i & 15]) * a0 + __uint_as_float(ob[i >> 4][i & 15]) * a1;
-            }
-            if (accf) {
-              const float4 f0 = reinterpret_cast<const float4*>(accf)[q8 * 2];
-              const float4 f1 = reinterpret_cast<const float4*>(accf)[q8 * 2 + 1];
-              v[0] = fmaf(f0.x, af, v[0]); v[1] = fmaf(f0.y, af, v[1]);
-              v[2] = fmaf(f0.z, af, v[2]); v[3] = fmaf(f0.w, af, v[3]);
-              v[4] = fmaf(f1.x, af, v[4]); v[5] = fmaf(f1.y, af, v[5]);
-              v[6] = fmaf(f1.z, af, v[6]); v[7] = fmaf(f1.w, af, v[7]);
-            }
-            uint4 o4;
-            o4.x = pack2<kBF16>(v[0] * inv, v[1] * inv);
-            o4.y = pack2<kBF16>(v[2] * inv, v[3] * inv);
-            o4.z = pack2<kBF16>(v[4] * inv, v[5] * inv);
-            o4.w = pack2<kBF16>(v[6] * inv, v[7] * inv);
-            *reinterpret_cast<uint4*>(orow + q8 * 8) = o4;
+          for (int q = 0; q < 4; ++q) {
+            const float4 f = reinterpret_cast<const float4*>(accf)[q];
+            acc[4 * q] = fmaf(f.x, af, acc[4 * q]);
+            acc[4 * q + 1] = fmaf(f.y, af, acc[4 * q + 1]);
+            acc[4 * q + 2] = fmaf(f.z, af, acc[4 * q + 2]);
+            acc[4 * q + 3] = fmaf(f.w, af, acc[4 * q + 3]);
           }
+        }
+        const float inv = 1.f / den;
+        const int bb = e.ubh / p.H, hh = e.ubh % p.H;
+        uint16_t* orow = p.o.data + bb * p.o.sb + hh * p.o.sh + (int64_t)e.r_out * p.o.sl + cg * 16;
+#pragma unroll
+        for (int q8 = 0; q8 < 2; ++q8) {
+          uint4 o4;
+          o4.x = pack2<kBF16>(acc[q8 * 8 + 0] * inv, acc[q8 * 8 + 1] * inv);
+          o4.y = pack2<kBF16>(acc[q8 * 8 + 2] * inv, acc[q8 * 8 + 3] * inv);
+          o4.z = pack2<kBF16>(acc[q8 * 8 + 4] * inv, acc[q8 * 8 + 5] * inv);
+          o4.w = pack2<kBF16>(acc[q8 * 8 + 6] * inv, acc[q8 * 8 + 7] * inv);
+          *reinterpret_cast<uint4*>(orow + q8 * 8) = o4;
         }
       }
       prof.mark(11);
@@ -558,51 +573,42 @@ __global__ void __launch_bounds__(kThreads, 1)
       float m = -INFINITY, l = 0.f;
       for (int j = 0; j < ntiles; ++j, ++g, ++n) {
         const uint32_t st = g % kStages, b = n & 1;
-        // S(n) complete implies (tcgen05.commit tracks all earlier tcgen05 ops of the MMA thread):
-        //  * P.V(n-2) of both halves done -> P[b][h] may be overwritten;
-        //  * the MMA warp had observed kv_full for this stage -> tile descriptor and bitmask landed.
+        // S(n) complete implies (tcgen05.commit tracks all earlier tcgen05 ops of the MMA thread)
+        // that the MMA warp had observed kv_full for this stage: tile descriptor and bitmask landed
         mbar_wait(bar(ctl->s_full[b]), (n >> 1) & 1);
         prof.mark(2);
         tc_fence_after();
         const int4 tri = ld_shared_v4(smem_u32(&ctl->tref[st]));   // {arg, kind, ncols, maskA}
         const int4 mw = ld_shared_v4(sM + st * kMaskBytes + t * 16);
-        const int ncols = tri.z;
+        const int nchunk = tri.z >> 4;                     // 16-column chunks of the tile: 2..8
+        const bool has0 = cg < nchunk, has1 = cg + 4 < nchunk;
         const bool partial = tri.w >= 0;
-        const int hc = ncols >> 1;                         // columns of this half: 16..64
-        const int nc = hc >> 4;                            // 16-column chunks: 1..4
-        const uint32_t tS = tl + b * 128 + h * hc;
-        uint32_t r0[16], r1[16], r2[16], r3[16];
-        if (active && !(p.debug_flags & 16)) {
-          tmem_ld16(tS, r0);
-          if (nc > 1) tmem_ld16(tS + 16, r1);
-          if (nc > 2) tmem_ld16(tS + 32, r2);
-          if (nc > 3) tmem_ld16(tS + 48, r3);
+        const uint32_t tS0 = tl + b * 128 + cg * 16, tS1 = tS0 + 64;
+        uint32_t r0[16], r1[16];
+        const bool ld = active && has0 && !(p.debug_flags & 16);
+        if (ld) {
+          tmem_ld16(tS0, r0);
+          if (has1) tmem_ld16(tS1, r1);
         }
-        uint64_t wd = ~0ull;
+        // validity bits of chunks cg (word 0) and cg + 4 (word 1)
+        uint32_t m0 = 0xffffu, m1 = 0xffffu;
         if (partial) {
           const uint64_t w0 = ((uint64_t)(uint32_t)mw.y << 32) | (uint32_t)mw.x;
           const uint64_t w1 = ((uint64_t)(uint32_t)mw.w << 32) | (uint32_t)mw.z;
-          const int off = h * hc;                          // 0, 16, 32, 48 or 64
-          wd = off == 0 ? w0 : (off >= 64 ? w1 : ((w0 >> off) | (w1 << (64 - off))));
+          m0 = (uint32_t)(w0 >> (16 * cg)) & 0xffffu;
+          m1 = (uint32_t)(w1 >> (16 * cg)) & 0xffffu;
         }
-        if (active && !(p.debug_flags & 16)) tmem_wait_ld();
+        if (ld) tmem_wait_ld();
         prof.mark(3);
-        tc_fence_before();                                 // S buffer free for tile n + 2
-        __syncwarp();
-        if (lane == 0) mbar_arrive(bar(ctl->s_free[b]));
         float tmax = -INFINITY;
-        if (active && !dry) {
+        if (active && has0 && !dry) {
           float mx0 = -INFINITY, mx1 = -INFINITY;
           if (partial) {
-            chunk_max<true>(r0, (uint32_t)wd & 0xffffu, mx0, mx1);
-            if (nc > 1) chunk_max<true>(r1, (uint32_t)(wd >> 16) & 0xffffu, mx0, mx1);
-            if (nc > 2) chunk_max<true>(r2, (uint32_t)(wd >> 32) & 0xffffu, mx0, mx1);
-            if (nc > 3) chunk_max<true>(r3, (uint32_t)(wd >> 48) & 0xffffu, mx0, mx1);
+            chunk_max<true>(r0, m0, mx0, mx1);
+            if (has1) chunk_max<true>(r1, m1, mx0, mx1);
           } else {
             chunk_max<false>(r0, 0xffffu, mx0, mx1);
-            if (nc > 1) chunk_max<false>(r1, 0xffffu, mx0, mx1);
-            if (nc > 2) chunk_max<false>(r2, 0xffffu, mx0, mx1);
-            if (nc > 3) chunk_max<false>(r3, 0xffffu, mx0, mx1);
+            if (has1) chunk_max<false>(r1, 0xffffu, mx0, mx1);
           }
           tmax = fmaxf(mx0, mx1);
         }
@@ -616,38 +622,33 @@ __global__ void __launch_bounds__(kThreads, 1)
         l *= alpha;
         prof.mark(4);
         if (j > 0 && __any_sync(0xffffffffu, need && alpha != 0.f)) {
-          // O_h holds tiles < n once P.V(n-1, h) is done; P.V(n, h) is not issued before p_full
-          mbar_wait(bar(ctl->pv_done[h][(n - 1) & 1]), ((n - 1) >> 1) & 1);
+          // O_cg holds tiles < n once P.V(n-1) is done; P.V(n) is not issued before p_full
+          mbar_wait(bar(ctl->pv_done[(n - 1) & 1]), ((n - 1) >> 1) & 1);
           tc_fence_after();
           if (active) {
 #pragma unroll
             for (int h2 = 0; h2 < 4; ++h2) {
               uint32_t r[16];
-              tmem_ld16(tl + kTmemO + h * 64 + h2 * 16, r);
+              tmem_ld16(tl + kTmemO + cg * 64 + h2 * 16, r);
               tmem_wait_ld();
 #pragma unroll
               for (int i = 0; i < 16; ++i) r[i] = __float_as_uint(__uint_as_float(r[i]) * alpha);
-              tmem_st16(tl + kTmemO + h * 64 + h2 * 16, r);
+              tmem_st16(tl + kTmemO + cg * 64 + h2 * 16, r);
             }
           }
         }
         prof.mark(5);
-        // p = 2^(s*c - m*c) (masked -> 0), packed to 16-bit pairs (A operand of P.V)
-        if (active && !dry) {
+        // p = 2^(s*c - m*c) (masked -> 0), packed to 16-bit pairs over the chunk's first 8 columns
+        if (active && has0 && !dry) {
           const float mu = (m == -INFINITY) ? 0.f : m;
           const float2 nb2 = make_float2(-mu * c, -mu * c);
           float2 rs0 = make_float2(0.f, 0.f), rs1 = make_float2(0.f, 0.f);
-          const uint32_t pb = tl + kTmemP + b * 64 + h * 32;
           if (partial) {
-            chunk_exp<true, kBF16>(r0, (uint32_t)wd & 0xffffu, c2, nb2, rs0, rs1, pb);
-            if (nc > 1) chunk_exp<true, kBF16>(r1, (uint32_t)(wd >> 16) & 0xffffu, c2, nb2, rs0, rs1, pb + 8);
-            if (nc > 2) chunk_exp<true, kBF16>(r2, (uint32_t)(wd >> 32) & 0xffffu, c2, nb2, rs0, rs1, pb + 16);
-            if (nc > 3) chunk_exp<true, kBF16>(r3, (uint32_t)(wd >> 48) & 0xffffu, c2, nb2, rs0, rs1, pb + 24);
+            chunk_exp<true, kBF16>(r0, m0, c2, nb2, rs0, rs1, tS0);
+            if (has1) chunk_exp<true, kBF16>(r1, m1, c2, nb2, rs0, rs1, tS1);
           } else {
-            chunk_exp<false, kBF16>(r0, 0xffffu, c2, nb2, rs0, rs1, pb);
-            if (nc > 1) chunk_exp<false, kBF16>(r1, 0xffffu, c2, nb2, rs0, rs1, pb + 8);
-            if (nc > 2) chunk_exp<false, kBF16>(r2, 0xffffu, c2, nb2, rs0, rs1, pb + 16);
-            if (nc > 3) chunk_exp<false, kBF16>(r3, 0xffffu, c2, nb2, rs0, rs1, pb + 24);
+            chunk_exp<false, kBF16>(r0, 0xffffu, c2, nb2, rs0, rs1, tS0);
+            if (has1) chunk_exp<false, kBF16>(r1, 0xffffu, c2, nb2, rs0, rs1, tS1);
           }
           l += (rs0.x + rs0.y) + (rs1.x + rs1.y);
           tmem_wait_st();
@@ -665,7 +666,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       pend = Epi{m, l, r_out, slot_f, ubh, n - 1, ipar, active, true};
     }
     if (pend.valid) epilogue(pend);
-    prof.flush(p, 2 + h);
+    prof.flush(p, 2 + (warp == 8));
   }
 
   tc_fence_before();

@@ -20,13 +20,13 @@ from workloads import get_config, make_qkv  # noqa: E402
 PHASES = {
     0: ("producer", ["item wait", "q_empty wait", "Q load/gather", "kv_empty wait", "K/V TMA issue",
                      "strip gather"]),
-    1: ("mma", ["item wait", "q_full wait", "kv_full wait", "s_free wait", "S issue", "o_free wait",
-                "p_full wait", "PV h0 issue", "-", "PV h1 issue"]),
-    2: ("softmax h0", ["item wait+meta", "-", "s_full wait", "tmem ld S", "s_free+max+decide",
+    1: ("mma", ["item wait", "q_full wait", "kv_full wait", "-", "S issue", "o_free wait",
+                "p_full wait", "PV issue", "-", "-"]),
+    2: ("softmax g0", ["item wait+meta", "-", "s_full wait", "tmem ld S", "max+decide",
                        "O rescale", "-", "exp+P store", "p_full arrive", "epi pv wait+xch",
                        "epi O ld+o_free", "epi store"]),
 }
-PHASES[3] = ("softmax h1", PHASES[2][1])
+PHASES[3] = ("softmax g1", PHASES[2][1])
 
 
 def main():
