@@ -39,6 +39,8 @@ def _compile(src: str, extra: list[str], verbose: bool) -> tuple[str, str]:
 def build(verbose: bool = False, ptxas_v: bool = False) -> str:
     os.makedirs(BUILD, exist_ok=True)
     extra = ["-Xptxas", "-v"] if ptxas_v else []
+    if os.environ.get("MG_TIMELINE"):
+        extra += ["-DMG_TIMELINE"]  # diagnostics build: per-item event clocks (tools/timeline_coarse.py)
     if os.environ.get("MG_TRACE"):
         extra += ["-DMG_TRACE"]  # diagnostics build: device event trace (tools/trace_coarse.py)
     with cf.ThreadPoolExecutor(max_workers=len(SOURCES)) as ex:

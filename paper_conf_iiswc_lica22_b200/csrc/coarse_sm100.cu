@@ -23,7 +23,8 @@
 //               row gathers (global rows, strip columns)
 //   warp 1      MMA issuer (lane 0): S(n), then P.V(n-1) of all groups
 //   warp 2      TMEM allocator, then scheduler: publishes work items, L2-prefetches their tiles
-//   warp 3      idle after setup
+//   warp 3      gatherer: row gathers (global-row Q tiles, strip K/V tiles) posted by the
+//               producer through a job ring, so gathers never stall the TMA stream
 //   warps 4..19 softmax: column group cg = (warp - 4) / 4, TMEM lane quarter = warp % 4
 // TMEM (512 columns): S/P[b] at b*128 (b = tile parity), O_cg at 256 + cg*64.
 #include <cuda_bf16.h>
@@ -49,7 +50,19 @@ struct __align__(16) ItemSlot {
   int32_t u, bh, pad0, pad1;
 };
 
+// A gather job for the gatherer warp: kind 0 = strip K/V tile into stage `dst`, 1 = Q rows into
+// Q buffer `dst`, 2 = stop.
+struct __align__(16) GatherJob {
+  const uint16_t* kbase;
+  const uint16_t* vbase;
+  const int32_t* idx;
+  int32_t kind, dst, nvalid, nfill, mask, pad;
+};
+constexpr int kJobs = 4;
+
 struct __align__(16) SmemCtl {
+  GatherJob job[kJobs];
+  uint64_t job_full[kJobs], job_empty[kJobs];
   TileRef tref[kStages];
   ItemSlot slot[2];
   float2 xch[2][4][128];                     // [item parity][group][row] (m, l) for the merge
@@ -190,6 +203,18 @@ struct Prof {
 #endif
 };
 
+// Diagnostics (MG_TIMELINE builds only): per-item event clocks (low 32 bits of clock64) of every
+// CTA, 16 fields per item, written by single lanes to p.trace (as uint32, after 256 uint64s):
+// 0 softmax item start, 1 first S ready, 2 last P stored, 3/4 epilogue start/end, 5 MMA Q ready,
+// 6 MMA first S issued, 7 MMA first P.V issued, 8 epilogue after (m, l) exchange, 9 epilogue
+// after last-P.V wait, 10 epilogue after O read. tools/timeline_coarse.py reads it.
+__device__ __forceinline__ void tl_rec(const CoarseParams& p, uint32_t idx, int field) {
+#ifdef MG_TIMELINE
+  if (p.trace == nullptr || idx >= 64 || p.trace_cap < 256 + 8 * 64 * (int)gridDim.x) return;
+  reinterpret_cast<uint32_t*>(p.trace + 256)[(blockIdx.x * 64 + idx) * 16 + field] = (uint32_t)clock64();
+#endif
+}
+
 }  // namespace
 
 template <bool kBF16>
@@ -220,6 +245,10 @@ __global__ void __launch_bounds__(kThreads, 1)
       mbar_init(bar(ctl->item_empty[b]), 18);       // producer + MMA + 16 softmax warps
     }
     mbar_init(bar(ctl->o_free), 16);
+    for (int j = 0; j < kJobs; ++j) {
+      mbar_init(bar(ctl->job_full[j]), 1);
+      mbar_init(bar(ctl->job_empty[j]), 1);
+    }
     for (int s = 0; s < kStages; ++s) {
       mbar_init(bar(ctl->kv_full[s]), 1);
       mbar_init(bar(ctl->kv_empty[s]), 1);
@@ -246,7 +275,17 @@ __global__ void __launch_bounds__(kThreads, 1)
     Prof prof(lane == 0 && blockIdx.x < 148);
     const uint64_t pol_kv = policy_evict_last();   // K/V tiles are re-read by neighbouring items
     const uint64_t pol_q = policy_evict_first();   // Q tiles are read once
-    uint32_t it = 0, g = 0;
+    uint32_t it = 0, g = 0, jc = 0;
+    auto post = [&](const GatherJob& jb) {             // hand a gather to the gatherer warp
+      if (lane == 0) {
+        const uint32_t js = jc % kJobs;
+        mbar_wait(bar(ctl->job_empty[js]), ((jc / kJobs) & 1) ^ 1);
+        ctl->job[js] = jb;
+        mbar_arrive(bar(ctl->job_full[js]));
+      }
+      __syncwarp();
+      ++jc;
+    };
     while (true) {
       const uint32_t slot = it & 1, ph = (it >> 1) & 1;
       mbar_wait(bar(ctl->item_full[slot]), ph);
@@ -268,11 +307,8 @@ __global__ void __launch_bounds__(kThreads, 1)
           tma_load_4d(dQ, &tmq, bar(ctl->q_full[qs]), 0, item.rowA, hh, bb, pol_q);
         }
       } else {
-        const uint16_t* qsrc = p.q.data + bb * p.q.sb + hh * p.q.sh;
-        gather_rows(dQ, qsrc, p.q.sl, p.global_rows + item.rowA, item.nrowsA, 128, lane);
-        fence_proxy_async_smem();
-        __syncwarp();
-        if (lane == 0) mbar_arrive(bar(ctl->q_full[qs]));
+        post(GatherJob{p.q.data + bb * p.q.sb + hh * p.q.sh, nullptr, p.global_rows + item.rowA, 1, (int32_t)qs,
+                       item.nrowsA, 128, -1, 0});
       }
       prof.mark(2);
       ++it;
@@ -296,19 +332,13 @@ __global__ void __launch_bounds__(kThreads, 1)
             if (mbytes) bulk_load(dM, p.masks + (size_t)tr.maskA * 256, kMaskBytes, kvf);
           }
         } else {
-          const int32_t* idx = p.strip_cols + tr.arg;
-          gather_rows(dK, p.k.data + bb * p.k.sb + hh * p.k.sh, p.k.sl, idx, tr.ncols, tr.ncols, lane);
-          gather_rows(dV, p.v.data + bb * p.v.sb + hh * p.v.sh, p.v.sl, idx, tr.ncols, tr.ncols, lane);
-          fence_proxy_async_smem();
-          __syncwarp();
-          if (lane == 0) {
-            mbar_arrive_expect_tx(kvf, mbytes);
-            if (mbytes) bulk_load(dM, p.masks + (size_t)tr.maskA * 256, kMaskBytes, kvf);
-          }
+          post(GatherJob{p.k.data + bb * p.k.sb + hh * p.k.sh, p.v.data + bb * p.v.sb + hh * p.v.sh,
+                         p.strip_cols + tr.arg, 0, (int32_t)st, tr.ncols, tr.ncols, tr.maskA, 0});
         }
         prof.mark(tr.kind == 0 ? 4 : 5);
       }
     }
+    post(GatherJob{nullptr, nullptr, nullptr, 2, 0, 0, 0, -1, 0});
     prof.flush(p, 0);
   } else if (warp == 2) {
     // ============================================================ scheduler
@@ -369,12 +399,13 @@ __global__ void __launch_bounds__(kThreads, 1)
       if (!pend) return;
       const uint32_t b = pend_n & 1, st = pend_st;
       if (pend_first) {
-        if (items_done > 0) mbar_wait(bar(ctl->o_free), (items_done - 1) & 1);
+        if (items_done > 0 && !(p.debug_flags & 64)) mbar_wait(bar(ctl->o_free), (items_done - 1) & 1);
+        if (leader) tl_rec(p, items_done, 7);
         ++items_done;
         started = 0;
       }
       prof.mark(5);
-      mbar_wait(bar(ctl->p_full[b]), (pend_n >> 1) & 1);
+      if (!(p.debug_flags & 64)) mbar_wait(bar(ctl->p_full[b]), (pend_n >> 1) & 1);
       prof.mark(6);
       tc_fence_after();
       if (leader && !(p.debug_flags & 2)) {
@@ -409,6 +440,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       const uint32_t qa = sQ + qs * kTileBytes;
       mbar_wait(bar(ctl->q_full[qs]), ph);
       prof.mark(1);
+      if (leader) tl_rec(p, it, 5);
       ++it;
       for (int j = 0; j < ntiles; ++j, ++g, ++n) {
         const uint32_t st = g % kStages, b = n & 1;
@@ -428,6 +460,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         }
         __syncwarp();
         prof.mark(4);
+        if (leader && j == 0) tl_rec(p, it - 1, 6);
         issue_pv();                                    // P.V of the previous tile
         pend = true;
         pend_first = j == 0;
@@ -439,7 +472,32 @@ __global__ void __launch_bounds__(kThreads, 1)
     issue_pv();
     prof.flush(p, 1);
   } else if (warp == 3) {
+    // ============================================================ gatherer
     asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(kRegsCtl) : "memory");
+    for (uint32_t jc = 0;; ++jc) {
+      const uint32_t js = jc % kJobs;
+      mbar_wait(bar(ctl->job_full[js]), (jc / kJobs) & 1);
+      const GatherJob jb = ctl->job[js];
+      __syncwarp();
+      if (lane == 0) mbar_arrive(bar(ctl->job_empty[js]));
+      if (jb.kind == 2) break;
+      if (jb.kind == 0) {                                  // strip K/V tile (+ its bitmask)
+        gather_rows(sK + jb.dst * kTileBytes, jb.kbase, p.k.sl, jb.idx, jb.nvalid, jb.nfill, lane);
+        gather_rows(sV + jb.dst * kTileBytes, jb.vbase, p.v.sl, jb.idx, jb.nvalid, jb.nfill, lane);
+        fence_proxy_async_smem();
+        __syncwarp();
+        if (lane == 0) {
+          const uint32_t kvf = bar(ctl->kv_full[jb.dst]);
+          mbar_arrive_expect_tx(kvf, jb.mask >= 0 ? kMaskBytes : 0);
+          if (jb.mask >= 0) bulk_load(sM + jb.dst * kMaskBytes, p.masks + (size_t)jb.mask * 256, kMaskBytes, kvf);
+        }
+      } else {                                             // gathered global-row Q tile
+        gather_rows(sQ + jb.dst * kTileBytes, jb.kbase, p.q.sl, jb.idx, jb.nvalid, jb.nfill, lane);
+        fence_proxy_async_smem();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(bar(ctl->q_full[jb.dst]));
+      }
+    }
   } else {
     // ============================================================ softmax + epilogue
     asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(kRegsSoftmax) : "memory");
@@ -461,17 +519,19 @@ __global__ void __launch_bounds__(kThreads, 1)
     struct Epi {
       float m, l;
       int r_out, slot_f, ubh;
-      uint32_t n_last, ipar;
+      uint32_t n_last, ipar, idx;
       bool active, valid;
     };
-    Epi pend{0.f, 0.f, -1, -1, 0, 0, 0, false, false};
+    Epi pend{0.f, 0.f, -1, -1, 0, 0, 0, 0, false, false};
+    const bool tlw = warp == 4 && lane == 0;
     auto epilogue = [&](const Epi& e) {
+      if (tlw) tl_rec(p, e.idx, 3);
       // the four groups' partial rows are merged; warp (cg, q4) writes output columns
       // [16cg, 16cg + 16) of its rows from O_0..O_3 (same TMEM lane), plus the fine partial if any.
       // (m, l) are final after the item's last tile: exchange them first, so that the only wait
       // between the item's last P.V and o_free is the O read itself.
       ctl->xch[e.ipar][cg][t] = make_float2(e.m, e.l);
-      named_bar_sync(1, 512);                              // (m, l) of all groups visible
+      named_bar_sync(1 + q4, 128);                         // (m, l) of the row's four groups visible
       float mg[4], lg[4];
 #pragma unroll
       for (int k = 0; k < 4; ++k) {
@@ -499,8 +559,10 @@ __global__ void __launch_bounds__(kThreads, 1)
       const float af = ex2((mf - mu) * c);
       den += lf * af;
       prof.mark(9);
+      if (tlw) tl_rec(p, e.idx, 8);
       mbar_wait(bar(ctl->pv_done[e.n_last & 1]), (e.n_last >> 1) & 1);   // the item's last P.V
       tc_fence_after();
+      if (tlw) tl_rec(p, e.idx, 9);
       float acc[16];
 #pragma unroll
       for (int i = 0; i < 16; ++i) acc[i] = 0.f;
@@ -520,6 +582,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       __syncwarp();
       if (lane == 0) mbar_arrive(bar(ctl->o_free));        // O may be overwritten by the next item
       prof.mark(10);
+      if (tlw) tl_rec(p, e.idx, 10);
       if (e.r_out >= 0 && mt != -INFINITY) {
         if (accf) {
 #pragma unroll
@@ -545,6 +608,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         }
       }
       prof.mark(11);
+      if (tlw) tl_rec(p, e.idx, 4);
     };
 
     uint32_t it = 0, g = 0, n = 0;                         // n: tiles processed (CTA lifetime)
@@ -570,6 +634,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         if (kind == 0) slot_f = __ldg(p.fine_slot + row0 + t);
       }
       prof.mark(0);
+      if (tlw) tl_rec(p, it - 1, 0);
       float m = -INFINITY, l = 0.f;
       for (int j = 0; j < ntiles; ++j, ++g, ++n) {
         const uint32_t st = g % kStages, b = n & 1;
@@ -577,6 +642,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         // that the MMA warp had observed kv_full for this stage: tile descriptor and bitmask landed
         mbar_wait(bar(ctl->s_full[b]), (n >> 1) & 1);
         prof.mark(2);
+        if (tlw && j == 0) tl_rec(p, it - 1, 1);
         tc_fence_after();
         const int4 tri = ld_shared_v4(smem_u32(&ctl->tref[st]));   // {arg, kind, ncols, maskA}
         const int4 mw = ld_shared_v4(sM + st * kMaskBytes + t * 16);
@@ -658,15 +724,17 @@ __global__ void __launch_bounds__(kThreads, 1)
         __syncwarp();
         if (lane == 0) mbar_arrive(bar(ctl->p_full[b]));
         prof.mark(8);
+        if (tlw && j == ntiles - 1) tl_rec(p, it - 1, 2);
         if (j == 0 && pend.valid) {                        // previous item's epilogue
           epilogue(pend);
           pend.valid = false;
         }
       }
-      pend = Epi{m, l, r_out, slot_f, ubh, n - 1, ipar, active, true};
+      pend = Epi{m, l, r_out, slot_f, ubh, n - 1, ipar, it - 1, active, true};
     }
     if (pend.valid) epilogue(pend);
     prof.flush(p, 2 + (warp == 8));
+
   }
 
   tc_fence_before();

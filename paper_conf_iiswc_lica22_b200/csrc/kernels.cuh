@@ -36,7 +36,8 @@ struct CoarseParams {
   float scale_log2;           // (1/sqrt(d)) * log2(e)
   unsigned long long* trace;  // diagnostics: event trace of CTA 0 (null = off)
   int32_t trace_cap;
-  int32_t debug_flags;        // diagnostics (env MG_DEBUG_FLAGS): 1 = no softmax arithmetic, 2 = no MMA, 4 = no loads
+  int32_t debug_flags;        // diagnostics (env MG_DEBUG_FLAGS): 1 = no softmax arithmetic, 2 = no MMA, 4 = no loads,
+                              // 16 = no S loads from TMEM, 64 = MMA ignores P-ready/O-free (timing only)
 };
 
 // Fine CSR kernel: warp per (row, batch*head); SDDMM -> online softmax -> SpMM on CUDA cores.
