@@ -39,11 +39,23 @@ using namespace ptx;
 
 namespace {
 
+#ifndef MG_GROUPS
+#define MG_GROUPS 4
+#endif
+// Column groups per tile (2 or 4): 4 * kGroups softmax warps; group cg owns the 16-column
+// chunks c = cg, cg + kGroups, ... of every tile. TMEM holds kSbuf S/P buffers (128 columns each)
+// and one 64-column O accumulator per group: 2 groups -> 3 buffers, 4 groups -> 2 buffers.
+constexpr int kGroups = MG_GROUPS;
+static_assert(kGroups == 2 || kGroups == 4, "column groups");
+constexpr int kChunks = 8 / kGroups;          // chunks per group of a 128-column tile
+constexpr int kSbuf = kGroups == 2 ? 3 : 2;   // S/P buffers
+constexpr int kLag = kSbuf - 1;               // tiles the MMA issuer runs S ahead of P.V
 constexpr int kStages = 5;
-constexpr int kThreads = 640;
+constexpr int kThreads = 128 + 128 * kGroups;
 constexpr uint32_t kTileBytes = 128 * 128;  // 128 rows x 64 x 16-bit
 constexpr uint32_t kMaskBytes = 128 * 16;   // 128 rows x 2 x u64
-constexpr uint32_t kTmemO = 256;
+constexpr uint32_t kTmemO = 128 * kSbuf;
+static_assert(kTmemO + 64 * kGroups <= 512, "TMEM columns");
 
 struct __align__(16) ItemSlot {
   Item item;
@@ -65,10 +77,10 @@ struct __align__(16) SmemCtl {
   uint64_t job_full[kJobs], job_empty[kJobs];
   TileRef tref[kStages];
   ItemSlot slot[2];
-  float2 xch[2][4][128];                     // [item parity][group][row] (m, l) for the merge
+  float2 xch[2][kGroups][128];               // [item parity][group][row] (m, l) for the merge
   uint64_t q_full[2], q_empty[2];
   uint64_t kv_full[kStages], kv_empty[kStages];
-  uint64_t s_full[2], p_full[2], pv_done[2];  // per S/P buffer
+  uint64_t s_full[kSbuf], p_full[kSbuf], pv_done[kSbuf];  // per S/P buffer
   uint64_t o_free;
   uint64_t item_full[2], item_empty[2];
   uint32_t tmem_base;
@@ -76,10 +88,11 @@ struct __align__(16) SmemCtl {
 
 constexpr size_t kSmemBytes = 1024 + kTileBytes * (2 + 2 * kStages) + kMaskBytes * kStages + sizeof(SmemCtl);
 static_assert(kSmemBytes <= 227 * 1024, "shared memory budget");
-// setmaxnreg.inc draws from the CTA's pool (96 x 640 = 61440 registers at launch):
-// 128 x kRegsCtl + 512 x kRegsSoftmax must not exceed it, or the inc blocks forever.
-constexpr int kRegsCtl = 56, kRegsSoftmax = 104;
-static_assert(128 * kRegsCtl + 512 * kRegsSoftmax <= 96 * 640, "register pool");
+// setmaxnreg.inc draws from the CTA's pool (launch registers x kThreads): 128 x kRegsCtl +
+// (kThreads - 128) x kRegsSoftmax must not exceed it, or the inc blocks forever.
+constexpr int kRegsLaunch = (65536 / kThreads) & ~7;
+constexpr int kRegsCtl = 56, kRegsSoftmax = kGroups == 2 ? 224 : 104;
+static_assert(128 * kRegsCtl + (kThreads - 128) * kRegsSoftmax <= kRegsLaunch * kThreads, "register pool");
 
 struct UnitInfo {
   int item, bh;
@@ -238,13 +251,15 @@ __global__ void __launch_bounds__(kThreads, 1)
     for (int b = 0; b < 2; ++b) {
       mbar_init(bar(ctl->q_full[b]), 1);
       mbar_init(bar(ctl->q_empty[b]), 1);
-      mbar_init(bar(ctl->s_full[b]), 1);
-      mbar_init(bar(ctl->p_full[b]), 16);           // all 16 softmax warps stored their P
-      mbar_init(bar(ctl->pv_done[b]), 1);
       mbar_init(bar(ctl->item_full[b]), 1);
-      mbar_init(bar(ctl->item_empty[b]), 18);       // producer + MMA + 16 softmax warps
+      mbar_init(bar(ctl->item_empty[b]), 2 + 4 * kGroups);   // producer + MMA + softmax warps
     }
-    mbar_init(bar(ctl->o_free), 16);
+    for (int b = 0; b < kSbuf; ++b) {
+      mbar_init(bar(ctl->s_full[b]), 1);
+      mbar_init(bar(ctl->p_full[b]), 4 * kGroups);  // every softmax warp stored its P
+      mbar_init(bar(ctl->pv_done[b]), 1);
+    }
+    mbar_init(bar(ctl->o_free), 4 * kGroups);
     for (int j = 0; j < kJobs; ++j) {
       mbar_init(bar(ctl->job_full[j]), 1);
       mbar_init(bar(ctl->job_empty[j]), 1);
@@ -382,41 +397,44 @@ __global__ void __launch_bounds__(kThreads, 1)
   } else if (warp == 1) {
     // ============================================================ MMA issuer (lane 0)
     asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(kRegsCtl) : "memory");
-    // Tile sequence over the CTA's lifetime: n = 0, 1, 2, ...; S(n) -> S/P[n&1]. Iteration n
-    // issues S(n), then P.V(n-1) once every softmax warp stored P(n-1). S(n) reuses the buffer of
-    // tile n-2, whose P.V was issued earlier by this thread (in-order execution). The first P.V of
-    // an item's column group (accumulate = 0) also waits until the previous item's epilogue has
+    // Tile sequence over the CTA's lifetime: n = 0, 1, 2, ...; S(n) -> S/P[n % kSbuf]. Iteration n
+    // issues S(n), then P.V(n - kLag) once every softmax warp stored that tile's P. S(n) reuses
+    // the buffer of tile n - kSbuf, whose P.V this thread issued earlier (in-order execution).
+    // The first P.V of an item (accumulate = 0) also waits until the previous item's epilogue has
     // read O (o_free).
     const bool leader = lane == 0;
     Prof prof(leader && blockIdx.x < 148);
     uint32_t it = 0, g = 0, n = 0, items_done = 0;
-    // pending P.V: the tile issued last (stage, width, tile index, first-of-item)
-    bool pend = false, pend_first = false;
-    uint32_t pend_st = 0, pend_n = 0;
-    int pend_ncols = 0;
-    uint32_t started = 0;                              // column groups with an accumulator this item
-    auto issue_pv = [&]() {
-      if (!pend) return;
-      const uint32_t b = pend_n & 1, st = pend_st;
-      if (pend_first) {
+    struct Pend {
+      uint32_t st, n;
+      int ncols;
+      bool first, valid;
+    };
+    Pend q[kLag];                                      // pending P.V, oldest first
+#pragma unroll
+    for (int i = 0; i < kLag; ++i) q[i].valid = false;
+    auto issue_pv = [&](const Pend& e) {
+      const uint32_t b = e.n % kSbuf, st = e.st;
+      if (e.first) {
         if (items_done > 0 && !(p.debug_flags & 64)) mbar_wait(bar(ctl->o_free), (items_done - 1) & 1);
         if (leader) tl_rec(p, items_done, 7);
         ++items_done;
-        started = 0;
       }
       prof.mark(5);
-      if (!(p.debug_flags & 64)) mbar_wait(bar(ctl->p_full[b]), (pend_n >> 1) & 1);
+      mbar_wait(bar(ctl->p_full[b]), (e.n / kSbuf) & 1);
       prof.mark(6);
       tc_fence_after();
       if (leader && !(p.debug_flags & 2)) {
         const uint32_t vA = sV + st * kTileBytes;
         const uint32_t idesc_pv = idesc_f16(kBF16, 128, 64, false, true);
-        // chunk c (16 keys): P at S/P[b] columns [16c, 16c + 8) (packed), V rows [16c, 16c + 16)
-        for (int c = 0; c < (pend_ncols >> 4); ++c) {
-          const int cg = c & 3;
+        // chunk c (16 keys): P at S/P[b] columns [16c, 16c + 8) (packed), V rows [16c, 16c + 16);
+        // group c % kGroups accumulates into its O; the first chunk of a group in an item
+        // overwrites (the item's first tile has all groups: tiles are >= 2 * kGroups chunks wide
+        // except strips, which come last)
+        for (int c = 0; c < (e.ncols >> 4); ++c) {
+          const int cg = c % kGroups;
           mma_ts(tmem + kTmemO + cg * 64, tmem + b * 128 + c * 16, smem_desc_sw128(vA + c * 2048, 8192, 1024),
-                 idesc_pv, (started >> cg) & 1u);
-          started |= 1u << cg;
+                 idesc_pv, (e.first && c < kGroups) ? 0u : 1u);
         }
       }
       if (leader) {
@@ -425,7 +443,6 @@ __global__ void __launch_bounds__(kThreads, 1)
       }
       __syncwarp();
       prof.mark(7);
-      pend = false;
     };
     while (true) {
       const uint32_t slot = it & 1, ph = (it >> 1) & 1;
@@ -443,7 +460,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       if (leader) tl_rec(p, it, 5);
       ++it;
       for (int j = 0; j < ntiles; ++j, ++g, ++n) {
-        const uint32_t st = g % kStages, b = n & 1;
+        const uint32_t st = g % kStages, b = n % kSbuf;
         mbar_wait(bar(ctl->kv_full[st]), (g / kStages) & 1);
         prof.mark(2);
         const int ncols = ctl->tref[st].ncols;
@@ -461,15 +478,15 @@ __global__ void __launch_bounds__(kThreads, 1)
         __syncwarp();
         prof.mark(4);
         if (leader && j == 0) tl_rec(p, it - 1, 6);
-        issue_pv();                                    // P.V of the previous tile
-        pend = true;
-        pend_first = j == 0;
-        pend_st = st;
-        pend_n = n;
-        pend_ncols = ncols;
+        if (q[0].valid) issue_pv(q[0]);               // P.V of tile n - kLag
+#pragma unroll
+        for (int i = 0; i + 1 < kLag; ++i) q[i] = q[i + 1];
+        q[kLag - 1] = Pend{st, n, ncols, j == 0, true};
       }
     }
-    issue_pv();
+#pragma unroll
+    for (int i = 0; i < kLag; ++i)
+      if (q[i].valid) issue_pv(q[i]);
     prof.flush(p, 1);
   } else if (warp == 3) {
     // ============================================================ gatherer
@@ -501,7 +518,7 @@ __global__ void __launch_bounds__(kThreads, 1)
   } else {
     // ============================================================ softmax + epilogue
     asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(kRegsSoftmax) : "memory");
-    const int cg = (warp - 4) >> 2;                        // column group: chunks cg, cg + 4
+    const int cg = (warp - 4) >> 2;                        // column group: chunks cg + kGroups*i
     const int q4 = warp & 3;                               // TMEM lane quarter
     const int t = q4 * 32 + lane;                          // row of the Q tile = TMEM lane
     const uint32_t tl = tmem + ((uint32_t)(q4 * 32) << 16);
@@ -512,10 +529,11 @@ __global__ void __launch_bounds__(kThreads, 1)
     // lazy rescaling (O accumulates in TMEM): the exponent uses a stale row max m until a tile's
     // max exceeds it by more than 2^8 in probability, so p <= 256 and O rarely needs a rescale
     const float thresh = 8.f / c;
+    constexpr int W = 64 / kGroups;                        // output columns written per warp
 
     // An item's epilogue runs after the NEXT item's first tile, by which time the item's last P.V
-    // (issued by the MMA warp after the next item's first S) has completed; the next item's first
-    // P.V (accumulate = 0) waits for it through o_free.
+    // (issued by the MMA warp after the next item's first S) has normally completed; the next
+    // item's first P.V (accumulate = 0) waits for it through o_free.
     struct Epi {
       float m, l;
       int r_out, slot_f, ubh;
@@ -526,15 +544,15 @@ __global__ void __launch_bounds__(kThreads, 1)
     const bool tlw = warp == 4 && lane == 0;
     auto epilogue = [&](const Epi& e) {
       if (tlw) tl_rec(p, e.idx, 3);
-      // the four groups' partial rows are merged; warp (cg, q4) writes output columns
-      // [16cg, 16cg + 16) of its rows from O_0..O_3 (same TMEM lane), plus the fine partial if any.
-      // (m, l) are final after the item's last tile: exchange them first, so that the only wait
-      // between the item's last P.V and o_free is the O read itself.
+      // the groups' partial rows are merged; warp (cg, q4) writes output columns [W*cg, W*cg + W)
+      // of its rows from every group's O (same TMEM lane), plus the fine partial if any. (m, l)
+      // are final after the item's last tile: exchange them first, so that the only wait between
+      // the item's last P.V and o_free is the O read itself.
       ctl->xch[e.ipar][cg][t] = make_float2(e.m, e.l);
-      named_bar_sync(1 + q4, 128);                         // (m, l) of the row's four groups visible
-      float mg[4], lg[4];
+      named_bar_sync(1 + q4, 32 * kGroups);                // (m, l) of the row's groups visible
+      float mg[kGroups], lg[kGroups];
 #pragma unroll
-      for (int k = 0; k < 4; ++k) {
+      for (int k = 0; k < kGroups; ++k) {
         const float2 v = ctl->xch[e.ipar][k][t];
         mg[k] = v.x;
         lg[k] = v.y;
@@ -546,13 +564,15 @@ __global__ void __launch_bounds__(kThreads, 1)
         const float2 ml = p.part_ml[idx];
         mf = ml.x;
         lf = ml.y;
-        accf = p.part_acc + idx * 64 + cg * 16;
+        accf = p.part_acc + idx * 64 + cg * W;
       }
-      const float mt = fmaxf(fmaxf(fmaxf(mg[0], mg[1]), fmaxf(mg[2], mg[3])), mf);
-      const float mu = mt == -INFINITY ? 0.f : mt;
-      float a[4], den = 0.f;
+      float mt = mf;
 #pragma unroll
-      for (int k = 0; k < 4; ++k) {
+      for (int k = 0; k < kGroups; ++k) mt = fmaxf(mt, mg[k]);
+      const float mu = mt == -INFINITY ? 0.f : mt;
+      float a[kGroups], den = 0.f;
+#pragma unroll
+      for (int k = 0; k < kGroups; ++k) {
         a[k] = ex2((mg[k] - mu) * c);                      // 0 for a group with no valid column
         den += lg[k] * a[k];
       }
@@ -560,22 +580,23 @@ __global__ void __launch_bounds__(kThreads, 1)
       den += lf * af;
       prof.mark(9);
       if (tlw) tl_rec(p, e.idx, 8);
-      mbar_wait(bar(ctl->pv_done[e.n_last & 1]), (e.n_last >> 1) & 1);   // the item's last P.V
+      mbar_wait(bar(ctl->pv_done[e.n_last % kSbuf]), (e.n_last / kSbuf) & 1);   // the item's last P.V
       tc_fence_after();
       if (tlw) tl_rec(p, e.idx, 9);
-      float acc[16];
+      float acc[W];
 #pragma unroll
-      for (int i = 0; i < 16; ++i) acc[i] = 0.f;
+      for (int i = 0; i < W; ++i) acc[i] = 0.f;
       if (e.active) {
 #pragma unroll
-        for (int k = 0; k < 4; k += 2) {
-          uint32_t o0[16], o1[16];
-          tmem_ld16(tl + kTmemO + k * 64 + cg * 16, o0);
-          tmem_ld16(tl + kTmemO + (k + 1) * 64 + cg * 16, o1);
-          tmem_wait_ld();
+        for (int k = 0; k < kGroups; ++k) {
 #pragma unroll
-          for (int i = 0; i < 16; ++i)
-            acc[i] += __uint_as_float(o0[i]) * a[k] + __uint_as_float(o1[i]) * a[k + 1];
+          for (int s16 = 0; s16 < W / 16; ++s16) {
+            uint32_t o[16];
+            tmem_ld16(tl + kTmemO + k * 64 + cg * W + s16 * 16, o);
+            tmem_wait_ld();
+#pragma unroll
+            for (int i = 0; i < 16; ++i) acc[s16 * 16 + i] = fmaf(__uint_as_float(o[i]), a[k], acc[s16 * 16 + i]);
+          }
         }
       }
       tc_fence_before();
@@ -586,7 +607,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       if (e.r_out >= 0 && mt != -INFINITY) {
         if (accf) {
 #pragma unroll
-          for (int q = 0; q < 4; ++q) {
+          for (int q = 0; q < W / 4; ++q) {
             const float4 f = reinterpret_cast<const float4*>(accf)[q];
             acc[4 * q] = fmaf(f.x, af, acc[4 * q]);
             acc[4 * q + 1] = fmaf(f.y, af, acc[4 * q + 1]);
@@ -594,11 +615,11 @@ __global__ void __launch_bounds__(kThreads, 1)
             acc[4 * q + 3] = fmaf(f.w, af, acc[4 * q + 3]);
           }
         }
-        const float inv = 1.f / den;
+        const float inv = __frcp_rn(den);
         const int bb = e.ubh / p.H, hh = e.ubh % p.H;
-        uint16_t* orow = p.o.data + bb * p.o.sb + hh * p.o.sh + (int64_t)e.r_out * p.o.sl + cg * 16;
+        uint16_t* orow = p.o.data + bb * p.o.sb + hh * p.o.sh + (int64_t)e.r_out * p.o.sl + cg * W;
 #pragma unroll
-        for (int q8 = 0; q8 < 2; ++q8) {
+        for (int q8 = 0; q8 < W / 8; ++q8) {
           uint4 o4;
           o4.x = pack2<kBF16>(acc[q8 * 8 + 0] * inv, acc[q8 * 8 + 1] * inv);
           o4.y = pack2<kBF16>(acc[q8 * 8 + 2] * inv, acc[q8 * 8 + 3] * inv);
@@ -637,44 +658,49 @@ __global__ void __launch_bounds__(kThreads, 1)
       if (tlw) tl_rec(p, it - 1, 0);
       float m = -INFINITY, l = 0.f;
       for (int j = 0; j < ntiles; ++j, ++g, ++n) {
-        const uint32_t st = g % kStages, b = n & 1;
+        const uint32_t st = g % kStages, b = n % kSbuf;
         // S(n) complete implies (tcgen05.commit tracks all earlier tcgen05 ops of the MMA thread)
         // that the MMA warp had observed kv_full for this stage: tile descriptor and bitmask landed
-        mbar_wait(bar(ctl->s_full[b]), (n >> 1) & 1);
+        mbar_wait(bar(ctl->s_full[b]), (n / kSbuf) & 1);
         prof.mark(2);
         if (tlw && j == 0) tl_rec(p, it - 1, 1);
         tc_fence_after();
         const int4 tri = ld_shared_v4(smem_u32(&ctl->tref[st]));   // {arg, kind, ncols, maskA}
         const int4 mw = ld_shared_v4(sM + st * kMaskBytes + t * 16);
         const int nchunk = tri.z >> 4;                     // 16-column chunks of the tile: 2..8
-        const bool has0 = cg < nchunk, has1 = cg + 4 < nchunk;
         const bool partial = tri.w >= 0;
-        const uint32_t tS0 = tl + b * 128 + cg * 16, tS1 = tS0 + 64;
-        uint32_t r0[16], r1[16];
-        const bool ld = active && has0 && !(p.debug_flags & 16);
+        const uint32_t tSb = tl + b * 128 + cg * 16;       // this group's first chunk
+        bool has[kChunks];
+#pragma unroll
+        for (int i = 0; i < kChunks; ++i) has[i] = cg + kGroups * i < nchunk;
+        uint32_t r[kChunks][16];
+        const bool ld = active && has[0] && !(p.debug_flags & 16);
         if (ld) {
-          tmem_ld16(tS0, r0);
-          if (has1) tmem_ld16(tS1, r1);
+#pragma unroll
+          for (int i = 0; i < kChunks; ++i)
+            if (has[i]) tmem_ld16(tSb + kGroups * 16 * i, r[i]);
         }
-        // validity bits of chunks cg (word 0) and cg + 4 (word 1)
-        uint32_t m0 = 0xffffu, m1 = 0xffffu;
-        if (partial) {
-          const uint64_t w0 = ((uint64_t)(uint32_t)mw.y << 32) | (uint32_t)mw.x;
-          const uint64_t w1 = ((uint64_t)(uint32_t)mw.w << 32) | (uint32_t)mw.z;
-          m0 = (uint32_t)(w0 >> (16 * cg)) & 0xffffu;
-          m1 = (uint32_t)(w1 >> (16 * cg)) & 0xffffu;
+        // validity bits of the group's chunks
+        uint32_t mk[kChunks];
+#pragma unroll
+        for (int i = 0; i < kChunks; ++i) {
+          const int ch = cg + kGroups * i;
+          const uint32_t word = (uint32_t)((ch & 4) ? (ch & 2 ? mw.w : mw.z) : (ch & 2 ? mw.y : mw.x));
+          mk[i] = partial ? (word >> (16 * (ch & 1))) & 0xffffu : 0xffffu;
         }
         if (ld) tmem_wait_ld();
         prof.mark(3);
         float tmax = -INFINITY;
-        if (active && has0 && !dry) {
+        if (active && has[0] && !dry) {
           float mx0 = -INFINITY, mx1 = -INFINITY;
           if (partial) {
-            chunk_max<true>(r0, m0, mx0, mx1);
-            if (has1) chunk_max<true>(r1, m1, mx0, mx1);
+#pragma unroll
+            for (int i = 0; i < kChunks; ++i)
+              if (has[i]) chunk_max<true>(r[i], mk[i], mx0, mx1);
           } else {
-            chunk_max<false>(r0, 0xffffu, mx0, mx1);
-            if (has1) chunk_max<false>(r1, 0xffffu, mx0, mx1);
+#pragma unroll
+            for (int i = 0; i < kChunks; ++i)
+              if (has[i]) chunk_max<false>(r[i], 0xffffu, mx0, mx1);
           }
           tmax = fmaxf(mx0, mx1);
         }
@@ -689,32 +715,34 @@ __global__ void __launch_bounds__(kThreads, 1)
         prof.mark(4);
         if (j > 0 && __any_sync(0xffffffffu, need && alpha != 0.f)) {
           // O_cg holds tiles < n once P.V(n-1) is done; P.V(n) is not issued before p_full
-          mbar_wait(bar(ctl->pv_done[(n - 1) & 1]), ((n - 1) >> 1) & 1);
+          mbar_wait(bar(ctl->pv_done[(n - 1) % kSbuf]), ((n - 1) / kSbuf) & 1);
           tc_fence_after();
           if (active) {
 #pragma unroll
             for (int h2 = 0; h2 < 4; ++h2) {
-              uint32_t r[16];
-              tmem_ld16(tl + kTmemO + cg * 64 + h2 * 16, r);
+              uint32_t rr[16];
+              tmem_ld16(tl + kTmemO + cg * 64 + h2 * 16, rr);
               tmem_wait_ld();
 #pragma unroll
-              for (int i = 0; i < 16; ++i) r[i] = __float_as_uint(__uint_as_float(r[i]) * alpha);
-              tmem_st16(tl + kTmemO + cg * 64 + h2 * 16, r);
+              for (int i = 0; i < 16; ++i) rr[i] = __float_as_uint(__uint_as_float(rr[i]) * alpha);
+              tmem_st16(tl + kTmemO + cg * 64 + h2 * 16, rr);
             }
           }
         }
         prof.mark(5);
         // p = 2^(s*c - m*c) (masked -> 0), packed to 16-bit pairs over the chunk's first 8 columns
-        if (active && has0 && !dry) {
+        if (active && has[0] && !dry) {
           const float mu = (m == -INFINITY) ? 0.f : m;
           const float2 nb2 = make_float2(-mu * c, -mu * c);
           float2 rs0 = make_float2(0.f, 0.f), rs1 = make_float2(0.f, 0.f);
           if (partial) {
-            chunk_exp<true, kBF16>(r0, m0, c2, nb2, rs0, rs1, tS0);
-            if (has1) chunk_exp<true, kBF16>(r1, m1, c2, nb2, rs0, rs1, tS1);
+#pragma unroll
+            for (int i = 0; i < kChunks; ++i)
+              if (has[i]) chunk_exp<true, kBF16>(r[i], mk[i], c2, nb2, rs0, rs1, tSb + kGroups * 16 * i);
           } else {
-            chunk_exp<false, kBF16>(r0, 0xffffu, c2, nb2, rs0, rs1, tS0);
-            if (has1) chunk_exp<false, kBF16>(r1, 0xffffu, c2, nb2, rs0, rs1, tS1);
+#pragma unroll
+            for (int i = 0; i < kChunks; ++i)
+              if (has[i]) chunk_exp<false, kBF16>(r[i], 0xffffu, c2, nb2, rs0, rs1, tSb + kGroups * 16 * i);
           }
           l += (rs0.x + rs0.y) + (rs1.x + rs1.y);
           tmem_wait_st();
@@ -734,7 +762,6 @@ __global__ void __launch_bounds__(kThreads, 1)
     }
     if (pend.valid) epilogue(pend);
     prof.flush(p, 2 + (warp == 8));
-
   }
 
   tc_fence_before();
