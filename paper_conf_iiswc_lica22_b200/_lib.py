@@ -5,7 +5,9 @@ import ctypes as C
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libmg.so")
+# MG_LIB_VARIANT=<name> loads a diagnostics build libmg_<name>.so (build.py --variant <name>)
+_VARIANT = os.environ.get("MG_LIB_VARIANT", "")
+LIB_PATH = os.path.join(_HERE, f"libmg_{_VARIANT}.so" if _VARIANT else "libmg.so")
 
 MG_OK, MG_ERR_INVALID_ARG, MG_ERR_UNSUPPORTED, MG_ERR_OUT_OF_MEMORY, MG_ERR_CUDA, MG_ERR_INTERNAL = range(6)
 MG_BF16, MG_FP16 = 0, 1

@@ -17,16 +17,18 @@ ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 BUILD = os.path.join(ROOT, "build", "mg")
 LIB = os.path.join(PKG, "libmg.so")
+# diagnostics variants: libmg_<name>.so with the matching -D flags, loaded via MG_LIB_VARIANT=<name>
+VARIANTS = {"watchdog": ["-DMG_WATCHDOG"], "timeline": ["-DMG_TIMELINE"], "trace": ["-DMG_TRACE"]}
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 
-SOURCES = ["plan.cpp", "api.cu", "coarse_sm100.cu", "fine_rows.cu", "selftest_umma.cu"]
+SOURCES = ["plan.cpp", "api.cu", "coarse_sm100.cu", "coarse_pp_sm100.cu", "fine_rows.cu", "selftest_umma.cu"]
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 COMMON = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC,-fvisibility=hidden",
           "-I", os.path.join(ROOT, "include"), "-I", CSRC]
 
 
-def _compile(src: str, extra: list[str], verbose: bool) -> tuple[str, str]:
-    obj = os.path.join(BUILD, os.path.splitext(src)[0] + ".o")
+def _compile(src: str, extra: list[str], verbose: bool, bdir: str = BUILD) -> tuple[str, str]:
+    obj = os.path.join(bdir, os.path.splitext(src)[0] + ".o")
     cmd = [NVCC, *ARCH, *COMMON, *extra, "-c", os.path.join(CSRC, src), "-o", obj]
     if verbose:
         print(" ".join(cmd))
@@ -36,21 +38,27 @@ def _compile(src: str, extra: list[str], verbose: bool) -> tuple[str, str]:
     return obj, r.stderr
 
 
-def build(verbose: bool = False, ptxas_v: bool = False) -> str:
-    os.makedirs(BUILD, exist_ok=True)
+def build(verbose: bool = False, ptxas_v: bool = False, variant: str = "") -> str:
+    bdir = os.path.join(BUILD, variant) if variant else BUILD
+    lib = os.path.join(PKG, f"libmg_{variant}.so") if variant else LIB
+    os.makedirs(bdir, exist_ok=True)
     extra = ["-Xptxas", "-v"] if ptxas_v else []
+    if variant:
+        extra += VARIANTS[variant]
     if os.environ.get("MG_TIMELINE"):
         extra += ["-DMG_TIMELINE"]  # diagnostics build: per-item event clocks (tools/timeline_coarse.py)
+    if os.environ.get("MG_WATCHDOG"):
+        extra += ["-DMG_WATCHDOG"]  # diagnostics build: barrier waits trap with a report instead of hanging
     if os.environ.get("MG_TRACE"):
         extra += ["-DMG_TRACE"]  # diagnostics build: device event trace (tools/trace_coarse.py)
     with cf.ThreadPoolExecutor(max_workers=len(SOURCES)) as ex:
-        results = list(ex.map(lambda s: _compile(s, extra, verbose), SOURCES))
+        results = list(ex.map(lambda s: _compile(s, extra, verbose, bdir), SOURCES))
     if ptxas_v:
         for _, log in results:
             if log.strip():
                 print(log)
     objs = [o for o, _ in results]
-    tmp = LIB + ".tmp"
+    tmp = lib + ".tmp"
     cmd = [NVCC, *ARCH, "-shared", "-cudart", "static", "-o", tmp, *objs,
            "-Xlinker", "--exclude-libs,ALL", "-lrt", "-ldl", "-lpthread"]
     if verbose:
@@ -58,14 +66,15 @@ def build(verbose: bool = False, ptxas_v: bool = False) -> str:
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         raise RuntimeError(f"link failed:\n{r.stdout}\n{r.stderr}")
-    os.replace(tmp, LIB)
-    return LIB
+    os.replace(tmp, lib)
+    return lib
 
 
 if __name__ == "__main__":
     ap = argparse.ArgumentParser()
     ap.add_argument("--verbose", action="store_true")
     ap.add_argument("--ptxas-v", action="store_true")
+    ap.add_argument("--variant", default="", choices=[""] + sorted(VARIANTS))
     a = ap.parse_args()
-    print(build(a.verbose, a.ptxas_v))
+    print(build(a.verbose, a.ptxas_v, a.variant))
     sys.exit(0)

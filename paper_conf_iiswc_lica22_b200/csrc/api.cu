@@ -235,6 +235,36 @@ bool encode_map(CUtensorMap* m, const mg_tensor* t) {
   return r == CUDA_SUCCESS;
 }
 
+// 2-D [rows, 64] view of a strided [B, H, L, 64] tensor for TMA row gathers (tile::gather4, box
+// 64 x 1): the row stride is the gcd of the element strides, which must be a multiple of 64
+// (true for dense [B,H,L,d] and [B,L,H,d]); row(b, h, l) = b * r.x + h * r.y + l * r.z.
+bool encode_map2d(CUtensorMap* m, const mg_tensor* t, longlong3* r) {
+  auto fn = tensor_map_encoder();
+  if (!fn) return false;
+  auto gcd = [](int64_t a, int64_t b) {
+    while (b) { const int64_t c = a % b; a = b; b = c; }
+    return a;
+  };
+  int64_t rs = 0;
+  for (int64_t s : {t->stride_b, t->stride_h, t->stride_l})
+    if (s > 0) rs = gcd(rs, s);
+  if (rs <= 0 || rs % 64) return false;
+  const int64_t span = (t->batch - 1) * t->stride_b + (t->heads - 1) * t->stride_h + (t->seq_len - 1) * t->stride_l + 64;
+  const int64_t rows = (span + rs - 1) / rs;
+  if (rows >= (int64_t(1) << 31)) return false;
+  cuuint64_t dims[2] = {64, (cuuint64_t)rows};
+  cuuint64_t strides[1] = {(cuuint64_t)rs * 2};
+  cuuint32_t box[2] = {64, 1};
+  cuuint32_t es[2] = {1, 1};
+  const CUtensorMapDataType dt =
+      t->dtype == MG_BF16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16;
+  if (fn(m, dt, 2, t->data, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+         CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+    return false;
+  *r = make_longlong3(t->stride_b / rs, t->stride_h / rs, t->stride_l / rs);
+  return true;
+}
+
 mg::TensorView view(const mg_tensor* t) {
   return mg::TensorView{static_cast<uint16_t*>(t->data), t->stride_b, t->stride_h, t->stride_l};
 }
@@ -322,10 +352,27 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
     if ((e = cudaMemsetAsync(p->d_counter, 0, sizeof(int32_t), stream)) != cudaSuccess)
       return cuda_fail(e, "cudaMemsetAsync");
     const int sms = p->num_sms_override > 0 ? std::min(p->num_sms_override, p->num_sms) : p->num_sms;
-    const int grid = std::min(sms, cp.total_units);
+    // MG_COARSE=v13 selects the previous single-CTA-per-SM kernel (A/B measurements only)
+    static const bool v13 = [] {
+      const char* e = std::getenv("MG_COARSE");
+      return e && std::strcmp(e, "v13") == 0;
+    }();
     if (p->profiling) cudaEventRecord(ev[2], stream);  // after the counter reset
-    if ((e = mg::launch_coarse(cp, tq, tk, tv, bf16, grid, stream)) != cudaSuccess)
-      return cuda_fail(e, "coarse kernel launch");
+    if (v13) {
+      if ((e = mg::launch_coarse(cp, tq, tk, tv, bf16, std::min(sms, cp.total_units), stream)) != cudaSuccess)
+        return cuda_fail(e, "coarse kernel launch");
+    } else {
+      CUtensorMap tq2, tk2, tv2;
+      std::memset(&tq2, 0, sizeof(tq2));
+      std::memset(&tk2, 0, sizeof(tk2));
+      std::memset(&tv2, 0, sizeof(tv2));
+      static const bool no_tma_gather = std::getenv("MG_NO_TMA_GATHER") != nullptr;   // A/B diagnostics
+      cp.gather_tma = !no_tma_gather && encode_map2d(&tq2, Q, &cp.rq) && encode_map2d(&tk2, K, &cp.rk) &&
+                      encode_map2d(&tv2, V, &cp.rv);
+      if ((e = mg::launch_coarse_pp(cp, tq, tk, tv, tq2, tk2, tv2, bf16, std::min(2 * sms, cp.total_units),
+                                    stream)) != cudaSuccess)
+        return cuda_fail(e, "coarse kernel launch");
+    }
   } else if (p->profiling) {
     cudaEventRecord(ev[2], stream);
   }

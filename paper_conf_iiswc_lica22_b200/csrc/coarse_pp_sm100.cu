@@ -1,0 +1,647 @@
+// Coarse-grained fused kernel for sm_100a, "paired pipelines" design: two co-resident CTAs per SM,
+// each an independent pipeline over the work items of the plan. One work item = one 128-row Q
+// tile (a band row block, or up to 128 gathered global rows) of one (batch, head) and its list of
+// K/V tiles:
+//   SDDMM   S = Q K_j^T            tcgen05.mma (SS), S in TMEM            (§3.2)
+//   scale + mask + online SpSoftmax  thread t owns row t of the Q tile   (§3.3)
+//   SpMM    O += P_j V_j           tcgen05.mma (TS: P from TMEM)         (§3.2)
+// The per-row running (max, sum) is carried across the row's tiles instead of re-reading S
+// (A14: the paper's 3-sweep SpSoftmax becomes an online softmax; same result).
+//   kind 0 items: a band row block with its BSR tiles (+ a gathered "strip" tile carrying the
+//     block's CSR residual on the tensor cores); the epilogue merges the fp32 partial statistics
+//     written by the CUDA-core fine kernel for any remaining CSR rows (compound SpSoftmax);
+//   kind 1 items: gathered global rows against every column tile (dense-row part).
+//
+// TMEM (256 columns per CTA, two CTAs fill the SM's 512): S [0,128) fp32, P [128,192) packed
+// 16-bit pairs, O [192,256) fp32. S and P are separate so that S(n+1) is issued as soon as the
+// softmax warps have *read* S(n) (s_free), i.e. while they compute the exponentials of tile n;
+// P(n) is stored at the end of the tile, after P.V(n-1) has consumed P(n-1) (pv_done).
+// While one CTA's softmax waits on its MMA chain, the other CTA's softmax owns the SM's MUFU and
+// FMA pipes: the two pipelines interleave without any shared barrier.
+//
+// Warp roles (256 threads = two warpgroups):
+//   warps 0-3  softmax + epilogue: thread t = row t of the Q tile = TMEM lane t (warp w owns the
+//              TMEM lane quarter w, as tcgen05.ld/st require)
+//   warp 4     producer: TMA of Q/K/V tiles (SWIZZLE_128B) and bitmasks; TMA row gathers
+//              (tile::gather4) for global-row Q tiles and strip K/V tiles
+//   warp 5     TMEM allocator; lane 0 issues the MMAs: S(n), then P.V(n-1)
+//   warp 6     scheduler: claims work items (atomic counter) into a 4-deep ring, L2 prefetch of
+//              each band item's Q tile
+//   warp 7     idle (completes the control warpgroup for setmaxnreg)
+// Shared memory: Q[2], K[2], V[2] 16 KB tiles (separate K and V rings: K(n+2) may load as soon
+// as S(n) has completed, V(n+2) after P.V(n)).
+#include <cuda_bf16.h>
+#include <cuda_fp16.h>
+
+#include "kernels.cuh"
+#include "sm100_ptx.cuh"
+
+namespace mg {
+
+using namespace ptx;
+
+namespace {
+
+constexpr int kThreads = 256;
+constexpr int kSt = 2;                       // K ring and V ring depth
+constexpr int kItems = 4;                    // work-item ring depth
+constexpr uint32_t kTileBytes = 128 * 128;   // 128 rows x 64 x 16-bit
+constexpr uint32_t kMaskBytes = 128 * 16;    // 128 rows x 128 validity bits
+constexpr uint32_t kTmemCols = 256;
+constexpr uint32_t kTS = 0, kTP = 128, kTO = 192;
+
+struct __align__(16) Slot {
+  Item item;
+  int32_t u, bh, pad0, pad1;
+};
+
+struct __align__(16) Ctl {
+  Slot slot[kItems];
+  int32_t kcols[kSt];                         // ncols of the tile in K stage s (producer -> MMA)
+  int2 vdesc[kSt];                            // {ncols, maskA} of the tile in V stage s (-> softmax)
+  uint64_t item_full[kItems], item_empty[kItems];
+  uint64_t q_full[2], q_empty[2];
+  uint64_t k_full[kSt], k_empty[kSt], v_full[kSt], v_empty[kSt];
+  uint64_t s_full, s_free, p_full, pv_done;
+  uint32_t tmem_base;
+};
+
+constexpr size_t kSmemBytes = 1024 + 6 * kTileBytes + kSt * kMaskBytes + sizeof(Ctl);
+static_assert(kSmemBytes <= 113 * 1024, "two CTAs per SM");
+// setmaxnreg applies per warpgroup: warps 0-3 (softmax) grow, warps 4-7 (control) shrink. The
+// pool of one CTA is (65536 / 2 / kThreads) x kThreads registers.
+constexpr int kRegsCtl = 64, kRegsSoftmax = 192;
+static_assert(128 * kRegsCtl + 128 * kRegsSoftmax <= (65536 / 2 / kThreads & ~7) * kThreads, "register pool");
+
+struct UnitInfo {
+  int item, bh;
+};
+
+// dense units first (long items start early), then band units in (b,h)-major, row-block order
+__device__ __forceinline__ UnitInfo decode_unit(const CoarseParams& p, int u) {
+  const int dense_units = p.n_dense_items * p.BH;
+  if (u < dense_units) return {u % p.n_dense_items, u / p.n_dense_items};
+  const int v = u - dense_units;
+  const int nband = p.n_items - p.n_dense_items;
+  return {p.n_dense_items + v % nband, v / nband};
+}
+
+// Copy rows idx[0..nvalid) (idx < 0 -> zeros) of a [*, 64] 16-bit matrix into a K-major
+// SWIZZLE_128B tile (row r at r*128 B, 16-byte chunk c at (c ^ (r & 7)) * 16); rows
+// [nvalid, nfill) are zero-filled. One warp; each lane keeps kBatch 16-byte loads in flight.
+__device__ __forceinline__ void gather_rows(uint32_t dst, const uint16_t* base, int64_t sl, const int32_t* idx,
+                                            int nvalid, int nfill, int lane) {
+  constexpr int kBatch = 4;
+  const int total = nfill * 8;
+  for (int e0 = 0; e0 < total; e0 += 32 * kBatch) {
+    int4 val[kBatch];
+#pragma unroll
+    for (int k = 0; k < kBatch; ++k) {
+      const int e = e0 + k * 32 + lane, r = e >> 3;
+      val[k] = make_int4(0, 0, 0, 0);
+      if (e < total && r < nvalid) {
+        const int src = __ldg(idx + r);
+        if (src >= 0) val[k] = ld_nc_v4(base + (int64_t)src * sl + (e & 7) * 8);
+      }
+    }
+#pragma unroll
+    for (int k = 0; k < kBatch; ++k) {
+      const int e = e0 + k * 32 + lane, r = e >> 3;
+      if (e < total) {
+        const uint32_t a = dst + r * 128 + (((e & 7) ^ (r & 7)) << 4);
+        asm volatile("st.shared.v4.s32 [%0], {%1, %2, %3, %4};" ::"r"(a), "r"(val[k].x), "r"(val[k].y),
+                     "r"(val[k].z), "r"(val[k].w)
+                     : "memory");
+      }
+    }
+  }
+}
+
+
+// 4 consecutive gather indices idx[i0 .. i0+4) (entries at or beyond n -> -1), 16-byte aligned
+__device__ __forceinline__ int4 load_idx4(const int32_t* idx, int i0, int n) {
+  int4 v = make_int4(-1, -1, -1, -1);
+  if (i0 + 3 < n) {
+    v = __ldg(reinterpret_cast<const int4*>(idx + i0));
+  } else if (i0 < n) {
+    v.x = __ldg(idx + i0);
+    if (i0 + 1 < n) v.y = __ldg(idx + i0 + 1);
+    if (i0 + 2 < n) v.z = __ldg(idx + i0 + 2);
+  }
+  return v;
+}
+
+// rows of the 2-D [rows, 64] view of a tensor: base + idx * step; idx < 0 -> -1 (out of bounds:
+// the TMA zero-fills the row)
+__device__ __forceinline__ int4 row_coords(int4 ix, int64_t base, int64_t step) {
+  auto f = [&](int i) { return i < 0 ? -1 : (int)(base + (int64_t)i * step); };
+  return make_int4(f(ix.x), f(ix.y), f(ix.z), f(ix.w));
+}
+
+// TMA row gather (tile::gather4): 4 rows of 64 16-bit elements into 4 consecutive 128-byte rows
+// of a SWIZZLE_128B tile at `dst` (the swizzle follows the shared address, as for tiled loads)
+__device__ __forceinline__ void gather4(uint32_t dst, const CUtensorMap* m, uint32_t bar, int4 rows,
+                                        uint64_t policy) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.tile::gather4.mbarrier::complete_tx::bytes.L2::cache_hint"
+      " [%0], [%1, {%2, %3, %4, %5, %6}], [%7], %8;" ::"r"(dst),
+      "l"(reinterpret_cast<uint64_t>(m)), "r"(0), "r"(rows.x), "r"(rows.y), "r"(rows.z), "r"(rows.w), "r"(bar),
+      "l"(policy)
+      : "memory");
+}
+
+template <bool kBF16>
+__device__ __forceinline__ uint32_t pack2(float lo, float hi) {
+  return kBF16 ? pack_bf16(lo, hi) : pack_f16(lo, hi);
+}
+
+__device__ __forceinline__ int4 ld_shared_v4(uint32_t a) {
+  int4 v;
+  asm volatile("ld.shared.v4.s32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(a));
+  return v;
+}
+
+// S values of one 32-column chunk with validity bits `bits` (bit i = column i): masked -> -inf.
+__device__ __forceinline__ void apply_mask(uint32_t (&r)[32], uint32_t bits) {
+#pragma unroll
+  for (int i = 0; i < 32; ++i)
+    if (!((bits >> i) & 1u)) r[i] = __float_as_uint(-INFINITY);
+}
+
+__device__ __forceinline__ float chunk_max(const uint32_t (&r)[32], float mx) {
+  float a = mx, b = -INFINITY, c = -INFINITY, d = -INFINITY;
+#pragma unroll
+  for (int i = 0; i < 32; i += 8) {
+    a = fmax3(a, __uint_as_float(r[i]), __uint_as_float(r[i + 1]));
+    b = fmax3(b, __uint_as_float(r[i + 2]), __uint_as_float(r[i + 3]));
+    c = fmax3(c, __uint_as_float(r[i + 4]), __uint_as_float(r[i + 5]));
+    d = fmax3(d, __uint_as_float(r[i + 6]), __uint_as_float(r[i + 7]));
+  }
+  return fmaxf(fmaxf(a, b), fmaxf(c, d));
+}
+
+// p = 2^(s*c - m*c) for 32 columns, packed to 16-bit pairs; row sum accumulated in rs[0..1]
+template <bool kBF16>
+__device__ __forceinline__ void chunk_exp(const uint32_t (&r)[32], float2 c2, float2 nb2, float2 (&rs)[2],
+                                          uint32_t (&pk)[16]) {
+#pragma unroll
+  for (int i = 0; i < 32; i += 2) {
+    const float2 x = __ffma2_rn(make_float2(__uint_as_float(r[i]), __uint_as_float(r[i + 1])), c2, nb2);
+    const float p0 = ex2(x.x), p1 = ex2(x.y);
+    rs[(i >> 1) & 1] = __fadd2_rn(rs[(i >> 1) & 1], make_float2(p0, p1));
+    pk[i >> 1] = pack2<kBF16>(p0, p1);
+  }
+}
+
+
+// Diagnostics (MG_TIMELINE builds only): per-tile event clocks (low 32 bits of clock64) of every
+// CTA for its first kTlTiles tiles, 8 fields per tile, after 256 uint64 header words of p.trace:
+// 0 softmax S(n)+V(n) ready, 1 softmax P.V(n-1) done, 2 softmax P(n) stored, 3 MMA S(n) issued,
+// 4 MMA P.V(n) issued, 5 producer K(n) issued, 6 producer V(n) issued, 7 SM id (tile 0 only).
+// tools/timeline_pp.py reads it.
+constexpr int kTlTiles = 128;
+__device__ __forceinline__ void tl_rec(const CoarseParams& p, uint32_t n, int field) {
+#ifdef MG_TIMELINE
+  if (p.trace == nullptr || n >= (uint32_t)kTlTiles ||
+      (int64_t)p.trace_cap < 256 + (int64_t)4 * kTlTiles * (int64_t)gridDim.x)
+    return;
+  reinterpret_cast<uint32_t*>(p.trace + 256)[((size_t)blockIdx.x * kTlTiles + n) * 8 + field] = (uint32_t)clock64();
+#endif
+}
+
+struct TileCtx {
+  uint32_t tl;          // TMEM address of this warp's lane quarter (column 0)
+  uint32_t mask_row;    // shared address of this row's 16 mask bytes
+  bool masked;          // the tile has a bitmask (else all columns valid)
+  uint32_t n;           // tile sequence number (CTA lifetime)
+  int j;                // tile index within the item
+  uint32_t s_free, pv_done, p_full;
+  float c, thresh;
+  const CoarseParams* prm;   // diagnostics only (tl_rec)
+};
+
+// One tile of the online SpSoftmax for this thread's row (NQ x 32 columns): read S(n) from TMEM
+// and release it, mask, row max, lazy rescale decision, then (after P.V(n-1)) rescale O if the
+// max moved and store P(n) = 2^(s*c - m*c) as packed 16-bit pairs, chunk by chunk.
+template <int NQ, bool kBF16>
+__device__ __forceinline__ void softmax_tile(const TileCtx& x, float& m, float& l) {
+  const uint32_t lane = threadIdx.x & 31;
+  uint32_t r[NQ][32];
+#pragma unroll
+  for (int q = 0; q < NQ; ++q) tmem_ld32(x.tl + kTS + q * 32, r[q]);
+  tmem_wait_ld();
+  tc_fence_before();
+  __syncwarp();
+  if (lane == 0) mbar_arrive(x.s_free);                 // S may be overwritten by S(n+1)
+  if (x.masked) {
+    const int4 mw = ld_shared_v4(x.mask_row);
+    const uint32_t w4[4] = {(uint32_t)mw.x, (uint32_t)mw.y, (uint32_t)mw.z, (uint32_t)mw.w};
+#pragma unroll
+    for (int q = 0; q < NQ; ++q) apply_mask(r[q], w4[q]);
+  }
+  float tmax = -INFINITY;
+#pragma unroll
+  for (int q = 0; q < NQ; ++q) tmax = chunk_max(r[q], tmax);
+  const bool need = tmax > m + x.thresh || (m == -INFINITY && tmax != -INFINITY);
+  float alpha = 1.f;
+  if (need) {
+    alpha = ex2((m - tmax) * x.c);                      // 0 when m = -inf
+    m = tmax;
+  }
+  l *= alpha;
+  const float mu = (m == -INFINITY) ? 0.f : m;
+  const float2 c2 = make_float2(x.c, x.c);
+  const float2 nb2 = make_float2(-mu * x.c, -mu * x.c);
+  float2 rs[2] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
+  // P.V(n-1) has consumed P(n-1) and updated O: rescale O if the max moved, then store P(n)
+  // chunk by chunk as it is produced (the other CTA on this SM keeps the pipes busy meanwhile)
+  if (x.n > 0) mbar_wait(x.pv_done, (x.n - 1) & 1);
+  if (threadIdx.x == 0) tl_rec(*x.prm, x.n, 1);
+  tc_fence_after();
+  if (x.j > 0 && __any_sync(0xffffffffu, need && alpha != 1.f)) {
+#pragma unroll 1
+    for (int h = 0; h < 4; ++h) {
+      uint32_t o[16];
+      tmem_ld16(x.tl + kTO + h * 16, o);
+      tmem_wait_ld();
+#pragma unroll
+      for (int i = 0; i < 16; ++i) o[i] = __float_as_uint(__uint_as_float(o[i]) * alpha);
+      tmem_st16(x.tl + kTO + h * 16, o);
+    }
+  }
+#pragma unroll
+  for (int q = 0; q < NQ; ++q) {
+    uint32_t pk[16];
+    chunk_exp<kBF16>(r[q], c2, nb2, rs, pk);
+    tmem_st16(x.tl + kTP + q * 16, pk);
+  }
+  l += (rs[0].x + rs[0].y) + (rs[1].x + rs[1].y);
+  tmem_wait_st();
+  tc_fence_before();
+  __syncwarp();
+  if (lane == 0) mbar_arrive(x.p_full);
+  if (threadIdx.x == 0) tl_rec(*x.prm, x.n, 2);
+}
+
+}  // namespace
+
+template <bool kBF16>
+__global__ void __launch_bounds__(kThreads, 2)
+    coarse_pp_kernel(const __grid_constant__ CUtensorMap tmq, const __grid_constant__ CUtensorMap tmk,
+                     const __grid_constant__ CUtensorMap tmv, const __grid_constant__ CUtensorMap tmq2,
+                     const __grid_constant__ CUtensorMap tmk2, const __grid_constant__ CUtensorMap tmv2,
+                     const CoarseParams p) {
+  extern __shared__ uint8_t smem_raw[];
+  const uint32_t sbase = (smem_u32(smem_raw) + 1023u) & ~1023u;
+  const uint32_t sQ = sbase;
+  const uint32_t sK = sQ + 2 * kTileBytes;
+  const uint32_t sV = sK + kSt * kTileBytes;
+  const uint32_t sMsk = sV + kSt * kTileBytes;            // [V stage] tile bitmasks
+  Ctl* ctl = reinterpret_cast<Ctl*>(smem_raw + (sMsk + kSt * kMaskBytes - smem_u32(smem_raw)));
+  const int warp = threadIdx.x >> 5;
+  const int lane = threadIdx.x & 31;
+  auto bar = [&](const uint64_t& b) { return smem_u32(&b); };
+
+  if (threadIdx.x == 0) {
+    for (int b = 0; b < kItems; ++b) {
+      mbar_init(bar(ctl->item_full[b]), 1);
+      mbar_init(bar(ctl->item_empty[b]), 2 + 4);   // producer + MMA thread + 4 softmax warps
+    }
+    for (int b = 0; b < 2; ++b) {
+      mbar_init(bar(ctl->q_full[b]), 1);
+      mbar_init(bar(ctl->q_empty[b]), 1);
+    }
+    for (int s = 0; s < kSt; ++s) {
+      mbar_init(bar(ctl->k_full[s]), 1);
+      mbar_init(bar(ctl->k_empty[s]), 1);
+      mbar_init(bar(ctl->v_full[s]), 1);
+      mbar_init(bar(ctl->v_empty[s]), 1);
+    }
+    mbar_init(bar(ctl->s_full), 1);
+    mbar_init(bar(ctl->s_free), 4);
+    mbar_init(bar(ctl->p_full), 4);
+    mbar_init(bar(ctl->pv_done), 1);
+    fence_barrier_init();
+  }
+  if (warp == 4 && lane == 0) {
+    prefetch_tmap(&tmq);
+    prefetch_tmap(&tmk);
+    prefetch_tmap(&tmv);
+    if (p.gather_tma) {
+      prefetch_tmap(&tmq2);
+      prefetch_tmap(&tmk2);
+      prefetch_tmap(&tmv2);
+    }
+  }
+  if (warp == 5) {
+    tmem_alloc(smem_u32(&ctl->tmem_base), kTmemCols);
+    tmem_relinquish();
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = ctl->tmem_base;
+
+  if (warp == 4) {
+    // ============================================================ producer
+    asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(kRegsCtl) : "memory");
+    const uint64_t pol_kv = policy_evict_last();   // K/V tiles are re-read by neighbouring items
+    const uint64_t pol_q = policy_evict_first();   // Q tiles are read once
+    uint32_t g = 0;
+    for (uint32_t it = 0;; ++it) {
+      const uint32_t slot = it % kItems;
+      mbar_wait(bar(ctl->item_full[slot]), (it / kItems) & 1);
+      const int u = ctl->slot[slot].u;
+      const Item item = ctl->slot[slot].item;
+      const int bh = ctl->slot[slot].bh;
+      __syncwarp();
+      if (lane == 0) mbar_arrive(bar(ctl->item_empty[slot]));
+      if (u >= p.total_units) break;
+      const int bb = bh / p.H, hh = bh % p.H;
+      const uint32_t qs = it & 1;
+      const uint32_t dQ = sQ + qs * kTileBytes;
+      const uint32_t qf = bar(ctl->q_full[qs]);
+      mbar_wait(bar(ctl->q_empty[qs]), ((it >> 1) & 1) ^ 1);
+      if (item.kind == 0) {
+        if (lane == 0) {
+          mbar_arrive_expect_tx(qf, kTileBytes);
+          tma_load_4d(dQ, &tmq, qf, 0, item.rowA, hh, bb, pol_q);
+        }
+      } else if (p.gather_tma) {
+        if (lane == 0) mbar_arrive_expect_tx(qf, kTileBytes);
+        __syncwarp();
+        const int4 ix = load_idx4(p.global_rows + item.rowA, 4 * lane, item.nrowsA);
+        gather4(dQ + lane * 512, &tmq2, qf, row_coords(ix, bb * p.rq.x + hh * p.rq.y, p.rq.z), pol_q);
+      } else {
+        gather_rows(dQ, p.q.data + bb * p.q.sb + hh * p.q.sh, p.q.sl, p.global_rows + item.rowA, item.nrowsA, 128,
+                    lane);
+        fence_proxy_async_smem();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(qf);
+      }
+      const int64_t krow0 = bb * p.rk.x + hh * p.rk.y, vrow0 = bb * p.rv.x + hh * p.rv.y;
+      for (int j0 = 0; j0 < item.ntiles; j0 += 32) {
+        // the item's tile references, 32 at a time (one per lane), broadcast per tile
+        int4 mine = make_int4(0, 0, 0, -1);
+        if (j0 + lane < item.ntiles) mine = __ldg(reinterpret_cast<const int4*>(p.trefs + item.tref_begin + j0 + lane));
+        const int nj = min(32, item.ntiles - j0);
+        for (int jj = 0; jj < nj; ++jj, ++g) {
+          const int arg = __shfl_sync(0xffffffffu, mine.x, jj), kind = __shfl_sync(0xffffffffu, mine.y, jj);
+          const int ncols = __shfl_sync(0xffffffffu, mine.z, jj), maskA = __shfl_sync(0xffffffffu, mine.w, jj);
+          const uint32_t st = g % kSt, sph = ((g / kSt) & 1) ^ 1;
+          const uint32_t dK = sK + st * kTileBytes, dV = sV + st * kTileBytes;
+          // strip tiles: the column indices of this lane's 4 gathered rows
+          int4 six = make_int4(-1, -1, -1, -1);
+          if (kind != 0 && p.gather_tma) six = load_idx4(p.strip_cols + arg, 4 * lane, ncols);
+          const uint32_t kf = bar(ctl->k_full[st]), vf = bar(ctl->v_full[st]);
+          mbar_wait(bar(ctl->k_empty[st]), sph);
+          if (lane == 0) {
+            ctl->kcols[st] = ncols;   // published by the k_full arrive
+            tl_rec(p, g, 5);
+          }
+          if (kind == 0) {
+            if (lane == 0) {
+              mbar_arrive_expect_tx(kf, kTileBytes);
+              tma_load_4d(dK, &tmk, kf, 0, arg, hh, bb, pol_kv);
+            }
+          } else if (p.gather_tma) {
+            if (lane == 0) mbar_arrive_expect_tx(kf, ncols * 128);
+            __syncwarp();
+            if (4 * lane < ncols) gather4(dK + lane * 512, &tmk2, kf, row_coords(six, krow0, p.rk.z), pol_kv);
+          } else {
+            gather_rows(dK, p.k.data + bb * p.k.sb + hh * p.k.sh, p.k.sl, p.strip_cols + arg, ncols, ncols, lane);
+            fence_proxy_async_smem();
+            __syncwarp();
+            if (lane == 0) mbar_arrive(kf);
+          }
+          mbar_wait(bar(ctl->v_empty[st]), sph);
+          const uint32_t mbytes = maskA >= 0 ? kMaskBytes : 0;
+          if (lane == 0) {
+            ctl->vdesc[st] = make_int2(ncols, maskA);   // published by the v_full arrive
+            tl_rec(p, g, 6);
+          }
+          if (kind == 0) {
+            if (lane == 0) {
+              mbar_arrive_expect_tx(vf, kTileBytes + mbytes);
+              tma_load_4d(dV, &tmv, vf, 0, arg, hh, bb, pol_kv);
+            }
+          } else if (p.gather_tma) {
+            if (lane == 0) mbar_arrive_expect_tx(vf, ncols * 128 + mbytes);
+            __syncwarp();
+            if (4 * lane < ncols) gather4(dV + lane * 512, &tmv2, vf, row_coords(six, vrow0, p.rv.z), pol_kv);
+          } else {
+            gather_rows(dV, p.v.data + bb * p.v.sb + hh * p.v.sh, p.v.sl, p.strip_cols + arg, ncols, ncols, lane);
+            fence_proxy_async_smem();
+            __syncwarp();
+            if (lane == 0) mbar_arrive_expect_tx(vf, mbytes);
+          }
+          if (lane == 0 && mbytes) bulk_load(sMsk + st * kMaskBytes, p.masks + (size_t)maskA * 256, kMaskBytes, vf);
+        }
+      }
+    }
+  } else if (warp == 6) {
+    // ============================================================ scheduler
+    asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(kRegsCtl) : "memory");
+    // Claims work items (dynamic counter) into a kItems-deep ring, i.e. up to kItems items ahead of
+    // the slowest consumer, and warms L2 with each band item's Q tile.
+    if (lane == 0) {
+      for (uint32_t it = 0;; ++it) {
+        const uint32_t slot = it % kItems;
+        mbar_wait(bar(ctl->item_empty[slot]), ((it / kItems) & 1) ^ 1);
+        const int u = atomicAdd(p.counter, 1);
+        Slot sl;
+        sl.u = u;
+        if (u < p.total_units) {
+          const UnitInfo ui = decode_unit(p, u);
+          sl.item = p.items[ui.item];
+          sl.bh = ui.bh;
+          if (sl.item.kind == 0) tma_prefetch_4d(&tmq, 0, sl.item.rowA, ui.bh % p.H, ui.bh / p.H);
+        }
+        ctl->slot[slot] = sl;
+        mbar_arrive(bar(ctl->item_full[slot]));
+        if (u >= p.total_units) break;
+      }
+    }
+    __syncwarp();
+  } else if (warp == 5) {
+    // ============================================================ MMA issuer (lane 0)
+    asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(kRegsCtl) : "memory");
+    if (lane == 0) {
+      // Tile sequence n = 0, 1, ... over the CTA's lifetime. Iteration n issues S(n) (after the
+      // softmax has read S(n-1)), then P.V(n-1) once its P is stored. P.V(n) of an item's first
+      // tile overwrites O (accumulate = 0): its P is stored only after the softmax warps have
+      // read the previous item's O in their epilogue, so no separate O barrier is needed.
+      const uint32_t idesc_pv = idesc_f16(kBF16, 128, 64, false, true);
+      uint32_t n = 0;
+      struct Pend {
+        uint32_t n, st;
+        int ncols;
+        bool first, valid;
+      } pend{0, 0, 0, false, false};
+      auto issue_pv = [&](const Pend& e) {
+        mbar_wait(bar(ctl->v_full[e.st]), (e.n / kSt) & 1);
+        mbar_wait(bar(ctl->p_full), e.n & 1);
+        tc_fence_after();
+        const uint32_t vA = sV + e.st * kTileBytes;
+        // chunk c (16 keys): P at columns [kTP + 8c, kTP + 8c + 8) (packed pairs), V rows [16c, 16c + 16)
+        for (int c = 0; c < (e.ncols >> 4); ++c)
+          mma_ts(tmem + kTO, tmem + kTP + c * 8, smem_desc_sw128(vA + c * 2048, 8192, 1024), idesc_pv,
+                 (e.first && c == 0) ? 0u : 1u);
+        mma_commit(bar(ctl->pv_done));
+        mma_commit(bar(ctl->v_empty[e.st]));
+        tl_rec(p, e.n, 4);
+      };
+      for (uint32_t it = 0;; ++it) {
+        const uint32_t slot = it % kItems;
+        mbar_wait(bar(ctl->item_full[slot]), (it / kItems) & 1);
+        const int u = ctl->slot[slot].u;
+        const int ntiles = ctl->slot[slot].item.ntiles;
+        mbar_arrive(bar(ctl->item_empty[slot]));
+        if (u >= p.total_units) break;
+        const uint32_t qs = it & 1;
+        // finish the previous item first unless this item's Q tile is already resident
+        if (pend.valid && !mbar_test_wait(bar(ctl->q_full[qs]), (it >> 1) & 1)) {
+          issue_pv(pend);
+          pend.valid = false;
+        }
+        mbar_wait(bar(ctl->q_full[qs]), (it >> 1) & 1);
+        const uint32_t qa = sQ + qs * kTileBytes;
+        for (int j = 0; j < ntiles; ++j, ++n) {
+          const uint32_t st = n % kSt;
+          mbar_wait(bar(ctl->k_full[st]), (n / kSt) & 1);
+          const int ncols = ctl->kcols[st];
+          if (n > 0) mbar_wait(bar(ctl->s_free), (n - 1) & 1);
+          tc_fence_after();
+          const uint32_t idesc_s = idesc_f16(kBF16, 128, ncols, false, false);
+          const uint32_t kA = sK + st * kTileBytes;
+#pragma unroll
+          for (int kk = 0; kk < 4; ++kk)
+            mma_ss(tmem + kTS, smem_desc_sw128(qa + kk * 32, 16, 1024), smem_desc_sw128(kA + kk * 32, 16, 1024),
+                   idesc_s, kk > 0);
+          mma_commit(bar(ctl->s_full));
+          mma_commit(bar(ctl->k_empty[st]));
+          tl_rec(p, n, 3);
+          if (j == ntiles - 1) mma_commit(bar(ctl->q_empty[qs]));
+          if (pend.valid) issue_pv(pend);
+          pend = Pend{n, st, ncols, j == 0, true};
+        }
+      }
+      if (pend.valid) issue_pv(pend);
+    }
+    __syncwarp();
+  } else if (warp == 7) {
+    asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(kRegsCtl) : "memory");
+  } else {
+    // ============================================================ softmax + epilogue
+    asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(kRegsSoftmax) : "memory");
+    const int t = warp * 32 + lane;                       // row of the Q tile = TMEM lane
+    const uint32_t tl = tmem + ((uint32_t)(warp * 32) << 16);
+    const float c = p.scale_log2;
+    // lazy rescaling (O accumulates in TMEM): the exponent keeps a stale row max m until a tile's
+    // max exceeds it by more than 2^8 in probability, so p <= 256 and O rarely needs a rescale
+    const float thresh = 8.f / c;
+    uint32_t n = 0;
+    for (uint32_t it = 0;; ++it) {
+      const uint32_t slot = it % kItems;
+      mbar_wait(bar(ctl->item_full[slot]), (it / kItems) & 1);
+      const int u = ctl->slot[slot].u;
+      const Item item = ctl->slot[slot].item;
+      const int ubh = ctl->slot[slot].bh;
+      __syncwarp();
+      if (lane == 0) mbar_arrive(bar(ctl->item_empty[slot]));
+      if (u >= p.total_units) break;
+      // epilogue metadata, loaded now so its latency hides behind the item's tiles
+      int r_out = -1, slot_f = -1;
+      if (t < item.nrowsA) {
+        r_out = item.kind == 0 ? item.rowA + t : __ldg(p.global_rows + item.rowA + t);
+        if (item.kind == 0) slot_f = __ldg(p.fine_slot + item.rowA + t);
+      }
+      float m = -INFINITY, l = 0.f;
+      for (int j = 0; j < item.ntiles; ++j, ++n) {
+        const uint32_t st = n % kSt;
+        mbar_wait(bar(ctl->s_full), n & 1);
+        // the tile's descriptor and bitmask travel with its V stage (freed only after P.V(n))
+        mbar_wait(bar(ctl->v_full[st]), (n / kSt) & 1);
+        tc_fence_after();
+        const int2 desc = ctl->vdesc[st];                 // {ncols, maskA}
+        const TileCtx tc{tl, sMsk + st * kMaskBytes + t * 16, desc.y >= 0, n, j, bar(ctl->s_free),
+                         bar(ctl->pv_done), bar(ctl->p_full), c, thresh, &p};
+        if (threadIdx.x == 0) tl_rec(p, n, 0);
+        switch (desc.x >> 5) {                            // 32-column chunks of the tile
+          case 4: softmax_tile<4, kBF16>(tc, m, l); break;
+          case 3: softmax_tile<3, kBF16>(tc, m, l); break;
+          case 2: softmax_tile<2, kBF16>(tc, m, l); break;
+          default: softmax_tile<1, kBF16>(tc, m, l); break;
+        }
+      }
+      // ---------------------------------------------------------------- epilogue (a-8)
+      float mf = -INFINITY, lf = 0.f;
+      const float4* accf = nullptr;
+      if (slot_f >= 0) {
+        const size_t idx = (size_t)ubh * p.n_fine_rows + slot_f;
+        const float2 ml = p.part_ml[idx];
+        mf = ml.x;
+        lf = ml.y;
+        accf = reinterpret_cast<const float4*>(p.part_acc + idx * 64);
+      }
+      const float mt = fmaxf(m, mf);
+      const float mu = mt == -INFINITY ? 0.f : mt;
+      const float ac = ex2((m - mu) * c), af = ex2((mf - mu) * c);
+      const float den = l * ac + lf * af;
+      mbar_wait(bar(ctl->pv_done), (n - 1) & 1);          // the item's last P.V
+      tc_fence_after();
+      uint32_t o[2][32];
+      tmem_ld32(tl + kTO, o[0]);
+      tmem_ld32(tl + kTO + 32, o[1]);
+      tmem_wait_ld();
+      tc_fence_before();
+      if (r_out >= 0 && mt != -INFINITY) {
+        const float inv = __frcp_rn(den);
+        const int bb = ubh / p.H, hh = ubh % p.H;
+        uint16_t* orow = p.o.data + bb * p.o.sb + hh * p.o.sh + (int64_t)r_out * p.o.sl;
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+#pragma unroll
+          for (int q8 = 0; q8 < 4; ++q8) {
+            float a[8];
+#pragma unroll
+            for (int i = 0; i < 8; ++i) a[i] = __uint_as_float(o[h][q8 * 8 + i]) * ac;
+            if (accf) {
+              const float4 f0 = accf[h * 8 + q8 * 2], f1 = accf[h * 8 + q8 * 2 + 1];
+              a[0] = fmaf(f0.x, af, a[0]);
+              a[1] = fmaf(f0.y, af, a[1]);
+              a[2] = fmaf(f0.z, af, a[2]);
+              a[3] = fmaf(f0.w, af, a[3]);
+              a[4] = fmaf(f1.x, af, a[4]);
+              a[5] = fmaf(f1.y, af, a[5]);
+              a[6] = fmaf(f1.z, af, a[6]);
+              a[7] = fmaf(f1.w, af, a[7]);
+            }
+            uint4 o4;
+            o4.x = pack2<kBF16>(a[0] * inv, a[1] * inv);
+            o4.y = pack2<kBF16>(a[2] * inv, a[3] * inv);
+            o4.z = pack2<kBF16>(a[4] * inv, a[5] * inv);
+            o4.w = pack2<kBF16>(a[6] * inv, a[7] * inv);
+            *reinterpret_cast<uint4*>(orow + h * 32 + q8 * 8) = o4;
+          }
+        }
+      }
+    }
+  }
+
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 5) tmem_dealloc(tmem, kTmemCols);
+}
+
+cudaError_t launch_coarse_pp(const CoarseParams& p, const CUtensorMap& tmq, const CUtensorMap& tmk,
+                             const CUtensorMap& tmv, const CUtensorMap& tmq2, const CUtensorMap& tmk2,
+                             const CUtensorMap& tmv2, bool bf16, int grid, cudaStream_t stream) {
+  auto kern = bf16 ? coarse_pp_kernel<true> : coarse_pp_kernel<false>;
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBytes);
+  if (e != cudaSuccess) return e;
+  kern<<<grid, kThreads, kSmemBytes, stream>>>(tmq, tmk, tmv, tmq2, tmk2, tmv2, p);
+  return cudaGetLastError();
+}
+
+}  // namespace mg

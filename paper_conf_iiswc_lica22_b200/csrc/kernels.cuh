@@ -36,6 +36,10 @@ struct CoarseParams {
   float scale_log2;           // (1/sqrt(d)) * log2(e)
   unsigned long long* trace;  // diagnostics: event trace of CTA 0 (null = off)
   int32_t trace_cap;
+  // 2-D [rows, 64] views for TMA row gathers (paired-pipeline kernel): row of (b, h, l) =
+  // b * r.x + h * r.y + l * r.z; gather_tma = 0 when the strides do not allow such a view
+  int32_t gather_tma;
+  longlong3 rq, rk, rv;
   int32_t debug_flags;        // diagnostics (env MG_DEBUG_FLAGS): 1 = no softmax arithmetic, 2 = no MMA, 4 = no loads,
                               // 16 = no S loads from TMEM, 64 = MMA ignores P-ready/O-free (timing only)
 };
@@ -54,6 +58,10 @@ struct FineParams {
 
 cudaError_t launch_coarse(const CoarseParams& p, const CUtensorMap& tmq, const CUtensorMap& tmk,
                           const CUtensorMap& tmv, bool bf16, int grid, cudaStream_t stream);
+// Paired-pipeline variant: two CTAs per SM (grid = 2 x SMs), see coarse_pp_sm100.cu.
+cudaError_t launch_coarse_pp(const CoarseParams& p, const CUtensorMap& tmq, const CUtensorMap& tmk,
+                             const CUtensorMap& tmv, const CUtensorMap& tmq2, const CUtensorMap& tmk2,
+                             const CUtensorMap& tmv2, bool bf16, int grid, cudaStream_t stream);
 cudaError_t launch_fine(const FineParams& p, bool bf16, cudaStream_t stream);
 cudaError_t launch_selftest_umma(int mode, const void* A, const void* B, float* D, cudaStream_t stream);
 

@@ -5,6 +5,7 @@
 
 #include <cuda.h>
 #include <cstdint>
+#include <cstdio>
 
 namespace mg {
 namespace ptx {
@@ -75,6 +76,19 @@ __device__ __forceinline__ bool mbar_try_wait_hint(uint32_t bar, uint32_t parity
 // Blocking wait for the phase with the given parity: the retry loop lives inside the asm (branch
 // on the predicate), which avoids the predicate -> register -> compare round trip of a C++ loop
 // (measured: ~51 vs ~101 cycles for an already-completed phase, tools/microbench/wait_lat.cu).
+#ifdef MG_WATCHDOG
+// Diagnostics build: a wait that has not completed after ~2^26 polls (about a second) reports the
+// barrier (shared-window offset) and parity, then traps.
+__device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
+  uint64_t spins = 0;
+  while (!mbar_test_wait(bar, parity)) {
+    if (++spins == (1ull << 26)) {
+      printf("MG_WATCHDOG block %d thread %d bar 0x%x parity %u\n", (int)blockIdx.x, (int)threadIdx.x, bar, parity);
+      asm volatile("trap;");
+    }
+  }
+}
+#else
 __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
   asm volatile(
       "{\n\t.reg .pred P;\n"
@@ -84,6 +98,7 @@ __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
       ::"r"(bar), "r"(parity)
       : "memory");
 }
+#endif
 
 // ------------------------------------------------------------------ TMA
 __device__ __forceinline__ void prefetch_tmap(const CUtensorMap* m) {
