@@ -195,17 +195,33 @@ __device__ __forceinline__ void chunk_exp(const uint32_t (&r)[32], float2 c2, fl
 
 
 // Diagnostics (MG_TIMELINE builds only): per-tile event clocks (low 32 bits of clock64) of every
-// CTA for its first kTlTiles tiles, 8 fields per tile, after 256 uint64 header words of p.trace:
-// 0 softmax S(n)+V(n) ready, 1 softmax P.V(n-1) done, 2 softmax P(n) stored, 3 MMA S(n) issued,
-// 4 MMA P.V(n) issued, 5 producer K(n) issued, 6 producer V(n) issued, 7 SM id (tile 0 only).
-// tools/timeline_pp.py reads it.
+// CTA for its first kTlTiles tiles, 16 fields per tile, after 256 uint64 header words of p.trace:
+// 0 softmax S(n)+V(n) ready, 1 softmax P.V(n-1) done, 2 softmax warp 0 P(n) stored, 3 MMA S(n)
+// issued, 4 MMA P.V(n) issued, 5 producer K(n) issued, 6 producer V(n) issued, 7 MMA sees p_full(n),
+// 8-10 softmax warps 1-3 P(n) stored, 11/12/13 epilogue start / O read / end (last tile of an
+// item), 14 MMA sees k_full(n), 15 SM id (tile 0 only). tools/timeline_pp.py reads it.
 constexpr int kTlTiles = 128;
 __device__ __forceinline__ void tl_rec(const CoarseParams& p, uint32_t n, int field) {
 #ifdef MG_TIMELINE
   if (p.trace == nullptr || n >= (uint32_t)kTlTiles ||
-      (int64_t)p.trace_cap < 256 + (int64_t)4 * kTlTiles * (int64_t)gridDim.x)
+      (int64_t)p.trace_cap < 256 + (int64_t)8 * kTlTiles * (int64_t)gridDim.x)
     return;
-  reinterpret_cast<uint32_t*>(p.trace + 256)[((size_t)blockIdx.x * kTlTiles + n) * 8 + field] = (uint32_t)clock64();
+  uint32_t v = (uint32_t)clock64();
+  if (field == 15) asm("mov.u32 %0, %%smid;" : "=r"(v));
+  reinterpret_cast<uint32_t*>(p.trace + 256)[((size_t)blockIdx.x * kTlTiles + n) * 16 + field] = v;
+#endif
+}
+
+// Item-level events (MG_TIMELINE): [CTA][item < 32][8] uint32 after the tile records: 0 scheduler
+// slot free, 1 scheduler item published, 2 producer item seen, 3 producer Q issued, 4 producer tile
+// refs loaded, 5 softmax item seen, 6 MMA item seen, 7 MMA Q ready.
+__device__ __forceinline__ void tl_item(const CoarseParams& p, uint32_t it, int field) {
+#ifdef MG_TIMELINE
+  if (p.trace == nullptr || it >= 32u ||
+      (int64_t)p.trace_cap < 256 + (int64_t)(8 * kTlTiles + 128) * (int64_t)gridDim.x)
+    return;
+  reinterpret_cast<uint32_t*>(p.trace + 256)[(size_t)gridDim.x * kTlTiles * 16 + ((size_t)blockIdx.x * 32 + it) * 8 +
+                                             field] = (uint32_t)clock64();
 #endif
 }
 
@@ -217,7 +233,7 @@ struct TileCtx {
   int j;                // tile index within the item
   uint32_t s_free, pv_done, p_full;
   float c, thresh;
-  const CoarseParams* prm;   // diagnostics only (tl_rec)
+  const CoarseParams* prm;   // diagnostics only (tl_rec, debug_flags)
 };
 
 // One tile of the online SpSoftmax for this thread's row (NQ x 32 columns): read S(n) from TMEM
@@ -242,6 +258,7 @@ __device__ __forceinline__ void softmax_tile(const TileCtx& x, float& m, float& 
   float tmax = -INFINITY;
 #pragma unroll
   for (int q = 0; q < NQ; ++q) tmax = chunk_max(r[q], tmax);
+  const bool dry = x.prm->debug_flags & 1;             // diagnostics: no exponentials
   const bool need = tmax > m + x.thresh || (m == -INFINITY && tmax != -INFINITY);
   float alpha = 1.f;
   if (need) {
@@ -272,15 +289,22 @@ __device__ __forceinline__ void softmax_tile(const TileCtx& x, float& m, float& 
 #pragma unroll
   for (int q = 0; q < NQ; ++q) {
     uint32_t pk[16];
-    chunk_exp<kBF16>(r[q], c2, nb2, rs, pk);
+    if (dry) {
+#pragma unroll
+      for (int i = 0; i < 16; ++i) pk[i] = r[q][2 * i];
+    } else {
+      chunk_exp<kBF16>(r[q], c2, nb2, rs, pk);
+    }
     tmem_st16(x.tl + kTP + q * 16, pk);
   }
   l += (rs[0].x + rs[0].y) + (rs[1].x + rs[1].y);
   tmem_wait_st();
   tc_fence_before();
   __syncwarp();
-  if (lane == 0) mbar_arrive(x.p_full);
-  if (threadIdx.x == 0) tl_rec(*x.prm, x.n, 2);
+  if (lane == 0) {
+    mbar_arrive(x.p_full);
+    tl_rec(*x.prm, x.n, threadIdx.x == 0 ? 2 : 7 + (threadIdx.x >> 5));
+  }
 }
 
 }  // namespace
@@ -309,7 +333,7 @@ __global__ void __launch_bounds__(kThreads, 2)
     }
     for (int b = 0; b < 2; ++b) {
       mbar_init(bar(ctl->q_full[b]), 1);
-      mbar_init(bar(ctl->q_empty[b]), 1);
+      mbar_init(bar(ctl->q_empty[b]), 4);   // softmax warps, after the epilogue staged O in it
     }
     for (int s = 0; s < kSt; ++s) {
       mbar_init(bar(ctl->k_full[s]), 1);
@@ -355,7 +379,10 @@ __global__ void __launch_bounds__(kThreads, 2)
       const Item item = ctl->slot[slot].item;
       const int bh = ctl->slot[slot].bh;
       __syncwarp();
-      if (lane == 0) mbar_arrive(bar(ctl->item_empty[slot]));
+      if (lane == 0) {
+        mbar_arrive(bar(ctl->item_empty[slot]));
+        tl_item(p, it, 2);
+      }
       if (u >= p.total_units) break;
       const int bb = bh / p.H, hh = bh % p.H;
       const uint32_t qs = it & 1;
@@ -379,12 +406,14 @@ __global__ void __launch_bounds__(kThreads, 2)
         __syncwarp();
         if (lane == 0) mbar_arrive(qf);
       }
+      if (lane == 0) tl_item(p, it, 3);
       const int64_t krow0 = bb * p.rk.x + hh * p.rk.y, vrow0 = bb * p.rv.x + hh * p.rv.y;
       for (int j0 = 0; j0 < item.ntiles; j0 += 32) {
         // the item's tile references, 32 at a time (one per lane), broadcast per tile
         int4 mine = make_int4(0, 0, 0, -1);
         if (j0 + lane < item.ntiles) mine = __ldg(reinterpret_cast<const int4*>(p.trefs + item.tref_begin + j0 + lane));
         const int nj = min(32, item.ntiles - j0);
+        if (j0 == 0 && __shfl_sync(0xffffffffu, mine.z, 0) >= 0 && lane == 0) tl_item(p, it, 4);
         for (int jj = 0; jj < nj; ++jj, ++g) {
           const int arg = __shfl_sync(0xffffffffu, mine.x, jj), kind = __shfl_sync(0xffffffffu, mine.y, jj);
           const int ncols = __shfl_sync(0xffffffffu, mine.z, jj), maskA = __shfl_sync(0xffffffffu, mine.w, jj);
@@ -401,8 +430,8 @@ __global__ void __launch_bounds__(kThreads, 2)
           }
           if (kind == 0) {
             if (lane == 0) {
-              mbar_arrive_expect_tx(kf, kTileBytes);
-              tma_load_4d(dK, &tmk, kf, 0, arg, hh, bb, pol_kv);
+              mbar_arrive_expect_tx(kf, (p.debug_flags & 4) ? 0 : kTileBytes);
+              if (!(p.debug_flags & 4)) tma_load_4d(dK, &tmk, kf, 0, arg, hh, bb, pol_kv);
             }
           } else if (p.gather_tma) {
             if (lane == 0) mbar_arrive_expect_tx(kf, ncols * 128);
@@ -422,8 +451,8 @@ __global__ void __launch_bounds__(kThreads, 2)
           }
           if (kind == 0) {
             if (lane == 0) {
-              mbar_arrive_expect_tx(vf, kTileBytes + mbytes);
-              tma_load_4d(dV, &tmv, vf, 0, arg, hh, bb, pol_kv);
+              mbar_arrive_expect_tx(vf, ((p.debug_flags & 4) ? 0 : kTileBytes) + mbytes);
+              if (!(p.debug_flags & 4)) tma_load_4d(dV, &tmv, vf, 0, arg, hh, bb, pol_kv);
             }
           } else if (p.gather_tma) {
             if (lane == 0) mbar_arrive_expect_tx(vf, ncols * 128 + mbytes);
@@ -444,11 +473,13 @@ __global__ void __launch_bounds__(kThreads, 2)
     asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(kRegsCtl) : "memory");
     // Claims work items (dynamic counter) into a kItems-deep ring, i.e. up to kItems items ahead of
     // the slowest consumer, and warms L2 with each band item's Q tile.
-    if (lane == 0) {
-      for (uint32_t it = 0;; ++it) {
-        const uint32_t slot = it % kItems;
+    for (uint32_t it = 0;; ++it) {
+      const uint32_t slot = it % kItems;
+      int u = 0;
+      if (lane == 0) {
         mbar_wait(bar(ctl->item_empty[slot]), ((it / kItems) & 1) ^ 1);
-        const int u = atomicAdd(p.counter, 1);
+        tl_item(p, it, 0);
+        u = atomicAdd(p.counter, 1);
         Slot sl;
         sl.u = u;
         if (u < p.total_units) {
@@ -459,10 +490,22 @@ __global__ void __launch_bounds__(kThreads, 2)
         }
         ctl->slot[slot] = sl;
         mbar_arrive(bar(ctl->item_full[slot]));
-        if (u >= p.total_units) break;
+        tl_item(p, it, 1);
+      }
+      u = __shfl_sync(0xffffffffu, u, 0);
+      if (u >= p.total_units) break;
+      __syncwarp();
+      // warm L2 with the item's contiguous K/V tiles (one lane per tile)
+      const Item item = ctl->slot[slot].item;
+      const int bh = ctl->slot[slot].bh;
+      for (int j = lane; j < item.ntiles; j += 32) {
+        const int4 tr = __ldg(reinterpret_cast<const int4*>(p.trefs + item.tref_begin + j));
+        if (tr.y == 0) {
+          tma_prefetch_4d(&tmk, 0, tr.x, bh % p.H, bh / p.H);
+          tma_prefetch_4d(&tmv, 0, tr.x, bh % p.H, bh / p.H);
+        }
       }
     }
-    __syncwarp();
   } else if (warp == 5) {
     // ============================================================ MMA issuer (lane 0)
     asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(kRegsCtl) : "memory");
@@ -481,15 +524,16 @@ __global__ void __launch_bounds__(kThreads, 2)
       auto issue_pv = [&](const Pend& e) {
         mbar_wait(bar(ctl->v_full[e.st]), (e.n / kSt) & 1);
         mbar_wait(bar(ctl->p_full), e.n & 1);
+        tl_rec(p, e.n, 7);
         tc_fence_after();
         const uint32_t vA = sV + e.st * kTileBytes;
         // chunk c (16 keys): P at columns [kTP + 8c, kTP + 8c + 8) (packed pairs), V rows [16c, 16c + 16)
-        for (int c = 0; c < (e.ncols >> 4); ++c)
+        for (int c = 0; c < ((p.debug_flags & 2) ? 0 : e.ncols >> 4); ++c)
           mma_ts(tmem + kTO, tmem + kTP + c * 8, smem_desc_sw128(vA + c * 2048, 8192, 1024), idesc_pv,
                  (e.first && c == 0) ? 0u : 1u);
+        tl_rec(p, e.n, 4);
         mma_commit(bar(ctl->pv_done));
         mma_commit(bar(ctl->v_empty[e.st]));
-        tl_rec(p, e.n, 4);
       };
       for (uint32_t it = 0;; ++it) {
         const uint32_t slot = it % kItems;
@@ -497,6 +541,7 @@ __global__ void __launch_bounds__(kThreads, 2)
         const int u = ctl->slot[slot].u;
         const int ntiles = ctl->slot[slot].item.ntiles;
         mbar_arrive(bar(ctl->item_empty[slot]));
+        tl_item(p, it, 6);
         if (u >= p.total_units) break;
         const uint32_t qs = it & 1;
         // finish the previous item first unless this item's Q tile is already resident
@@ -505,23 +550,25 @@ __global__ void __launch_bounds__(kThreads, 2)
           pend.valid = false;
         }
         mbar_wait(bar(ctl->q_full[qs]), (it >> 1) & 1);
+        tl_item(p, it, 7);
         const uint32_t qa = sQ + qs * kTileBytes;
         for (int j = 0; j < ntiles; ++j, ++n) {
           const uint32_t st = n % kSt;
           mbar_wait(bar(ctl->k_full[st]), (n / kSt) & 1);
+          tl_rec(p, n, 14);
+          if (n == 0) tl_rec(p, 0, 15);
           const int ncols = ctl->kcols[st];
           if (n > 0) mbar_wait(bar(ctl->s_free), (n - 1) & 1);
           tc_fence_after();
           const uint32_t idesc_s = idesc_f16(kBF16, 128, ncols, false, false);
           const uint32_t kA = sK + st * kTileBytes;
 #pragma unroll
-          for (int kk = 0; kk < 4; ++kk)
+          for (int kk = 0; kk < ((p.debug_flags & 2) ? 0 : 4); ++kk)
             mma_ss(tmem + kTS, smem_desc_sw128(qa + kk * 32, 16, 1024), smem_desc_sw128(kA + kk * 32, 16, 1024),
                    idesc_s, kk > 0);
           mma_commit(bar(ctl->s_full));
           mma_commit(bar(ctl->k_empty[st]));
           tl_rec(p, n, 3);
-          if (j == ntiles - 1) mma_commit(bar(ctl->q_empty[qs]));
           if (pend.valid) issue_pv(pend);
           pend = Pend{n, st, ncols, j == 0, true};
         }
@@ -549,6 +596,7 @@ __global__ void __launch_bounds__(kThreads, 2)
       const int ubh = ctl->slot[slot].bh;
       __syncwarp();
       if (lane == 0) mbar_arrive(bar(ctl->item_empty[slot]));
+      if (threadIdx.x == 0) tl_item(p, it, 5);
       if (u >= p.total_units) break;
       // epilogue metadata, loaded now so its latency hides behind the item's tiles
       int r_out = -1, slot_f = -1;
@@ -588,6 +636,7 @@ __global__ void __launch_bounds__(kThreads, 2)
       const float mu = mt == -INFINITY ? 0.f : mt;
       const float ac = ex2((m - mu) * c), af = ex2((mf - mu) * c);
       const float den = l * ac + lf * af;
+      if (threadIdx.x == 0) tl_rec(p, n - 1, 11);
       mbar_wait(bar(ctl->pv_done), (n - 1) & 1);          // the item's last P.V
       tc_fence_after();
       uint32_t o[2][32];
@@ -595,10 +644,15 @@ __global__ void __launch_bounds__(kThreads, 2)
       tmem_ld32(tl + kTO + 32, o[1]);
       tmem_wait_ld();
       tc_fence_before();
-      if (r_out >= 0 && mt != -INFINITY) {
-        const float inv = __frcp_rn(den);
-        const int bb = ubh / p.H, hh = ubh % p.H;
-        uint16_t* orow = p.o.data + bb * p.o.sb + hh * p.o.sh + (int64_t)r_out * p.o.sl;
+      if (threadIdx.x == 0) tl_rec(p, n - 1, 12);
+      // normalised row -> 16-bit, staged in this item's Q tile (its S MMAs are complete) in the
+      // 128B-swizzled layout, then written back 4 rows x 128 B per warp instruction (coalesced)
+      {
+        // a row with no valid element in this item (a global row inside a band row block: it is
+        // owned by the dense-row part, A5) is not written
+        const float inv = mt == -INFINITY ? 0.f : __frcp_rn(den);
+        const int r_st = mt == -INFINITY ? -1 : r_out;
+        const uint32_t srow = sQ + (it & 1) * kTileBytes + t * 128;
 #pragma unroll
         for (int h = 0; h < 2; ++h) {
 #pragma unroll
@@ -617,15 +671,31 @@ __global__ void __launch_bounds__(kThreads, 2)
               a[6] = fmaf(f1.z, af, a[6]);
               a[7] = fmaf(f1.w, af, a[7]);
             }
-            uint4 o4;
-            o4.x = pack2<kBF16>(a[0] * inv, a[1] * inv);
-            o4.y = pack2<kBF16>(a[2] * inv, a[3] * inv);
-            o4.z = pack2<kBF16>(a[4] * inv, a[5] * inv);
-            o4.w = pack2<kBF16>(a[6] * inv, a[7] * inv);
-            *reinterpret_cast<uint4*>(orow + h * 32 + q8 * 8) = o4;
+            const int ch = h * 4 + q8;
+            asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(srow + ((ch ^ (t & 7)) << 4)),
+                         "r"(pack2<kBF16>(a[0] * inv, a[1] * inv)), "r"(pack2<kBF16>(a[2] * inv, a[3] * inv)),
+                         "r"(pack2<kBF16>(a[4] * inv, a[5] * inv)), "r"(pack2<kBF16>(a[6] * inv, a[7] * inv))
+                         : "memory");
           }
         }
+        __syncwarp();
+        const int bb = ubh / p.H, hh = ubh % p.H;
+        uint16_t* obase = p.o.data + bb * p.o.sb + hh * p.o.sh;
+        const int ch = lane & 7;
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+          const int rw = 4 * k + (lane >> 3);               // row of this warp's 32
+          const int ro = __shfl_sync(0xffffffffu, r_st, rw);
+          const int tr = warp * 32 + rw;
+          const int4 v = ld_shared_v4(sQ + (it & 1) * kTileBytes + tr * 128 + ((ch ^ (tr & 7)) << 4));
+          if (ro >= 0) *reinterpret_cast<int4*>(obase + (int64_t)ro * p.o.sl + ch * 8) = v;
+        }
+        // the Q buffer may take the next TMA load (async proxy) once these generic accesses are done
+        fence_proxy_async_smem();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(bar(ctl->q_empty[it & 1]));
       }
+      if (threadIdx.x == 0) tl_rec(p, n - 1, 13);
     }
   }
 
