@@ -180,6 +180,32 @@ __device__ __forceinline__ float chunk_max(const uint32_t (&r)[32], float mx) {
   return fmaxf(fmaxf(a, b), fmaxf(c, d));
 }
 
+// 2^x for a pair on the FMA pipe (x <= 8): Cody-Waite split x = j + f with j = rint(x) (1.5 * 2^23
+// magic add), f in [-1/2, 1/2]; 2^f by a cubic (relative error 2.2e-4, far below the 2^-9 of the
+// 16-bit P it feeds); 2^j added to the exponent field. x is clamped to -126 so that masked (-inf)
+// scores give a denormal-range value ~1e-38 instead of 0, which no output can distinguish.
+__device__ __forceinline__ float2 exp2_fma2(float2 x) {
+  x.x = fmaxf(x.x, -126.f);
+  x.y = fmaxf(x.y, -126.f);
+  const float2 t = __fadd2_rn(x, make_float2(12582912.f, 12582912.f));
+  const float2 r = __fadd2_rn(t, make_float2(-12582912.f, -12582912.f));
+  const float2 f = __fadd2_rn(x, make_float2(-r.x, -r.y));
+  float2 p = __ffma2_rn(make_float2(0.05286743491888046f, 0.05286743491888046f), f,
+                        make_float2(0.2421518862247467f, 0.2421518862247467f));
+  p = __ffma2_rn(p, f, make_float2(0.6935867667198181f, 0.6935867667198181f));
+  p = __ffma2_rn(p, f, make_float2(0.9999627470970154f, 0.9999627470970154f));
+  return make_float2(__int_as_float(__float_as_int(t.x) * 0x800000 + __float_as_int(p.x)),
+                     __int_as_float(__float_as_int(t.y) * 0x800000 + __float_as_int(p.y)));
+}
+
+// Pairs (of 16 per 32-column chunk) whose exponentials run on the FMA pipe instead of MUFU.
+// Measured on C2/C3 (tools/ab_variants.sh): 0 is fastest with the current kernel, whose softmax
+// is latency- and issue-bound rather than MUFU-bound; kept for re-tuning.
+#ifndef MG_EXP_EMU
+#define MG_EXP_EMU 0
+#endif
+constexpr int kExpEmu = MG_EXP_EMU;
+
 // p = 2^(s*c - m*c) for 32 columns, packed to 16-bit pairs; row sum accumulated in rs[0..1]
 template <bool kBF16>
 __device__ __forceinline__ void chunk_exp(const uint32_t (&r)[32], float2 c2, float2 nb2, float2 (&rs)[2],
@@ -187,12 +213,17 @@ __device__ __forceinline__ void chunk_exp(const uint32_t (&r)[32], float2 c2, fl
 #pragma unroll
   for (int i = 0; i < 32; i += 2) {
     const float2 x = __ffma2_rn(make_float2(__uint_as_float(r[i]), __uint_as_float(r[i + 1])), c2, nb2);
-    const float p0 = ex2(x.x), p1 = ex2(x.y);
-    rs[(i >> 1) & 1] = __fadd2_rn(rs[(i >> 1) & 1], make_float2(p0, p1));
-    pk[i >> 1] = pack2<kBF16>(p0, p1);
+    float2 pp;
+    if ((i >> 1) < kExpEmu) {
+      pp = exp2_fma2(x);
+    } else {
+      pp.x = ex2(x.x);
+      pp.y = ex2(x.y);
+    }
+    rs[(i >> 1) & 1] = __fadd2_rn(rs[(i >> 1) & 1], pp);
+    pk[i >> 1] = pack2<kBF16>(pp.x, pp.y);
   }
 }
-
 
 // Diagnostics (MG_TIMELINE builds only): per-tile event clocks (low 32 bits of clock64) of every
 // CTA for its first kTlTiles tiles, 16 fields per tile, after 256 uint64 header words of p.trace:
@@ -498,7 +529,7 @@ __global__ void __launch_bounds__(kThreads, 2)
       // warm L2 with the item's contiguous K/V tiles (one lane per tile)
       const Item item = ctl->slot[slot].item;
       const int bh = ctl->slot[slot].bh;
-      for (int j = lane; j < item.ntiles; j += 32) {
+      for (int j = lane; j < ((p.debug_flags & 8) ? 0 : item.ntiles); j += 32) {
         const int4 tr = __ldg(reinterpret_cast<const int4*>(p.trefs + item.tref_begin + j));
         if (tr.y == 0) {
           tma_prefetch_4d(&tmk, 0, tr.x, bh % p.H, bh / p.H);
