@@ -20,7 +20,10 @@ LIB = os.path.join(PKG, "libmg.so")
 # diagnostics variants: libmg_<name>.so with the matching -D flags, loaded via MG_LIB_VARIANT=<name>
 VARIANTS = {"watchdog": ["-DMG_WATCHDOG"], "timeline": ["-DMG_TIMELINE"], "trace": ["-DMG_TRACE"],
             # A/B of the share of exponentials emulated on the FMA pipe (pairs of 16 per chunk)
-            "e0": ["-DMG_EXP_EMU=0"], "e4": ["-DMG_EXP_EMU=4"], "e8": ["-DMG_EXP_EMU=8"]}
+            "e0": ["-DMG_EXP_EMU=0"], "e4": ["-DMG_EXP_EMU=4"], "e8": ["-DMG_EXP_EMU=8"],
+            "maxpass": ["-DMG_SKIP_MAX=0"],
+            # skeleton cost: no exponentials / no MMAs / no loads (results are garbage)
+            "dbg1": ["-DMG_DBG=1"], "dbg3": ["-DMG_DBG=3"], "dbg7": ["-DMG_DBG=7"]}
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 
 SOURCES = ["plan.cpp", "api.cu", "coarse_sm100.cu", "coarse_pp_sm100.cu", "fine_rows.cu", "selftest_umma.cu"]

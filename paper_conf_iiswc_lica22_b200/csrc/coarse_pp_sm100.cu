@@ -206,6 +206,16 @@ __device__ __forceinline__ float2 exp2_fma2(float2 x) {
 #endif
 constexpr int kExpEmu = MG_EXP_EMU;
 
+// Diagnostics builds (MG_DBG=bits, results are garbage): 1 = no exponentials, 2 = no MMAs,
+// 4 = no K/V loads. Compile-time so that the measured build carries no runtime checks.
+#ifndef MG_DBG
+#define MG_DBG 0
+#endif
+constexpr bool kDbgNoExp = MG_DBG & 1, kDbgNoMma = MG_DBG & 2, kDbgNoLoads = MG_DBG & 4;
+#ifndef MG_SKIP_MAX
+#define MG_SKIP_MAX 1
+#endif
+
 // p = 2^(s*c - m*c) for 32 columns, packed to 16-bit pairs; row sum accumulated in rs[0..1]
 template <bool kBF16>
 __device__ __forceinline__ void chunk_exp(const uint32_t (&r)[32], float2 c2, float2 nb2, float2 (&rs)[2],
@@ -222,6 +232,24 @@ __device__ __forceinline__ void chunk_exp(const uint32_t (&r)[32], float2 c2, fl
     }
     rs[(i >> 1) & 1] = __fadd2_rn(rs[(i >> 1) & 1], pp);
     pk[i >> 1] = pack2<kBF16>(pp.x, pp.y);
+  }
+}
+
+// p = 2^(s*c - m*c) for 32 columns in place (fp32); row sum accumulated in rs[0..1]
+__device__ __forceinline__ void chunk_exp_f32(uint32_t (&r)[32], float2 c2, float2 nb2, float2 (&rs)[2]) {
+#pragma unroll
+  for (int i = 0; i < 32; i += 2) {
+    const float2 x = __ffma2_rn(make_float2(__uint_as_float(r[i]), __uint_as_float(r[i + 1])), c2, nb2);
+    float2 pp;
+    if ((i >> 1) < kExpEmu) {
+      pp = exp2_fma2(x);
+    } else {
+      pp.x = ex2(x.x);
+      pp.y = ex2(x.y);
+    }
+    rs[(i >> 1) & 1] = __fadd2_rn(rs[(i >> 1) & 1], pp);
+    r[i] = __float_as_uint(pp.x);
+    r[i + 1] = __float_as_uint(pp.y);
   }
 }
 
@@ -289,7 +317,6 @@ __device__ __forceinline__ void softmax_tile(const TileCtx& x, float& m, float& 
   float tmax = -INFINITY;
 #pragma unroll
   for (int q = 0; q < NQ; ++q) tmax = chunk_max(r[q], tmax);
-  const bool dry = x.prm->debug_flags & 1;             // diagnostics: no exponentials
   const bool need = tmax > m + x.thresh || (m == -INFINITY && tmax != -INFINITY);
   float alpha = 1.f;
   if (need) {
@@ -320,12 +347,7 @@ __device__ __forceinline__ void softmax_tile(const TileCtx& x, float& m, float& 
 #pragma unroll
   for (int q = 0; q < NQ; ++q) {
     uint32_t pk[16];
-    if (dry) {
-#pragma unroll
-      for (int i = 0; i < 16; ++i) pk[i] = r[q][2 * i];
-    } else {
-      chunk_exp<kBF16>(r[q], c2, nb2, rs, pk);
-    }
+    chunk_exp<kBF16>(r[q], c2, nb2, rs, pk);
     tmem_st16(x.tl + kTP + q * 16, pk);
   }
   l += (rs[0].x + rs[0].y) + (rs[1].x + rs[1].y);
@@ -364,7 +386,7 @@ __global__ void __launch_bounds__(kThreads, 2)
     }
     for (int b = 0; b < 2; ++b) {
       mbar_init(bar(ctl->q_full[b]), 1);
-      mbar_init(bar(ctl->q_empty[b]), 4);   // softmax warps, after the epilogue staged O in it
+      mbar_init(bar(ctl->q_empty[b]), 1);
     }
     for (int s = 0; s < kSt; ++s) {
       mbar_init(bar(ctl->k_full[s]), 1);
@@ -461,8 +483,8 @@ __global__ void __launch_bounds__(kThreads, 2)
           }
           if (kind == 0) {
             if (lane == 0) {
-              mbar_arrive_expect_tx(kf, (p.debug_flags & 4) ? 0 : kTileBytes);
-              if (!(p.debug_flags & 4)) tma_load_4d(dK, &tmk, kf, 0, arg, hh, bb, pol_kv);
+              mbar_arrive_expect_tx(kf, kDbgNoLoads ? 0 : kTileBytes);
+              if (!kDbgNoLoads) tma_load_4d(dK, &tmk, kf, 0, arg, hh, bb, pol_kv);
             }
           } else if (p.gather_tma) {
             if (lane == 0) mbar_arrive_expect_tx(kf, ncols * 128);
@@ -482,8 +504,8 @@ __global__ void __launch_bounds__(kThreads, 2)
           }
           if (kind == 0) {
             if (lane == 0) {
-              mbar_arrive_expect_tx(vf, ((p.debug_flags & 4) ? 0 : kTileBytes) + mbytes);
-              if (!(p.debug_flags & 4)) tma_load_4d(dV, &tmv, vf, 0, arg, hh, bb, pol_kv);
+              mbar_arrive_expect_tx(vf, (kDbgNoLoads ? 0 : kTileBytes) + mbytes);
+              if (!kDbgNoLoads) tma_load_4d(dV, &tmv, vf, 0, arg, hh, bb, pol_kv);
             }
           } else if (p.gather_tma) {
             if (lane == 0) mbar_arrive_expect_tx(vf, ncols * 128 + mbytes);
@@ -526,16 +548,6 @@ __global__ void __launch_bounds__(kThreads, 2)
       u = __shfl_sync(0xffffffffu, u, 0);
       if (u >= p.total_units) break;
       __syncwarp();
-      // warm L2 with the item's contiguous K/V tiles (one lane per tile)
-      const Item item = ctl->slot[slot].item;
-      const int bh = ctl->slot[slot].bh;
-      for (int j = lane; j < ((p.debug_flags & 8) ? 0 : item.ntiles); j += 32) {
-        const int4 tr = __ldg(reinterpret_cast<const int4*>(p.trefs + item.tref_begin + j));
-        if (tr.y == 0) {
-          tma_prefetch_4d(&tmk, 0, tr.x, bh % p.H, bh / p.H);
-          tma_prefetch_4d(&tmv, 0, tr.x, bh % p.H, bh / p.H);
-        }
-      }
     }
   } else if (warp == 5) {
     // ============================================================ MMA issuer (lane 0)
@@ -559,7 +571,7 @@ __global__ void __launch_bounds__(kThreads, 2)
         tc_fence_after();
         const uint32_t vA = sV + e.st * kTileBytes;
         // chunk c (16 keys): P at columns [kTP + 8c, kTP + 8c + 8) (packed pairs), V rows [16c, 16c + 16)
-        for (int c = 0; c < ((p.debug_flags & 2) ? 0 : e.ncols >> 4); ++c)
+        for (int c = 0; c < (kDbgNoMma ? 0 : e.ncols >> 4); ++c)
           mma_ts(tmem + kTO, tmem + kTP + c * 8, smem_desc_sw128(vA + c * 2048, 8192, 1024), idesc_pv,
                  (e.first && c == 0) ? 0u : 1u);
         tl_rec(p, e.n, 4);
@@ -594,11 +606,12 @@ __global__ void __launch_bounds__(kThreads, 2)
           const uint32_t idesc_s = idesc_f16(kBF16, 128, ncols, false, false);
           const uint32_t kA = sK + st * kTileBytes;
 #pragma unroll
-          for (int kk = 0; kk < ((p.debug_flags & 2) ? 0 : 4); ++kk)
+          for (int kk = 0; kk < (kDbgNoMma ? 0 : 4); ++kk)
             mma_ss(tmem + kTS, smem_desc_sw128(qa + kk * 32, 16, 1024), smem_desc_sw128(kA + kk * 32, 16, 1024),
                    idesc_s, kk > 0);
           mma_commit(bar(ctl->s_full));
           mma_commit(bar(ctl->k_empty[st]));
+          if (j == ntiles - 1) mma_commit(bar(ctl->q_empty[qs]));   // last S of the item
           tl_rec(p, n, 3);
           if (pend.valid) issue_pv(pend);
           pend = Pend{n, st, ncols, j == 0, true};
@@ -676,14 +689,14 @@ __global__ void __launch_bounds__(kThreads, 2)
       tmem_wait_ld();
       tc_fence_before();
       if (threadIdx.x == 0) tl_rec(p, n - 1, 12);
-      // normalised row -> 16-bit, staged in this item's Q tile (its S MMAs are complete) in the
-      // 128B-swizzled layout, then written back 4 rows x 128 B per warp instruction (coalesced)
-      {
-        // a row with no valid element in this item (a global row inside a band row block: it is
-        // owned by the dense-row part, A5) is not written
-        const float inv = mt == -INFINITY ? 0.f : __frcp_rn(den);
-        const int r_st = mt == -INFINITY ? -1 : r_out;
-        const uint32_t srow = sQ + (it & 1) * kTileBytes + t * 128;
+      // normalised row -> 16-bit, 8 x 16-byte stores of this thread's row. A row with no valid
+      // element in this item (a global row inside a band row block: it is owned by the dense-row
+      // part, A5) is not written. (Staging the tile through shared memory for 4-rows-per-
+      // instruction stores measured 10% slower: tools/experiments/.)
+      if (r_out >= 0 && mt != -INFINITY) {
+        const float inv = __frcp_rn(den);
+        const int bb = ubh / p.H, hh = ubh % p.H;
+        uint16_t* orow = p.o.data + bb * p.o.sb + hh * p.o.sh + (int64_t)r_out * p.o.sl;
 #pragma unroll
         for (int h = 0; h < 2; ++h) {
 #pragma unroll
@@ -702,29 +715,14 @@ __global__ void __launch_bounds__(kThreads, 2)
               a[6] = fmaf(f1.z, af, a[6]);
               a[7] = fmaf(f1.w, af, a[7]);
             }
-            const int ch = h * 4 + q8;
-            asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(srow + ((ch ^ (t & 7)) << 4)),
-                         "r"(pack2<kBF16>(a[0] * inv, a[1] * inv)), "r"(pack2<kBF16>(a[2] * inv, a[3] * inv)),
-                         "r"(pack2<kBF16>(a[4] * inv, a[5] * inv)), "r"(pack2<kBF16>(a[6] * inv, a[7] * inv))
-                         : "memory");
+            uint4 o4;
+            o4.x = pack2<kBF16>(a[0] * inv, a[1] * inv);
+            o4.y = pack2<kBF16>(a[2] * inv, a[3] * inv);
+            o4.z = pack2<kBF16>(a[4] * inv, a[5] * inv);
+            o4.w = pack2<kBF16>(a[6] * inv, a[7] * inv);
+            *reinterpret_cast<uint4*>(orow + h * 32 + q8 * 8) = o4;
           }
         }
-        __syncwarp();
-        const int bb = ubh / p.H, hh = ubh % p.H;
-        uint16_t* obase = p.o.data + bb * p.o.sb + hh * p.o.sh;
-        const int ch = lane & 7;
-#pragma unroll
-        for (int k = 0; k < 8; ++k) {
-          const int rw = 4 * k + (lane >> 3);               // row of this warp's 32
-          const int ro = __shfl_sync(0xffffffffu, r_st, rw);
-          const int tr = warp * 32 + rw;
-          const int4 v = ld_shared_v4(sQ + (it & 1) * kTileBytes + tr * 128 + ((ch ^ (tr & 7)) << 4));
-          if (ro >= 0) *reinterpret_cast<int4*>(obase + (int64_t)ro * p.o.sl + ch * 8) = v;
-        }
-        // the Q buffer may take the next TMA load (async proxy) once these generic accesses are done
-        fence_proxy_async_smem();
-        __syncwarp();
-        if (lane == 0) mbar_arrive(bar(ctl->q_empty[it & 1]));
       }
       if (threadIdx.x == 0) tl_rec(p, n - 1, 13);
     }
