@@ -52,6 +52,6 @@ for W in ("C2", "C4"):
     src = os.path.join(OUT, f"launches_{W}.csv")
     if not os.path.exists(src):
         continue
-    rows = [l for l in open(src) if l.startswith('"ID"') or "mg::" in l or "coarse_kernel" in l or "fine_rows" in l]
+    rows = [l for l in open(src) if l.startswith('"ID"') or "mg::" in l or "coarse" in l or "fine_rows" in l]
     open(os.path.join(PROF, f"{tag}_launches_{W}.csv"), "w").writelines(rows)
 print("written", sorted(os.listdir(PROF)))
