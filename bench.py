@@ -44,6 +44,8 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-flush", action="store_true")
     ap.add_argument("--strip-max-cols", type=int, default=0)
+    ap.add_argument("--fine-kernel", type=int, default=0, choices=[0, 1],
+                    help="CSR rows: 0 = warp-level tensor-core kernel, 1 = CUDA-core kernel (A/B)")
     return ap.parse_args()
 
 
@@ -234,7 +236,7 @@ def main():
 
     cfg = get_config(args.workload)
     plan = mg.Plan(cfg.L, cfg.H, cfg.d, cfg.window, cfg.global_idx, cfg.extra_idx,
-                   strip_max_cols=args.strip_max_cols)
+                   strip_max_cols=args.strip_max_cols, fine_kernel=args.fine_kernel)
     info = plan.info()
     BH = cfg.B * cfg.H
     useful = 4.0 * info["nnz_total"] * cfg.d * BH

@@ -110,7 +110,9 @@ typedef struct {
   int32_t strip_max_cols; /* max gathered columns per row block for the tensor-core strip path of
                              the CSR residual; 0 -> default (128); -1 disables the strip path */
   int32_t num_sms;        /* persistent grid size override; 0 -> device SM count */
-  int32_t reserved[4];
+  int32_t fine_kernel;    /* CSR rows outside strip tiles: 0 -> warp-level tensor-core kernel
+                             (mma.sync, default), 1 -> CUDA-core shuffle-reduction kernel (A/B) */
+  int32_t reserved[3];
 } mg_plan_opts;
 
 MG_API mg_status mg_plan_create_ex(int64_t L, int32_t heads, int32_t d, int32_t window,
@@ -167,7 +169,7 @@ MG_API mg_status mg_plan_export(mg_plan_t plan, int32_t* bsr_row_ptr, int32_t* b
  * so one plan must not be used by two concurrent forwards on different streams.
  * Errors: INVALID_ARG (null, shape/dtype mismatch with the plan or between tensors,
  * head_dim stride != 1, misaligned data or strides), UNSUPPORTED (block != 128,
- * dtypes that differ), CUDA.
+ * dtypes that differ, (L - 1) * stride_l of K or V >= 2^32 elements), CUDA.
  * ---------------------------------------------------------------------------------- */
 MG_API mg_status mg_sparse_attention_fwd(mg_plan_t plan, const mg_tensor* Q, const mg_tensor* K,
                                   const mg_tensor* V, mg_tensor* O, void* stream);

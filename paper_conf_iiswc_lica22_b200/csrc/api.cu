@@ -48,6 +48,7 @@ struct mg_plan_s {
   bool uploaded = false;
   int num_sms = 0;
   int num_sms_override = 0;
+  int fine_kernel = 0;   // 0: mma.sync kernel (fine_mma.cu), 1: CUDA-core kernel (fine_rows.cu)
   std::vector<void*> allocs;
   mg::Item* d_items = nullptr;
   mg::TileRef* d_trefs = nullptr;
@@ -135,7 +136,7 @@ mg_status create_impl(int64_t L, int32_t heads, int32_t d, int32_t window, const
   if (!plan_out) return fail(MG_ERR_INVALID_ARG, "plan_out is null");
   *plan_out = nullptr;
   mg::PlanOptions po;
-  int sms_override = 0;
+  int sms_override = 0, fine_kernel = 0;
   if (opts) {
     if (opts->block != 0) po.block = opts->block;
     po.force_all_fine = opts->force_all_fine != 0;
@@ -143,6 +144,8 @@ mg_status create_impl(int64_t L, int32_t heads, int32_t d, int32_t window, const
     if (po.strip_max_cols > 128) return fail(MG_ERR_INVALID_ARG, "strip_max_cols must be <= 128");
     if (opts->num_sms < 0) return fail(MG_ERR_INVALID_ARG, "num_sms must be >= 0");
     sms_override = opts->num_sms;
+    if (opts->fine_kernel < 0 || opts->fine_kernel > 1) return fail(MG_ERR_INVALID_ARG, "fine_kernel must be 0 or 1");
+    fine_kernel = opts->fine_kernel;
   }
   mg_plan_s* p = new (std::nothrow) mg_plan_s();
   if (!p) return fail(MG_ERR_OUT_OF_MEMORY, "host allocation failed");
@@ -162,6 +165,7 @@ mg_status create_impl(int64_t L, int32_t heads, int32_t d, int32_t window, const
     return fail(unsupported ? MG_ERR_UNSUPPORTED : MG_ERR_INVALID_ARG, err);
   }
   p->num_sms_override = sms_override;
+  p->fine_kernel = fine_kernel;
   int ndev = 0;
   if (cudaGetDeviceCount(&ndev) != cudaSuccess) {
     ndev = 0;
@@ -214,6 +218,9 @@ mg_status check_all(const mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, 
   if (!p->hp.kernel_ready) return fail(MG_ERR_UNSUPPORTED, "the forward requires block == 128");
   if ((int64_t)Q->batch * p->hp.heads >= (int64_t(1) << 31) / std::max<int64_t>(1, (int64_t)p->hp.items.size()))
     return fail(MG_ERR_UNSUPPORTED, "batch * heads * work items exceeds int32");
+  // the fine kernels address a gathered row as (uint32) col * stride_l elements
+  if ((p->hp.L - 1) * std::max(K->stride_l, V->stride_l) >= (int64_t(1) << 32))
+    return fail(MG_ERR_UNSUPPORTED, "(L - 1) * stride_l exceeds 2^32 elements");
   return MG_OK;
 }
 
@@ -315,7 +322,8 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
     fp.q = view(Q); fp.k = view(K); fp.v = view(V); fp.o = view(O);
     fp.H = h.heads; fp.BH = BH; fp.n_fine_rows = nf;
     fp.scale_log2 = scale_log2;
-    if ((e = mg::launch_fine(fp, bf16, stream)) != cudaSuccess) return cuda_fail(e, "fine kernel launch");
+    e = p->fine_kernel == 1 ? mg::launch_fine(fp, bf16, stream) : mg::launch_fine_mma(fp, bf16, stream);
+    if (e != cudaSuccess) return cuda_fail(e, "fine kernel launch");
   }
   if (p->profiling) cudaEventRecord(ev[1], stream);
   if (!h.items.empty()) {

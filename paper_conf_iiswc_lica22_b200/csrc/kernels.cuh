@@ -63,6 +63,8 @@ cudaError_t launch_coarse_pp(const CoarseParams& p, const CUtensorMap& tmq, cons
                              const CUtensorMap& tmv, const CUtensorMap& tmq2, const CUtensorMap& tmk2,
                              const CUtensorMap& tmv2, bool bf16, int grid, cudaStream_t stream);
 cudaError_t launch_fine(const FineParams& p, bool bf16, cudaStream_t stream);
+// Warp-level tensor-core variant (mma.sync m16n8k16), the default; see fine_mma.cu.
+cudaError_t launch_fine_mma(const FineParams& p, bool bf16, cudaStream_t stream);
 cudaError_t launch_selftest_umma(int mode, const void* A, const void* B, float* D, cudaStream_t stream);
 
 }  // namespace mg

@@ -49,6 +49,58 @@ __global__ void __launch_bounds__(256) gather(const uint16_t* K, const uint16_t*
   if (acc == 0x12345678) out[gw] = acc;
 }
 
+// same gathers through cp.async.cg into a warp-private shared-memory ring (NS stages), lane-private
+// chunks read back with ld.shared after cp.async.wait_group
+template <int LPR, int NS>
+__global__ void __launch_bounds__(128) gather_cpasync(const uint16_t* K, const uint16_t* V, const int* cols, int* out) {
+  extern __shared__ __align__(16) uint8_t sm[];
+  const int lane = threadIdx.x & 31;
+  const int gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  if (gw >= BH * L) return;
+  const int bh = gw / L, r = gw % L;
+  const uint16_t* Kb = K + (size_t)bh * L * D;
+  const uint16_t* Vb = V + (size_t)bh * L * D;
+  const int* c = cols + (size_t)r * NNZ;
+  constexpr int RPI = 32 / LPR, V4 = 8 / LPR;
+  constexpr int CH = 2 * V4 * (32 / RPI) / 4;   // 16-byte chunks per lane per quarter-window (8 rows)
+  const int sub = lane / LPR, part = lane % LPR;
+  const uint32_t ring = (uint32_t)__cvta_generic_to_shared(sm) + (threadIdx.x >> 5) * NS * CH * 512 + lane * 16;
+  int acc = 0;
+  // a "step" = 8 rows of the 32-index window
+  const int nsteps = (NNZ + 7) / 8;
+  auto issue = [&](int s) {
+    if (s < nsteps) {
+      const int idx = s * 8 + (lane & 7);
+      const int col = idx < NNZ ? __ldg(c + idx) : 0;
+      const uint32_t dst = ring + (s % NS) * CH * 512;
+      int k = 0;
+#pragma unroll
+      for (int q = 0; q < 8 / RPI; ++q) {
+        const int cc = __shfl_sync(0xffffffffu, col, q * RPI + sub);
+#pragma unroll
+        for (int u = 0; u < V4; ++u) {
+          asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dst + (k++) * 512), "l"(Kb + (size_t)cc * D + part * (8 * V4) + u * 8) : "memory");
+          asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dst + (k++) * 512), "l"(Vb + (size_t)cc * D + part * (8 * V4) + u * 8) : "memory");
+        }
+      }
+    }
+    asm volatile("cp.async.commit_group;" ::: "memory");
+  };
+  for (int s = 0; s < NS - 1; ++s) issue(s);
+  for (int s = 0; s < nsteps; ++s) {
+    issue(s + NS - 1);
+    asm volatile("cp.async.wait_group %0;" ::"n"(NS - 1) : "memory");
+    const uint32_t src = ring + (s % NS) * CH * 512;
+#pragma unroll
+    for (int k = 0; k < CH; ++k) {
+      int4 v;
+      asm volatile("ld.shared.v4.s32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(src + k * 512));
+      acc ^= v.x ^ v.y ^ v.z ^ v.w;
+    }
+  }
+  if (acc == 0x12345678) out[gw] = acc;
+}
+
 __global__ void mma_rate(float* out, int iters) {
   uint32_t a0 = threadIdx.x, a1 = a0 * 3, a2 = a0 * 5, a3 = a0 * 7, b0 = a0 ^ 9, b1 = a0 ^ 11;
   float c[8][4] = {};
@@ -101,6 +153,27 @@ int main() {
   run(gather<4>, "4 lanes/row (32 B each)");
   run(gather<2>, "2 lanes/row (64 B each)");
   run(gather<1>, "1 lane/row (128 B each)");
+  auto runc = [&](auto kern, int ns, int lpr, const char* name) {
+    const int CH = 2 * (8 / lpr) * (lpr * 8 / 32 > 0 ? lpr * 8 / 32 : 1) ;
+    const int smem = 4 * ns * 4 * 512;   // 4 warps x NS stages x 4 chunks x 512 B
+    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    const int blocks = BH * L / 4;
+    for (int i = 0; i < 3; ++i) kern<<<blocks, 128, smem>>>(K, V, cols, out);
+    cudaEventRecord(e0);
+    for (int i = 0; i < 10; ++i) kern<<<blocks, 128, smem>>>(K, V, cols, out);
+    cudaEventRecord(e1);
+    cudaEventSynchronize(e1);
+    float ms;
+    cudaEventElapsedTime(&ms, e0, e1);
+    ms /= 10;
+    (void)CH;
+    printf("%-28s %.3f ms  %.0f GB/s gathered (%s, smem %d)\n", name, ms, bytes / ms / 1e6,
+           cudaGetErrorString(cudaGetLastError()), smem);
+  };
+  runc(gather_cpasync<8, 2>, 2, 8, "cp.async 8 lanes/row NS=2");
+  runc(gather_cpasync<8, 4>, 4, 8, "cp.async 8 lanes/row NS=4");
+  runc(gather_cpasync<4, 4>, 4, 4, "cp.async 4 lanes/row NS=4");
+  runc(gather_cpasync<8, 8>, 8, 8, "cp.async 8 lanes/row NS=8");
   float* f;
   cudaMalloc(&f, 64);
   for (int warps = 4; warps <= 32; warps *= 2) {
