@@ -182,6 +182,49 @@ MG_API mg_status mg_sparse_attention_fwd_host(mg_plan_t plan, const mg_tensor* Q
                                        const mg_tensor* V, mg_tensor* O, void* stream);
 
 /* ------------------------------------------------------------------------------------
+ * Staged forward ("paper dataflow"): the steps of the method as separate calls with
+ * the scores S and probabilities P materialised in the plan's formats, so that each step can be
+ * checked on its own and the fused forward can be compared with the paper's dataflow. Same
+ * result as mg_sparse_attention_fwd (within the tolerance; P is rounded to 16 bits here).
+ *
+ * Formats, per (batch, head) unit u = b * heads + h, all row-major device arrays:
+ *   S_tiles  float  [B*H][n_tiles][128][128]  coarse scores Q_I K_J^T / sqrt(d) of each BSR tile
+ *            (BSR order of mg_plan_export), -inf where the canonical tile bit is 0      (a-2)
+ *   S_csr    float  [B*H][nnz_fine]           CSR residual scores, canonical CSR order   (a-3)
+ *   S_global float  [B*H][n_global][Lpad]     dense-row scores, -inf at columns >= L     (a-4)
+ *   P_tiles / P_csr / P_global: the same shapes in the tensor dtype (bf16 / fp16, RNE):
+ *            the compound SpSoftmax of each row over its tiles and CSR elements (global rows:
+ *            over their dense row), three sweeps max / sum / normalise as in P:128-131  (a-5)
+ *   O_csr    float  [B*H][L][64]              sum_c P(r,c) V[c] over each row's CSR part (a-6);
+ *            rows without CSR elements are not written
+ *   O        the caller's output tensor: sum_J P_IJ V_J + O_csr (global rows: P_g V)  (a-7, a-8)
+ * with Lpad = 128 * ceil(L / 128). mg_staged_get_sizes returns the per-unit element counts
+ * (a zero-size part may be passed as NULL). Requires block == 128. All calls are asynchronous
+ * on `stream`; buffers belong to the caller. Errors: INVALID_ARG (null plan / tensors / a
+ * required buffer, shape mismatch), UNSUPPORTED (block != 128), CUDA.
+ * mg_sparse_attention_fwd_staged runs the three calls with plan-owned buffers (grown
+ * stream-ordered like the fused forward's workspace).
+ * ---------------------------------------------------------------------------------- */
+typedef struct {
+  int64_t tile_elems;    /* n_tiles * 128 * 128 */
+  int64_t csr_elems;     /* nnz_fine */
+  int64_t global_elems;  /* n_global * Lpad */
+  int64_t ocsr_elems;    /* L * 64 */
+  int64_t lpad;
+} mg_staged_sizes;
+
+MG_API mg_status mg_staged_get_sizes(mg_plan_t plan, mg_staged_sizes* out);
+MG_API mg_status mg_staged_sddmm(mg_plan_t plan, const mg_tensor* Q, const mg_tensor* K, float* S_tiles,
+                                 float* S_csr, float* S_global, void* stream);
+MG_API mg_status mg_staged_softmax(mg_plan_t plan, int64_t batch, mg_dtype dtype, const float* S_tiles,
+                                   const float* S_csr, const float* S_global, void* P_tiles, void* P_csr,
+                                   void* P_global, void* stream);
+MG_API mg_status mg_staged_spmm(mg_plan_t plan, const void* P_tiles, const void* P_csr, const void* P_global,
+                                const mg_tensor* V, mg_tensor* O, float* O_csr, void* stream);
+MG_API mg_status mg_sparse_attention_fwd_staged(mg_plan_t plan, const mg_tensor* Q, const mg_tensor* K,
+                                                const mg_tensor* V, mg_tensor* O, void* stream);
+
+/* ------------------------------------------------------------------------------------
  * Profiling (tracing subsystem). When enabled, every forward records CUDA events on its
  * stream around each kernel it launches; mg_plan_get_profile() synchronises on the recorded
  * events, returns the summed device durations since the last enable/reset, and resets.

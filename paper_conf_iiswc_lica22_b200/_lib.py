@@ -18,6 +18,7 @@ EXPORTED = [
     "mg_plan_create", "mg_plan_create_ex", "mg_plan_destroy", "mg_last_error", "mg_plan_info_get",
     "mg_plan_export", "mg_sparse_attention_fwd", "mg_sparse_attention_fwd_host", "mg_selftest_umma",
     "mg_abi_version", "mg_plan_set_profiling", "mg_plan_get_profile", "mg_plan_set_trace",
+    "mg_staged_get_sizes", "mg_staged_sddmm", "mg_staged_softmax", "mg_staged_spmm", "mg_sparse_attention_fwd_staged",
 ]
 
 
@@ -44,6 +45,11 @@ class mg_plan_info(C.Structure):
 
 class mg_profile(C.Structure):
     _fields_ = [("calls", C.c_int64), ("fine_ms", C.c_double), ("coarse_ms", C.c_double), ("total_ms", C.c_double)]
+
+
+class mg_staged_sizes(C.Structure):
+    _fields_ = [("tile_elems", C.c_int64), ("csr_elems", C.c_int64), ("global_elems", C.c_int64),
+                ("ocsr_elems", C.c_int64), ("lpad", C.c_int64)]
 
 
 _lib = None
@@ -76,6 +82,11 @@ def load() -> C.CDLL:
     lib.mg_plan_set_profiling.argtypes = [P, C.c_int32]
     lib.mg_plan_get_profile.argtypes = [P, C.POINTER(mg_profile)]
     lib.mg_plan_set_trace.argtypes = [P, P, C.c_int64]
+    lib.mg_staged_get_sizes.argtypes = [P, C.POINTER(mg_staged_sizes)]
+    lib.mg_staged_sddmm.argtypes = [P, tp, tp, P, P, P, P]
+    lib.mg_staged_softmax.argtypes = [P, C.c_int64, C.c_int32, P, P, P, P, P, P, P]
+    lib.mg_staged_spmm.argtypes = [P, P, P, P, tp, tp, P, P]
+    lib.mg_sparse_attention_fwd_staged.argtypes = [P, tp, tp, tp, tp, P]
     lib.mg_abi_version.restype = C.c_int32
     lib.mg_abi_version.argtypes = []
     for name in EXPORTED:

@@ -145,6 +145,66 @@ def sparse_attention_fwd_host(plan: Plan, Q, K, V, O, stream=None):
     return O
 
 
+def staged_sizes(plan: Plan) -> dict:
+    """mg_staged_get_sizes: per-(batch, head) element counts of the staged buffers."""
+    z = _lib.mg_staged_sizes()
+    check(plan._lib.mg_staged_get_sizes(plan.handle, C.byref(z)))
+    return {name: getattr(z, name) for name, _ in z._fields_}
+
+
+def _ptr(t):
+    return None if t is None or t.numel() == 0 else C.c_void_p(t.data_ptr())
+
+
+def staged_buffers(plan: Plan, batch: int, dtype, device="cuda") -> dict:
+    """Allocate the staged-mode buffers (S fp32, P in `dtype`, O_csr fp32) for `batch`."""
+    import torch
+    z = staged_sizes(plan)
+    BH = batch * plan.heads
+    f32 = dict(dtype=torch.float32, device=device)
+    return {"S_tiles": torch.empty(BH, z["tile_elems"], **f32), "S_csr": torch.empty(BH, z["csr_elems"], **f32),
+            "S_global": torch.empty(BH, z["global_elems"], **f32),
+            "P_tiles": torch.empty(BH, z["tile_elems"], dtype=dtype, device=device),
+            "P_csr": torch.empty(BH, z["csr_elems"], dtype=dtype, device=device),
+            "P_global": torch.empty(BH, z["global_elems"], dtype=dtype, device=device),
+            "O_csr": torch.empty(BH, z["ocsr_elems"], **f32), "lpad": z["lpad"]}
+
+
+def staged_sddmm(plan: Plan, Q, K, bufs: dict, stream=None):
+    """mg_staged_sddmm: coarse, fine and dense-row scores into bufs S_tiles / S_csr / S_global."""
+    dq, dk = tensor_desc(Q), tensor_desc(K)
+    check(plan._lib.mg_staged_sddmm(plan.handle, C.byref(dq), C.byref(dk), _ptr(bufs["S_tiles"]),
+                                    _ptr(bufs["S_csr"]), _ptr(bufs["S_global"]), _stream_ptr(stream)))
+
+
+def staged_softmax(plan: Plan, batch: int, bufs: dict, stream=None):
+    """mg_staged_softmax: compound SpSoftmax of the S buffers into the P buffers."""
+    import torch
+    dt = _lib.MG_BF16 if bufs["P_tiles"].dtype == torch.bfloat16 else _lib.MG_FP16
+    check(plan._lib.mg_staged_softmax(plan.handle, batch, dt, _ptr(bufs["S_tiles"]), _ptr(bufs["S_csr"]),
+                                      _ptr(bufs["S_global"]), _ptr(bufs["P_tiles"]), _ptr(bufs["P_csr"]),
+                                      _ptr(bufs["P_global"]), _stream_ptr(stream)))
+
+
+def staged_spmm(plan: Plan, V, O, bufs: dict, stream=None):
+    """mg_staged_spmm: O = P V over the tiles, the CSR part (via O_csr) and the dense rows."""
+    dv, do = tensor_desc(V), tensor_desc(O)
+    check(plan._lib.mg_staged_spmm(plan.handle, _ptr(bufs["P_tiles"]), _ptr(bufs["P_csr"]), _ptr(bufs["P_global"]),
+                                   C.byref(dv), C.byref(do), _ptr(bufs["O_csr"]), _stream_ptr(stream)))
+    return O
+
+
+def sparse_attention_fwd_staged(plan: Plan, Q, K, V, O=None, stream=None):
+    """mg_sparse_attention_fwd_staged: the paper's dataflow (SDDMM -> SpSoftmax -> SpMM kernels)."""
+    import torch
+    if O is None:
+        O = torch.empty(Q.shape, dtype=Q.dtype, device=Q.device)
+    dq, dk, dv, do = tensor_desc(Q), tensor_desc(K), tensor_desc(V), tensor_desc(O)
+    check(plan._lib.mg_sparse_attention_fwd_staged(plan.handle, C.byref(dq), C.byref(dk), C.byref(dv),
+                                                   C.byref(do), _stream_ptr(stream)))
+    return O
+
+
 def selftest_umma(mode: int, A, B, D, stream=None):
     """mg_selftest_umma: one tcgen05 MMA on device buffers (diagnostics)."""
     check(load().mg_selftest_umma(mode, C.c_void_p(A.data_ptr()), C.c_void_p(B.data_ptr()),

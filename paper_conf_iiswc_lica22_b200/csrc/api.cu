@@ -65,6 +65,14 @@ struct mg_plan_s {
   size_t part_cap = 0;      // in (row, bh) partial slots
   uint8_t* d_stage = nullptr;
   size_t stage_cap = 0;     // bytes
+  // staged (paper-dataflow) path: canonical plan on the device, uploaded on first use
+  bool staged_uploaded = false;
+  int32_t *d_bsr_row_ptr = nullptr, *d_bsr_col = nullptr, *d_tile_row = nullptr, *d_csr_row_ptr = nullptr,
+          *d_csr_col = nullptr;
+  uint64_t* d_tile_masks = nullptr;
+  uint8_t* d_row_is_global = nullptr;
+  uint8_t* d_staged_ws = nullptr;   // S, P and O_csr buffers of mg_sparse_attention_fwd_staged
+  size_t staged_ws_cap = 0;
   // diagnostics: device event-trace buffer of the coarse kernel (CTA 0)
   unsigned long long* trace = nullptr;
   int32_t trace_cap = 0;
@@ -88,6 +96,7 @@ struct mg_plan_s {
     for (void* p : allocs) cudaFree(p);
     if (d_part) cudaFree(d_part);
     if (d_stage) cudaFree(d_stage);
+    if (d_staged_ws) cudaFree(d_staged_ws);
   }
 };
 
@@ -388,6 +397,118 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
   return MG_OK;
 }
 
+
+// ------------------------------------------------------------------ staged (paper dataflow) path
+mg_status staged_upload(mg_plan_s* p) {
+  mg_status s = upload(p);
+  if (s != MG_OK) return s;
+  if (p->staged_uploaded) return MG_OK;
+  const mg::HostPlan& h = p->hp;
+  std::vector<int32_t> tile_row(h.bsr_col.size());
+  for (int64_t I = 0; I < h.nb(); ++I)
+    for (int32_t t = h.bsr_row_ptr[I]; t < h.bsr_row_ptr[I + 1]; ++t) tile_row[t] = (int32_t)I;
+  std::vector<uint8_t> is_g(h.L, 0);
+  for (int32_t r : h.global_rows) is_g[r] = 1;
+  cudaError_t e;
+  if ((e = upload_vec(p, &p->d_bsr_row_ptr, h.bsr_row_ptr)) != cudaSuccess ||
+      (e = upload_vec(p, &p->d_bsr_col, h.bsr_col)) != cudaSuccess ||
+      (e = upload_vec(p, &p->d_tile_row, tile_row)) != cudaSuccess ||
+      (e = upload_vec(p, &p->d_tile_masks, h.tile_masks)) != cudaSuccess ||
+      (e = upload_vec(p, &p->d_csr_row_ptr, h.csr_row_ptr)) != cudaSuccess ||
+      (e = upload_vec(p, &p->d_csr_col, h.csr_col)) != cudaSuccess ||
+      (e = upload_vec(p, &p->d_row_is_global, is_g)) != cudaSuccess)
+    return e == cudaErrorMemoryAllocation ? fail(MG_ERR_OUT_OF_MEMORY, "device allocation failed")
+                                          : cuda_fail(e, "staged plan upload");
+  p->staged_uploaded = true;
+  return MG_OK;
+}
+
+mg_staged_sizes staged_sizes(const mg::HostPlan& h) {
+  mg_staged_sizes z;
+  z.lpad = h.nb() * 128;
+  z.tile_elems = (int64_t)h.bsr_col.size() * 128 * 128;
+  z.csr_elems = (int64_t)h.csr_col.size();
+  z.global_elems = (int64_t)h.global_rows.size() * z.lpad;
+  z.ocsr_elems = h.L * 64;
+  return z;
+}
+
+mg::StagedParams staged_params(const mg_plan_s* p, int64_t batch) {
+  const mg::HostPlan& h = p->hp;
+  mg::StagedParams sp{};
+  sp.bsr_row_ptr = p->d_bsr_row_ptr;
+  sp.bsr_col = p->d_bsr_col;
+  sp.tile_row = p->d_tile_row;
+  sp.tile_masks = p->d_tile_masks;
+  sp.csr_row_ptr = p->d_csr_row_ptr;
+  sp.csr_col = p->d_csr_col;
+  sp.global_rows = p->d_global_rows;
+  sp.row_is_global = p->d_row_is_global;
+  sp.L = h.L;
+  sp.nnz_csr = (int64_t)h.csr_col.size();
+  sp.Lpad = h.nb() * 128;
+  sp.H = h.heads;
+  sp.BH = (int32_t)(batch * h.heads);
+  sp.nb = (int32_t)h.nb();
+  sp.n_tiles = (int32_t)h.bsr_col.size();
+  sp.n_global = (int32_t)h.global_rows.size();
+  sp.sf = (float)(1.0 / std::sqrt((double)h.d));
+  return sp;
+}
+
+mg_status staged_check(mg_plan_s* p, const mg_tensor* t, const char* name) {
+  mg_status s = check_tensor(t, name, p, false);
+  if (s != MG_OK) return s;
+  if (!p->hp.kernel_ready) return fail(MG_ERR_UNSUPPORTED, "the staged forward requires block == 128");
+  if ((int64_t)t->batch * p->hp.heads >= 65536) return fail(MG_ERR_UNSUPPORTED, "batch * heads must be < 65536");
+  return staged_upload(p);
+}
+
+mg_status staged_buffers_ok(const mg_plan_s* p, const void* tiles, const void* csr, const void* glob) {
+  const mg_staged_sizes z = staged_sizes(p->hp);
+  if ((z.tile_elems && !tiles) || (z.csr_elems && !csr) || (z.global_elems && !glob))
+    return fail(MG_ERR_INVALID_ARG, "a staged buffer of non-zero size is null");
+  return MG_OK;
+}
+
+mg_status staged_sddmm_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, float* St, float* Sf, float* Sg,
+                            cudaStream_t stream) {
+  mg::StagedParams sp = staged_params(p, Q->batch);
+  sp.q = view(Q);
+  sp.k = view(K);
+  sp.S_t = St;
+  sp.S_f = Sf;
+  sp.S_g = Sg;
+  cudaError_t e = mg::launch_staged_sddmm(sp, Q->dtype == MG_BF16, stream);
+  return e == cudaSuccess ? MG_OK : cuda_fail(e, "staged SDDMM launch");
+}
+
+mg_status staged_softmax_impl(mg_plan_s* p, int64_t batch, mg_dtype dt, const float* St, const float* Sf,
+                              const float* Sg, void* Pt, void* Pf, void* Pg, cudaStream_t stream) {
+  mg::StagedParams sp = staged_params(p, batch);
+  sp.S_t = const_cast<float*>(St);
+  sp.S_f = const_cast<float*>(Sf);
+  sp.S_g = const_cast<float*>(Sg);
+  sp.P_t = static_cast<uint16_t*>(Pt);
+  sp.P_f = static_cast<uint16_t*>(Pf);
+  sp.P_g = static_cast<uint16_t*>(Pg);
+  cudaError_t e = mg::launch_staged_softmax(sp, dt == MG_BF16, stream);
+  return e == cudaSuccess ? MG_OK : cuda_fail(e, "staged SpSoftmax launch");
+}
+
+mg_status staged_spmm_impl(mg_plan_s* p, const void* Pt, const void* Pf, const void* Pg, const mg_tensor* V,
+                           mg_tensor* O, float* Of, cudaStream_t stream) {
+  mg::StagedParams sp = staged_params(p, V->batch);
+  sp.v = view(V);
+  sp.o = view(O);
+  sp.P_t = static_cast<uint16_t*>(const_cast<void*>(Pt));
+  sp.P_f = static_cast<uint16_t*>(const_cast<void*>(Pf));
+  sp.P_g = static_cast<uint16_t*>(const_cast<void*>(Pg));
+  sp.O_f = Of;
+  cudaError_t e = mg::launch_staged_spmm(sp, V->dtype == MG_BF16, stream);
+  return e == cudaSuccess ? MG_OK : cuda_fail(e, "staged SpMM launch");
+}
+
 }  // namespace
 
 extern "C" {
@@ -501,6 +622,92 @@ mg_status mg_sparse_attention_fwd_host(mg_plan_t plan, const mg_tensor* Q, const
   if ((e = cudaMemcpyAsync(O->data, dO.data, bytes, cudaMemcpyDeviceToHost, stream)) != cudaSuccess)
     return cuda_fail(e, "D2H copy");
   return MG_OK;
+}
+
+
+mg_status mg_staged_get_sizes(mg_plan_t plan, mg_staged_sizes* out) {
+  g_err.clear();
+  if (!plan || !out) return fail(MG_ERR_INVALID_ARG, "null argument");
+  *out = staged_sizes(plan->hp);
+  return MG_OK;
+}
+
+mg_status mg_staged_sddmm(mg_plan_t plan, const mg_tensor* Q, const mg_tensor* K, float* S_tiles, float* S_csr,
+                          float* S_global, void* stream) {
+  g_err.clear();
+  if (!plan) return fail(MG_ERR_INVALID_ARG, "plan is null");
+  mg_status s;
+  if ((s = staged_check(plan, Q, "Q")) != MG_OK || (s = staged_check(plan, K, "K")) != MG_OK) return s;
+  if (K->batch != Q->batch || K->dtype != Q->dtype) return fail(MG_ERR_INVALID_ARG, "Q/K batch or dtype differ");
+  if ((s = staged_buffers_ok(plan, S_tiles, S_csr, S_global)) != MG_OK) return s;
+  return staged_sddmm_impl(plan, Q, K, S_tiles, S_csr, S_global, static_cast<cudaStream_t>(stream));
+}
+
+mg_status mg_staged_softmax(mg_plan_t plan, int64_t batch, mg_dtype dtype, const float* S_tiles, const float* S_csr,
+                            const float* S_global, void* P_tiles, void* P_csr, void* P_global, void* stream) {
+  g_err.clear();
+  if (!plan) return fail(MG_ERR_INVALID_ARG, "plan is null");
+  if (batch <= 0) return fail(MG_ERR_INVALID_ARG, "batch must be > 0");
+  if (dtype != MG_BF16 && dtype != MG_FP16) return fail(MG_ERR_INVALID_ARG, "dtype is not bf16/fp16");
+  if (!plan->hp.kernel_ready) return fail(MG_ERR_UNSUPPORTED, "the staged forward requires block == 128");
+  mg_status s;
+  if ((s = staged_upload(plan)) != MG_OK) return s;
+  if ((s = staged_buffers_ok(plan, S_tiles, S_csr, S_global)) != MG_OK ||
+      (s = staged_buffers_ok(plan, P_tiles, P_csr, P_global)) != MG_OK)
+    return s;
+  return staged_softmax_impl(plan, batch, dtype, S_tiles, S_csr, S_global, P_tiles, P_csr, P_global,
+                             static_cast<cudaStream_t>(stream));
+}
+
+mg_status mg_staged_spmm(mg_plan_t plan, const void* P_tiles, const void* P_csr, const void* P_global,
+                         const mg_tensor* V, mg_tensor* O, float* O_csr, void* stream) {
+  g_err.clear();
+  if (!plan) return fail(MG_ERR_INVALID_ARG, "plan is null");
+  mg_status s;
+  if ((s = staged_check(plan, V, "V")) != MG_OK || (s = staged_check(plan, O, "O")) != MG_OK) return s;
+  if (O->batch != V->batch || O->dtype != V->dtype) return fail(MG_ERR_INVALID_ARG, "V/O batch or dtype differ");
+  if ((s = staged_buffers_ok(plan, P_tiles, P_csr, P_global)) != MG_OK) return s;
+  if (!plan->hp.csr_col.empty() && !O_csr) return fail(MG_ERR_INVALID_ARG, "O_csr is null");
+  return staged_spmm_impl(plan, P_tiles, P_csr, P_global, V, O, O_csr, static_cast<cudaStream_t>(stream));
+}
+
+mg_status mg_sparse_attention_fwd_staged(mg_plan_t plan, const mg_tensor* Q, const mg_tensor* K, const mg_tensor* V,
+                                         mg_tensor* O, void* stream_) {
+  g_err.clear();
+  if (!plan) return fail(MG_ERR_INVALID_ARG, "plan is null");
+  mg_status s = check_all(plan, Q, K, V, O, false);
+  if (s != MG_OK) return s;
+  if ((s = staged_check(plan, Q, "Q")) != MG_OK) return s;
+  cudaStream_t stream = static_cast<cudaStream_t>(stream_);
+  const mg_staged_sizes z = staged_sizes(plan->hp);
+  const size_t BH = (size_t)Q->batch * plan->hp.heads;
+  auto al = [](size_t b) { return (b + 255) & ~size_t(255); };
+  const size_t bt = al(BH * z.tile_elems * 4), bf = al(BH * z.csr_elems * 4), bg = al(BH * z.global_elems * 4);
+  const size_t pt = al(BH * z.tile_elems * 2), pf = al(BH * z.csr_elems * 2), pg = al(BH * z.global_elems * 2);
+  const size_t bo = al(BH * z.ocsr_elems * 4);
+  const size_t need = bt + bf + bg + pt + pf + pg + bo;
+  cudaError_t e;
+  if (need > plan->staged_ws_cap) {
+    if (plan->d_staged_ws) {
+      if ((e = cudaFreeAsync(plan->d_staged_ws, stream)) != cudaSuccess) return cuda_fail(e, "cudaFreeAsync");
+      plan->d_staged_ws = nullptr;
+    }
+    if ((e = cudaMallocAsync(reinterpret_cast<void**>(&plan->d_staged_ws), need, stream)) != cudaSuccess)
+      return e == cudaErrorMemoryAllocation ? fail(MG_ERR_OUT_OF_MEMORY, "staged workspace allocation failed")
+                                            : cuda_fail(e, "cudaMallocAsync");
+    plan->staged_ws_cap = need;
+  }
+  uint8_t* w = plan->d_staged_ws;
+  float* St = reinterpret_cast<float*>(w);
+  float* Sf = reinterpret_cast<float*>(w + bt);
+  float* Sg = reinterpret_cast<float*>(w + bt + bf);
+  void* Pt = w + bt + bf + bg;
+  void* Pf = w + bt + bf + bg + pt;
+  void* Pg = w + bt + bf + bg + pt + pf;
+  float* Of = reinterpret_cast<float*>(w + bt + bf + bg + pt + pf + pg);
+  if ((s = staged_sddmm_impl(plan, Q, K, St, Sf, Sg, stream)) != MG_OK) return s;
+  if ((s = staged_softmax_impl(plan, Q->batch, (mg_dtype)Q->dtype, St, Sf, Sg, Pt, Pf, Pg, stream)) != MG_OK) return s;
+  return staged_spmm_impl(plan, Pt, Pf, Pg, V, O, Of, stream);
 }
 
 mg_status mg_plan_set_profiling(mg_plan_t plan, int32_t enable) {

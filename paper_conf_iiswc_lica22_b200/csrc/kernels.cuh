@@ -56,6 +56,33 @@ struct FineParams {
   float scale_log2;
 };
 
+// Staged (paper dataflow) kernels: S and P materialised in the plan's formats; see staged.cu.
+struct StagedParams {
+  const int32_t* bsr_row_ptr;   // canonical plan (block 128)
+  const int32_t* bsr_col;
+  const int32_t* tile_row;      // [n_tiles] row block of each tile
+  const uint64_t* tile_masks;   // [n_tiles][128][2]
+  const int32_t* csr_row_ptr;   // [L + 1]
+  const int32_t* csr_col;
+  const int32_t* global_rows;
+  const uint8_t* row_is_global; // [L]
+  TensorView q, k, v, o;
+  float* S_t;
+  float* S_f;
+  float* S_g;
+  uint16_t* P_t;
+  uint16_t* P_f;
+  uint16_t* P_g;
+  float* O_f;
+  int64_t L, nnz_csr, Lpad;
+  int32_t H, BH, nb, n_tiles, n_global;
+  float sf;                     // 1 / sqrt(d)
+};
+
+cudaError_t launch_staged_sddmm(const StagedParams& p, bool bf16, cudaStream_t stream);
+cudaError_t launch_staged_softmax(const StagedParams& p, bool bf16, cudaStream_t stream);
+cudaError_t launch_staged_spmm(const StagedParams& p, bool bf16, cudaStream_t stream);
+
 cudaError_t launch_coarse(const CoarseParams& p, const CUtensorMap& tmq, const CUtensorMap& tmk,
                           const CUtensorMap& tmv, bool bf16, int grid, cudaStream_t stream);
 // Paired-pipeline variant: two CTAs per SM (grid = 2 x SMs), see coarse_pp_sm100.cu.
