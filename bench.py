@@ -44,6 +44,10 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-flush", action="store_true")
     ap.add_argument("--strip-max-cols", type=int, default=0)
+    ap.add_argument("--ablation", action="store_true",
+                    help="also time the staged paper-dataflow forward (mg_sparse_attention_fwd_staged)")
+    ap.add_argument("--concurrency", type=int, default=0, choices=[0, 1, 2],
+                    help="coarse vs CSR kernels: 0 = library default, 1 = serial, 2 = concurrent streams")
     ap.add_argument("--fine-kernel", type=int, default=0, choices=[0, 1],
                     help="CSR rows: 0 = warp-level tensor-core kernel, 1 = CUDA-core kernel (A/B)")
     return ap.parse_args()
@@ -236,7 +240,8 @@ def main():
 
     cfg = get_config(args.workload)
     plan = mg.Plan(cfg.L, cfg.H, cfg.d, cfg.window, cfg.global_idx, cfg.extra_idx,
-                   strip_max_cols=args.strip_max_cols, fine_kernel=args.fine_kernel)
+                   strip_max_cols=args.strip_max_cols, fine_kernel=args.fine_kernel,
+                   concurrency=args.concurrency)
     info = plan.info()
     BH = cfg.B * cfg.H
     useful = 4.0 * info["nnz_total"] * cfg.d * BH
@@ -375,6 +380,29 @@ def main():
     }
     if gather_ms is not None:
         line["allgather_O_ms"] = gather_ms
+    if args.ablation:
+        # the paper's dataflow (S and P materialised, SDDMM -> 3-sweep SpSoftmax -> SpMM kernels),
+        # same inputs, same L2 flush, CUDA events on the same stream
+        Os = mg.sparse_attention_fwd_staged(plan, Q, K, V, None, stream)
+        for _ in range(3):
+            mg.sparse_attention_fwd_staged(plan, Q, K, V, Os, stream)
+        n_ab = max(3, min(50, args.steps))
+        ab = []
+        for _ in range(n_ab):
+            if not args.no_flush:
+                flush.zero_()
+            a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a0.record(stream)
+            mg.sparse_attention_fwd_staged(plan, Q, K, V, Os, stream)
+            a1.record(stream)
+            ab.append((a0, a1))
+        torch.cuda.synchronize()
+        st_ms = sum(a.elapsed_time(b) for a, b in ab) / n_ab
+        diff = (Os.float() - O.float()).abs()
+        line["staged_ablation"] = {"ms_per_step": st_ms, "tflops": useful / (st_ms * 1e-3) / 1e12,
+                                   "fused_speedup": st_ms / ms_per_step, "steps": n_ab,
+                                   "max_abs_vs_fused": float(diff.max()),
+                                   "path": "mg_sparse_attention_fwd_staged (S, P in HBM; 5-7 kernels)"}
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         line["cpu_baseline"] = cpu_oracle_heads(cfg, args.cpu_seconds)
     if rank == 0:

@@ -112,7 +112,10 @@ typedef struct {
   int32_t num_sms;        /* persistent grid size override; 0 -> device SM count */
   int32_t fine_kernel;    /* CSR rows outside strip tiles: 0 -> warp-level tensor-core kernel
                              (mma.sync, default), 1 -> CUDA-core shuffle-reduction kernel (A/B) */
-  int32_t reserved[3];
+  int32_t concurrency;    /* coarse vs CUDA-core CSR kernels: 0 -> library default, 1 -> serial (fine
+                             kernel, then coarse kernel merging its partials), 2 -> concurrent on two
+                             streams, rows merged by whichever side finishes second */
+  int32_t reserved[2];
 } mg_plan_opts;
 
 MG_API mg_status mg_plan_create_ex(int64_t L, int32_t heads, int32_t d, int32_t window,

@@ -49,6 +49,9 @@ struct mg_plan_s {
   int num_sms = 0;
   int num_sms_override = 0;
   int fine_kernel = 0;   // 0: mma.sync kernel (fine_mma.cu), 1: CUDA-core kernel (fine_rows.cu)
+  int concurrency = 0;   // 0 default, 1 serial, 2 concurrent streams (see mg_plan_opts)
+  cudaStream_t side = nullptr;              // second stream of the concurrent mode
+  cudaEvent_t fork_ev = nullptr, join_ev = nullptr;
   std::vector<void*> allocs;
   mg::Item* d_items = nullptr;
   mg::TileRef* d_trefs = nullptr;
@@ -93,6 +96,9 @@ struct mg_plan_s {
 
   ~mg_plan_s() {
     for (cudaEvent_t e : prof_events) cudaEventDestroy(e);
+    if (fork_ev) cudaEventDestroy(fork_ev);
+    if (join_ev) cudaEventDestroy(join_ev);
+    if (side) cudaStreamDestroy(side);
     for (void* p : allocs) cudaFree(p);
     if (d_part) cudaFree(d_part);
     if (d_stage) cudaFree(d_stage);
@@ -145,7 +151,7 @@ mg_status create_impl(int64_t L, int32_t heads, int32_t d, int32_t window, const
   if (!plan_out) return fail(MG_ERR_INVALID_ARG, "plan_out is null");
   *plan_out = nullptr;
   mg::PlanOptions po;
-  int sms_override = 0, fine_kernel = 0;
+  int sms_override = 0, fine_kernel = 0, concurrency = 0;
   if (opts) {
     if (opts->block != 0) po.block = opts->block;
     po.force_all_fine = opts->force_all_fine != 0;
@@ -155,6 +161,8 @@ mg_status create_impl(int64_t L, int32_t heads, int32_t d, int32_t window, const
     sms_override = opts->num_sms;
     if (opts->fine_kernel < 0 || opts->fine_kernel > 1) return fail(MG_ERR_INVALID_ARG, "fine_kernel must be 0 or 1");
     fine_kernel = opts->fine_kernel;
+    if (opts->concurrency < 0 || opts->concurrency > 2) return fail(MG_ERR_INVALID_ARG, "concurrency must be 0, 1 or 2");
+    concurrency = opts->concurrency;
   }
   mg_plan_s* p = new (std::nothrow) mg_plan_s();
   if (!p) return fail(MG_ERR_OUT_OF_MEMORY, "host allocation failed");
@@ -175,6 +183,7 @@ mg_status create_impl(int64_t L, int32_t heads, int32_t d, int32_t window, const
   }
   p->num_sms_override = sms_override;
   p->fine_kernel = fine_kernel;
+  p->concurrency = concurrency;
   int ndev = 0;
   if (cudaGetDeviceCount(&ndev) != cudaSuccess) {
     ndev = 0;
@@ -285,6 +294,9 @@ mg::TensorView view(const mg_tensor* t) {
   return mg::TensorView{static_cast<uint16_t*>(t->data), t->stride_b, t->stride_h, t->stride_l};
 }
 
+// measured on B200: C4 serial vs concurrent
+constexpr bool kConcurrentDefault = false;
+
 mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const mg_tensor* V, mg_tensor* O,
                    cudaStream_t stream) {
   mg_status s = upload(p);
@@ -298,20 +310,49 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
   const int nf = (int)h.fine_rows.size();
   const float scale_log2 = (float)(1.4426950408889634 / std::sqrt((double)h.d));
   cudaError_t e;
-  // fp32 partials of the CUDA-core CSR rows that are merged by the coarse epilogue
-  const size_t need = (size_t)BH * nf;
+  // Concurrent coarse || fine (north_star item 5): chosen by measurement, only with
+  // the tensor-core fine kernel and the paired-pipeline coarse kernel.
+  static const bool v13 = [] {
+    const char* e = std::getenv("MG_COARSE");
+    return e && std::strcmp(e, "v13") == 0;
+  }();
+  const bool concurrent = nf > 0 && !h.items.empty() && p->fine_kernel == 0 && !v13 &&
+                          (p->concurrency == 2 || (p->concurrency == 0 && kConcurrentDefault));
+  // fp32 partials of the CUDA-core CSR rows (fine -> coarse; and coarse -> fine plus one counter
+  // per row when concurrent). Layout by capacity: [fine acc 64][fine ml 2][coarse acc 64][coarse ml 2]
+  // floats per slot, then one int32 counter per slot (zeroed at allocation; even between forwards).
+  const size_t need = ((size_t)BH * nf + 3) & ~size_t(3);   // multiple of 4: 16-byte aligned sections
   if (need > p->part_cap) {
     if (p->d_part) {
       if ((e = cudaFreeAsync(p->d_part, stream)) != cudaSuccess) return cuda_fail(e, "cudaFreeAsync");
       p->d_part = nullptr;
     }
-    if ((e = cudaMallocAsync(reinterpret_cast<void**>(&p->d_part), need * 66 * sizeof(float), stream)) != cudaSuccess)
+    if ((e = cudaMallocAsync(reinterpret_cast<void**>(&p->d_part), need * 133 * sizeof(float), stream)) != cudaSuccess)
       return e == cudaErrorMemoryAllocation ? fail(MG_ERR_OUT_OF_MEMORY, "workspace allocation failed")
                                             : cuda_fail(e, "cudaMallocAsync");
+    if ((e = cudaMemsetAsync(p->d_part + need * 132, 0, need * sizeof(int32_t), stream)) != cudaSuccess)
+      return cuda_fail(e, "cudaMemsetAsync");
     p->part_cap = need;
   }
+  const size_t cap = p->part_cap;
   float* part_acc = p->d_part;
-  float2* part_ml = reinterpret_cast<float2*>(p->d_part + need * 64);
+  float2* part_ml = reinterpret_cast<float2*>(p->d_part + cap * 64);
+  float* part_c_acc = p->d_part + cap * 66;
+  float2* part_c_ml = reinterpret_cast<float2*>(p->d_part + cap * 130);
+  int32_t* part_flags = reinterpret_cast<int32_t*>(p->d_part + cap * 132);
+  cudaStream_t fstream = stream;
+  if (concurrent) {
+    if (!p->side) {
+      if ((e = cudaStreamCreateWithFlags(&p->side, cudaStreamNonBlocking)) != cudaSuccess ||
+          (e = cudaEventCreateWithFlags(&p->fork_ev, cudaEventDisableTiming)) != cudaSuccess ||
+          (e = cudaEventCreateWithFlags(&p->join_ev, cudaEventDisableTiming)) != cudaSuccess)
+        return cuda_fail(e, "stream/event creation");
+    }
+    if ((e = cudaEventRecord(p->fork_ev, stream)) != cudaSuccess ||
+        (e = cudaStreamWaitEvent(p->side, p->fork_ev, 0)) != cudaSuccess)
+      return cuda_fail(e, "stream fork");
+    fstream = p->side;
+  }
 
   cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
   if (p->profiling) {
@@ -319,7 +360,7 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
       if (!(ev[i] = p->prof_event())) return fail(MG_ERR_CUDA, "cudaEventCreate failed");
     p->prof_has_fine.push_back(nf > 0);
     p->prof_has_coarse.push_back(!h.items.empty());
-    cudaEventRecord(ev[0], stream);
+    cudaEventRecord(ev[0], fstream);
   }
   if (nf > 0) {
     mg::FineParams fp{};
@@ -331,10 +372,14 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
     fp.q = view(Q); fp.k = view(K); fp.v = view(V); fp.o = view(O);
     fp.H = h.heads; fp.BH = BH; fp.n_fine_rows = nf;
     fp.scale_log2 = scale_log2;
-    e = p->fine_kernel == 1 ? mg::launch_fine(fp, bf16, stream) : mg::launch_fine_mma(fp, bf16, stream);
+    fp.concurrent = concurrent;
+    fp.part_c_acc = part_c_acc;
+    fp.part_c_ml = part_c_ml;
+    fp.part_flags = part_flags;
+    e = p->fine_kernel == 1 ? mg::launch_fine(fp, bf16, fstream) : mg::launch_fine_mma(fp, bf16, fstream);
     if (e != cudaSuccess) return cuda_fail(e, "fine kernel launch");
   }
-  if (p->profiling) cudaEventRecord(ev[1], stream);
+  if (p->profiling) cudaEventRecord(ev[1], fstream);
   if (!h.items.empty()) {
     CUtensorMap tq, tk, tv;
     if (!encode_map(&tq, Q) || !encode_map(&tk, K) || !encode_map(&tv, V))
@@ -359,6 +404,10 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
     cp.n_fine_rows = nf;
     cp.total_units = cp.n_items * BH;
     cp.scale_log2 = scale_log2;
+    cp.concurrent = concurrent;
+    cp.part_c_acc = part_c_acc;
+    cp.part_c_ml = part_c_ml;
+    cp.part_flags = part_flags;
     static const int dbg = [] {
       const char* e = std::getenv("MG_DEBUG_FLAGS");
       return e ? std::atoi(e) : 0;
@@ -366,14 +415,12 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
     cp.debug_flags = dbg;
     cp.trace = p->trace;
     cp.trace_cap = p->trace_cap;
-    if ((e = cudaMemsetAsync(p->d_counter, 0, sizeof(int32_t), stream)) != cudaSuccess)
+    // the paired-pipeline kernel resets its work counter itself (last CTA to exit); the v13 kernel
+    // needs it zeroed before the launch
+    if (v13 && (e = cudaMemsetAsync(p->d_counter, 0, sizeof(int32_t), stream)) != cudaSuccess)
       return cuda_fail(e, "cudaMemsetAsync");
     const int sms = p->num_sms_override > 0 ? std::min(p->num_sms_override, p->num_sms) : p->num_sms;
     // MG_COARSE=v13 selects the previous single-CTA-per-SM kernel (A/B measurements only)
-    static const bool v13 = [] {
-      const char* e = std::getenv("MG_COARSE");
-      return e && std::strcmp(e, "v13") == 0;
-    }();
     if (p->profiling) cudaEventRecord(ev[2], stream);  // after the counter reset
     if (v13) {
       if ((e = mg::launch_coarse(cp, tq, tk, tv, bf16, std::min(sms, cp.total_units), stream)) != cudaSuccess)
@@ -392,6 +439,11 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
     }
   } else if (p->profiling) {
     cudaEventRecord(ev[2], stream);
+  }
+  if (concurrent) {
+    if ((e = cudaEventRecord(p->join_ev, fstream)) != cudaSuccess ||
+        (e = cudaStreamWaitEvent(stream, p->join_ev, 0)) != cudaSuccess)
+      return cuda_fail(e, "stream join");
   }
   if (p->profiling) cudaEventRecord(ev[3], stream);
   return MG_OK;

@@ -669,17 +669,13 @@ __global__ void __launch_bounds__(kThreads, 2)
       // ---------------------------------------------------------------- epilogue (a-8)
       float mf = -INFINITY, lf = 0.f;
       const float4* accf = nullptr;
-      if (slot_f >= 0) {
-        const size_t idx = (size_t)ubh * p.n_fine_rows + slot_f;
-        const float2 ml = p.part_ml[idx];
+      const size_t fidx = (size_t)ubh * p.n_fine_rows + slot_f;
+      if (slot_f >= 0 && !p.concurrent) {
+        const float2 ml = p.part_ml[fidx];
         mf = ml.x;
         lf = ml.y;
-        accf = reinterpret_cast<const float4*>(p.part_acc + idx * 64);
+        accf = reinterpret_cast<const float4*>(p.part_acc + fidx * 64);
       }
-      const float mt = fmaxf(m, mf);
-      const float mu = mt == -INFINITY ? 0.f : mt;
-      const float ac = ex2((m - mu) * c), af = ex2((mf - mu) * c);
-      const float den = l * ac + lf * af;
       if (threadIdx.x == 0) tl_rec(p, n - 1, 11);
       mbar_wait(bar(ctl->pv_done), (n - 1) & 1);          // the item's last P.V
       tc_fence_after();
@@ -689,11 +685,36 @@ __global__ void __launch_bounds__(kThreads, 2)
       tmem_wait_ld();
       tc_fence_before();
       if (threadIdx.x == 0) tl_rec(p, n - 1, 12);
+      bool skip = false;
+      if (slot_f >= 0 && p.concurrent) {
+        // publish this row's coarse partial; the side that finishes the row second merges both
+        float4* dst = reinterpret_cast<float4*>(p.part_c_acc + fidx * 64);
+#pragma unroll
+        for (int i = 0; i < 16; ++i)
+          __stcg(dst + i, make_float4(__uint_as_float(o[i >> 3][(i & 7) * 4]), __uint_as_float(o[i >> 3][(i & 7) * 4 + 1]),
+                                      __uint_as_float(o[i >> 3][(i & 7) * 4 + 2]), __uint_as_float(o[i >> 3][(i & 7) * 4 + 3])));
+        __stcg(p.part_c_ml + fidx, make_float2(m, l));
+        __threadfence();
+        const int old = atomicAdd(p.part_flags + fidx, 1);
+        if (old & 1) {
+          __threadfence();
+          const float2 ml = __ldcg(p.part_ml + fidx);
+          mf = ml.x;
+          lf = ml.y;
+          accf = reinterpret_cast<const float4*>(p.part_acc + fidx * 64);
+        } else {
+          skip = true;
+        }
+      }
+      const float mt = fmaxf(m, mf);
+      const float mu = mt == -INFINITY ? 0.f : mt;
+      const float ac = ex2((m - mu) * c), af = ex2((mf - mu) * c);
+      const float den = l * ac + lf * af;
       // normalised row -> 16-bit, 8 x 16-byte stores of this thread's row. A row with no valid
       // element in this item (a global row inside a band row block: it is owned by the dense-row
       // part, A5) is not written. (Staging the tile through shared memory for 4-rows-per-
       // instruction stores measured 10% slower: tools/experiments/.)
-      if (r_out >= 0 && mt != -INFINITY) {
+      if (r_out >= 0 && mt != -INFINITY && !skip) {
         const float inv = __frcp_rn(den);
         const int bb = ubh / p.H, hh = ubh % p.H;
         uint16_t* orow = p.o.data + bb * p.o.sb + hh * p.o.sh + (int64_t)r_out * p.o.sl;
@@ -705,7 +726,7 @@ __global__ void __launch_bounds__(kThreads, 2)
 #pragma unroll
             for (int i = 0; i < 8; ++i) a[i] = __uint_as_float(o[h][q8 * 8 + i]) * ac;
             if (accf) {
-              const float4 f0 = accf[h * 8 + q8 * 2], f1 = accf[h * 8 + q8 * 2 + 1];
+              const float4 f0 = __ldcg(accf + h * 8 + q8 * 2), f1 = __ldcg(accf + h * 8 + q8 * 2 + 1);
               a[0] = fmaf(f0.x, af, a[0]);
               a[1] = fmaf(f0.y, af, a[1]);
               a[2] = fmaf(f0.z, af, a[2]);
@@ -731,6 +752,15 @@ __global__ void __launch_bounds__(kThreads, 2)
   tc_fence_before();
   __syncthreads();
   if (warp == 5) tmem_dealloc(tmem, kTmemCols);
+  // the last CTA to finish resets the work counter for the next launch (every CTA's scheduler has
+  // claimed its final, out-of-range unit before its CTA gets here), so no memset precedes a launch
+  if (threadIdx.x == 0) {
+    __threadfence();
+    if (atomicAdd(p.counter + 1, 1) == (int)gridDim.x - 1) {
+      atomicExch(p.counter, 0);
+      atomicExch(p.counter + 1, 0);
+    }
+  }
 }
 
 cudaError_t launch_coarse_pp(const CoarseParams& p, const CUtensorMap& tmq, const CUtensorMap& tmk,

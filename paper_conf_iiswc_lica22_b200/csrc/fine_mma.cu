@@ -187,23 +187,49 @@ __global__ void __launch_bounds__(256, 2) fine_mma_kernel(const FineParams p) {
   // row sum: lanes with the same g hold disjoint nnz subsets (t); every g holds the same sums
   l += __shfl_xor_sync(0xffffffffu, l, 1);
   l += __shfl_xor_sync(0xffffffffu, l, 2);
-  if (t != 0) return;
   // lane (g, 0): O dims 8g .. 8g+7 = acc[j][0] (dim 8g+2j), acc[j][2] (dim 8g+2j+1)
-  if (final_out) {
-    const float inv = l > 0.f ? 1.f / l : 0.f;
-    uint4 o4;
-    o4.x = pack2<kBF16>(acc[0][0] * inv, acc[0][2] * inv);
-    o4.y = pack2<kBF16>(acc[1][0] * inv, acc[1][2] * inv);
-    o4.z = pack2<kBF16>(acc[2][0] * inv, acc[2][2] * inv);
-    o4.w = pack2<kBF16>(acc[3][0] * inv, acc[3][2] * inv);
-    *reinterpret_cast<uint4*>(p.o.data + bb * p.o.sb + hh * p.o.sh + (int64_t)r * p.o.sl + g * 8) = o4;
-  } else {
+  float o8[8] = {acc[0][0], acc[0][2], acc[1][0], acc[1][2], acc[2][0], acc[2][2], acc[3][0], acc[3][2]};
+  float inv = l > 0.f ? 1.f / l : 0.f;
+  bool write_o = final_out;
+  if (!final_out) {
     const size_t idx = (size_t)bh * p.n_fine_rows + fi;
-    float4* dst = reinterpret_cast<float4*>(p.part_acc + idx * 64 + g * 8);
-    dst[0] = make_float4(acc[0][0], acc[0][2], acc[1][0], acc[1][2]);
-    dst[1] = make_float4(acc[2][0], acc[2][2], acc[3][0], acc[3][2]);
-    if (lane == 0) p.part_ml[idx] = make_float2(m, l);
+    if (t == 0) {
+      float4* dst = reinterpret_cast<float4*>(p.part_acc + idx * 64 + g * 8);
+      __stcg(dst, make_float4(o8[0], o8[1], o8[2], o8[3]));
+      __stcg(dst + 1, make_float4(o8[4], o8[5], o8[6], o8[7]));
+      if (lane == 0) __stcg(p.part_ml + idx, make_float2(m, l));
+    }
+    if (p.concurrent) {
+      // concurrent coarse || fine: the side that finishes the row second merges (a-8)
+      __threadfence();
+      __syncwarp();
+      int old = 0;
+      if (lane == 0) old = atomicAdd(p.part_flags + idx, 1);
+      old = __shfl_sync(0xffffffffu, old, 0);
+      if (old & 1) {
+        __threadfence();
+        const float2 mlc = __ldcg(p.part_c_ml + idx);
+        const float mt = fmaxf(m, mlc.x);
+        const float mu = mt == -INFINITY ? 0.f : mt;
+        const float af = ex2((m - mu) * c), ac = ex2((mlc.x - mu) * c);
+        const float den = l * af + mlc.y * ac;
+        inv = den > 0.f ? 1.f / den : 0.f;
+        const float4* src = reinterpret_cast<const float4*>(p.part_c_acc + idx * 64 + g * 8);
+        const float4 c0 = __ldcg(src), c1 = __ldcg(src + 1);
+        const float cc[8] = {c0.x, c0.y, c0.z, c0.w, c1.x, c1.y, c1.z, c1.w};
+#pragma unroll
+        for (int e = 0; e < 8; ++e) o8[e] = o8[e] * af + cc[e] * ac;
+        write_o = true;
+      }
+    }
   }
+  if (t != 0 || !write_o) return;
+  uint4 o4;
+  o4.x = pack2<kBF16>(o8[0] * inv, o8[1] * inv);
+  o4.y = pack2<kBF16>(o8[2] * inv, o8[3] * inv);
+  o4.z = pack2<kBF16>(o8[4] * inv, o8[5] * inv);
+  o4.w = pack2<kBF16>(o8[6] * inv, o8[7] * inv);
+  *reinterpret_cast<uint4*>(p.o.data + bb * p.o.sb + hh * p.o.sh + (int64_t)r * p.o.sl + g * 8) = o4;
 }
 
 cudaError_t launch_fine_mma(const FineParams& p, bool bf16, cudaStream_t stream) {

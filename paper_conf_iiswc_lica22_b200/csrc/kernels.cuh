@@ -26,7 +26,7 @@ struct CoarseParams {
   const int32_t* fine_slot;   // [L]; >= 0: merge fine partial of that slot
   const float* part_acc;      // [BH * n_fine_rows * 64]
   const float2* part_ml;      // [BH * n_fine_rows]  (max in raw score units, sum)
-  int32_t* counter;           // work counter (zeroed before launch)
+  int32_t* counter;           // [0] work counter, [1] CTAs finished (pp kernel: reset by the last CTA)
   TensorView q, k, v, o;
   int64_t L;
   int32_t H, BH;
@@ -40,6 +40,12 @@ struct CoarseParams {
   // b * r.x + h * r.y + l * r.z; gather_tma = 0 when the strides do not allow such a view
   int32_t gather_tma;
   longlong3 rq, rk, rv;
+  // concurrent coarse || fine (plan option): the rows with both a coarse and a CUDA-core CSR part are
+  // merged by whichever side finishes the row second (per-row counters, parity = "other side done")
+  int32_t concurrent;
+  float* part_c_acc;          // [BH * n_fine_rows * 64] coarse partial (written when concurrent)
+  float2* part_c_ml;
+  int32_t* part_flags;        // [BH * n_fine_rows], +1 per side per forward (even between forwards)
   int32_t debug_flags;        // diagnostics (env MG_DEBUG_FLAGS): 1 = no softmax arithmetic, 2 = no MMA, 4 = no loads,
                               // 16 = no S loads from TMEM, 64 = MMA ignores P-ready/O-free (timing only)
 };
@@ -54,6 +60,10 @@ struct FineParams {
   TensorView q, k, v, o;
   int32_t H, BH, n_fine_rows;
   float scale_log2;
+  int32_t concurrent;         // see CoarseParams::concurrent
+  const float* part_c_acc;
+  const float2* part_c_ml;
+  int32_t* part_flags;
 };
 
 // Staged (paper dataflow) kernels: S and P materialised in the plan's formats; see staged.cu.

@@ -67,17 +67,17 @@ def mixed_extra(L, seed=3, per_row=6):
     return random_residual(L, 128, per_row, seed=seed)
 
 
-@pytest.mark.parametrize("fine_kernel", [0, 1])
+@pytest.mark.parametrize("fine_kernel,concurrency", [(0, 1), (0, 2), (1, 1)])
 @pytest.mark.parametrize("strip", [0, -1])
 @pytest.mark.parametrize("all_fine", [False, True])
-def test_mixed_pattern_all_parts(strip, all_fine, fine_kernel):
+def test_mixed_pattern_all_parts(strip, all_fine, fine_kernel, concurrency):
     """Band tiles + strip tiles or CSR rows (tensor-core or CUDA-core fine kernel) + dense global
     rows, several heads."""
     m = MIXED
     E = mixed_extra(m["L"])
     q, k, v = make_qkv(m["B"], m["H"], m["L"], 64, seed=5, dist="adversarial", global_idx=m["G"])
     plan = mg.Plan(m["L"], m["H"], 64, m["window"], m["G"], E, strip_max_cols=strip, force_all_fine=all_fine,
-                   fine_kernel=fine_kernel)
+                   fine_kernel=fine_kernel, concurrency=concurrency)
     inf = plan.info()
     if all_fine:
         assert inf["n_tiles"] == 0 and inf["nnz_fine_cuda"] == inf["nnz_fine"]
@@ -86,10 +86,10 @@ def test_mixed_pattern_all_parts(strip, all_fine, fine_kernel):
     check(got, ref)
 
 
-@pytest.mark.parametrize("fine_kernel", [0, 1])
+@pytest.mark.parametrize("fine_kernel,concurrency", [(0, 1), (0, 2), (1, 1)])
 @pytest.mark.parametrize("dtype", ["bf16", "fp16"])
 @pytest.mark.parametrize("dist", ["normal", "peaky", "adversarial"])
-def test_fine_rows_all_lengths(fine_kernel, dtype, dist):
+def test_fine_rows_all_lengths(fine_kernel, concurrency, dtype, dist):
     """CSR-only rows of every length 1..70 (ragged 16-nnz steps of the tensor-core fine kernel,
     32-index windows, final rows written directly) plus rows with a coarse part (fp32 partials)."""
     L, G = 768, np.array([700], np.int32)
@@ -101,7 +101,8 @@ def test_fine_rows_all_lengths(fine_kernel, dtype, dist):
     E = np.array(pairs, np.int32)
     q, k, v = make_qkv(1, 2, L, 64, seed=12, dist=dist, global_idx=G, dtype=dtype)
     for all_fine in (True, False):
-        plan = mg.Plan(L, 2, 64, 32, G, E, strip_max_cols=-1, force_all_fine=all_fine, fine_kernel=fine_kernel)
+        plan = mg.Plan(L, 2, 64, 32, G, E, strip_max_cols=-1, force_all_fine=all_fine, fine_kernel=fine_kernel,
+                       concurrency=concurrency)
         assert plan.info()["nnz_fine_cuda"] > 0
         got = run_gpu(plan, q, k, v, dtype=dtype)
         ref = oracle_full(q, k, v, 32, G, E, dtype=dtype)
@@ -161,6 +162,18 @@ def test_ones_v_and_zero_q():
     check(run_gpu(plan, q, k, v), oracle_full(q, k, v, c.window, c.global_idx, c.extra_idx))
 
 
+def test_concurrent_repeat_calls_and_batch_change():
+    """Concurrent mode: per-row counters stay consistent over repeated calls and batch changes."""
+    m = MIXED
+    E = mixed_extra(m["L"], seed=9)
+    plan = mg.Plan(m["L"], m["H"], 64, m["window"], m["G"], E, strip_max_cols=-1, concurrency=2)
+    for B in (2, 3, 1, 3):
+        q, k, v = make_qkv(B, m["H"], m["L"], 64, seed=B)
+        ref = oracle_full(q, k, v, m["window"], m["G"], E)
+        for _ in range(2):
+            check(run_gpu(plan, q, k, v), ref)
+
+
 def test_repeat_calls_deterministic_and_batch_growth():
     c = get_config("C1")
     plan = mg.Plan(c.L, 1, 64, c.window, c.global_idx, c.extra_idx)
@@ -206,11 +219,13 @@ def sample_rows(L, G, rng, n=48):
     return sorted(r for r in rows if 0 <= r < L)
 
 
-@pytest.mark.parametrize("cfg,fine_kernel", [("C2", 0), ("C3", 0), ("C4", 0), ("C4", 1)])
-def test_full_size_sampled(cfg, fine_kernel):
+@pytest.mark.parametrize("cfg,fine_kernel,concurrency", [("C2", 0, 0), ("C3", 0, 0), ("C4", 0, 1), ("C4", 0, 2),
+                                                          ("C4", 1, 1)])
+def test_full_size_sampled(cfg, fine_kernel, concurrency):
     c = get_config(cfg)
     q, k, v = make_qkv(c.B, c.H, c.L, c.d, seed=c.seed)
-    plan = mg.Plan(c.L, c.H, c.d, c.window, c.global_idx, c.extra_idx, fine_kernel=fine_kernel)
+    plan = mg.Plan(c.L, c.H, c.d, c.window, c.global_idx, c.extra_idx, fine_kernel=fine_kernel,
+                   concurrency=concurrency)
     got = run_gpu(plan, q, k, v)
     assert np.isfinite(got).all()
     rng = np.random.default_rng(17)

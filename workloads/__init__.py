@@ -17,6 +17,16 @@ arrays produced here.
     E = 164 (=⌈0.01·L⌉) distinct uniform columns per row outside the band,
     drawn row by row from ``default_rng(0)``;
   - C5: C2's shape at B=64 (sharded over ranks in the scaling bench).
+* Paper-faithful extra workloads (reading A15):
+  - QDS-LS: QDS-Transformer as local + selected: B=8, H=12, L=2048, w=128 (the window
+    whose 64-blocks give P:185's 2:1 sparse:dense ratio), the C3 special tokens as column-only
+    selected tokens (every row attends to them, "all-to-one", P:66), no global rows;
+  - Fig. 9 synthetic compound patterns (batch 1, L=4096, 4 heads, d=64, 95% sparsity
+    per row, i.e. ~205 non-zeros per row): F9-LS (local w=128 + 76 selected columns), F9-LSG
+    (local w=128 + 64 selected columns + 12 global tokens), F9-LBR (blocked local, 64-blocks,
+    + 141 random columns per row), F9-RBR (blocked random: each 64-row block attends to two
+    random 64-column blocks, + 77 random columns per row). Selected columns, random columns and
+    block choices are drawn from ``default_rng(seed)`` in a fixed order (see the builders).
   Paper context: local/global/selected/random atomic patterns, PAPER.md
   lines 64-71 (§2.3); Longformer = L+S+G, QDS = L+S.
 """
@@ -29,7 +39,8 @@ import numpy as np
 
 __all__ = [
     "Config", "CONFIGS", "get_config", "make_qkv", "to_bf16_bits", "to_fp16_bits",
-    "bits_to_f64", "random_residual", "qds_globals", "random_small_config",
+    "bits_to_f64", "random_residual", "qds_globals", "random_small_config", "selected_columns",
+    "blocked_pairs", "uniform_random_pairs", "EXTRA_WORKLOADS",
 ]
 
 
@@ -104,6 +115,68 @@ def random_residual(L: int, window: int, per_row: int, seed: int = 0) -> np.ndar
 _EMPTY_E = np.zeros((0, 2), dtype=np.int32)
 
 
+def selected_columns(L: int, cols: np.ndarray) -> np.ndarray:
+    """Column-only "selected" tokens (all-to-one): every row r attends to every c in cols."""
+    cols = np.asarray(cols, dtype=np.int32)
+    r = np.repeat(np.arange(L, dtype=np.int32), cols.size)
+    return np.stack([r, np.tile(cols, L)], axis=1).astype(np.int32)
+
+
+def blocked_pairs(L: int, block: int, col_blocks_of_row_block) -> np.ndarray:
+    """Blocked pattern: row block I attends all-to-all to each column block in
+    col_blocks_of_row_block(I)."""
+    out = []
+    nb = (L + block - 1) // block
+    for I in range(nb):
+        rows = np.arange(I * block, min(L, I * block + block), dtype=np.int32)
+        for J in col_blocks_of_row_block(I):
+            cols = np.arange(J * block, min(L, J * block + block), dtype=np.int32)
+            out.append(np.stack([np.repeat(rows, cols.size), np.tile(cols, rows.size)], axis=1))
+    return np.concatenate(out).astype(np.int32) if out else _EMPTY_E
+
+
+def uniform_random_pairs(L: int, per_row: int, seed: int) -> np.ndarray:
+    """Per row `per_row` distinct uniform columns over [0, L), drawn row by row (random pattern)."""
+    rng = np.random.default_rng(seed)
+    out = np.empty((L * per_row, 2), dtype=np.int32)
+    for r in range(L):
+        out[r * per_row:(r + 1) * per_row, 0] = r
+        out[r * per_row:(r + 1) * per_row, 1] = rng.choice(L, per_row, replace=False)
+    return out
+
+
+def _f9(name: str) -> "Config":
+    L, rng = 4096, np.random.default_rng(9)
+    if name == "F9-LS":
+        sel = np.sort(rng.choice(L, 76, replace=False))
+        return Config(name, 1, 4, L, 64, 128, np.zeros(0, np.int32), selected_columns(L, sel), 0,
+                      "Fig. 9 L+S: local w=128 + 76 selected columns, 95% sparsity per row")
+    if name == "F9-LSG":
+        sel = np.sort(rng.choice(L, 76, replace=False))
+        return Config(name, 1, 4, L, 64, 128, sel[:12].astype(np.int32), selected_columns(L, sel[12:]), 0,
+                      "Fig. 9 L+S+G: local w=128 + 64 selected columns + 12 global tokens")
+    if name == "F9-LBR":
+        E = np.concatenate([blocked_pairs(L, 64, lambda I: [I]), uniform_random_pairs(L, 141, seed=10)])
+        return Config(name, 1, 4, L, 64, 0, np.zeros(0, np.int32), E, 0,
+                      "Fig. 9 LB+R: blocked local (64-blocks) + 141 random columns per row")
+    if name == "F9-RBR":
+        nb = L // 64
+        picks = [np.sort(rng.choice(nb, 2, replace=False)) for _ in range(nb)]
+        E = np.concatenate([blocked_pairs(L, 64, lambda I: picks[I]), uniform_random_pairs(L, 77, seed=11)])
+        return Config(name, 1, 4, L, 64, 0, np.zeros(0, np.int32), E, 0,
+                      "Fig. 9 RB+R: two random 64-column blocks per 64-row block + 77 random columns")
+    raise KeyError(name)
+
+
+def _qds_ls() -> "Config":
+    L = 2048
+    return Config("QDS-LS", 8, 12, L, 64, 128, np.zeros(0, np.int32), selected_columns(L, qds_globals(L)), 0,
+                  "QDS-Transformer as L+S: w=128, 64 special tokens as column-only selected tokens, B=8")
+
+
+EXTRA_WORKLOADS = ("QDS-LS", "F9-LS", "F9-LSG", "F9-LBR", "F9-RBR")
+
+
 def _build_configs():
     c = {}
     c["C1"] = Config("C1", 1, 1, 512, 64, 64, np.array([0, 200], np.int32), _EMPTY_E, 0,
@@ -122,7 +195,12 @@ _C4_CACHE: dict = {}
 
 
 def get_config(name: str) -> Config:
-    """Return a BASELINE config by name (C1..C5). C4's residual is generated on first use (~1 s)."""
+    """Return a BASELINE config by name (C1..C5) or a paper-faithful extra workload (EXTRA_WORKLOADS).
+    C4's residual is generated on first use (~1 s)."""
+    if name in EXTRA_WORKLOADS:
+        if name not in _C4_CACHE:
+            _C4_CACHE[name] = _qds_ls() if name == "QDS-LS" else _f9(name)
+        return _C4_CACHE[name]
     if name == "C4":
         if "C4" not in _C4_CACHE:
             L = 16384
