@@ -79,11 +79,17 @@ struct mg_plan_s {
   // diagnostics: device event-trace buffer of the coarse kernel (CTA 0)
   unsigned long long* trace = nullptr;
   int32_t trace_cap = 0;
-  // profiling: 4 events per recorded call (start, after fine, after coarse, end)
+  // profiling: per recorded call as few events as the call's kernels need (every timing event is
+  // a point the stream must drain to, ~2-3 us each on B200, so a single-kernel call records 2):
+  //   serial: E0 [fine] E1 [coarse] E2 (E1 only with both kernels);
+  //   concurrent: E0 fork [fine on side] E1(side) [coarse] E2 join E3.
+  struct ProfCall {
+    int32_t first, last, fb, fe, cb, ce;   // event indices (-1: kernel absent)
+  };
   bool profiling = false;
   std::vector<cudaEvent_t> prof_events;
   size_t prof_used = 0;
-  std::vector<uint8_t> prof_has_fine, prof_has_coarse;
+  std::vector<ProfCall> prof_calls;
 
   cudaEvent_t prof_event() {
     if (prof_used == prof_events.size()) {
@@ -354,13 +360,20 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
     fstream = p->side;
   }
 
-  cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
+  // profiling events (see mg_plan_s::ProfCall)
+  const bool has_f = nf > 0, has_c = !h.items.empty();
+  mg_plan_s::ProfCall pc{-1, -1, -1, -1, -1, -1};
+  auto prof_rec = [&](cudaStream_t st) -> int32_t {
+    cudaEvent_t ev = p->prof_event();
+    if (!ev) return -1;
+    cudaEventRecord(ev, st);
+    return (int32_t)p->prof_used - 1;
+  };
   if (p->profiling) {
-    for (int i = 0; i < 4; ++i)
-      if (!(ev[i] = p->prof_event())) return fail(MG_ERR_CUDA, "cudaEventCreate failed");
-    p->prof_has_fine.push_back(nf > 0);
-    p->prof_has_coarse.push_back(!h.items.empty());
-    cudaEventRecord(ev[0], fstream);
+    pc.first = prof_rec(stream);
+    if (concurrent) cudaStreamWaitEvent(fstream, p->prof_events[pc.first], 0);
+    if (has_f) pc.fb = pc.first;
+    if (has_c && !has_f) pc.cb = pc.first;
   }
   if (nf > 0) {
     mg::FineParams fp{};
@@ -379,7 +392,14 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
     e = p->fine_kernel == 1 ? mg::launch_fine(fp, bf16, fstream) : mg::launch_fine_mma(fp, bf16, fstream);
     if (e != cudaSuccess) return cuda_fail(e, "fine kernel launch");
   }
-  if (p->profiling) cudaEventRecord(ev[1], fstream);
+  if (p->profiling && has_f) {
+    if (concurrent) {
+      pc.fe = prof_rec(fstream);
+      pc.cb = pc.first;
+    } else if (has_c) {
+      pc.fe = pc.cb = prof_rec(stream);
+    }
+  }
   if (!h.items.empty()) {
     CUtensorMap tq, tk, tv;
     if (!encode_map(&tq, Q) || !encode_map(&tk, K) || !encode_map(&tv, V))
@@ -421,7 +441,6 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
       return cuda_fail(e, "cudaMemsetAsync");
     const int sms = p->num_sms_override > 0 ? std::min(p->num_sms_override, p->num_sms) : p->num_sms;
     // MG_COARSE=v13 selects the previous single-CTA-per-SM kernel (A/B measurements only)
-    if (p->profiling) cudaEventRecord(ev[2], stream);  // after the counter reset
     if (v13) {
       if ((e = mg::launch_coarse(cp, tq, tk, tv, bf16, std::min(sms, cp.total_units), stream)) != cudaSuccess)
         return cuda_fail(e, "coarse kernel launch");
@@ -437,15 +456,20 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
                                     stream)) != cudaSuccess)
         return cuda_fail(e, "coarse kernel launch");
     }
-  } else if (p->profiling) {
-    cudaEventRecord(ev[2], stream);
   }
+  if (p->profiling && concurrent) pc.ce = prof_rec(stream);
   if (concurrent) {
     if ((e = cudaEventRecord(p->join_ev, fstream)) != cudaSuccess ||
         (e = cudaStreamWaitEvent(stream, p->join_ev, 0)) != cudaSuccess)
       return cuda_fail(e, "stream join");
   }
-  if (p->profiling) cudaEventRecord(ev[3], stream);
+  if (p->profiling) {
+    pc.last = prof_rec(stream);
+    if (has_f && pc.fe < 0) pc.fe = pc.last;
+    if (has_c && pc.ce < 0) pc.ce = pc.last;
+    if (pc.first < 0 || pc.last < 0) return fail(MG_ERR_CUDA, "cudaEventCreate failed");
+    p->prof_calls.push_back(pc);
+  }
   return MG_OK;
 }
 
@@ -767,8 +791,7 @@ mg_status mg_plan_set_profiling(mg_plan_t plan, int32_t enable) {
   if (!plan) return fail(MG_ERR_INVALID_ARG, "plan is null");
   plan->profiling = enable != 0;
   plan->prof_used = 0;
-  plan->prof_has_fine.clear();
-  plan->prof_has_coarse.clear();
+  plan->prof_calls.clear();
   return MG_OK;
 }
 
@@ -776,23 +799,21 @@ mg_status mg_plan_get_profile(mg_plan_t plan, mg_profile* out) {
   g_err.clear();
   if (!plan || !out) return fail(MG_ERR_INVALID_ARG, "null argument");
   std::memset(out, 0, sizeof(*out));
-  const size_t calls = plan->prof_used / 4;
-  for (size_t c = 0; c < calls; ++c) {
-    cudaEvent_t* ev = plan->prof_events.data() + 4 * c;
-    cudaError_t e = cudaEventSynchronize(ev[3]);
+  auto ms = [&](int32_t a, int32_t b) {
+    float t = 0.f;
+    if (a >= 0 && b >= 0) cudaEventElapsedTime(&t, plan->prof_events[a], plan->prof_events[b]);
+    return (double)t;
+  };
+  for (const auto& c : plan->prof_calls) {
+    cudaError_t e = cudaEventSynchronize(plan->prof_events[c.last]);
     if (e != cudaSuccess) return cuda_fail(e, "cudaEventSynchronize");
-    float a = 0.f, b = 0.f, t = 0.f;
-    cudaEventElapsedTime(&a, ev[0], ev[1]);
-    cudaEventElapsedTime(&b, ev[2], ev[3]);
-    cudaEventElapsedTime(&t, ev[0], ev[3]);
-    if (plan->prof_has_fine[c]) out->fine_ms += a;
-    if (plan->prof_has_coarse[c]) out->coarse_ms += b;
-    out->total_ms += t;
+    out->fine_ms += ms(c.fb, c.fe);
+    out->coarse_ms += ms(c.cb, c.ce);
+    out->total_ms += ms(c.first, c.last);
   }
-  out->calls = (int64_t)calls;
+  out->calls = (int64_t)plan->prof_calls.size();
   plan->prof_used = 0;
-  plan->prof_has_fine.clear();
-  plan->prof_has_coarse.clear();
+  plan->prof_calls.clear();
   return MG_OK;
 }
 

@@ -220,7 +220,8 @@ def sample_rows(L, G, rng, n=48):
 
 
 @pytest.mark.parametrize("cfg,fine_kernel,concurrency", [("C2", 0, 0), ("C3", 0, 0), ("C4", 0, 1), ("C4", 0, 2),
-                                                          ("C4", 1, 1)])
+                                                          ("C4", 1, 1), ("QDS-LS", 0, 0), ("F9-LS", 0, 0),
+                                                          ("F9-LSG", 0, 0), ("F9-LBR", 0, 0), ("F9-RBR", 0, 0)])
 def test_full_size_sampled(cfg, fine_kernel, concurrency):
     c = get_config(cfg)
     q, k, v = make_qkv(c.B, c.H, c.L, c.d, seed=c.seed)

@@ -1,0 +1,54 @@
+"""Paper-faithful extra workloads: the recipes produce the patterns the paper
+describes, and the C-ABI plan of each is bit-identical to the oracle's canonical plan (no GPU).
+
+* Fig. 9: batch 1, L = 4096, 4 heads, d = 64, "95% sparsity in each row";
+* QDS-Transformer = local + selected, selected tokens all-to-one, and the window
+  whose 64-blocks give P:185's 2:1 sparse:dense block ratio.
+"""
+import numpy as np
+import pytest
+
+import paper_conf_iiswc_lica22_b200 as mg
+from oracle import ExtraIndex, canonical_plan, global_flags, mask_row_cols
+from workloads import EXTRA_WORKLOADS, get_config, qds_globals
+
+
+def row_nnz(c, rows):
+    g = global_flags(c.L, c.global_idx)
+    ex = ExtraIndex(c.L, c.extra_idx)
+    return np.array([mask_row_cols(r, c.L, c.window, g, ex).size for r in rows])
+
+
+@pytest.mark.parametrize("name", ["F9-LS", "F9-LSG", "F9-LBR", "F9-RBR"])
+def test_fig9_shape_and_row_sparsity(name):
+    c = get_config(name)
+    assert (c.B, c.H, c.L, c.d) == (1, 4, 4096, 64)
+    rows = np.arange(0, c.L, 37)
+    g = set(np.asarray(c.global_idx).tolist())
+    rows = np.array([r for r in rows if r not in g])
+    dens = row_nnz(c, rows) / c.L
+    # 95% sparsity per row (5% density), up to the overlaps of the random draws with the rest
+    assert 0.046 <= dens.mean() <= 0.051, dens.mean()
+    assert dens.min() >= 0.03 and dens.max() <= 0.06   # edge rows have a one-sided band
+
+
+def test_qds_ls_selected_columns_all_to_one():
+    c = get_config("QDS-LS")
+    sel = qds_globals(c.L)
+    assert len(c.global_idx) == 0 and c.window == 128
+    for r in (0, 1, 500, 1999, 2047):
+        cols = set(mask_row_cols(r, c.L, c.window, global_flags(c.L, c.global_idx), ExtraIndex(c.L, c.extra_idx)).tolist())
+        assert set(sel.tolist()) <= cols
+    # w = 128 with 64-blocks gives sparse:dense band blocks of about 2:1
+    p = canonical_plan(c.L, c.window, c.global_idx, np.zeros((0, 2), np.int32), 64)
+    full = p.n_full_tiles()
+    assert 1.7 <= (p.n_tiles - full) / full <= 2.3
+
+
+@pytest.mark.parametrize("name", EXTRA_WORKLOADS)
+def test_extra_workload_plan_bit_exact(name):
+    c = get_config(name)
+    ref = canonical_plan(c.L, c.window, c.global_idx, c.extra_idx, 128)
+    got = mg.Plan(c.L, c.H, c.d, c.window, c.global_idx, c.extra_idx).export()
+    for f in ("bsr_row_ptr", "bsr_col", "tile_masks", "csr_row_ptr", "csr_col", "global_rows"):
+        assert np.array_equal(got[f], getattr(ref, f)), f
