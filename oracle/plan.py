@@ -11,7 +11,10 @@ Integer-exact rules (readings A4-A7), block b:
 
 * global_rows = sorted unique G.
 * T = {(I, J) : exists r in [Ib, Ib+b) \\ G, c in [Jb, Jb+b), |r-c| <= w/2}
-  (every tile touched by the band of a non-global row is coarse; tau = 0).
+  (every tile touched by the band of a non-global row is coarse; tau = 0), or, with a density
+  threshold tau > 0 (reading A17: "sparse blocks with low sparsity"
+  favour the fine kernel, dense blocks the coarse one),
+  T = {(I, J) : #{(r, c) in tile : M(r, c), r not in G} >= tau * b * b}.
 * BSR: bsr_row_ptr[nb+1], bsr_col[] ascending J within each row block.
 * tile mask bit (a, beta) = M(Ib+a, Jb+beta) AND NOT G[Ib+a], zero outside [0, L);
   row-major, ceil(b/64) uint64 words per tile row, LSB = lowest column.
@@ -61,6 +64,8 @@ class CanonicalPlan:
         return np.unpackbits(by, axis=1, bitorder="little").astype(bool)[:, :b]
 
     def tile_popcount(self) -> np.ndarray:
+        if self.n_tiles == 0:
+            return np.zeros(0, dtype=np.int64)
         by = self.tile_masks.reshape(self.n_tiles, -1).view(np.uint8)
         return np.unpackbits(by, axis=1).sum(axis=1)
 
@@ -68,9 +73,12 @@ class CanonicalPlan:
         return int((self.tile_popcount() == self.block * self.block).sum())
 
 
-def canonical_plan(L: int, window: int, global_idx, extra_idx, block: int = 128) -> CanonicalPlan:
+def canonical_plan(L: int, window: int, global_idx, extra_idx, block: int = 128,
+                   tau: float = 0.0) -> CanonicalPlan:
     if block < 1 or (block > 64 and block % 64):
         raise ValueError("block must be <= 64 or a multiple of 64")
+    if not 0.0 <= tau <= 1.0:
+        raise ValueError("tau must be in [0, 1]")
     b = block
     wpr = _words_per_row(b)
     w1 = window // 2
@@ -85,15 +93,20 @@ def canonical_plan(L: int, window: int, global_idx, extra_idx, block: int = 128)
     csr_cols = []
     for I in range(nb):
         r0, r1 = I * b, min(I * b + b, L)
-        # Tile set of this row block: band of every non-global row.
-        in_T = np.zeros(nb, dtype=bool)
-        for r in range(r0, r1):
-            if g[r]:
-                continue
-            in_T[max(0, r - w1) // b: min(L - 1, r + w1) // b + 1] = True
-        Js = np.nonzero(in_T)[0]
         M = mask_rows(r0, r1, L, window, g, extra)          # (r1-r0) x L
         Mc = M & ~g[r0:r1, None]                            # global rows leave tiles and CSR
+        in_T = np.zeros(nb, dtype=bool)
+        if tau == 0.0:
+            # Tile set of this row block: band of every non-global row.
+            for r in range(r0, r1):
+                if g[r]:
+                    continue
+                in_T[max(0, r - w1) // b: min(L - 1, r + w1) // b + 1] = True
+        else:
+            # Tile set by density: union elements of non-global rows in the tile >= tau * b^2.
+            for J in range(nb):
+                in_T[J] = Mc[:, J * b: min(J * b + b, L)].sum() >= tau * b * b
+        Js = np.nonzero(in_T)[0]
         for J in Js:
             c0, c1 = J * b, min(J * b + b, L)
             bits = np.zeros((b, wpr * 64), dtype=bool)

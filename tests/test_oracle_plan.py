@@ -252,3 +252,56 @@ def test_c4_counts():
     # exact for any seed: band + 164 per row (the residual is drawn outside the band)
     assert p.tile_popcount().sum() + p.csr_col.size == band_nnz(c.L, 256) + 164 * c.L == 11_026_176
     assert p.n_tiles == 634 and p.n_full_tiles() == 382
+
+
+# ---------------------------------------------------------------- density threshold tau (f-2)
+def _tau_brute(L, window, G, E, b, tau):
+    """Independent tile classification by density, straight from the union mask."""
+    M = union_mask_dense(L, window, G, E)
+    g = np.zeros(L, bool)
+    g[np.asarray(G, dtype=np.int64)] = True
+    Mc = M & ~g[:, None]
+    nb = -(-L // b)
+    T = set()
+    for I in range(nb):
+        for J in range(nb):
+            if Mc[I * b:(I + 1) * b, J * b:(J + 1) * b].sum() >= tau * b * b:
+                T.add((I, J))
+    return Mc, T
+
+
+@pytest.mark.parametrize("seed", range(12))
+@pytest.mark.parametrize("tau", [0.05, 0.3, 0.75, 1.0])
+def test_tau_plan_brute_force(seed, tau):
+    rng = np.random.default_rng(100 + seed)
+    L, window, G, E = random_small_config(rng, 64)
+    b = int(rng.choice([2, 4, 8]))
+    p = canonical_plan(L, window, G, E, b, tau=tau)
+    Mc, T = _tau_brute(L, window, G, E, b, tau)
+    got_T = {(I, int(J)) for I in range(p.nb) for J in p.bsr_col[p.bsr_row_ptr[I]:p.bsr_row_ptr[I + 1]]}
+    assert got_T == T
+    # every union element of a non-global row is in exactly one part
+    rebuilt = np.zeros_like(Mc)
+    for t in range(p.n_tiles):
+        I = int(np.searchsorted(p.bsr_row_ptr, t, side="right") - 1)
+        J = int(p.bsr_col[t])
+        bits = p.tile_bits(t)
+        r1, c1 = min(b, L - I * b), min(b, L - J * b)
+        assert not (rebuilt[I * b:I * b + r1, J * b:J * b + c1] & bits[:r1, :c1]).any()
+        rebuilt[I * b:I * b + r1, J * b:J * b + c1] |= bits[:r1, :c1]
+        assert not bits[r1:].any() and not bits[:, c1:].any()
+    for r in range(L):
+        cols = p.csr_col[p.csr_row_ptr[r]:p.csr_row_ptr[r + 1]]
+        assert not rebuilt[r, cols].any()
+        rebuilt[r, cols] = True
+    assert np.array_equal(rebuilt, Mc)
+
+
+def test_tau_one_keeps_only_full_tiles_and_band_rule_differs():
+    c = get_config("C1")
+    p1 = canonical_plan(c.L, c.window, c.global_idx, c.extra_idx, 64, tau=1.0)
+    assert p1.n_tiles == p1.n_full_tiles()
+    p0 = canonical_plan(c.L, c.window, c.global_idx, c.extra_idx, 64)
+    # C1 at b=64 has no full tile (SURVEY Appendix A): tau = 1 leaves everything to the CSR
+    assert p0.n_full_tiles() == 0 and p1.n_tiles == 0
+    assert p1.csr_col.size == p0.tile_popcount().sum() + p0.csr_col.size
