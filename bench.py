@@ -49,6 +49,7 @@ def parse():
                     help="also time the staged paper-dataflow forward (mg_sparse_attention_fwd_staged)")
     ap.add_argument("--concurrency", type=int, default=0, choices=[0, 1, 2],
                     help="coarse vs CSR kernels: 0 = library default, 1 = serial, 2 = concurrent streams")
+    ap.add_argument("--tau", type=float, default=0.0, help="tile density threshold (0 = band rule)")
     ap.add_argument("--fine-kernel", type=int, default=0, choices=[0, 1],
                     help="CSR rows: 0 = warp-level tensor-core kernel, 1 = CUDA-core kernel (A/B)")
     return ap.parse_args()
@@ -242,7 +243,7 @@ def main():
     cfg = get_config(args.workload)
     plan = mg.Plan(cfg.L, cfg.H, cfg.d, cfg.window, cfg.global_idx, cfg.extra_idx,
                    strip_max_cols=args.strip_max_cols, fine_kernel=args.fine_kernel,
-                   concurrency=args.concurrency)
+                   concurrency=args.concurrency, tau=args.tau)
     info = plan.info()
     BH = cfg.B * cfg.H
     useful = 4.0 * info["nnz_total"] * cfg.d * BH

@@ -93,7 +93,8 @@ typedef struct {
  * residual; global rows are dense and owned by the dense-row part.
  * If a CUDA device is present the metadata is uploaded synchronously to the current device;
  * otherwise the upload is deferred to the first forward call.
- * Errors: INVALID_ARG (L <= 0, heads <= 0, d <= 0, window < 0 or odd, index out of range,
+ * Errors: INVALID_ARG (L <= 0, heads <= 0, d <= 0, window < 0 or odd, index out of range, tau
+ * outside [0, 1],
  * null array with a non-zero count, null plan), UNSUPPORTED (d != 64, CSR nnz >= 2^31),
  * OUT_OF_MEMORY, CUDA.
  * ---------------------------------------------------------------------------------- */
@@ -115,7 +116,10 @@ typedef struct {
   int32_t concurrency;    /* coarse vs CUDA-core CSR kernels: 0 -> library default, 1 -> serial (fine
                              kernel, then coarse kernel merging its partials), 2 -> concurrent on two
                              streams, rows merged by whichever side finishes second */
-  int32_t reserved[2];
+  float tau;              /* tile rule: 0 -> every tile touched by the band of a non-global row is
+                             coarse (default, A7); (0, 1] -> a tile is coarse iff its
+                             non-global union elements number >= tau * block^2 (A17) */
+  int32_t reserved[1];
 } mg_plan_opts;
 
 MG_API mg_status mg_plan_create_ex(int64_t L, int32_t heads, int32_t d, int32_t window,

@@ -169,6 +169,8 @@ mg_status create_impl(int64_t L, int32_t heads, int32_t d, int32_t window, const
     fine_kernel = opts->fine_kernel;
     if (opts->concurrency < 0 || opts->concurrency > 2) return fail(MG_ERR_INVALID_ARG, "concurrency must be 0, 1 or 2");
     concurrency = opts->concurrency;
+    if (!(opts->tau >= 0.f && opts->tau <= 1.f)) return fail(MG_ERR_INVALID_ARG, "tau must be in [0, 1]");
+    po.tau = opts->tau;
   }
   mg_plan_s* p = new (std::nothrow) mg_plan_s();
   if (!p) return fail(MG_ERR_OUT_OF_MEMORY, "host allocation failed");

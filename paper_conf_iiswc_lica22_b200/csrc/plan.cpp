@@ -3,7 +3,8 @@
 // Canonical partition (must be bit-identical to oracle/plan.py; readings A2-A7):
 //   M(r,c) = |r-c| <= w/2 or G[r] or G[c] or (r,c) in E
 //   T = {(I,J): some non-global r in row block I has band columns in column block J}
-//       ("local pattern -> coarse BSR"; tau = 0)
+//       ("local pattern -> coarse BSR"; tau = 0), or with tau > 0 (A17)
+//   T = {(I,J): #non-global union elements in the tile >= tau * b^2}
 //   tile bits = M restricted to the tile, global rows cleared
 //   CSR = non-global union elements outside T ("selected -> fine CSR")
 #include "plan.hpp"
@@ -33,6 +34,7 @@ std::string build_plan(HostPlan& p, int64_t L, int32_t heads, int32_t d, int32_t
   if (n_extra > 0 && !extra_idx) return "extra_idx is null";
   const int b = opts.block;
   if (b < 1 || (b > 64 && b % 64) || b > 1024) return "block must be <= 64 or a multiple of 64 (<= 1024)";
+  if (!(opts.tau >= 0.0 && opts.tau <= 1.0)) return "tau must be in [0, 1]";
   if (d != 64) { *unsupported = true; return "v1 supports head_dim == 64 only"; }
   for (int64_t i = 0; i < n_global; ++i)
     if (global_idx[i] < 0 || global_idx[i] >= L) return "global index out of range";
@@ -64,26 +66,56 @@ std::string build_plan(HostPlan& p, int64_t L, int32_t heads, int32_t d, int32_t
   std::vector<int32_t> tile_of_J(nb, -1);
   std::vector<int64_t> csr_ptr(L + 1, 0);
   p.bsr_row_ptr.push_back(0);
-  std::vector<int32_t> outside;  // scratch: sorted off-band columns of one row
+  std::vector<std::vector<int32_t>> outs(b);   // off-band union columns of each row of the block
+  std::vector<int64_t> cnt(nb, 0);
   for (int64_t I = 0; I < nb; ++I) {
     const int64_t r0 = I * b, r1 = std::min<int64_t>(L, r0 + b);
+    // off-band columns from globals and extras, merged ascending, unique
+    for (int64_t r = r0; r < r1; ++r) {
+      std::vector<int32_t>& outside = outs[r - r0];
+      outside.clear();
+      if (isG[r]) continue;
+      const int64_t lo = std::max<int64_t>(0, r - w1), hi = std::min<int64_t>(L - 1, r + w1);
+      size_t gi = 0;
+      int64_t ei = ext_ptr[r], ee = ext_ptr[r + 1];
+      while (gi < gcols.size() || ei < ee) {
+        int64_t c;
+        if (ei >= ee || (gi < gcols.size() && gcols[gi] <= keys[ei] % L)) {
+          c = gcols[gi++];
+          if (ei < ee && keys[ei] % L == c) ++ei;
+        } else {
+          c = keys[ei++] % L;
+        }
+        if (c < lo || c > hi) outside.push_back((int32_t)c);
+      }
+    }
     std::vector<uint8_t> inT(nb, 0);
-    if (!opts.force_all_fine) {
+    if (!opts.force_all_fine && opts.tau <= 0.0) {
       for (int64_t r = r0; r < r1; ++r) {
         if (isG[r]) continue;
         const int64_t jlo = std::max<int64_t>(0, r - w1) / b;
         const int64_t jhi = std::min<int64_t>(L - 1, r + w1) / b;
         for (int64_t J = jlo; J <= jhi; ++J) inT[J] = 1;
       }
+    } else if (!opts.force_all_fine) {
+      // density rule: count the union elements of the block's non-global rows per column block
+      std::fill(cnt.begin(), cnt.end(), 0);
+      for (int64_t r = r0; r < r1; ++r) {
+        if (isG[r]) continue;
+        const int64_t lo = std::max<int64_t>(0, r - w1), hi = std::min<int64_t>(L - 1, r + w1);
+        for (int64_t J = lo / b; J <= hi / b; ++J)
+          cnt[J] += std::min<int64_t>(hi, J * b + b - 1) - std::max<int64_t>(lo, J * b) + 1;
+        for (int32_t c : outs[r - r0]) cnt[c / b]++;
+      }
+      const double thr = opts.tau * (double)b * (double)b;
+      for (int64_t J = 0; J < nb; ++J) inT[J] = (double)cnt[J] >= thr;
     }
-    const int64_t tbase = (int64_t)p.bsr_col.size();
     for (int64_t J = 0; J < nb; ++J) {
       tile_of_J[J] = -1;
       if (inT[J]) { tile_of_J[J] = (int32_t)p.bsr_col.size(); p.bsr_col.push_back((int32_t)J); }
     }
     p.bsr_row_ptr.push_back((int32_t)p.bsr_col.size());
     p.tile_masks.resize(p.bsr_col.size() * (size_t)b * wpr, 0ull);
-    (void)tbase;
 
     for (int64_t r = r0; r < r1; ++r) {
       if (isG[r]) continue;  // global rows: owned by the dense-row part
@@ -100,20 +132,7 @@ std::string build_plan(HostPlan& p, int64_t L, int32_t heads, int32_t d, int32_t
         }
       };
       const int64_t lo = std::max<int64_t>(0, r - w1), hi = std::min<int64_t>(L - 1, r + w1);
-      // off-band columns from globals and extras, merged ascending, unique
-      outside.clear();
-      size_t gi = 0;
-      int64_t ei = ext_ptr[r], ee = ext_ptr[r + 1];
-      while (gi < gcols.size() || ei < ee) {
-        int64_t c;
-        if (ei >= ee || (gi < gcols.size() && gcols[gi] <= keys[ei] % L)) {
-          c = gcols[gi++];
-          if (ei < ee && keys[ei] % L == c) ++ei;
-        } else {
-          c = keys[ei++] % L;
-        }
-        if (c < lo || c > hi) outside.push_back((int32_t)c);
-      }
+      const std::vector<int32_t>& outside = outs[a];
       // emit in ascending column order: outside-left, band, outside-right
       size_t oi = 0;
       while (oi < outside.size() && outside[oi] < lo) take(outside[oi++]);

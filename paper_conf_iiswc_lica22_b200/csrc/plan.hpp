@@ -14,6 +14,7 @@ struct PlanOptions {
   int block = 128;
   bool force_all_fine = false;
   int strip_max_cols = 128;  // <= 0 disables the tensor-core strip path for the CSR residual
+  double tau = 0.0;          // 0: band rule; > 0: a tile is coarse iff its density >= tau (A17)
 };
 
 // Device work-list encodings. The tensor-core kernel processes one 128-row

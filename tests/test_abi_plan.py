@@ -35,8 +35,8 @@ def test_library_loads_and_exports_header_symbols():
     assert lib.mg_abi_version() == 1
 
 
-def compare(plan: "mg.Plan", L, window, G, E, b):
-    ref = canonical_plan(L, window, G, E, b)
+def compare(plan: "mg.Plan", L, window, G, E, b, tau=0.0):
+    ref = canonical_plan(L, window, G, E, b, tau=tau)
     got = plan.export()
     assert np.array_equal(got["bsr_row_ptr"], ref.bsr_row_ptr)
     assert np.array_equal(got["bsr_col"], ref.bsr_col)
@@ -134,6 +134,8 @@ def status_of(fn):
     (dict(L=64, heads=1, d=128, window=2), _lib.MG_ERR_UNSUPPORTED),
     (dict(L=64, heads=1, d=64, window=2, block=96), _lib.MG_ERR_INVALID_ARG),
     (dict(L=64, heads=1, d=64, window=2, strip_max_cols=256), _lib.MG_ERR_INVALID_ARG),
+    (dict(L=64, heads=1, d=64, window=2, tau=1.5), _lib.MG_ERR_INVALID_ARG),
+    (dict(L=64, heads=1, d=64, window=2, tau=-0.1), _lib.MG_ERR_INVALID_ARG),
 ])
 def test_plan_create_validation(kwargs, status):
     assert status_of(lambda: mg.Plan(**kwargs)) == status
@@ -160,3 +162,30 @@ def test_duplicates_collapse():
     a, b = p1.export(), p2.export()
     for k in a:
         assert np.array_equal(a[k], b[k]), k
+
+
+# ---------------------------------------------------------------- density threshold tau (f-2)
+def f32(x):
+    """tau as the C ABI sees it (mg_plan_opts.tau is a float)."""
+    return float(np.float32(x))
+
+
+@pytest.mark.parametrize("seed", range(16))
+@pytest.mark.parametrize("tau", [0.05, 0.25, 0.5, 1.0])
+def test_tau_plan_export_matches_oracle_random(seed, tau):
+    rng = np.random.default_rng(500 + seed)
+    L, window, G, E = random_small_config(rng, 64)
+    b = int(rng.choice([2, 4, 8, 16]))
+    plan = mg.Plan(L, 1, 64, window, G, E, block=b, tau=tau)
+    compare(plan, L, window, G, E, b, tau=f32(tau))
+
+
+@pytest.mark.parametrize("cfg,tau", [("C1", 0.1), ("C1", 0.6), ("C3", 0.3), ("F9-RBR", 0.2), ("F9-LBR", 0.2),
+                                     ("QDS-LS", 0.5)])
+def test_tau_plan_export_matches_oracle_configs(cfg, tau):
+    c = get_config(cfg)
+    plan = mg.Plan(c.L, c.H, c.d, c.window, c.global_idx, c.extra_idx, tau=tau)
+    inf = compare(plan, c.L, c.window, c.global_idx, c.extra_idx, 128, tau=f32(tau))
+    if cfg == "F9-RBR":
+        # the 64 x 64 random blocks (25% of a 128-tile) become coarse at tau = 0.2
+        assert inf["nnz_coarse"] > 64 * 64 * 64

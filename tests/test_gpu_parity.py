@@ -109,6 +109,20 @@ def test_fine_rows_all_lengths(fine_kernel, concurrency, dtype, dist):
         check(got, ref, tol_max=2e-2 * max(1.0, np.abs(ref).max() / 4))
 
 
+@pytest.mark.parametrize("tau", [0.1, 0.5, 1.0])
+def test_density_threshold_plans(tau):
+    """tau > 0 tile rule (A17): band-edge tiles below the threshold move to the CSR part, dense
+    random blocks become coarse; every part still runs and merges correctly."""
+    L, G = 1024, np.array([3, 600], np.int32)
+    rng = np.random.default_rng(4)
+    blocks = [(int(rng.integers(0, 16)), int(rng.integers(0, 16))) for _ in range(10)]
+    E = np.array([(I * 64 + a, J * 64 + c) for I, J in blocks for a in range(64) for c in range(64)], np.int32)
+    E = np.concatenate([E, random_residual(L, 96, 5, seed=6)])
+    q, k, v = make_qkv(2, 2, L, 64, seed=13, dist="adversarial", global_idx=G)
+    plan = mg.Plan(L, 2, 64, 96, G, E, tau=tau)
+    check(run_gpu(plan, q, k, v), oracle_full(q, k, v, 96, G, E))
+
+
 def test_strip_path_c2_pattern_small():
     """C2-like globals [0, 32) with fewer blocks: the CSR residual runs as tensor-core strips."""
     L, G = 1024, np.arange(32, dtype=np.int32)
@@ -221,12 +235,15 @@ def sample_rows(L, G, rng, n=48):
 
 @pytest.mark.parametrize("cfg,fine_kernel,concurrency", [("C2", 0, 0), ("C3", 0, 0), ("C4", 0, 1), ("C4", 0, 2),
                                                           ("C4", 1, 1), ("QDS-LS", 0, 0), ("F9-LS", 0, 0),
-                                                          ("F9-LSG", 0, 0), ("F9-LBR", 0, 0), ("F9-RBR", 0, 0)])
+                                                          ("F9-LSG", 0, 0), ("F9-LBR", 0, 0), ("F9-RBR", 0, 0),
+                                                          ("F9-RBR", 0, 0.2)])
 def test_full_size_sampled(cfg, fine_kernel, concurrency):
     c = get_config(cfg)
     q, k, v = make_qkv(c.B, c.H, c.L, c.d, seed=c.seed)
+    # (a float in the concurrency column is a tau for the density tile rule, with the default mode)
+    tau = concurrency if isinstance(concurrency, float) else 0.0
     plan = mg.Plan(c.L, c.H, c.d, c.window, c.global_idx, c.extra_idx, fine_kernel=fine_kernel,
-                   concurrency=concurrency)
+                   concurrency=0 if tau else concurrency, tau=tau)
     got = run_gpu(plan, q, k, v)
     assert np.isfinite(got).all()
     rng = np.random.default_rng(17)
