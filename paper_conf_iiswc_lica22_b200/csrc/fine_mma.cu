@@ -60,20 +60,45 @@ __device__ __forceinline__ uint32_t pack2(float lo, float hi) {
   return kBF16 ? pack_bf16(lo, hi) : pack_f16(lo, hi);
 }
 
-// the gathered rows of one 16-nnz step
-struct Step {
-  int4 k[4];   // K rows of chunk A nnz g (k[0], k[1]) and chunk B nnz g (k[2], k[3])
-  int4 v[4];   // V rows of nnz A 2t, A 2t+1, B 2t, B 2t+1 (dims 8g..8g+7)
-};
+__device__ __forceinline__ void cp_async16(uint32_t dst, const void* src) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dst), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() {
+  asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
+}
+__device__ __forceinline__ void ldsm_x4(uint32_t (&r)[4], uint32_t addr) {
+  asm volatile("ldmatrix.sync.aligned.m8n8.x4.shared.b16 {%0,%1,%2,%3}, [%4];"
+               : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3])
+               : "r"(addr));
+}
+__device__ __forceinline__ void ldsm_x4_t(uint32_t (&r)[4], uint32_t addr) {
+  asm volatile("ldmatrix.sync.aligned.m8n8.x4.trans.shared.b16 {%0,%1,%2,%3}, [%4];"
+               : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3])
+               : "r"(addr));
+}
+
+#ifndef MG_FINE_STAGES
+#define MG_FINE_STAGES 3
+#endif
+constexpr int kWarps = 4;                   // warps per block, one (row, b*h) each
+constexpr int kStages = MG_FINE_STAGES;     // smem ring stages per warp (kStages - 1 steps in flight)
+constexpr int kStageBytes = 32 * 128;       // 16 K rows + 16 V rows of 128 bytes
+constexpr int kSmemBytes = kWarps * kStages * kStageBytes;
 
 }  // namespace
 
-// The gathers of step i+1 are issued into registers before step i is computed (one step in flight
-// per warp, 16 warps per SM). A shared-memory ring filled by cp.async measured 6x slower: cp.async
-// of 16-byte pieces that cover only part of a 128-byte line per instruction is pathological on
-// sm_100 (tools/microbench/gather_bw.cu: 2.4 TB/s vs 17.6 TB/s for the same loads into registers).
+// The 16 K rows and 16 V rows of a step are gathered with cp.async into a warp-private shared-memory
+// ring, kStages - 1 steps ahead of the computation: 8 lanes copy one full 128-byte row per
+// instruction (the pattern the L2 serves at ~15 TB/s through cp.async; partial-line pieces are 6x
+// slower, tools/microbench/gather_bw.cu), and the copies hold no registers while in flight. Rows
+// are stored with the 16-byte-chunk XOR swizzle (chunk c of row r at (c ^ (r & 7)) * 16), and the
+// MMA fragments come from ldmatrix: non-transposed for the SDDMM's B operand (K rows = columns n,
+// dims = k), transposed for the SpMM's A operand (V^T: dims = rows m, nnz = k).
 template <bool kBF16>
-__global__ void __launch_bounds__(256, 2) fine_mma_kernel(const FineParams p) {
+__global__ void __launch_bounds__(kWarps * 32) fine_mma_kernel(const FineParams p) {
+  extern __shared__ __align__(128) uint8_t fsm[];
   const int lane = threadIdx.x & 31;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   if (gw >= (int64_t)p.BH * p.n_fine_rows) return;
@@ -85,38 +110,50 @@ __global__ void __launch_bounds__(256, 2) fine_mma_kernel(const FineParams p) {
   const int bb = bh / p.H, hh = bh % p.H;
   const int g = lane >> 2, t = lane & 3;
   const float c = p.scale_log2;
+  const uint32_t ring = (uint32_t)__cvta_generic_to_shared(fsm) + (threadIdx.x >> 5) * (kStages * kStageBytes);
 
-  const uint16_t* Kb = p.k.data + bb * p.k.sb + hh * p.k.sh + t * 8;   // + 32 for the second half
-  const uint16_t* Vb = p.v.data + bb * p.v.sb + hh * p.v.sh + g * 8;
-  const uint16_t* qrow = p.q.data + bb * p.q.sb + hh * p.q.sh + (int64_t)r * p.q.sl + t * 8;
-  const int4 q0 = ld_nc_v4(qrow), q1 = ld_nc_v4(qrow + 32);
-  const uint32_t qr[8] = {(uint32_t)q0.x, (uint32_t)q0.y, (uint32_t)q0.z, (uint32_t)q0.w,
-                          (uint32_t)q1.x, (uint32_t)q1.y, (uint32_t)q1.z, (uint32_t)q1.w};
-
+  // q as the SDDMM's A operand (every row = q): k16 step j uses dims 16j + 2t (+1) and 16j + 8 + 2t (+1)
+  const uint16_t* qrow = p.q.data + bb * p.q.sb + hh * p.q.sh + (int64_t)r * p.q.sl;
+  uint32_t qa[4], qb[4];
+#pragma unroll
+  for (int j = 0; j < 4; ++j) {
+    qa[j] = __ldg(reinterpret_cast<const uint32_t*>(qrow + 16 * j + 2 * t));
+    qb[j] = __ldg(reinterpret_cast<const uint32_t*>(qrow + 16 * j + 8 + 2 * t));
+  }
+  const uint16_t* Kb = p.k.data + bb * p.k.sb + hh * p.k.sh + (lane & 7) * 8;
+  const uint16_t* Vb = p.v.data + bb * p.v.sb + hh * p.v.sh + (lane & 7) * 8;
   const int beg = __ldg(p.row_ptr + fi), end = __ldg(p.row_ptr + fi + 1);
   // row strides fit 32 bits (checked by the forward's validation: (L - 1) * stride_l < 2^32)
   const uint32_t ksl = (uint32_t)p.k.sl, vsl = (uint32_t)p.v.sl;
 
-  // step loader: the 16 column indices of a step come from `col` (lane i holds index base0 + i of
-  // a 32-index window; `off` = 0 or 16 selects the half). Indices past the row's end are -1 and
-  // read row 0 (the values are masked / multiplied by p = 0).
-  auto load_step = [&](Step& st, int col, int off) {
-    const int ca = __shfl_sync(0xffffffffu, col, off + g), cb = __shfl_sync(0xffffffffu, col, off + 8 + g);
-    const int va0 = __shfl_sync(0xffffffffu, col, off + 2 * t), va1 = __shfl_sync(0xffffffffu, col, off + 2 * t + 1);
-    const int vb0 = __shfl_sync(0xffffffffu, col, off + 8 + 2 * t);
-    const int vb1 = __shfl_sync(0xffffffffu, col, off + 9 + 2 * t);
-    const uint16_t* ka = Kb + (uint32_t)max(ca, 0) * ksl;
-    const uint16_t* kb = Kb + (uint32_t)max(cb, 0) * ksl;
-    st.k[0] = ld_nc_v4(ka);
-    st.k[1] = ld_nc_v4(ka + 32);
-    st.k[2] = ld_nc_v4(kb);
-    st.k[3] = ld_nc_v4(kb + 32);
-    st.v[0] = ld_nc_v4(Vb + (uint32_t)max(va0, 0) * vsl);
-    st.v[1] = ld_nc_v4(Vb + (uint32_t)max(va1, 0) * vsl);
-    st.v[2] = ld_nc_v4(Vb + (uint32_t)max(vb0, 0) * vsl);
-    st.v[3] = ld_nc_v4(Vb + (uint32_t)max(vb1, 0) * vsl);
+  // issue the gathers of step s (nnz beg + 16 s ..) into ring stage `stg`: lane copies chunk
+  // (lane & 7) of the rows R = (lane >> 3) + 4 i, i = 0..3, of K and of V. Indices come from `col`
+  // (lane i holds index beg + 32 w + i of window w; steps 2w, 2w + 1 use it); past the row's end
+  // they are -1 and read row 0 (masked scores, p = 0).
+  uint32_t doff[4];   // swizzled destination of this lane's chunk in rows R_i
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    const int R = (lane >> 3) + 4 * i;
+    doff[i] = R * 128 + (((lane & 7) ^ (R & 7)) << 4);
+  }
+  int col = -1;
+  auto issue_step = [&](int s, uint32_t stg) {
+    const int nb0 = beg + 16 * s;
+    if ((s & 1) == 0) col = nb0 + lane < end ? __ldg(p.cols + nb0 + lane) : -1;
+    const int off = (s & 1) * 16 + (lane >> 3);
+    int cc[4];
+#pragma unroll
+    for (int i = 0; i < 4; ++i) cc[i] = max(__shfl_sync(0xffffffffu, col, off + 4 * i), 0);
+    if (nb0 < end) {   // warp-uniform
+      const uint32_t st = ring + stg * kStageBytes;
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        cp_async16(st + doff[i], Kb + (uint32_t)cc[i] * ksl);
+        cp_async16(st + doff[i] + 2048, Vb + (uint32_t)cc[i] * vsl);
+      }
+    }
+    cp_async_commit();   // (an empty group past the end keeps the wait count uniform)
   };
-  auto load_cols = [&](int base) { return base + lane < end ? __ldg(p.cols + base + lane) : -1; };
 
   float m = -INFINITY, l = 0.f;
   float acc[4][4];
@@ -126,32 +163,39 @@ __global__ void __launch_bounds__(256, 2) fine_mma_kernel(const FineParams p) {
     for (int e = 0; e < 4; ++e) acc[j][e] = 0.f;
   const float thresh = 8.f / c;
 
-  Step cur;
-  int col = load_cols(beg);
-  if (beg < end) load_step(cur, col, 0);
-  for (int base = beg; base < end; base += 16) {
-    // prefetch the next step's rows (the 32-index window advances every other step)
-    Step nxt;
-    const int nb = base + 16;
-    const int off_next = ((nb - beg) & 16);
-    if (off_next == 0) col = load_cols(nb);
-    load_step(nxt, col, off_next);
-
-    // ---- SDDMM: chunk A -> sa, chunk B -> sb (lane holds nnz 2t, 2t+1 of each)
-    float sa[4] = {0.f, 0.f, 0.f, 0.f}, sb[4] = {0.f, 0.f, 0.f, 0.f};
-    const uint32_t ka[8] = {(uint32_t)cur.k[0].x, (uint32_t)cur.k[0].y, (uint32_t)cur.k[0].z, (uint32_t)cur.k[0].w,
-                            (uint32_t)cur.k[1].x, (uint32_t)cur.k[1].y, (uint32_t)cur.k[1].z, (uint32_t)cur.k[1].w};
-    const uint32_t kb[8] = {(uint32_t)cur.k[2].x, (uint32_t)cur.k[2].y, (uint32_t)cur.k[2].z, (uint32_t)cur.k[2].w,
-                            (uint32_t)cur.k[3].x, (uint32_t)cur.k[3].y, (uint32_t)cur.k[3].z, (uint32_t)cur.k[3].w};
 #pragma unroll
-    for (int j = 0; j < 4; ++j) {
-      mma16816<kBF16>(sa, qr[2 * j], qr[2 * j], qr[2 * j + 1], qr[2 * j + 1], ka[2 * j], ka[2 * j + 1]);
-      mma16816<kBF16>(sb, qr[2 * j], qr[2 * j], qr[2 * j + 1], qr[2 * j + 1], kb[2 * j], kb[2 * j + 1]);
+  for (int s = 0; s < kStages - 1; ++s) issue_step(s, s);
+  uint32_t stage = 0, istage = kStages - 1;
+  const uint32_t a_row = (lane & 7) * 128, b_row = a_row + 8 * 128;
+  const uint32_t vr = (lane & 7) + 8 * (lane >> 4);
+  int step = 0;
+  for (int base = beg; base < end; base += 16, ++step) {
+    issue_step(step + kStages - 1, istage);
+    istage = istage == kStages - 1 ? 0 : istage + 1;
+    cp_async_wait<kStages - 1>();
+    __syncwarp();
+    const uint32_t st = ring + stage * kStageBytes;
+    stage = stage == kStages - 1 ? 0 : stage + 1;
+
+    // ---- SDDMM: chunk A (rows 0-7) -> sa, chunk B (rows 8-15) -> sb; lane holds nnz 2t, 2t+1 of
+    // each; two independent accumulators per chunk (dims 0-31, 32-63) shorten the MMA chains
+    float sa[2][4] = {{0.f, 0.f, 0.f, 0.f}, {0.f, 0.f, 0.f, 0.f}};
+    float sb[2][4] = {{0.f, 0.f, 0.f, 0.f}, {0.f, 0.f, 0.f, 0.f}};
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {   // dims 32h .. 32h + 31 = k16 steps 2h, 2h + 1
+      uint32_t ka[4], kb[4];
+      const uint32_t sw = ((uint32_t)(((lane >> 3) + 4 * h) ^ (lane & 7))) << 4;
+      ldsm_x4(ka, st + a_row + sw);
+      ldsm_x4(kb, st + b_row + sw);
+      mma16816<kBF16>(sa[h], qa[2 * h], qa[2 * h], qb[2 * h], qb[2 * h], ka[0], ka[1]);
+      mma16816<kBF16>(sb[h], qa[2 * h], qa[2 * h], qb[2 * h], qb[2 * h], kb[0], kb[1]);
+      mma16816<kBF16>(sa[h], qa[2 * h + 1], qa[2 * h + 1], qb[2 * h + 1], qb[2 * h + 1], ka[2], ka[3]);
+      mma16816<kBF16>(sb[h], qa[2 * h + 1], qa[2 * h + 1], qb[2 * h + 1], qb[2 * h + 1], kb[2], kb[3]);
     }
     // this lane's score positions: nnz base + 2t, + 2t+1 (chunk A), + 8 + 2t, + 9 + 2t (chunk B)
     const int rem = end - base - 2 * t;
-    float s[4] = {rem > 0 ? sa[0] : -INFINITY, rem > 1 ? sa[1] : -INFINITY, rem > 8 ? sb[0] : -INFINITY,
-                  rem > 9 ? sb[1] : -INFINITY};
+    float s[4] = {rem > 0 ? sa[0][0] + sa[1][0] : -INFINITY, rem > 1 ? sa[0][1] + sa[1][1] : -INFINITY,
+                  rem > 8 ? sb[0][0] + sb[1][0] : -INFINITY, rem > 9 ? sb[0][1] + sb[1][1] : -INFINITY};
     // ---- online softmax over the step (warp-uniform max: lanes with equal t hold equal values)
     float mx = fmaxf(fmaxf(s[0], s[1]), fmaxf(s[2], s[3]));
     mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, 1));
@@ -173,32 +217,36 @@ __global__ void __launch_bounds__(256, 2) fine_mma_kernel(const FineParams p) {
       l += pr[i];
     }
     const uint32_t pb0 = pack2<kBF16>(pr[0], pr[1]), pb1 = pack2<kBF16>(pr[2], pr[3]);
-    // ---- SpMM: O^T[dims 8g+2j, 8g+2j+1] += V^T . p
-    const uint32_t v0[4] = {(uint32_t)cur.v[0].x, (uint32_t)cur.v[0].y, (uint32_t)cur.v[0].z, (uint32_t)cur.v[0].w};
-    const uint32_t v1[4] = {(uint32_t)cur.v[1].x, (uint32_t)cur.v[1].y, (uint32_t)cur.v[1].z, (uint32_t)cur.v[1].w};
-    const uint32_t v2[4] = {(uint32_t)cur.v[2].x, (uint32_t)cur.v[2].y, (uint32_t)cur.v[2].z, (uint32_t)cur.v[2].w};
-    const uint32_t v3[4] = {(uint32_t)cur.v[3].x, (uint32_t)cur.v[3].y, (uint32_t)cur.v[3].z, (uint32_t)cur.v[3].w};
+    // ---- SpMM: O^T[dims 16j + g, 16j + g + 8] += V^T . p (A = V^T from ldmatrix.trans)
 #pragma unroll
-    for (int j = 0; j < 4; ++j)
-      mma16816<kBF16>(acc[j], prmt(v0[j], v1[j], 0x5410), prmt(v0[j], v1[j], 0x7632), prmt(v2[j], v3[j], 0x5410),
-                      prmt(v2[j], v3[j], 0x7632), pb0, pb1);
-    cur = nxt;
+    for (int j = 0; j < 4; ++j) {
+      uint32_t a[4];
+      const uint32_t ch = 2 * j + ((lane >> 3) & 1);
+      ldsm_x4_t(a, st + 2048 + vr * 128 + ((ch ^ (vr & 7)) << 4));
+      mma16816<kBF16>(acc[j], a[0], a[1], a[2], a[3], pb0, pb1);
+    }
+    __syncwarp();   // every lane has read this stage before it is refilled
   }
+  cp_async_wait<0>();
   // row sum: lanes with the same g hold disjoint nnz subsets (t); every g holds the same sums
   l += __shfl_xor_sync(0xffffffffu, l, 1);
   l += __shfl_xor_sync(0xffffffffu, l, 2);
-  // lane (g, 0): O dims 8g .. 8g+7 = acc[j][0] (dim 8g+2j), acc[j][2] (dim 8g+2j+1)
-  float o8[8] = {acc[0][0], acc[0][2], acc[1][0], acc[1][2], acc[2][0], acc[2][2], acc[3][0], acc[3][2]};
+  // lane (g, t) owns output dims d0 = 16t + g and d1 = d0 + 8: acc[t][0] and acc[t][2]
+  float v0 = acc[0][0], v1 = acc[0][2];
+#pragma unroll
+  for (int j = 1; j < 4; ++j)
+    if (t == j) {
+      v0 = acc[j][0];
+      v1 = acc[j][2];
+    }
+  const int d0 = 16 * t + g, d1 = d0 + 8;
   float inv = l > 0.f ? 1.f / l : 0.f;
   bool write_o = final_out;
   if (!final_out) {
     const size_t idx = (size_t)bh * p.n_fine_rows + fi;
-    if (t == 0) {
-      float4* dst = reinterpret_cast<float4*>(p.part_acc + idx * 64 + g * 8);
-      __stcg(dst, make_float4(o8[0], o8[1], o8[2], o8[3]));
-      __stcg(dst + 1, make_float4(o8[4], o8[5], o8[6], o8[7]));
-      if (lane == 0) __stcg(p.part_ml + idx, make_float2(m, l));
-    }
+    __stcg(p.part_acc + idx * 64 + d0, v0);
+    __stcg(p.part_acc + idx * 64 + d1, v1);
+    if (lane == 0) __stcg(p.part_ml + idx, make_float2(m, l));
     if (p.concurrent) {
       // concurrent coarse || fine: the side that finishes the row second merges (a-8)
       __threadfence();
@@ -214,32 +262,27 @@ __global__ void __launch_bounds__(256, 2) fine_mma_kernel(const FineParams p) {
         const float af = ex2((m - mu) * c), ac = ex2((mlc.x - mu) * c);
         const float den = l * af + mlc.y * ac;
         inv = den > 0.f ? 1.f / den : 0.f;
-        const float4* src = reinterpret_cast<const float4*>(p.part_c_acc + idx * 64 + g * 8);
-        const float4 c0 = __ldcg(src), c1 = __ldcg(src + 1);
-        const float cc[8] = {c0.x, c0.y, c0.z, c0.w, c1.x, c1.y, c1.z, c1.w};
-#pragma unroll
-        for (int e = 0; e < 8; ++e) o8[e] = o8[e] * af + cc[e] * ac;
+        v0 = v0 * af + __ldcg(p.part_c_acc + idx * 64 + d0) * ac;
+        v1 = v1 * af + __ldcg(p.part_c_acc + idx * 64 + d1) * ac;
         write_o = true;
       }
     }
   }
-  if (t != 0 || !write_o) return;
-  uint4 o4;
-  o4.x = pack2<kBF16>(o8[0] * inv, o8[1] * inv);
-  o4.y = pack2<kBF16>(o8[2] * inv, o8[3] * inv);
-  o4.z = pack2<kBF16>(o8[4] * inv, o8[5] * inv);
-  o4.w = pack2<kBF16>(o8[6] * inv, o8[7] * inv);
-  *reinterpret_cast<uint4*>(p.o.data + bb * p.o.sb + hh * p.o.sh + (int64_t)r * p.o.sl + g * 8) = o4;
+  if (!write_o) return;
+  uint16_t* orow = p.o.data + bb * p.o.sb + hh * p.o.sh + (int64_t)r * p.o.sl;
+  const uint32_t pk = pack2<kBF16>(v0 * inv, v1 * inv);
+  orow[d0] = (uint16_t)(pk & 0xffffu);
+  orow[d1] = (uint16_t)(pk >> 16);
 }
 
 cudaError_t launch_fine_mma(const FineParams& p, bool bf16, cudaStream_t stream) {
   const int64_t warps = (int64_t)p.BH * p.n_fine_rows;
   if (warps == 0) return cudaSuccess;
-  const int64_t blocks = (warps + 7) / 8;
-  if (bf16)
-    fine_mma_kernel<true><<<(unsigned)blocks, 256, 0, stream>>>(p);
-  else
-    fine_mma_kernel<false><<<(unsigned)blocks, 256, 0, stream>>>(p);
+  const int64_t blocks = (warps + kWarps - 1) / kWarps;
+  auto kern = bf16 ? fine_mma_kernel<true> : fine_mma_kernel<false>;
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytes);
+  if (e != cudaSuccess) return e;
+  kern<<<(unsigned)blocks, kWarps * 32, kSmemBytes, stream>>>(p);
   return cudaGetLastError();
 }
 
