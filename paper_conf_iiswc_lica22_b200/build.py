@@ -22,8 +22,9 @@ VARIANTS = {"watchdog": ["-DMG_WATCHDOG"], "timeline": ["-DMG_TIMELINE"], "trace
             # A/B of the share of exponentials emulated on the FMA pipe (pairs of 16 per chunk)
             "e0": ["-DMG_EXP_EMU=0"], "e4": ["-DMG_EXP_EMU=4"], "e8": ["-DMG_EXP_EMU=8"],
             "maxpass": ["-DMG_SKIP_MAX=0"],
-            # fine tensor-core kernel: cp.async ring stages per warp (default 3)
-            "fs2": ["-DMG_FINE_STAGES=2"], "fs4": ["-DMG_FINE_STAGES=4"],
+            # fine tensor-core kernel: cp.async ring stages per warp (default 2), min blocks per SM
+            "fs3": ["-DMG_FINE_STAGES=3"], "fb4": ["-DMG_FINE_MINB=4"], "fb6": ["-DMG_FINE_MINB=6"],
+            "fb8": ["-DMG_FINE_MINB=8"],
             # skeleton cost: no exponentials / no MMAs / no loads (results are garbage)
             "dbg1": ["-DMG_DBG=1"], "dbg3": ["-DMG_DBG=3"], "dbg7": ["-DMG_DBG=7"]}
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")

@@ -20,6 +20,8 @@
 // p is rounded to the operand dtype for the SpMM (as in the coarse kernel, A9); s, the
 // running max/sum and O accumulate in fp32. Lazy rescaling: the exponent keeps a stale max until
 // a step's max exceeds it by 8/c (p <= 256), warp-uniform because all lanes see the same max.
+#include <algorithm>
+
 #include <cuda_bf16.h>
 #include <cuda_fp16.h>
 
@@ -80,7 +82,10 @@ __device__ __forceinline__ void ldsm_x4_t(uint32_t (&r)[4], uint32_t addr) {
 }
 
 #ifndef MG_FINE_STAGES
-#define MG_FINE_STAGES 3
+#define MG_FINE_STAGES 2
+#endif
+#ifndef MG_FINE_MINB
+#define MG_FINE_MINB 5
 #endif
 constexpr int kWarps = 4;                   // warps per block, one (row, b*h) each
 constexpr int kStages = MG_FINE_STAGES;     // smem ring stages per warp (kStages - 1 steps in flight)
@@ -96,192 +101,226 @@ constexpr int kSmemBytes = kWarps * kStages * kStageBytes;
 // are stored with the 16-byte-chunk XOR swizzle (chunk c of row r at (c ^ (r & 7)) * 16), and the
 // MMA fragments come from ldmatrix: non-transposed for the SDDMM's B operand (K rows = columns n,
 // dims = k), transposed for the SpMM's A operand (V^T: dims = rows m, nnz = k).
+// Persistent warps: warp w processes the rows w, w + W, w + 2W, ... of the (b*h, CSR row) space (W =
+// warps in the grid; neighbouring warps stay on neighbouring rows of the same head, so the head's
+// K/V stay in L2), and the gather pointer runs ahead across row boundaries, so a row's first gathers
+// are in flight while the previous row is computed (one row is only ~11 steps).
 template <bool kBF16>
-__global__ void __launch_bounds__(kWarps * 32) fine_mma_kernel(const FineParams p) {
+__global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(const FineParams p) {
   extern __shared__ __align__(128) uint8_t fsm[];
   const int lane = threadIdx.x & 31;
-  const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  if (gw >= (int64_t)p.BH * p.n_fine_rows) return;
-  const int bh = (int)(gw / p.n_fine_rows);
-  const int fi = (int)(gw % p.n_fine_rows);
-  const int enc = __ldg(p.fine_rows + fi);
-  const int r = enc & 0x7fffffff;
-  const bool final_out = enc < 0;
-  const int bb = bh / p.H, hh = bh % p.H;
   const int g = lane >> 2, t = lane & 3;
   const float c = p.scale_log2;
+  const float thresh = 8.f / c;
+  const int64_t nrows = (int64_t)p.BH * p.n_fine_rows;
+  const int64_t W = (int64_t)gridDim.x * kWarps;
+  const int64_t w0 = (int64_t)blockIdx.x * kWarps + (threadIdx.x >> 5);
   const uint32_t ring = (uint32_t)__cvta_generic_to_shared(fsm) + (threadIdx.x >> 5) * (kStages * kStageBytes);
-
-  // q as the SDDMM's A operand (every row = q): k16 step j uses dims 16j + 2t (+1) and 16j + 8 + 2t (+1)
-  const uint16_t* qrow = p.q.data + bb * p.q.sb + hh * p.q.sh + (int64_t)r * p.q.sl;
-  uint32_t qa[4], qb[4];
-#pragma unroll
-  for (int j = 0; j < 4; ++j) {
-    qa[j] = __ldg(reinterpret_cast<const uint32_t*>(qrow + 16 * j + 2 * t));
-    qb[j] = __ldg(reinterpret_cast<const uint32_t*>(qrow + 16 * j + 8 + 2 * t));
-  }
-  const uint16_t* Kb = p.k.data + bb * p.k.sb + hh * p.k.sh + (lane & 7) * 8;
-  const uint16_t* Vb = p.v.data + bb * p.v.sb + hh * p.v.sh + (lane & 7) * 8;
-  const int beg = __ldg(p.row_ptr + fi), end = __ldg(p.row_ptr + fi + 1);
   // row strides fit 32 bits (checked by the forward's validation: (L - 1) * stride_l < 2^32)
   const uint32_t ksl = (uint32_t)p.k.sl, vsl = (uint32_t)p.v.sl;
-
-  // issue the gathers of step s (nnz beg + 16 s ..) into ring stage `stg`: lane copies chunk
-  // (lane & 7) of the rows R = (lane >> 3) + 4 i, i = 0..3, of K and of V. Indices come from `col`
-  // (lane i holds index beg + 32 w + i of window w; steps 2w, 2w + 1 use it); past the row's end
-  // they are -1 and read row 0 (masked scores, p = 0).
-  uint32_t doff[4];   // swizzled destination of this lane's chunk in rows R_i
+  uint32_t doff[4];   // swizzled destination of this lane's chunk in rows R_i = (lane >> 3) + 4 i
 #pragma unroll
   for (int i = 0; i < 4; ++i) {
     const int R = (lane >> 3) + 4 * i;
     doff[i] = R * 128 + (((lane & 7) ^ (R & 7)) << 4);
   }
-  int col = -1;
-  auto issue_step = [&](int s, uint32_t stg) {
-    const int nb0 = beg + 16 * s;
-    if ((s & 1) == 0) col = nb0 + lane < end ? __ldg(p.cols + nb0 + lane) : -1;
-    const int off = (s & 1) * 16 + (lane >> 3);
-    int cc[4];
-#pragma unroll
-    for (int i = 0; i < 4; ++i) cc[i] = max(__shfl_sync(0xffffffffu, col, off + 4 * i), 0);
-    if (nb0 < end) {   // warp-uniform
+
+  // ---- gather pointer: row gi (global work index), step is of [ibeg, iend)
+  int64_t gi = w0;
+  int ibeg = 0, iend = 0, is = 0, icol = -1;
+  const uint16_t *iK = nullptr, *iV = nullptr;
+  auto open_issue_row = [&]() {
+    if (gi < nrows) {
+      const int bh = (int)(gi / p.n_fine_rows), fi = (int)(gi % p.n_fine_rows);
+      ibeg = __ldg(p.row_ptr + fi);
+      iend = __ldg(p.row_ptr + fi + 1);
+      const int bb = bh / p.H, hh = bh % p.H;
+      iK = p.k.data + bb * p.k.sb + hh * p.k.sh + (lane & 7) * 8;
+      iV = p.v.data + bb * p.v.sb + hh * p.v.sh + (lane & 7) * 8;
+    }
+    is = 0;
+  };
+  // issue the gathers of the pointer's step into ring stage `stg` and advance the pointer. Indices
+  // come from `icol` (lane i holds index ibeg + 32 w + i of window w; steps 2w, 2w + 1 use it); past
+  // the row's end they are -1 and read row 0 (masked scores, p = 0).
+  auto issue_step = [&](uint32_t stg) {
+    if (gi < nrows) {   // warp-uniform
+      const int nb0 = ibeg + 16 * is;
+      if ((is & 1) == 0) icol = nb0 + lane < iend ? __ldg(p.cols + nb0 + lane) : -1;
+      const int off = (is & 1) * 16 + (lane >> 3);
       const uint32_t st = ring + stg * kStageBytes;
 #pragma unroll
       for (int i = 0; i < 4; ++i) {
-        cp_async16(st + doff[i], Kb + (uint32_t)cc[i] * ksl);
-        cp_async16(st + doff[i] + 2048, Vb + (uint32_t)cc[i] * vsl);
+        const uint32_t cc = (uint32_t)max(__shfl_sync(0xffffffffu, icol, off + 4 * i), 0);
+        cp_async16(st + doff[i], iK + cc * ksl);
+        cp_async16(st + doff[i] + 2048, iV + cc * vsl);
+      }
+      if (nb0 + 16 < iend) {
+        ++is;
+      } else {
+        gi += W;
+        open_issue_row();
       }
     }
     cp_async_commit();   // (an empty group past the end keeps the wait count uniform)
   };
 
-  float m = -INFINITY, l = 0.f;
-  float acc[4][4];
+  open_issue_row();
 #pragma unroll
-  for (int j = 0; j < 4; ++j)
-#pragma unroll
-    for (int e = 0; e < 4; ++e) acc[j][e] = 0.f;
-  const float thresh = 8.f / c;
-
-#pragma unroll
-  for (int s = 0; s < kStages - 1; ++s) issue_step(s, s);
+  for (int s = 0; s < kStages - 1; ++s) issue_step(s);
   uint32_t stage = 0, istage = kStages - 1;
   const uint32_t a_row = (lane & 7) * 128, b_row = a_row + 8 * 128;
   const uint32_t vr = (lane & 7) + 8 * (lane >> 4);
-  int step = 0;
-  for (int base = beg; base < end; base += 16, ++step) {
-    issue_step(step + kStages - 1, istage);
-    istage = istage == kStages - 1 ? 0 : istage + 1;
-    cp_async_wait<kStages - 1>();
-    __syncwarp();
-    const uint32_t st = ring + stage * kStageBytes;
-    stage = stage == kStages - 1 ? 0 : stage + 1;
 
-    // ---- SDDMM: chunk A (rows 0-7) -> sa, chunk B (rows 8-15) -> sb; lane holds nnz 2t, 2t+1 of
-    // each; two independent accumulators per chunk (dims 0-31, 32-63) shorten the MMA chains
-    float sa[2][4] = {{0.f, 0.f, 0.f, 0.f}, {0.f, 0.f, 0.f, 0.f}};
-    float sb[2][4] = {{0.f, 0.f, 0.f, 0.f}, {0.f, 0.f, 0.f, 0.f}};
-#pragma unroll
-    for (int h = 0; h < 2; ++h) {   // dims 32h .. 32h + 31 = k16 steps 2h, 2h + 1
-      uint32_t ka[4], kb[4];
-      const uint32_t sw = ((uint32_t)(((lane >> 3) + 4 * h) ^ (lane & 7))) << 4;
-      ldsm_x4(ka, st + a_row + sw);
-      ldsm_x4(kb, st + b_row + sw);
-      mma16816<kBF16>(sa[h], qa[2 * h], qa[2 * h], qb[2 * h], qb[2 * h], ka[0], ka[1]);
-      mma16816<kBF16>(sb[h], qa[2 * h], qa[2 * h], qb[2 * h], qb[2 * h], kb[0], kb[1]);
-      mma16816<kBF16>(sa[h], qa[2 * h + 1], qa[2 * h + 1], qb[2 * h + 1], qb[2 * h + 1], ka[2], ka[3]);
-      mma16816<kBF16>(sb[h], qa[2 * h + 1], qa[2 * h + 1], qb[2 * h + 1], qb[2 * h + 1], kb[2], kb[3]);
-    }
-    // this lane's score positions: nnz base + 2t, + 2t+1 (chunk A), + 8 + 2t, + 9 + 2t (chunk B)
-    const int rem = end - base - 2 * t;
-    float s[4] = {rem > 0 ? sa[0][0] + sa[1][0] : -INFINITY, rem > 1 ? sa[0][1] + sa[1][1] : -INFINITY,
-                  rem > 8 ? sb[0][0] + sb[1][0] : -INFINITY, rem > 9 ? sb[0][1] + sb[1][1] : -INFINITY};
-    // ---- online softmax over the step (warp-uniform max: lanes with equal t hold equal values)
-    float mx = fmaxf(fmaxf(s[0], s[1]), fmaxf(s[2], s[3]));
-    mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, 1));
-    mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, 2));
-    if (mx > m + thresh) {   // also taken on the first step (m = -inf); mx is finite (>= 1 valid nnz)
-      const float alpha = ex2((m - mx) * c);
-      l *= alpha;
-#pragma unroll
-      for (int j = 0; j < 4; ++j)
-#pragma unroll
-        for (int e = 0; e < 4; ++e) acc[j][e] *= alpha;
-      m = mx;
-    }
-    const float nbias = -m * c;
-    float pr[4];
-#pragma unroll
-    for (int i = 0; i < 4; ++i) {
-      pr[i] = ex2(fmaf(s[i], c, nbias));
-      l += pr[i];
-    }
-    const uint32_t pb0 = pack2<kBF16>(pr[0], pr[1]), pb1 = pack2<kBF16>(pr[2], pr[3]);
-    // ---- SpMM: O^T[dims 16j + g, 16j + g + 8] += V^T . p (A = V^T from ldmatrix.trans)
+  for (int64_t gw = w0; gw < nrows; gw += W) {
+    const int bh = (int)(gw / p.n_fine_rows);
+    const int fi = (int)(gw % p.n_fine_rows);
+    const int enc = __ldg(p.fine_rows + fi);
+    const int r = enc & 0x7fffffff;
+    const bool final_out = enc < 0;
+    const int bb = bh / p.H, hh = bh % p.H;
+    // q as the SDDMM's A operand (every row = q): k16 step j uses dims 16j + 2t (+1), 16j + 8 + 2t (+1)
+    const uint16_t* qrow = p.q.data + bb * p.q.sb + hh * p.q.sh + (int64_t)r * p.q.sl;
+    uint32_t qa[4], qb[4];
 #pragma unroll
     for (int j = 0; j < 4; ++j) {
-      uint32_t a[4];
-      const uint32_t ch = 2 * j + ((lane >> 3) & 1);
-      ldsm_x4_t(a, st + 2048 + vr * 128 + ((ch ^ (vr & 7)) << 4));
-      mma16816<kBF16>(acc[j], a[0], a[1], a[2], a[3], pb0, pb1);
+      qa[j] = __ldg(reinterpret_cast<const uint32_t*>(qrow + 16 * j + 2 * t));
+      qb[j] = __ldg(reinterpret_cast<const uint32_t*>(qrow + 16 * j + 8 + 2 * t));
     }
-    __syncwarp();   // every lane has read this stage before it is refilled
-  }
-  cp_async_wait<0>();
-  // row sum: lanes with the same g hold disjoint nnz subsets (t); every g holds the same sums
-  l += __shfl_xor_sync(0xffffffffu, l, 1);
-  l += __shfl_xor_sync(0xffffffffu, l, 2);
-  // lane (g, t) owns output dims d0 = 16t + g and d1 = d0 + 8: acc[t][0] and acc[t][2]
-  float v0 = acc[0][0], v1 = acc[0][2];
+    const int beg = __ldg(p.row_ptr + fi), end = __ldg(p.row_ptr + fi + 1);
+
+    float m = -INFINITY, l = 0.f;
+    float acc[4][4];
 #pragma unroll
-  for (int j = 1; j < 4; ++j)
-    if (t == j) {
-      v0 = acc[j][0];
-      v1 = acc[j][2];
-    }
-  const int d0 = 16 * t + g, d1 = d0 + 8;
-  float inv = l > 0.f ? 1.f / l : 0.f;
-  bool write_o = final_out;
-  if (!final_out) {
-    const size_t idx = (size_t)bh * p.n_fine_rows + fi;
-    __stcg(p.part_acc + idx * 64 + d0, v0);
-    __stcg(p.part_acc + idx * 64 + d1, v1);
-    if (lane == 0) __stcg(p.part_ml + idx, make_float2(m, l));
-    if (p.concurrent) {
-      // concurrent coarse || fine: the side that finishes the row second merges (a-8)
-      __threadfence();
+    for (int j = 0; j < 4; ++j)
+#pragma unroll
+      for (int e = 0; e < 4; ++e) acc[j][e] = 0.f;
+
+    for (int base = beg; base < end; base += 16) {
+      issue_step(istage);
+      istage = istage == kStages - 1 ? 0 : istage + 1;
+      cp_async_wait<kStages - 1>();
       __syncwarp();
-      int old = 0;
-      if (lane == 0) old = atomicAdd(p.part_flags + idx, 1);
-      old = __shfl_sync(0xffffffffu, old, 0);
-      if (old & 1) {
+      const uint32_t st = ring + stage * kStageBytes;
+      stage = stage == kStages - 1 ? 0 : stage + 1;
+
+      // ---- SDDMM: chunk A (rows 0-7) -> sa, chunk B (rows 8-15) -> sb; lane holds nnz 2t, 2t+1 of
+      // each; two independent accumulators per chunk (dims 0-31, 32-63) shorten the MMA chains
+      float sa[2][4] = {{0.f, 0.f, 0.f, 0.f}, {0.f, 0.f, 0.f, 0.f}};
+      float sb[2][4] = {{0.f, 0.f, 0.f, 0.f}, {0.f, 0.f, 0.f, 0.f}};
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {   // dims 32h .. 32h + 31 = k16 steps 2h, 2h + 1
+        uint32_t ka[4], kb[4];
+        const uint32_t sw = ((uint32_t)(((lane >> 3) + 4 * h) ^ (lane & 7))) << 4;
+        ldsm_x4(ka, st + a_row + sw);
+        ldsm_x4(kb, st + b_row + sw);
+        mma16816<kBF16>(sa[h], qa[2 * h], qa[2 * h], qb[2 * h], qb[2 * h], ka[0], ka[1]);
+        mma16816<kBF16>(sb[h], qa[2 * h], qa[2 * h], qb[2 * h], qb[2 * h], kb[0], kb[1]);
+        mma16816<kBF16>(sa[h], qa[2 * h + 1], qa[2 * h + 1], qb[2 * h + 1], qb[2 * h + 1], ka[2], ka[3]);
+        mma16816<kBF16>(sb[h], qa[2 * h + 1], qa[2 * h + 1], qb[2 * h + 1], qb[2 * h + 1], kb[2], kb[3]);
+      }
+      // this lane's score positions: nnz base + 2t, + 2t+1 (chunk A), + 8 + 2t, + 9 + 2t (chunk B)
+      const int rem = end - base - 2 * t;
+      float s[4] = {rem > 0 ? sa[0][0] + sa[1][0] : -INFINITY, rem > 1 ? sa[0][1] + sa[1][1] : -INFINITY,
+                    rem > 8 ? sb[0][0] + sb[1][0] : -INFINITY, rem > 9 ? sb[0][1] + sb[1][1] : -INFINITY};
+      // ---- online softmax over the step (warp-uniform max: lanes with equal t hold equal values)
+      float mx = fmaxf(fmaxf(s[0], s[1]), fmaxf(s[2], s[3]));
+      mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, 1));
+      mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, 2));
+      if (mx > m + thresh) {   // also taken on the first step (m = -inf); mx is finite (>= 1 valid nnz)
+        const float alpha = ex2((m - mx) * c);
+        l *= alpha;
+#pragma unroll
+        for (int j = 0; j < 4; ++j)
+#pragma unroll
+          for (int e = 0; e < 4; ++e) acc[j][e] *= alpha;
+        m = mx;
+      }
+      const float nbias = -m * c;
+      float pr[4];
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        pr[i] = ex2(fmaf(s[i], c, nbias));
+        l += pr[i];
+      }
+      const uint32_t pb0 = pack2<kBF16>(pr[0], pr[1]), pb1 = pack2<kBF16>(pr[2], pr[3]);
+      // ---- SpMM: O^T[dims 16j + g, 16j + g + 8] += V^T . p (A = V^T from ldmatrix.trans)
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        uint32_t a[4];
+        const uint32_t ch = 2 * j + ((lane >> 3) & 1);
+        ldsm_x4_t(a, st + 2048 + vr * 128 + ((ch ^ (vr & 7)) << 4));
+        mma16816<kBF16>(acc[j], a[0], a[1], a[2], a[3], pb0, pb1);
+      }
+      __syncwarp();   // every lane has read this stage before it is refilled
+    }
+    // ---- row epilogue. Row sum: lanes with the same g hold disjoint nnz subsets (t).
+    l += __shfl_xor_sync(0xffffffffu, l, 1);
+    l += __shfl_xor_sync(0xffffffffu, l, 2);
+    // lane (g, t) owns output dims d0 = 16t + g and d1 = d0 + 8: acc[t][0] and acc[t][2]
+    float v0 = acc[0][0], v1 = acc[0][2];
+#pragma unroll
+    for (int j = 1; j < 4; ++j)
+      if (t == j) {
+        v0 = acc[j][0];
+        v1 = acc[j][2];
+      }
+    const int d0 = 16 * t + g, d1 = d0 + 8;
+    float inv = l > 0.f ? 1.f / l : 0.f;
+    bool write_o = final_out;
+    if (!final_out) {
+      const size_t idx = (size_t)bh * p.n_fine_rows + fi;
+      __stcg(p.part_acc + idx * 64 + d0, v0);
+      __stcg(p.part_acc + idx * 64 + d1, v1);
+      if (lane == 0) __stcg(p.part_ml + idx, make_float2(m, l));
+      if (p.concurrent) {
+        // concurrent coarse || fine: the side that finishes the row second merges (a-8)
         __threadfence();
-        const float2 mlc = __ldcg(p.part_c_ml + idx);
-        const float mt = fmaxf(m, mlc.x);
-        const float mu = mt == -INFINITY ? 0.f : mt;
-        const float af = ex2((m - mu) * c), ac = ex2((mlc.x - mu) * c);
-        const float den = l * af + mlc.y * ac;
-        inv = den > 0.f ? 1.f / den : 0.f;
-        v0 = v0 * af + __ldcg(p.part_c_acc + idx * 64 + d0) * ac;
-        v1 = v1 * af + __ldcg(p.part_c_acc + idx * 64 + d1) * ac;
-        write_o = true;
+        __syncwarp();
+        int old = 0;
+        if (lane == 0) old = atomicAdd(p.part_flags + idx, 1);
+        old = __shfl_sync(0xffffffffu, old, 0);
+        if (old & 1) {
+          __threadfence();
+          const float2 mlc = __ldcg(p.part_c_ml + idx);
+          const float mt = fmaxf(m, mlc.x);
+          const float mu = mt == -INFINITY ? 0.f : mt;
+          const float af = ex2((m - mu) * c), ac = ex2((mlc.x - mu) * c);
+          const float den = l * af + mlc.y * ac;
+          inv = den > 0.f ? 1.f / den : 0.f;
+          v0 = v0 * af + __ldcg(p.part_c_acc + idx * 64 + d0) * ac;
+          v1 = v1 * af + __ldcg(p.part_c_acc + idx * 64 + d1) * ac;
+          write_o = true;
+        }
       }
     }
+    if (write_o) {
+      uint16_t* orow = p.o.data + bb * p.o.sb + hh * p.o.sh + (int64_t)r * p.o.sl;
+      const uint32_t pk = pack2<kBF16>(v0 * inv, v1 * inv);
+      orow[d0] = (uint16_t)(pk & 0xffffu);
+      orow[d1] = (uint16_t)(pk >> 16);
+    }
   }
-  if (!write_o) return;
-  uint16_t* orow = p.o.data + bb * p.o.sb + hh * p.o.sh + (int64_t)r * p.o.sl;
-  const uint32_t pk = pack2<kBF16>(v0 * inv, v1 * inv);
-  orow[d0] = (uint16_t)(pk & 0xffffu);
-  orow[d1] = (uint16_t)(pk >> 16);
+  cp_async_wait<0>();
 }
 
 cudaError_t launch_fine_mma(const FineParams& p, bool bf16, cudaStream_t stream) {
   const int64_t warps = (int64_t)p.BH * p.n_fine_rows;
   if (warps == 0) return cudaSuccess;
-  const int64_t blocks = (warps + kWarps - 1) / kWarps;
   auto kern = bf16 ? fine_mma_kernel<true> : fine_mma_kernel<false>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytes);
   if (e != cudaSuccess) return e;
+  // persistent grid: every resident block slot of every SM, or fewer if the rows are few
+  static int per_sm = 0, sms = 0;
+  if (per_sm == 0) {
+    int dev = 0;
+    if ((e = cudaGetDevice(&dev)) != cudaSuccess ||
+        (e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev)) != cudaSuccess ||
+        (e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kWarps * 32, kSmemBytes)) != cudaSuccess)
+      return e;
+    per_sm = std::max(per_sm, 1);
+  }
+  const int64_t blocks = std::min<int64_t>((warps + kWarps - 1) / kWarps, (int64_t)per_sm * sms);
   kern<<<(unsigned)blocks, kWarps * 32, kSmemBytes, stream>>>(p);
   return cudaGetLastError();
 }
