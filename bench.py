@@ -340,7 +340,7 @@ def main():
         flops = 4.0 * coarse_nnz * cfg.d * BH
         achieved = flops / (coarse_avg * 1e-3) / 1e12
         peak = peaks["bf16_tflops"]
-        roof = {"kernel": "coarse_kernel (tcgen05 SDDMM + online SpSoftmax + SpMM)", "bound": "tensor",
+        roof = {"kernel": "coarse_pp_kernel (tcgen05 SDDMM + online SpSoftmax + SpMM)", "bound": "tensor",
                 "achieved": achieved, "peak": peak, "unit": "TFLOP/s", "frac": achieved / peak,
                 "avg_launch_ms": coarse_avg, "algorithmic_per_launch": flops,
                 "algorithmic_rule": "4*d flops per valid element it owns (coarse + strip + dense-row)",
@@ -349,7 +349,9 @@ def main():
         nbytes_f = info["nnz_fine_cuda"] * BH * (2 * cfg.d * 2 + 4) + info["n_fine_rows"] * BH * (2 * cfg.d + 264)
         achieved = nbytes_f / (fine_avg * 1e-3) / 1e9
         peak = peaks["hbm_gbs"]
-        roof = {"kernel": "fine_rows_kernel (CUDA-core CSR)", "bound": "hbm", "achieved": achieved, "peak": peak,
+        kname = ("fine_mma_kernel (warp-level tensor-core CSR)" if args.fine_kernel == 0
+                 else "fine_rows_kernel (CUDA-core CSR)")
+        roof = {"kernel": kname, "bound": "hbm", "achieved": achieved, "peak": peak,
                 "unit": "GB/s", "frac": achieved / peak, "avg_launch_ms": fine_avg,
                 "algorithmic_per_launch": nbytes_f,
                 "algorithmic_rule": "per nnz: K row + V row (2*d*2 B) + 4 B index; per row: Q read + partial write",

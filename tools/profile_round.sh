@@ -8,7 +8,7 @@ for W in C2 C4; do
 done
 timeout -s KILL 400 ncu --set full --clock-control none --import-source on -k regex:coarse -s 3 -c 1 -o gpurun_out/full_c2_coarse \
   python bench.py --workload C2 --steps 4 --warmup 2 --no-cpu-baseline --e2e-steps 1 > /dev/null 2>&1
-timeout -s KILL 400 ncu --set full --clock-control none --import-source on -k regex:fine_rows -s 2 -c 1 -o gpurun_out/full_c4_fine \
+timeout -s KILL 400 ncu --set full --clock-control none --import-source on -k regex:fine_ -s 2 -c 1 -o gpurun_out/full_c4_fine \
   python bench.py --workload C4 --steps 3 --warmup 2 --no-cpu-baseline --e2e-steps 1 > /dev/null 2>&1
 timeout -s KILL 400 ncu --set full --clock-control none --import-source on -k regex:coarse -s 2 -c 1 -o gpurun_out/full_c4_coarse \
   python bench.py --workload C4 --steps 3 --warmup 2 --no-cpu-baseline --e2e-steps 1 > /dev/null 2>&1
