@@ -50,6 +50,7 @@ def parse():
     ap.add_argument("--concurrency", type=int, default=0, choices=[0, 1, 2],
                     help="coarse vs CSR kernels: 0 = library default, 1 = serial, 2 = concurrent streams")
     ap.add_argument("--tau", type=float, default=0.0, help="tile density threshold (0 = band rule)")
+    ap.add_argument("--dense-chunk", type=int, default=0, help="column tiles per dense-row item (-1: no split)")
     ap.add_argument("--fine-kernel", type=int, default=0, choices=[0, 1],
                     help="CSR rows: 0 = warp-level tensor-core kernel, 1 = CUDA-core kernel (A/B)")
     return ap.parse_args()
@@ -243,7 +244,7 @@ def main():
     cfg = get_config(args.workload)
     plan = mg.Plan(cfg.L, cfg.H, cfg.d, cfg.window, cfg.global_idx, cfg.extra_idx,
                    strip_max_cols=args.strip_max_cols, fine_kernel=args.fine_kernel,
-                   concurrency=args.concurrency, tau=args.tau)
+                   concurrency=args.concurrency, tau=args.tau, dense_chunk=args.dense_chunk)
     info = plan.info()
     BH = cfg.B * cfg.H
     useful = 4.0 * info["nnz_total"] * cfg.d * BH

@@ -119,7 +119,8 @@ typedef struct {
   float tau;              /* tile rule: 0 -> every tile touched by the band of a non-global row is
                              coarse (default, A7); (0, 1] -> a tile is coarse iff its
                              non-global union elements number >= tau * block^2 (A17) */
-  int32_t reserved[1];
+  int32_t dense_chunk;    /* column tiles per dense-row (global-row) work item: 0 -> default (8),
+                             -1 -> one item per 128-row group; chunks are merged by log-sum-exp */
 } mg_plan_opts;
 
 MG_API mg_status mg_plan_create_ex(int64_t L, int32_t heads, int32_t d, int32_t window,

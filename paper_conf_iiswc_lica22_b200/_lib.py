@@ -31,7 +31,7 @@ class mg_tensor(C.Structure):
 class mg_plan_opts(C.Structure):
     _fields_ = [("block", C.c_int32), ("force_all_fine", C.c_int32), ("strip_max_cols", C.c_int32),
                 ("num_sms", C.c_int32), ("fine_kernel", C.c_int32), ("concurrency", C.c_int32),
-                ("tau", C.c_float), ("reserved", C.c_int32 * 1)]
+                ("tau", C.c_float), ("dense_chunk", C.c_int32)]
 
 
 class mg_plan_info(C.Structure):

@@ -24,19 +24,21 @@ class Plan:
     Options (test/ablation): block, force_all_fine, strip_max_cols, num_sms, fine_kernel
     (0 = warp-level tensor-core CSR kernel, 1 = CUDA-core CSR kernel), concurrency (0 = default,
     1 = serial fine -> coarse, 2 = concurrent streams with last-finisher row merge), tau (tile
-    density threshold; 0 = band rule).
+    density threshold; 0 = band rule), dense_chunk (column tiles per dense-row item; 0 = default 8,
+    -1 = no split).
     """
 
     def __init__(self, L: int, heads: int, d: int, window: int, global_idx=(), extra_idx=None, *,
                  block: int = 0, force_all_fine: bool = False, strip_max_cols: int = 0, num_sms: int = 0,
-                 fine_kernel: int = 0, concurrency: int = 0, tau: float = 0.0):
+                 fine_kernel: int = 0, concurrency: int = 0, tau: float = 0.0, dense_chunk: int = 0):
         lib = load()
         g = _i32(list(global_idx) if not isinstance(global_idx, np.ndarray) else global_idx).reshape(-1)
         e = _i32(np.zeros((0, 2)) if extra_idx is None else extra_idx).reshape(-1, 2)
         self._handle = C.c_void_p()
         self._lib = lib
-        opts = mg_plan_opts(block, int(force_all_fine), strip_max_cols, num_sms, fine_kernel, concurrency, tau)
-        if block or force_all_fine or strip_max_cols or num_sms or fine_kernel or concurrency or tau:
+        opts = mg_plan_opts(block, int(force_all_fine), strip_max_cols, num_sms, fine_kernel, concurrency, tau,
+                            dense_chunk)
+        if block or force_all_fine or strip_max_cols or num_sms or fine_kernel or concurrency or tau or dense_chunk:
             st = lib.mg_plan_create_ex(L, heads, d, window, _ptr_i32(g), g.size, _ptr_i32(e), e.shape[0],
                                        C.byref(opts), C.byref(self._handle))
         else:

@@ -54,6 +54,7 @@ struct mg_plan_s {
   cudaEvent_t fork_ev = nullptr, join_ev = nullptr;
   std::vector<void*> allocs;
   mg::Item* d_items = nullptr;
+  mg::Item* d_items_split = nullptr;   // dense items split into column chunks (chosen per forward)
   mg::TileRef* d_trefs = nullptr;
   uint64_t* d_masks = nullptr;
   int32_t* d_strip_cols = nullptr;
@@ -68,6 +69,8 @@ struct mg_plan_s {
   size_t part_cap = 0;      // in (row, bh) partial slots
   uint8_t* d_stage = nullptr;
   size_t stage_cap = 0;     // bytes
+  uint8_t* d_dense = nullptr;   // split dense items: partials, then counters (zeroed at allocation)
+  size_t dense_cap = 0;         // in (b*h) units
   // staged (paper-dataflow) path: canonical plan on the device, uploaded on first use
   bool staged_uploaded = false;
   int32_t *d_bsr_row_ptr = nullptr, *d_bsr_col = nullptr, *d_tile_row = nullptr, *d_csr_row_ptr = nullptr,
@@ -108,6 +111,7 @@ struct mg_plan_s {
     for (void* p : allocs) cudaFree(p);
     if (d_part) cudaFree(d_part);
     if (d_stage) cudaFree(d_stage);
+    if (d_dense) cudaFree(d_dense);
     if (d_staged_ws) cudaFree(d_staged_ws);
   }
 };
@@ -136,6 +140,7 @@ mg_status upload(mg_plan_s* p) {
   if (major != 10) return fail(MG_ERR_UNSUPPORTED, "this library is built for sm_100a (B200) only");
   const mg::HostPlan& h = p->hp;
   if ((e = upload_vec(p, &p->d_items, h.items)) != cudaSuccess ||
+      (e = upload_vec(p, &p->d_items_split, h.items_split)) != cudaSuccess ||
       (e = upload_vec(p, &p->d_trefs, h.trefs)) != cudaSuccess ||
       (e = upload_vec(p, &p->d_masks, h.dev_masks)) != cudaSuccess ||
       (e = upload_vec(p, &p->d_strip_cols, h.strip_cols)) != cudaSuccess ||
@@ -171,6 +176,12 @@ mg_status create_impl(int64_t L, int32_t heads, int32_t d, int32_t window, const
     concurrency = opts->concurrency;
     if (!(opts->tau >= 0.f && opts->tau <= 1.f)) return fail(MG_ERR_INVALID_ARG, "tau must be in [0, 1]");
     po.tau = opts->tau;
+    if (opts->dense_chunk < -1) return fail(MG_ERR_INVALID_ARG, "dense_chunk must be >= -1");
+    if (opts->dense_chunk < 0) po.dense_split = 1;
+    if (opts->dense_chunk > 0) {
+      po.dense_split = 2;
+      po.dense_chunk = opts->dense_chunk;
+    }
   }
   mg_plan_s* p = new (std::nothrow) mg_plan_s();
   if (!p) return fail(MG_ERR_OUT_OF_MEMORY, "host allocation failed");
@@ -242,7 +253,8 @@ mg_status check_all(const mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, 
   if (K->dtype != Q->dtype || V->dtype != Q->dtype || O->dtype != Q->dtype)
     return fail(MG_ERR_UNSUPPORTED, "Q/K/V/O dtypes differ");
   if (!p->hp.kernel_ready) return fail(MG_ERR_UNSUPPORTED, "the forward requires block == 128");
-  if ((int64_t)Q->batch * p->hp.heads >= (int64_t(1) << 31) / std::max<int64_t>(1, (int64_t)p->hp.items.size()))
+  if ((int64_t)Q->batch * p->hp.heads >=
+      (int64_t(1) << 31) / std::max<int64_t>(1, (int64_t)std::max(p->hp.items.size(), p->hp.items_split.size())))
     return fail(MG_ERR_UNSUPPORTED, "batch * heads * work items exceeds int32");
   // the fine kernels address a gathered row as (uint32) col * stride_l elements
   if ((p->hp.L - 1) * std::max(K->stride_l, V->stride_l) >= (int64_t(1) << 32))
@@ -348,6 +360,33 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
   float* part_c_acc = p->d_part + cap * 66;
   float2* part_c_ml = reinterpret_cast<float2*>(p->d_part + cap * 130);
   int32_t* part_flags = reinterpret_cast<int32_t*>(p->d_part + cap * 132);
+  // split dense-row items (a work list with the global rows' column tiles in chunks): chosen when
+  // the unsplit dense items would be few against the SMs (each would be a long serial chain), or
+  // forced by the plan option; per (b*h, row group) chunk partials + monotone counters
+  const bool use_split = h.dense_nsplit > 1 && h.n_dense_groups > 0 &&
+                         (h.opts.dense_split == 2 ||
+                          (h.opts.dense_split == 0 && (int64_t)h.n_dense_groups * BH * 2 <= p->num_sms));
+  float* dense_part = nullptr;
+  int32_t* dense_ctr = nullptr;
+  if (use_split) {
+    const size_t per_bh_part = (size_t)h.n_dense_groups * h.dense_nsplit * 128 * 68 * sizeof(float);
+    const size_t per_bh_ctr = (size_t)h.n_dense_groups * sizeof(int32_t);
+    if ((size_t)BH > p->dense_cap) {
+      if (p->d_dense) {
+        if ((e = cudaFreeAsync(p->d_dense, stream)) != cudaSuccess) return cuda_fail(e, "cudaFreeAsync");
+        p->d_dense = nullptr;
+      }
+      const size_t bytes = (size_t)BH * (per_bh_part + per_bh_ctr);
+      if ((e = cudaMallocAsync(reinterpret_cast<void**>(&p->d_dense), bytes, stream)) != cudaSuccess)
+        return e == cudaErrorMemoryAllocation ? fail(MG_ERR_OUT_OF_MEMORY, "workspace allocation failed")
+                                              : cuda_fail(e, "cudaMallocAsync");
+      if ((e = cudaMemsetAsync(p->d_dense + (size_t)BH * per_bh_part, 0, (size_t)BH * per_bh_ctr, stream)) != cudaSuccess)
+        return cuda_fail(e, "cudaMemsetAsync");
+      p->dense_cap = (size_t)BH;
+    }
+    dense_part = reinterpret_cast<float*>(p->d_dense);
+    dense_ctr = reinterpret_cast<int32_t*>(p->d_dense + p->dense_cap * per_bh_part);
+  }
   cudaStream_t fstream = stream;
   if (concurrent) {
     if (!p->side) {
@@ -407,7 +446,7 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
     if (!encode_map(&tq, Q) || !encode_map(&tk, K) || !encode_map(&tv, V))
       return fail(MG_ERR_CUDA, "cuTensorMapEncodeTiled failed (driver entry point unavailable or bad layout)");
     mg::CoarseParams cp{};
-    cp.items = p->d_items;
+    cp.items = use_split ? p->d_items_split : p->d_items;
     cp.trefs = p->d_trefs;
     cp.masks = p->d_masks;
     cp.strip_cols = p->d_strip_cols;
@@ -420,8 +459,8 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
     cp.L = h.L;
     cp.H = h.heads;
     cp.BH = BH;
-    cp.n_items = (int)h.items.size();
-    cp.n_dense_items = h.n_dense_items;
+    cp.n_items = (int)(use_split ? h.items_split.size() : h.items.size());
+    cp.n_dense_items = use_split ? h.n_dense_items_split : h.n_dense_items;
     cp.n_global = (int)h.global_rows.size();
     cp.n_fine_rows = nf;
     cp.total_units = cp.n_items * BH;
@@ -430,6 +469,10 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
     cp.part_c_acc = part_c_acc;
     cp.part_c_ml = part_c_ml;
     cp.part_flags = part_flags;
+    cp.dense_part = dense_part;
+    cp.dense_ctr = dense_ctr;
+    cp.n_dense_groups = h.n_dense_groups;
+    cp.dense_nsplit = h.dense_nsplit;
     static const int dbg = [] {
       const char* e = std::getenv("MG_DEBUG_FLAGS");
       return e ? std::atoi(e) : 0;
@@ -454,7 +497,7 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
       static const bool no_tma_gather = std::getenv("MG_NO_TMA_GATHER") != nullptr;   // A/B diagnostics
       cp.gather_tma = !no_tma_gather && encode_map2d(&tq2, Q, &cp.rq) && encode_map2d(&tk2, K, &cp.rk) &&
                       encode_map2d(&tv2, V, &cp.rv);
-      if ((e = mg::launch_coarse_pp(cp, tq, tk, tv, tq2, tk2, tv2, bf16, std::min(2 * sms, cp.total_units),
+      if ((e = mg::launch_coarse_pp(cp, tq, tk, tv, tq2, tk2, tv2, bf16, use_split, std::min(2 * sms, cp.total_units),
                                     stream)) != cudaSuccess)
         return cuda_fail(e, "coarse kernel launch");
     }

@@ -64,6 +64,7 @@ struct __align__(16) Ctl {
   uint64_t k_full[kSt], k_empty[kSt], v_full[kSt], v_empty[kSt];
   uint64_t s_full, s_free, p_full, pv_done;
   uint32_t tmem_base;
+  int32_t dense_last;                         // split dense item: this chunk finished its row group last
 };
 
 constexpr size_t kSmemBytes = 1024 + 6 * kTileBytes + kSt * kMaskBytes + sizeof(Ctl);
@@ -362,7 +363,7 @@ __device__ __forceinline__ void softmax_tile(const TileCtx& x, float& m, float& 
 
 }  // namespace
 
-template <bool kBF16>
+template <bool kBF16, bool kSplit>
 __global__ void __launch_bounds__(kThreads, 2)
     coarse_pp_kernel(const __grid_constant__ CUtensorMap tmq, const __grid_constant__ CUtensorMap tmk,
                      const __grid_constant__ CUtensorMap tmv, const __grid_constant__ CUtensorMap tmq2,
@@ -686,6 +687,57 @@ __global__ void __launch_bounds__(kThreads, 2)
       tc_fence_before();
       if (threadIdx.x == 0) tl_rec(p, n - 1, 12);
       bool skip = false;
+      if (kSplit && item.kind == 1 && item.nrowsB > 1) {
+        // split dense-row item: publish this chunk's (m, l, acc) per row; the chunk that finishes
+        // its row group last merges all chunks by log-sum-exp and writes O (a-4 over column chunks)
+        const size_t gidx = (size_t)ubh * p.n_dense_groups + item.rowB;
+        float* part = p.dense_part + ((gidx * p.dense_nsplit + item.turns) * 128 + t) * 68;
+        if (t < item.nrowsA) {
+          float4* dst = reinterpret_cast<float4*>(part);
+#pragma unroll
+          for (int i = 0; i < 16; ++i)
+            __stcg(dst + i, make_float4(__uint_as_float(o[i >> 3][(i & 7) * 4]), __uint_as_float(o[i >> 3][(i & 7) * 4 + 1]),
+                                        __uint_as_float(o[i >> 3][(i & 7) * 4 + 2]),
+                                        __uint_as_float(o[i >> 3][(i & 7) * 4 + 3])));
+          __stcg(reinterpret_cast<float2*>(part + 64), make_float2(m, l));
+        }
+        __threadfence();
+        named_bar_sync(1, 128);
+        if (threadIdx.x == 0)
+          ctl->dense_last = (atomicAdd(p.dense_ctr + gidx, 1) % item.nrowsB) == item.nrowsB - 1;
+        named_bar_sync(1, 128);
+        skip = !ctl->dense_last;
+        if (!skip && t < item.nrowsA) {
+          __threadfence();
+          const float* base = p.dense_part + (gidx * p.dense_nsplit * 128 + t) * 68;
+          float mm = -INFINITY;
+          for (int k = 0; k < item.nrowsB; ++k) mm = fmaxf(mm, __ldcg(base + (size_t)k * 128 * 68 + 64));
+          const float mu0 = mm == -INFINITY ? 0.f : mm;
+          // merged row accumulated in place of this chunk's O registers
+#pragma unroll
+          for (int i = 0; i < 64; ++i) o[i >> 5][i & 31] = 0u;
+          float den0 = 0.f;
+          for (int k = 0; k < item.nrowsB; ++k) {
+            const float* pk = base + (size_t)k * 128 * 68;
+            const float2 ml = __ldcg(reinterpret_cast<const float2*>(pk + 64));
+            const float a = ex2((ml.x - mu0) * c);
+            den0 += ml.y * a;
+            const float4* src = reinterpret_cast<const float4*>(pk);
+#pragma unroll
+            for (int i = 0; i < 16; ++i) {
+              const float4 v = __ldcg(src + i);
+              uint32_t* q4 = &o[i >> 3][(i & 7) * 4];
+              q4[0] = __float_as_uint(fmaf(v.x, a, __uint_as_float(q4[0])));
+              q4[1] = __float_as_uint(fmaf(v.y, a, __uint_as_float(q4[1])));
+              q4[2] = __float_as_uint(fmaf(v.z, a, __uint_as_float(q4[2])));
+              q4[3] = __float_as_uint(fmaf(v.w, a, __uint_as_float(q4[3])));
+            }
+          }
+          // hand the merged row to the common store below: O = o (scale 1), l = den0, m = mm
+          m = mm;
+          l = den0;
+        }
+      }
       if (slot_f >= 0 && p.concurrent) {
         // publish this row's coarse partial; the side that finishes the row second merges both
         float4* dst = reinterpret_cast<float4*>(p.part_c_acc + fidx * 64);
@@ -765,8 +817,11 @@ __global__ void __launch_bounds__(kThreads, 2)
 
 cudaError_t launch_coarse_pp(const CoarseParams& p, const CUtensorMap& tmq, const CUtensorMap& tmk,
                              const CUtensorMap& tmv, const CUtensorMap& tmq2, const CUtensorMap& tmk2,
-                             const CUtensorMap& tmv2, bool bf16, int grid, cudaStream_t stream) {
-  auto kern = bf16 ? coarse_pp_kernel<true> : coarse_pp_kernel<false>;
+                             const CUtensorMap& tmv2, bool bf16, bool split_dense, int grid, cudaStream_t stream) {
+  // the split-dense-item epilogue is compiled only into the instantiation that needs it (its code
+  // costs the common path registers)
+  auto kern = bf16 ? (split_dense ? coarse_pp_kernel<true, true> : coarse_pp_kernel<true, false>)
+                   : (split_dense ? coarse_pp_kernel<false, true> : coarse_pp_kernel<false, false>);
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBytes);
   if (e != cudaSuccess) return e;
   kern<<<grid, kThreads, kSmemBytes, stream>>>(tmq, tmk, tmv, tmq2, tmk2, tmv2, p);

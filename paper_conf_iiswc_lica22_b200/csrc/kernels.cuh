@@ -46,6 +46,10 @@ struct CoarseParams {
   float* part_c_acc;          // [BH * n_fine_rows * 64] coarse partial (written when concurrent)
   float2* part_c_ml;
   int32_t* part_flags;        // [BH * n_fine_rows], +1 per side per forward (even between forwards)
+  // split dense-row items (Item::nrowsB > 1): per (b*h, row group) chunk partials and counters
+  float* dense_part;          // [BH][n_dense_groups][dense_nsplit][128][68]: acc[64], m, l, pad (16-B rows)
+  int32_t* dense_ctr;         // [BH][n_dense_groups], +1 per finished chunk (monotone, mod nsplit)
+  int32_t n_dense_groups, dense_nsplit;
   int32_t debug_flags;        // diagnostics (env MG_DEBUG_FLAGS): 1 = no softmax arithmetic, 2 = no MMA, 4 = no loads,
                               // 16 = no S loads from TMEM, 64 = MMA ignores P-ready/O-free (timing only)
 };
@@ -98,7 +102,7 @@ cudaError_t launch_coarse(const CoarseParams& p, const CUtensorMap& tmq, const C
 // Paired-pipeline variant: two CTAs per SM (grid = 2 x SMs), see coarse_pp_sm100.cu.
 cudaError_t launch_coarse_pp(const CoarseParams& p, const CUtensorMap& tmq, const CUtensorMap& tmk,
                              const CUtensorMap& tmv, const CUtensorMap& tmq2, const CUtensorMap& tmk2,
-                             const CUtensorMap& tmv2, bool bf16, int grid, cudaStream_t stream);
+                             const CUtensorMap& tmv2, bool bf16, bool split_dense, int grid, cudaStream_t stream);
 cudaError_t launch_fine(const FineParams& p, bool bf16, cudaStream_t stream);
 // Warp-level tensor-core variant (mma.sync m16n8k16), the default; see fine_mma.cu.
 cudaError_t launch_fine_mma(const FineParams& p, bool bf16, cudaStream_t stream);

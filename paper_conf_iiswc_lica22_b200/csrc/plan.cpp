@@ -186,14 +186,29 @@ std::string build_plan(HostPlan& p, int64_t L, int32_t heads, int32_t d, int32_t
   const int64_t G = (int64_t)p.global_rows.size();
   for (int64_t k = 0; k < G; k += 128) {
     const int32_t nr = (int32_t)std::min<int64_t>(128, G - k);
-    Item it{1, (int32_t)k, 0, (int32_t)nb, (int32_t)p.trefs.size(), nr, 0, 0, 0ull, 0ull};
+    Item it{1, (int32_t)k, (int32_t)(k / 128), (int32_t)nb, (int32_t)p.trefs.size(), nr, 1, 0, 0ull, 0ull};
     for (int64_t J = 0; J < nb; ++J) {
       const int32_t m = (J == nb - 1) ? ragged_mask : kMaskFull;
       p.trefs.push_back(TileRef{(int32_t)(J * B), 0, 128, m, kMaskSkip, 0, 0, 0});
       count(m, 128, nr);
     }
     p.items.push_back(it);
+    p.n_dense_groups++;
   }
+  // the same rows split into chunks of <= dense_chunk column tiles (a separate work list, chosen
+  // per forward when the dense items would be too few to spread over the SMs); the chunks' fp32
+  // partials are merged by the last chunk to finish. The chunks reuse the unsplit items' tile refs.
+  const int64_t chunk = std::max<int64_t>(1, std::min<int64_t>(opts.dense_chunk, nb));
+  const int32_t nsplit = (int32_t)((nb + chunk - 1) / chunk);
+  p.dense_nsplit = nsplit;
+  for (const Item& d : p.items) {
+    for (int32_t sc = 0; sc < nsplit; ++sc) {
+      const int64_t J0 = sc * chunk, J1 = std::min<int64_t>(nb, J0 + chunk);
+      p.items_split.push_back(Item{1, d.rowA, d.rowB, (int32_t)(J1 - J0), d.tref_begin + (int32_t)J0, d.nrowsA,
+                                   nsplit, sc, 0ull, 0ull});
+    }
+  }
+  p.n_dense_items_split = (int32_t)p.items_split.size();
   p.n_dense_items = (int32_t)p.items.size();
 
   // distinct CSR columns of each row block
@@ -260,6 +275,7 @@ std::string build_plan(HostPlan& p, int64_t L, int32_t heads, int32_t d, int32_t
     }
     it.ntiles = (int32_t)p.trefs.size() - it.tref_begin;
     p.items.push_back(it);
+    p.items_split.push_back(it);
   }
 
   // CSR rows left to the CUDA-core fine kernel

@@ -15,14 +15,19 @@ struct PlanOptions {
   bool force_all_fine = false;
   int strip_max_cols = 128;  // <= 0 disables the tensor-core strip path for the CSR residual
   double tau = 0.0;          // 0: band rule; > 0: a tile is coarse iff its density >= tau (A17)
+  int dense_chunk = 8;       // column tiles per split dense-row work item
+  int dense_split = 0;       // 0: split dense items when the forward has few of them, 1: never, 2: always
 };
 
 // Device work-list encodings. The tensor-core kernel processes one 128-row
 // Q tile per work item against the item's list of K/V tiles.
 //   Item {kind, rowA, -, ntiles, tref_begin, nrowsA, ...}:
 //     kind 0: band row block starting at row rowA (a block with coarse tiles);
-//     kind 1: gathered global rows global_rows[rowA ..) against every column tile (dense part);
-//     nrowsA = valid rows of the Q tile. rowB, nrowsB, turns, useA, useB are reserved (0).
+//     kind 1: gathered global rows global_rows[rowA ..) against column tiles (dense part); the
+//       row group's nb column tiles are split into nrowsB chunks of <= dense_chunk tiles, one item
+//       each: rowB = row group, turns = chunk index; with nrowsB > 1 every chunk writes an fp32
+//       partial and the last chunk to finish merges them;
+//     nrowsA = valid rows of the Q tile. useA, useB are reserved (0).
 //   TileRef {arg, kind, ncols, maskA, -}: one K/V tile of the item:
 //     kind 0 = contiguous column tile at column `arg`; kind 1 = gathered strip whose column list
 //     starts at strip_cols[arg] (ncols a multiple of 32); maskA = index of a 128 x 2-word bitmask,
@@ -49,6 +54,10 @@ struct HostPlan {
   std::vector<uint64_t> dev_masks;   // 128 x 2 words per entry: tiles, then strip/ragged masks
   std::vector<Item> items;           // dense items first, then band items in row-block order
   int32_t n_dense_items = 0;
+  int32_t n_dense_groups = 0, dense_nsplit = 1;
+  // alternative work list with the dense items split into chunks (same band items after them)
+  std::vector<Item> items_split;
+  int32_t n_dense_items_split = 0;
   std::vector<TileRef> trefs;
   std::vector<int32_t> strip_cols;   // gathered column lists (padded with -1)
   std::vector<int32_t> fine_rows;    // rows executed by the CUDA-core fine kernel; bit 31 = write final O

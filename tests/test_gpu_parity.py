@@ -123,6 +123,19 @@ def test_density_threshold_plans(tau):
     check(run_gpu(plan, q, k, v), oracle_full(q, k, v, 96, G, E))
 
 
+@pytest.mark.parametrize("dense_chunk", [-1, 1, 3, 8])
+@pytest.mark.parametrize("L,G", [(1024, list(range(40))), (1000, [0, 5, 999]), (640, list(range(0, 640, 4)))])
+def test_dense_row_split_chunks(dense_chunk, L, G):
+    """Global rows split over column-tile chunks (a-4) merged by the last chunk; repeated calls keep
+    the per-group counters consistent; >128 global rows give several row groups."""
+    G = np.array(G, np.int32)
+    q, k, v = make_qkv(2, 3, L, 64, seed=31, dist="adversarial", global_idx=G)
+    plan = mg.Plan(L, 3, 64, 64, G, None, dense_chunk=dense_chunk)
+    ref = oracle_full(q, k, v, 64, G, np.zeros((0, 2), np.int32))
+    for _ in range(3):
+        check(run_gpu(plan, q, k, v), ref)
+
+
 def test_strip_path_c2_pattern_small():
     """C2-like globals [0, 32) with fewer blocks: the CSR residual runs as tensor-core strips."""
     L, G = 1024, np.arange(32, dtype=np.int32)
