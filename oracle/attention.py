@@ -49,11 +49,15 @@ def _softmax_rows(S: np.ndarray):
 
 
 def dense_masked_attention(Q, K, V, window: int, global_idx, extra_idx, *, M=None,
-                           chunk: int = 256, return_P: bool = False):
+                           chunk: int = 256, return_P: bool = False, valid_len: int | None = None):
     """O-4: S = QK^T/sqrt(d); S[~M] = -inf; P = softmax(S); O = P V, for one head (fp64).
 
     Rows are processed in chunks so that L = 16384 fits in memory. If ``M`` (L x L bool)
     is given it is used instead of the pattern arguments.
+
+    ``valid_len`` = n (padding, "zero-padding ... masked with -inf"; reading A18):
+    tokens at positions >= n are padding, so M(r, c) additionally requires r < n and c < n; the
+    padded rows have no valid element and get O = 0 (reading A10).
     """
     L, d = Q.shape
     sf = 1.0 / math.sqrt(d)
@@ -65,6 +69,8 @@ def dense_masked_attention(Q, K, V, window: int, global_idx, extra_idx, *, M=Non
     for r0 in range(0, L, chunk):
         r1 = min(L, r0 + chunk)
         Mb = M[r0:r1] if M is not None else mask_rows(r0, r1, L, window, g, extra)
+        if valid_len is not None:
+            Mb = Mb & (np.arange(r0, r1) < valid_len)[:, None] & (np.arange(L) < valid_len)[None, :]
         S = (Q[r0:r1] @ K.T) * sf
         S = np.where(Mb, S, -np.inf)
         P = _softmax_rows(S)
@@ -99,13 +105,19 @@ def csr_reference(Q, K, V, window: int, global_idx, extra_idx):
     return O
 
 
-def attention_rows(Q, K, V, rows, window: int, gflags: np.ndarray, extra: ExtraIndex):
-    """The same definition evaluated only at the given rows (for sampled full-size parity)."""
+def attention_rows(Q, K, V, rows, window: int, gflags: np.ndarray, extra: ExtraIndex,
+                   valid_len: int | None = None):
+    """The same definition evaluated only at the given rows (for sampled full-size parity);
+    ``valid_len`` as in dense_masked_attention."""
     L, d = Q.shape
     sf = 1.0 / math.sqrt(d)
     out = np.zeros((len(rows), V.shape[1]))
     for i, r in enumerate(rows):
+        if valid_len is not None and r >= valid_len:
+            continue
         c = mask_row_cols(int(r), L, window, gflags, extra)
+        if valid_len is not None:
+            c = c[c < valid_len]
         if c.size == 0:
             continue
         s = (K[c] @ Q[r]) * sf

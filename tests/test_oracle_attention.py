@@ -189,3 +189,27 @@ def test_bf16_inputs_exact_upcast():
     # every value is exactly representable in bf16: 8 significant bits
     m, e = np.frexp(x[x != 0])
     assert np.all((m * 2**8) == np.round(m * 2**8))
+
+
+# ---------------------------------------------------------------- padding (valid length, A18)
+@pytest.mark.parametrize("seed", range(6))
+def test_padding_equals_truncated_problem(seed):
+    """Padding to L with n valid tokens = the same pattern on the first n tokens only (a problem of
+    length n, computed without any padding), and O = 0 on the padded rows."""
+    rng = np.random.default_rng(700 + seed)
+    L = int(rng.integers(40, 160))
+    n = int(rng.integers(1, L + 1))
+    window = 2 * int(rng.integers(0, 20))
+    G = np.unique(rng.integers(0, L, size=int(rng.integers(0, 4)))).astype(np.int32)
+    E = rng.integers(0, L, size=(int(rng.integers(0, 3 * L)), 2)).astype(np.int32)
+    Q, K, V = (rng.standard_normal((L, 64)) for _ in range(3))
+    got = dense_masked_attention(Q, K, V, window, G, E, valid_len=n)
+    Gn = G[G < n]
+    En = E[(E[:, 0] < n) & (E[:, 1] < n)]
+    ref = dense_masked_attention(Q[:n], K[:n], V[:n], window, Gn, En)
+    np.testing.assert_allclose(got[:n], ref, rtol=0, atol=1e-12)
+    assert (got[n:] == 0).all()
+    g = global_flags(L, G)
+    rows = list(range(0, L, 7))
+    np.testing.assert_allclose(attention_rows(Q, K, V, rows, window, g, ExtraIndex(L, E), valid_len=n),
+                               got[rows], rtol=0, atol=1e-12)
