@@ -182,6 +182,15 @@ MG_API mg_status mg_plan_export(mg_plan_t plan, int32_t* bsr_row_ptr, int32_t* b
 MG_API mg_status mg_sparse_attention_fwd(mg_plan_t plan, const mg_tensor* Q, const mg_tensor* K,
                                   const mg_tensor* V, mg_tensor* O, void* stream);
 
+/* Padded batch ("zero-padding ... masked with -inf"; reading A18): valid_len is a
+ * DEVICE int32 array [batch] (values clamped to [0, L]); for batch element b with n = valid_len[b]
+ * the mask is M(r,c) AND r < n AND c < n, and the rows r >= n of O are written as 0. Same
+ * arguments, asynchrony and errors as mg_sparse_attention_fwd (INVALID_ARG also for a null
+ * valid_len). The staged entry points do not take a padding mask. */
+MG_API mg_status mg_sparse_attention_fwd_padded(mg_plan_t plan, const mg_tensor* Q, const mg_tensor* K,
+                                         const mg_tensor* V, mg_tensor* O, const int32_t* valid_len,
+                                         void* stream);
+
 /* Same computation with HOST tensors: copies Q/K/V host->device into plan-owned staging
  * buffers on `stream`, runs the forward, copies O device->host, all stream-ordered and
  * asynchronous (host buffers should be pinned for the copies to overlap; the caller

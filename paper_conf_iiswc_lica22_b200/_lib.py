@@ -18,7 +18,7 @@ EXPORTED = [
     "mg_plan_create", "mg_plan_create_ex", "mg_plan_destroy", "mg_last_error", "mg_plan_info_get",
     "mg_plan_export", "mg_sparse_attention_fwd", "mg_sparse_attention_fwd_host", "mg_selftest_umma",
     "mg_abi_version", "mg_plan_set_profiling", "mg_plan_get_profile", "mg_plan_set_trace",
-    "mg_staged_get_sizes", "mg_staged_sddmm", "mg_staged_softmax", "mg_staged_spmm", "mg_sparse_attention_fwd_staged",
+    "mg_sparse_attention_fwd_padded", "mg_staged_get_sizes", "mg_staged_sddmm", "mg_staged_softmax", "mg_staged_spmm", "mg_sparse_attention_fwd_staged",
 ]
 
 
@@ -79,6 +79,7 @@ def load() -> C.CDLL:
     tp = C.POINTER(mg_tensor)
     lib.mg_sparse_attention_fwd.argtypes = [P, tp, tp, tp, tp, P]
     lib.mg_sparse_attention_fwd_host.argtypes = [P, tp, tp, tp, tp, P]
+    lib.mg_sparse_attention_fwd_padded.argtypes = [P, tp, tp, tp, tp, P, P]
     lib.mg_selftest_umma.argtypes = [C.c_int32, P, P, P, P]
     lib.mg_plan_set_profiling.argtypes = [P, C.c_int32]
     lib.mg_plan_get_profile.argtypes = [P, C.POINTER(mg_profile)]

@@ -140,6 +140,20 @@ def sparse_attention_fwd(plan: Plan, Q, K, V, O=None, stream=None):
     return O
 
 
+def sparse_attention_fwd_padded(plan: Plan, Q, K, V, valid_len, O=None, stream=None):
+    """mg_sparse_attention_fwd_padded: valid_len is a device int32 tensor [B] (tokens >= valid_len[b]
+    are padding: masked as columns, zero output rows)."""
+    import torch
+    if O is None:
+        O = torch.empty(Q.shape, dtype=Q.dtype, device=Q.device)
+    if valid_len.dtype != torch.int32 or not valid_len.is_cuda or valid_len.numel() != Q.shape[0]:
+        raise ValueError("valid_len must be a CUDA int32 tensor with one entry per batch element")
+    dq, dk, dv, do = tensor_desc(Q), tensor_desc(K), tensor_desc(V), tensor_desc(O)
+    check(plan._lib.mg_sparse_attention_fwd_padded(plan.handle, C.byref(dq), C.byref(dk), C.byref(dv), C.byref(do),
+                                                   C.c_void_p(valid_len.data_ptr()), _stream_ptr(stream)))
+    return O
+
+
 def sparse_attention_fwd_host(plan: Plan, Q, K, V, O, stream=None):
     """mg_sparse_attention_fwd_host on dense HOST tensors (pinned for async copies). Asynchronous:
     synchronise `stream` before reading O."""

@@ -318,7 +318,7 @@ mg::TensorView view(const mg_tensor* t) {
 constexpr bool kConcurrentDefault = false;
 
 mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const mg_tensor* V, mg_tensor* O,
-                   cudaStream_t stream) {
+                   cudaStream_t stream, const int32_t* valid_len = nullptr) {
   mg_status s = upload(p);
   if (s != MG_OK) return s;
   int dev = -1;
@@ -427,6 +427,7 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
     fp.H = h.heads; fp.BH = BH; fp.n_fine_rows = nf;
     fp.scale_log2 = scale_log2;
     fp.concurrent = concurrent;
+    fp.valid_len = valid_len;
     fp.part_c_acc = part_c_acc;
     fp.part_c_ml = part_c_ml;
     fp.part_flags = part_flags;
@@ -466,6 +467,7 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
     cp.total_units = cp.n_items * BH;
     cp.scale_log2 = scale_log2;
     cp.concurrent = concurrent;
+    cp.valid_len = valid_len;
     cp.part_c_acc = part_c_acc;
     cp.part_c_ml = part_c_ml;
     cp.part_flags = part_flags;
@@ -708,6 +710,16 @@ mg_status mg_sparse_attention_fwd(mg_plan_t plan, const mg_tensor* Q, const mg_t
   mg_status s = check_all(plan, Q, K, V, O, false);
   if (s != MG_OK) return s;
   return fwd_impl(plan, Q, K, V, O, static_cast<cudaStream_t>(stream));
+}
+
+mg_status mg_sparse_attention_fwd_padded(mg_plan_t plan, const mg_tensor* Q, const mg_tensor* K, const mg_tensor* V,
+                                         mg_tensor* O, const int32_t* valid_len, void* stream) {
+  g_err.clear();
+  if (!plan) return fail(MG_ERR_INVALID_ARG, "plan is null");
+  if (!valid_len) return fail(MG_ERR_INVALID_ARG, "valid_len is null");
+  mg_status s = check_all(plan, Q, K, V, O, false);
+  if (s != MG_OK) return s;
+  return fwd_impl(plan, Q, K, V, O, static_cast<cudaStream_t>(stream), valid_len);
 }
 
 mg_status mg_sparse_attention_fwd_host(mg_plan_t plan, const mg_tensor* Q, const mg_tensor* K, const mg_tensor* V,

@@ -59,6 +59,7 @@ struct __align__(16) Ctl {
   Slot slot[kItems];
   int32_t kcols[kSt];                         // ncols of the tile in K stage s (producer -> MMA)
   int2 vdesc[kSt];                            // {ncols, maskA} of the tile in V stage s (-> softmax)
+  uint32_t cmask[kSt][4];                     // padding: valid columns of the tile in V stage s
   uint64_t item_full[kItems], item_empty[kItems];
   uint64_t q_full[2], q_empty[2];
   uint64_t k_full[kSt], k_empty[kSt], v_full[kSt], v_empty[kSt];
@@ -289,6 +290,7 @@ struct TileCtx {
   uint32_t tl;          // TMEM address of this warp's lane quarter (column 0)
   uint32_t mask_row;    // shared address of this row's 16 mask bytes
   bool masked;          // the tile has a bitmask (else all columns valid)
+  const uint32_t* cmask;  // padding: 4 words of valid columns (shared memory), or null
   uint32_t n;           // tile sequence number (CTA lifetime)
   int j;                // tile index within the item
   uint32_t s_free, pv_done, p_full;
@@ -309,9 +311,19 @@ __device__ __forceinline__ void softmax_tile(const TileCtx& x, float& m, float& 
   tc_fence_before();
   __syncwarp();
   if (lane == 0) mbar_arrive(x.s_free);                 // S may be overwritten by S(n+1)
-  if (x.masked) {
-    const int4 mw = ld_shared_v4(x.mask_row);
-    const uint32_t w4[4] = {(uint32_t)mw.x, (uint32_t)mw.y, (uint32_t)mw.z, (uint32_t)mw.w};
+  if (x.masked || x.cmask) {
+    uint32_t w4[4] = {~0u, ~0u, ~0u, ~0u};
+    if (x.masked) {
+      const int4 mw = ld_shared_v4(x.mask_row);
+      w4[0] = (uint32_t)mw.x;
+      w4[1] = (uint32_t)mw.y;
+      w4[2] = (uint32_t)mw.z;
+      w4[3] = (uint32_t)mw.w;
+    }
+    if (x.cmask) {
+#pragma unroll
+      for (int q = 0; q < NQ; ++q) w4[q] &= x.cmask[q];
+    }
 #pragma unroll
     for (int q = 0; q < NQ; ++q) apply_mask(r[q], w4[q]);
   }
@@ -363,7 +375,7 @@ __device__ __forceinline__ void softmax_tile(const TileCtx& x, float& m, float& 
 
 }  // namespace
 
-template <bool kBF16, bool kSplit>
+template <bool kBF16, bool kSplit, bool kPad>
 __global__ void __launch_bounds__(kThreads, 2)
     coarse_pp_kernel(const __grid_constant__ CUtensorMap tmq, const __grid_constant__ CUtensorMap tmk,
                      const __grid_constant__ CUtensorMap tmv, const __grid_constant__ CUtensorMap tmq2,
@@ -499,6 +511,39 @@ __global__ void __launch_bounds__(kThreads, 2)
           }
           mbar_wait(bar(ctl->v_empty[st]), sph);
           const uint32_t mbytes = maskA >= 0 ? kMaskBytes : 0;
+          if (kPad) {
+            // padding: the tile's columns below n_b (published with vdesc by the v_full arrive)
+            const int nvalid = min(max(__ldg(p.valid_len + bb), 0), (int)p.L);
+            uint32_t w[4];
+            if (kind == 0) {
+#pragma unroll
+              for (int q = 0; q < 4; ++q) {
+                const int lim = nvalid - (arg + 32 * q);
+                w[q] = lim >= 32 ? ~0u : (lim <= 0 ? 0u : (1u << lim) - 1u);
+              }
+            } else {
+              const int4 cx = load_idx4(p.strip_cols + arg, 4 * lane, ncols);
+              const uint32_t b0 = __ballot_sync(0xffffffffu, cx.x >= 0 && cx.x < nvalid);
+              const uint32_t b1 = __ballot_sync(0xffffffffu, cx.y >= 0 && cx.y < nvalid);
+              const uint32_t b2 = __ballot_sync(0xffffffffu, cx.z >= 0 && cx.z < nvalid);
+              const uint32_t b3 = __ballot_sync(0xffffffffu, cx.w >= 0 && cx.w < nvalid);
+              // column 32q + i is entry i % 4 of lane 8q + i / 4
+#pragma unroll
+              for (int q = 0; q < 4; ++q) {
+                uint32_t v = 0;
+#pragma unroll
+                for (int i = 0; i < 32; ++i) {
+                  const uint32_t bk = (i & 3) == 0 ? b0 : (i & 3) == 1 ? b1 : (i & 3) == 2 ? b2 : b3;
+                  v |= ((bk >> (8 * q + (i >> 2))) & 1u) << i;
+                }
+                w[q] = v;
+              }
+            }
+            if (lane == 0) {
+#pragma unroll
+              for (int q = 0; q < 4; ++q) ctl->cmask[st][q] = w[q];
+            }
+          }
           if (lane == 0) {
             ctl->vdesc[st] = make_int2(ncols, maskA);   // published by the v_full arrive
             tl_rec(p, g, 6);
@@ -657,7 +702,8 @@ __global__ void __launch_bounds__(kThreads, 2)
         mbar_wait(bar(ctl->v_full[st]), (n / kSt) & 1);
         tc_fence_after();
         const int2 desc = ctl->vdesc[st];                 // {ncols, maskA}
-        const TileCtx tc{tl, sMsk + st * kMaskBytes + t * 16, desc.y >= 0, n, j, bar(ctl->s_free),
+        const TileCtx tc{tl, sMsk + st * kMaskBytes + t * 16, desc.y >= 0, kPad ? ctl->cmask[st] : nullptr,
+                         n, j, bar(ctl->s_free),
                          bar(ctl->pv_done), bar(ctl->p_full), c, thresh, &p};
         if (threadIdx.x == 0) tl_rec(p, n, 0);
         switch (desc.x >> 5) {                            // 32-column chunks of the tile
@@ -766,7 +812,16 @@ __global__ void __launch_bounds__(kThreads, 2)
       // element in this item (a global row inside a band row block: it is owned by the dense-row
       // part, A5) is not written. (Staging the tile through shared memory for 4-rows-per-
       // instruction stores measured 10% slower: tools/experiments/.)
-      if (r_out >= 0 && mt != -INFINITY && !skip) {
+      // padding (A18): rows at or beyond the batch element's valid length are written as 0 by
+      // every item that holds them (whatever the merge protocol decided)
+      const bool pad_row = kPad && r_out >= 0 &&
+                           r_out >= min(max(__ldg(p.valid_len + ubh / p.H), 0), (int)p.L);
+      if (pad_row) {
+        const int bb = ubh / p.H, hh = ubh % p.H;
+        uint4* orow = reinterpret_cast<uint4*>(p.o.data + bb * p.o.sb + hh * p.o.sh + (int64_t)r_out * p.o.sl);
+#pragma unroll
+        for (int i = 0; i < 8; ++i) orow[i] = make_uint4(0u, 0u, 0u, 0u);
+      } else if (r_out >= 0 && mt != -INFINITY && !skip) {
         const float inv = __frcp_rn(den);
         const int bb = ubh / p.H, hh = ubh % p.H;
         uint16_t* orow = p.o.data + bb * p.o.sb + hh * p.o.sh + (int64_t)r_out * p.o.sl;
@@ -818,10 +873,15 @@ __global__ void __launch_bounds__(kThreads, 2)
 cudaError_t launch_coarse_pp(const CoarseParams& p, const CUtensorMap& tmq, const CUtensorMap& tmk,
                              const CUtensorMap& tmv, const CUtensorMap& tmq2, const CUtensorMap& tmk2,
                              const CUtensorMap& tmv2, bool bf16, bool split_dense, int grid, cudaStream_t stream) {
-  // the split-dense-item epilogue is compiled only into the instantiation that needs it (its code
-  // costs the common path registers)
-  auto kern = bf16 ? (split_dense ? coarse_pp_kernel<true, true> : coarse_pp_kernel<true, false>)
-                   : (split_dense ? coarse_pp_kernel<false, true> : coarse_pp_kernel<false, false>);
+  // the split-dense-item epilogue and the padding masks are compiled only into the instantiations
+  // that need them (their code costs the common path registers)
+  using K = void (*)(const CUtensorMap, const CUtensorMap, const CUtensorMap, const CUtensorMap, const CUtensorMap,
+                     const CUtensorMap, const CoarseParams);
+  static const K table[8] = {coarse_pp_kernel<false, false, false>, coarse_pp_kernel<false, false, true>,
+                             coarse_pp_kernel<false, true, false>,  coarse_pp_kernel<false, true, true>,
+                             coarse_pp_kernel<true, false, false>,  coarse_pp_kernel<true, false, true>,
+                             coarse_pp_kernel<true, true, false>,   coarse_pp_kernel<true, true, true>};
+  const K kern = table[(bf16 ? 4 : 0) + (split_dense ? 2 : 0) + (p.valid_len ? 1 : 0)];
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBytes);
   if (e != cudaSuccess) return e;
   kern<<<grid, kThreads, kSmemBytes, stream>>>(tmq, tmk, tmv, tmq2, tmk2, tmv2, p);

@@ -105,7 +105,7 @@ constexpr int kSmemBytes = kWarps * kStages * kStageBytes;
 // warps in the grid; neighbouring warps stay on neighbouring rows of the same head, so the head's
 // K/V stay in L2), and the gather pointer runs ahead across row boundaries, so a row's first gathers
 // are in flight while the previous row is computed (one row is only ~11 steps).
-template <bool kBF16>
+template <bool kBF16, bool kPad>
 __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(const FineParams p) {
   extern __shared__ __align__(128) uint8_t fsm[];
   const int lane = threadIdx.x & 31;
@@ -188,6 +188,10 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(con
       qb[j] = __ldg(reinterpret_cast<const uint32_t*>(qrow + 16 * j + 8 + 2 * t));
     }
     const int beg = __ldg(p.row_ptr + fi), end = __ldg(p.row_ptr + fi + 1);
+    // padding (A18): columns >= n_b are masked; a row >= n_b is written as 0 if it is final (a row
+    // with a coarse part is zeroed by the coarse kernel)
+    const int nvalid = kPad ? max(__ldg(p.valid_len + bb), 0) : 0x7fffffff;
+    const bool pad_row = kPad && r >= nvalid;
 
     float m = -INFINITY, l = 0.f;
     float acc[4][4];
@@ -223,11 +227,18 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(con
       const int rem = end - base - 2 * t;
       float s[4] = {rem > 0 ? sa[0][0] + sa[1][0] : -INFINITY, rem > 1 ? sa[0][1] + sa[1][1] : -INFINITY,
                     rem > 8 ? sb[0][0] + sb[1][0] : -INFINITY, rem > 9 ? sb[0][1] + sb[1][1] : -INFINITY};
+      if (kPad) {   // padding: mask the columns at or beyond n_b (index loads hit L1)
+        const int o4[4] = {0, 1, 8, 9};
+#pragma unroll
+        for (int i = 0; i < 4; ++i)
+          if (rem > o4[i] && __ldg(p.cols + base + 2 * t + o4[i]) >= nvalid) s[i] = -INFINITY;
+      }
       // ---- online softmax over the step (warp-uniform max: lanes with equal t hold equal values)
       float mx = fmaxf(fmaxf(s[0], s[1]), fmaxf(s[2], s[3]));
       mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, 1));
       mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, 2));
-      if (mx > m + thresh) {   // also taken on the first step (m = -inf); mx is finite (>= 1 valid nnz)
+      // (mx = -inf only when padding masked the whole step: nothing to add)
+      if (mx > m + thresh) {   // also taken on the first step (m = -inf) unless mx = -inf
         const float alpha = ex2((m - mx) * c);
         l *= alpha;
 #pragma unroll
@@ -236,7 +247,7 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(con
           for (int e = 0; e < 4; ++e) acc[j][e] *= alpha;
         m = mx;
       }
-      const float nbias = -m * c;
+      const float nbias = m == -INFINITY ? 0.f : -m * c;   // (all-masked steps: every p is 0)
       float pr[4];
 #pragma unroll
       for (int i = 0; i < 4; ++i) {
@@ -294,6 +305,10 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(con
         }
       }
     }
+    if (pad_row) {
+      write_o = final_out;   // rows with a coarse part are zeroed by the coarse kernel
+      v0 = v1 = 0.f;
+    }
     if (write_o) {
       uint16_t* orow = p.o.data + bb * p.o.sb + hh * p.o.sh + (int64_t)r * p.o.sl;
       const uint32_t pk = pack2<kBF16>(v0 * inv, v1 * inv);
@@ -307,20 +322,22 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(con
 cudaError_t launch_fine_mma(const FineParams& p, bool bf16, cudaStream_t stream) {
   const int64_t warps = (int64_t)p.BH * p.n_fine_rows;
   if (warps == 0) return cudaSuccess;
-  auto kern = bf16 ? fine_mma_kernel<true> : fine_mma_kernel<false>;
+  auto kern = bf16 ? (p.valid_len ? fine_mma_kernel<true, true> : fine_mma_kernel<true, false>)
+                   : (p.valid_len ? fine_mma_kernel<false, true> : fine_mma_kernel<false, false>);
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytes);
   if (e != cudaSuccess) return e;
   // persistent grid: every resident block slot of every SM, or fewer if the rows are few
-  static int per_sm = 0, sms = 0;
-  if (per_sm == 0) {
-    int dev = 0;
+  static int per_sm[4] = {0, 0, 0, 0}, sms = 0;   // per kernel variant
+  const int vi = (bf16 ? 2 : 0) + (p.valid_len ? 1 : 0);
+  if (per_sm[vi] == 0) {
+    int dev = 0, n = 0;
     if ((e = cudaGetDevice(&dev)) != cudaSuccess ||
         (e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev)) != cudaSuccess ||
-        (e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kWarps * 32, kSmemBytes)) != cudaSuccess)
+        (e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kern, kWarps * 32, kSmemBytes)) != cudaSuccess)
       return e;
-    per_sm = std::max(per_sm, 1);
+    per_sm[vi] = std::max(n, 1);
   }
-  const int64_t blocks = std::min<int64_t>((warps + kWarps - 1) / kWarps, (int64_t)per_sm * sms);
+  const int64_t blocks = std::min<int64_t>((warps + kWarps - 1) / kWarps, (int64_t)per_sm[vi] * sms);
   kern<<<(unsigned)blocks, kWarps * 32, kSmemBytes, stream>>>(p);
   return cudaGetLastError();
 }

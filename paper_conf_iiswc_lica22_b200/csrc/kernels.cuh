@@ -46,6 +46,9 @@ struct CoarseParams {
   float* part_c_acc;          // [BH * n_fine_rows * 64] coarse partial (written when concurrent)
   float2* part_c_ml;
   int32_t* part_flags;        // [BH * n_fine_rows], +1 per side per forward (even between forwards)
+  // padding (A18): valid length per batch element (device [B]) or null; columns >= n_b are masked
+  // for every row, rows >= n_b are written as 0
+  const int32_t* valid_len;
   // split dense-row items (Item::nrowsB > 1): per (b*h, row group) chunk partials and counters
   float* dense_part;          // [BH][n_dense_groups][dense_nsplit][128][68]: acc[64], m, l, pad (16-B rows)
   int32_t* dense_ctr;         // [BH][n_dense_groups], +1 per finished chunk (monotone, mod nsplit)
@@ -65,6 +68,7 @@ struct FineParams {
   int32_t H, BH, n_fine_rows;
   float scale_log2;
   int32_t concurrent;         // see CoarseParams::concurrent
+  const int32_t* valid_len;   // see CoarseParams::valid_len
   const float* part_c_acc;
   const float2* part_c_ml;
   int32_t* part_flags;

@@ -270,3 +270,35 @@ def test_full_size_sampled(cfg, fine_kernel, concurrency):
         errs.append(np.abs(got[b, h, rows] - ref))
     e = np.concatenate(errs)
     assert e.max() <= TOL_MAX and e.mean() <= TOL_MEAN, (e.max(), e.mean())
+
+
+# ------------------------------------------------------------------ padding (valid length, A18)
+@pytest.mark.parametrize("case", ["mixed", "c1", "fine_only", "dense_split", "concurrent"])
+def test_padded_batch(case):
+    """mg_sparse_attention_fwd_padded: per-sample valid lengths (including 0, full, and cuts inside
+    row blocks and strips); every part (tiles, strips, CSR rows, dense rows, split dense chunks,
+    concurrent merge) masks the padded columns and zeroes the padded rows."""
+    if case == "c1":
+        c = get_config("C1")
+        B, H, L, window, G, E = 4, 1, c.L, c.window, c.global_idx, c.extra_idx
+        kw = {}
+    else:
+        m = MIXED
+        B, H, L, window, G = 4, m["H"], m["L"], m["window"], m["G"]
+        E = mixed_extra(L, seed=12)
+        kw = {"fine_only": dict(strip_max_cols=-1), "dense_split": dict(dense_chunk=2),
+              "concurrent": dict(strip_max_cols=-1, concurrency=2), "mixed": {}}[case]
+    q, k, v = make_qkv(B, H, L, 64, seed=41, dist="adversarial", global_idx=G)
+    plan = mg.Plan(L, H, 64, window, G, E, **kw)
+    lens = np.array([L, 0, L // 2 + 37, 129][:B], np.int32)
+    Q, K, V = (to_device(x) for x in (q, k, v))
+    vl = torch.from_numpy(lens).cuda()
+    got = from_device(mg.sparse_attention_fwd_padded(plan, Q, K, V, vl))
+    for b in range(B):
+        for h in range(H):
+            Qh, Kh, Vh = head_inputs_f64(q, k, v, b, h)
+            ref = dense_masked_attention(Qh, Kh, Vh, window, G, E, valid_len=int(lens[b]))
+            mx, mean = err_stats(got[b, h], ref)
+            # adversarial inputs: bf16 output rounding grows with |O| (as for the peaky case)
+            assert mx <= TOL_MAX * max(1.0, np.abs(ref).max() / 4) and mean <= TOL_MEAN, (case, b, h, mx, mean)
+            assert (got[b, h, lens[b]:] == 0).all()
