@@ -499,7 +499,11 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
       static const bool no_tma_gather = std::getenv("MG_NO_TMA_GATHER") != nullptr;   // A/B diagnostics
       cp.gather_tma = !no_tma_gather && encode_map2d(&tq2, Q, &cp.rq) && encode_map2d(&tk2, K, &cp.rk) &&
                       encode_map2d(&tv2, V, &cp.rv);
-      if ((e = mg::launch_coarse_pp(cp, tq, tk, tv, tq2, tk2, tv2, bf16, use_split, std::min(2 * sms, cp.total_units),
+      CUtensorMap to;
+      std::memset(&to, 0, sizeof(to));
+      static const bool no_tma_store = std::getenv("MG_NO_TMA_STORE") != nullptr;   // A/B diagnostics
+      cp.tma_store = !no_tma_store && encode_map(&to, O);
+      if ((e = mg::launch_coarse_pp(cp, tq, tk, tv, tq2, tk2, tv2, to, bf16, use_split, std::min(2 * sms, cp.total_units),
                                     stream)) != cudaSuccess)
         return cuda_fail(e, "coarse kernel launch");
     }

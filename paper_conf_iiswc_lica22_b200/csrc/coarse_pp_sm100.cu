@@ -380,7 +380,7 @@ __global__ void __launch_bounds__(kThreads, 2)
     coarse_pp_kernel(const __grid_constant__ CUtensorMap tmq, const __grid_constant__ CUtensorMap tmk,
                      const __grid_constant__ CUtensorMap tmv, const __grid_constant__ CUtensorMap tmq2,
                      const __grid_constant__ CUtensorMap tmk2, const __grid_constant__ CUtensorMap tmv2,
-                     const CoarseParams p) {
+                     const __grid_constant__ CUtensorMap tmo, const CoarseParams p) {
   extern __shared__ uint8_t smem_raw[];
   const uint32_t sbase = (smem_u32(smem_raw) + 1023u) & ~1023u;
   const uint32_t sQ = sbase;
@@ -657,7 +657,7 @@ __global__ void __launch_bounds__(kThreads, 2)
                    idesc_s, kk > 0);
           mma_commit(bar(ctl->s_full));
           mma_commit(bar(ctl->k_empty[st]));
-          if (j == ntiles - 1) mma_commit(bar(ctl->q_empty[qs]));   // last S of the item
+          // (q_empty is arrived by the softmax epilogue: the Q buffer also stages the item's O tile)
           tl_rec(p, n, 3);
           if (pend.valid) issue_pv(pend);
           pend = Pend{n, st, ncols, j == 0, true};
@@ -816,7 +816,36 @@ __global__ void __launch_bounds__(kThreads, 2)
       // every item that holds them (whatever the merge protocol decided)
       const bool pad_row = kPad && r_out >= 0 &&
                            r_out >= min(max(__ldg(p.valid_len + ubh / p.H), 0), (int)p.L);
-      if (pad_row) {
+      // (only blocks without global rows and without CUDA-core CSR rows: no other writer, no partial
+      // to merge; measured: merging partials in this path costs C2 3% and gains nothing on C4)
+      const bool tma_out = !kPad && p.tma_store && item.kind == 0 && (item.useA & 3) == 3;   // uniform per item
+      if (tma_out) {
+        // normalised rows into the item's Q buffer (SWIZZLE_128B layout of the O tensor map), then one
+        // TMA store of the 128 x 64 tile (rows beyond L are clipped by the map)
+        const uint32_t sO = sQ + (it & 1) * kTileBytes;
+        const float inv = (r_out >= 0 && mt != -INFINITY) ? __frcp_rn(den) : 0.f;
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+#pragma unroll
+          for (int q8 = 0; q8 < 4; ++q8) {
+            float a[8];
+#pragma unroll
+            for (int i = 0; i < 8; ++i) a[i] = __uint_as_float(o[h][q8 * 8 + i]) * (ac * inv);
+            const int ch = h * 4 + q8;
+            asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(sO + t * 128 + ((ch ^ (t & 7)) << 4)),
+                         "r"(pack2<kBF16>(a[0], a[1])), "r"(pack2<kBF16>(a[2], a[3])), "r"(pack2<kBF16>(a[4], a[5])),
+                         "r"(pack2<kBF16>(a[6], a[7]))
+                         : "memory");
+          }
+        }
+        fence_proxy_async_smem();
+        named_bar_sync(1, 128);
+        if (threadIdx.x == 0) {
+          tma_store_4d(&tmo, sO, 0, item.rowA, ubh % p.H, ubh / p.H);
+          bulk_commit_group();
+          bulk_wait_group_read0();   // the buffer is reloaded with a later item's Q after q_empty
+        }
+      } else if (pad_row) {
         const int bb = ubh / p.H, hh = ubh % p.H;
         uint4* orow = reinterpret_cast<uint4*>(p.o.data + bb * p.o.sb + hh * p.o.sh + (int64_t)r_out * p.o.sl);
 #pragma unroll
@@ -852,7 +881,12 @@ __global__ void __launch_bounds__(kThreads, 2)
           }
         }
       }
-      if (threadIdx.x == 0) tl_rec(p, n - 1, 13);
+      // the item's Q buffer is free (its last S MMA has completed: pv_done above; its O tile, if
+      // staged there, has been read by the TMA store)
+      if (threadIdx.x == 0) {
+        mbar_arrive(bar(ctl->q_empty[it & 1]));
+        tl_rec(p, n - 1, 13);
+      }
     }
   }
 
@@ -872,11 +906,12 @@ __global__ void __launch_bounds__(kThreads, 2)
 
 cudaError_t launch_coarse_pp(const CoarseParams& p, const CUtensorMap& tmq, const CUtensorMap& tmk,
                              const CUtensorMap& tmv, const CUtensorMap& tmq2, const CUtensorMap& tmk2,
-                             const CUtensorMap& tmv2, bool bf16, bool split_dense, int grid, cudaStream_t stream) {
+                             const CUtensorMap& tmv2, const CUtensorMap& tmo, bool bf16, bool split_dense, int grid,
+                             cudaStream_t stream) {
   // the split-dense-item epilogue and the padding masks are compiled only into the instantiations
   // that need them (their code costs the common path registers)
   using K = void (*)(const CUtensorMap, const CUtensorMap, const CUtensorMap, const CUtensorMap, const CUtensorMap,
-                     const CUtensorMap, const CoarseParams);
+                     const CUtensorMap, const CUtensorMap, const CoarseParams);
   static const K table[8] = {coarse_pp_kernel<false, false, false>, coarse_pp_kernel<false, false, true>,
                              coarse_pp_kernel<false, true, false>,  coarse_pp_kernel<false, true, true>,
                              coarse_pp_kernel<true, false, false>,  coarse_pp_kernel<true, false, true>,
@@ -884,7 +919,7 @@ cudaError_t launch_coarse_pp(const CoarseParams& p, const CUtensorMap& tmq, cons
   const K kern = table[(bf16 ? 4 : 0) + (split_dense ? 2 : 0) + (p.valid_len ? 1 : 0)];
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBytes);
   if (e != cudaSuccess) return e;
-  kern<<<grid, kThreads, kSmemBytes, stream>>>(tmq, tmk, tmv, tmq2, tmk2, tmv2, p);
+  kern<<<grid, kThreads, kSmemBytes, stream>>>(tmq, tmk, tmv, tmq2, tmk2, tmv2, tmo, p);
   return cudaGetLastError();
 }
 

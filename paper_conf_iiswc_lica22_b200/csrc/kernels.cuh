@@ -53,6 +53,9 @@ struct CoarseParams {
   float* dense_part;          // [BH][n_dense_groups][dense_nsplit][128][68]: acc[64], m, l, pad (16-B rows)
   int32_t* dense_ctr;         // [BH][n_dense_groups], +1 per finished chunk (monotone, mod nsplit)
   int32_t n_dense_groups, dense_nsplit;
+  // band items whose rows are all theirs to write (Item::useA) store O by TMA from shared memory
+  // (the item's Q buffer) instead of per-thread row stores
+  int32_t tma_store;
   int32_t debug_flags;        // diagnostics (env MG_DEBUG_FLAGS): 1 = no softmax arithmetic, 2 = no MMA, 4 = no loads,
                               // 16 = no S loads from TMEM, 64 = MMA ignores P-ready/O-free (timing only)
 };
@@ -106,7 +109,8 @@ cudaError_t launch_coarse(const CoarseParams& p, const CUtensorMap& tmq, const C
 // Paired-pipeline variant: two CTAs per SM (grid = 2 x SMs), see coarse_pp_sm100.cu.
 cudaError_t launch_coarse_pp(const CoarseParams& p, const CUtensorMap& tmq, const CUtensorMap& tmk,
                              const CUtensorMap& tmv, const CUtensorMap& tmq2, const CUtensorMap& tmk2,
-                             const CUtensorMap& tmv2, bool bf16, bool split_dense, int grid, cudaStream_t stream);
+                             const CUtensorMap& tmv2, const CUtensorMap& tmo, bool bf16, bool split_dense, int grid,
+                             cudaStream_t stream);
 cudaError_t launch_fine(const FineParams& p, bool bf16, cudaStream_t stream);
 // Warp-level tensor-core variant (mma.sync m16n8k16), the default; see fine_mma.cu.
 cudaError_t launch_fine_mma(const FineParams& p, bool bf16, cudaStream_t stream);

@@ -290,6 +290,19 @@ std::string build_plan(HostPlan& p, int64_t L, int32_t heads, int32_t d, int32_t
       p.fine_rows.push_back((int32_t)r | (has_tiles ? 0 : (int32_t)0x80000000));
     }
   }
+  // band items whose rows are all written by this item (bit 0: no global row; bit 1: no CUDA-core
+  // CSR row, which the concurrent mode may let the fine kernel write)
+  for (auto* list : {&p.items, &p.items_split}) {
+    for (Item& it : *list) {
+      if (it.kind != 0) continue;
+      bool no_global = true, no_fine = true;
+      for (int64_t r = it.rowA; r < it.rowA + it.nrowsA; ++r) {
+        no_global = no_global && !isG[r];
+        no_fine = no_fine && p.fine_slot[r] < 0;
+      }
+      it.useA = (no_global ? 1ull : 0ull) | (no_fine ? 2ull : 0ull);
+    }
+  }
   p.fine_row_ptr.assign(1, 0);
   for (int32_t enc : p.fine_rows) {
     const int32_t r = enc & 0x7fffffff;

@@ -27,7 +27,10 @@ struct PlanOptions {
 //       row group's nb column tiles are split into nrowsB chunks of <= dense_chunk tiles, one item
 //       each: rowB = row group, turns = chunk index; with nrowsB > 1 every chunk writes an fp32
 //       partial and the last chunk to finish merges them;
-//     nrowsA = valid rows of the Q tile. useA, useB are reserved (0).
+//     nrowsA = valid rows of the Q tile. useA (kind 0): bit 0 = no global row in the block, bit 1 =
+//     no CUDA-core CSR row (then every row is written by this item alone, so O may be stored as a
+//     tile; bit 1 matters only in the concurrent mode).
+//     useB is reserved (0).
 //   TileRef {arg, kind, ncols, maskA, -}: one K/V tile of the item:
 //     kind 0 = contiguous column tile at column `arg`; kind 1 = gathered strip whose column list
 //     starts at strip_cols[arg] (ncols a multiple of 32); maskA = index of a 128 x 2-word bitmask,
