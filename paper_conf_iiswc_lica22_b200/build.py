@@ -22,6 +22,8 @@ VARIANTS = {"watchdog": ["-DMG_WATCHDOG"], "timeline": ["-DMG_TIMELINE"], "trace
             # A/B of the share of exponentials emulated on the FMA pipe (pairs of 16 per chunk)
             "e0": ["-DMG_EXP_EMU=0"], "e4": ["-DMG_EXP_EMU=4"], "e8": ["-DMG_EXP_EMU=8"],
             "maxpass": ["-DMG_SKIP_MAX=0"],
+            # coarse softmax: 32-column chunks whose exponentials precede the P.V(n-1) wait
+            "pre0": ["-DMG_PRE_CHUNKS=0"], "pre1": ["-DMG_PRE_CHUNKS=1"], "pre2": ["-DMG_PRE_CHUNKS=2"],
             # fine tensor-core kernel: cp.async ring stages per warp (default 2), min blocks per SM
             "fs3": ["-DMG_FINE_STAGES=3"], "fb4": ["-DMG_FINE_MINB=4"], "fb6": ["-DMG_FINE_MINB=6"],
             "fb8": ["-DMG_FINE_MINB=8"],

@@ -286,6 +286,11 @@ __device__ __forceinline__ void tl_item(const CoarseParams& p, uint32_t it, int 
 #endif
 }
 
+#ifndef MG_PRE_CHUNKS
+#define MG_PRE_CHUNKS 4
+#endif
+constexpr int kPre = MG_PRE_CHUNKS;   // chunks whose exponentials precede the P.V(n-1) wait
+
 struct TileCtx {
   uint32_t tl;          // TMEM address of this warp's lane quarter (column 0)
   uint32_t mask_row;    // shared address of this row's 16 mask bytes
@@ -341,6 +346,12 @@ __device__ __forceinline__ void softmax_tile(const TileCtx& x, float& m, float& 
   const float2 c2 = make_float2(x.c, x.c);
   const float2 nb2 = make_float2(-mu * x.c, -mu * x.c);
   float2 rs[2] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
+  // the first kPre chunks' exponentials are computed before waiting for P.V(n-1) (they overlap its
+  // issue and execution; their packed P waits in registers)
+  constexpr int kPreN = kPre < NQ ? kPre : NQ;
+  uint32_t pre[kPreN > 0 ? kPreN : 1][16];
+#pragma unroll
+  for (int q = 0; q < kPreN; ++q) chunk_exp<kBF16>(r[q], c2, nb2, rs, pre[q]);
   // P.V(n-1) has consumed P(n-1) and updated O: rescale O if the max moved, then store P(n)
   // chunk by chunk as it is produced (the other CTA on this SM keeps the pipes busy meanwhile)
   if (x.n > 0) mbar_wait(x.pv_done, (x.n - 1) & 1);
@@ -358,7 +369,9 @@ __device__ __forceinline__ void softmax_tile(const TileCtx& x, float& m, float& 
     }
   }
 #pragma unroll
-  for (int q = 0; q < NQ; ++q) {
+  for (int q = 0; q < kPreN; ++q) tmem_st16(x.tl + kTP + q * 16, pre[q]);
+#pragma unroll
+  for (int q = kPreN; q < NQ; ++q) {
     uint32_t pk[16];
     chunk_exp<kBF16>(r[q], c2, nb2, rs, pk);
     tmem_st16(x.tl + kTP + q * 16, pk);
