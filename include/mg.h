@@ -172,6 +172,7 @@ MG_API mg_status mg_plan_export(mg_plan_t plan, int32_t* bsr_row_ptr, int32_t* b
  *   O        device tensor, same shape; written for every (b, h, row).
  *   stream   a cudaStream_t (passed as void*); 0 = legacy default stream.
  * Asynchronous: returns after enqueueing; no host synchronisation on the steady-state path.
+ * O must not alias Q, K or V (Q/K/V tiles of later work items are read while O rows are written).
  * Q/K/V/O must stay alive until the stream work completes. The plan's fwd workspace (fp32
  * partial statistics of the CSR part) is plan-owned and grown stream-ordered on `stream`,
  * so one plan must not be used by two concurrent forwards on different streams.

@@ -7,16 +7,14 @@
 // while the gathers alone would run at ~22 TB/s from L2 (tools/microbench/gather_bw.cu).
 //
 // A step handles 16 nnz of the row, as two chunks A and B of 8. Lane = 4g + t.
-//   SDDMM  s^T = q . K_c^T as mma(M=16 x N=8 x K=16) x 4 (64 dims): A = q broadcast to all 16
-//          rows, B column n = gathered K row c_{chunk[n]}. The contraction order over d is free,
-//          so lane t owns dims {8t..8t+7} and {32+8t..32+8t+7} of both q and the K row it loads
-//          (two 16-byte loads, half-line contiguous per 4 lanes); mma j uses the lane's register
-//          pairs 2j, 2j+1 for k {2t,2t+1} and {2t+8,2t+9}. D: lane (g,t) gets s of chunk nnz 2t, 2t+1.
+//   SDDMM  s^T = q . K_c^T as mma(M=16 x N=8 x K=16) x 4 per chunk (64 dims): A = q broadcast to
+//          all 16 rows (lane registers straight from global memory), B column n = gathered K row
+//          of chunk nnz n (ldmatrix from the swizzled stage). D: lane (g,t) gets the scores of
+//          chunk nnz 2t and 2t+1.
 //   SpMM   O^T = V_c^T . p as mma(M=16 dims x N=8 x K=16 nnz) x 4 (64 dims): k = nnz (chunk A
 //          nnz 2t,2t+1 -> k 2t,2t+1; chunk B -> k 2t+8, 2t+9), which is exactly where the SDDMM
-//          left each lane's p, so P never moves between lanes; the M (dim) order is free too: lane
-//          g owns dims 8g..8g+7, i.e. one 16-byte load per gathered V row, and the A fragment is
-//          built from the four rows with byte permutes.
+//          left each lane's p, so P never moves between lanes; A = V^T from ldmatrix.trans. D:
+//          lane (g,t) holds output dims 16j+g, 16j+g+8 (all N columns equal), and writes j = t.
 // p is rounded to the operand dtype for the SpMM (as in the coarse kernel, A9); s, the
 // running max/sum and O accumulate in fp32. Lazy rescaling: the exponent keeps a stale max until
 // a step's max exceeds it by 8/c (p <= 256), warp-uniform because all lanes see the same max.
@@ -49,12 +47,6 @@ __device__ __forceinline__ void mma16816(float (&d)[4], uint32_t a0, uint32_t a1
         "{%0,%1,%2,%3};"
         : "+f"(d[0]), "+f"(d[1]), "+f"(d[2]), "+f"(d[3])
         : "r"(a0), "r"(a1), "r"(a2), "r"(a3), "r"(b0), "r"(b1));
-}
-
-__device__ __forceinline__ uint32_t prmt(uint32_t a, uint32_t b, uint32_t sel) {
-  uint32_t r;
-  asm("prmt.b32 %0, %1, %2, %3;" : "=r"(r) : "r"(a), "r"(b), "r"(sel));
-  return r;
 }
 
 template <bool kBF16>
