@@ -79,6 +79,14 @@ struct mg_plan_s {
   uint8_t* d_row_is_global = nullptr;
   uint8_t* d_staged_ws = nullptr;   // S, P and O_csr buffers of mg_sparse_attention_fwd_staged
   size_t staged_ws_cap = 0;
+  // TMA descriptors of the last forward's Q/K/V/O (re-encoded only when a tensor descriptor changes:
+  // cuTensorMapEncodeTiled is host work on every call otherwise)
+  struct Maps {
+    mg_tensor q, k, v, o;
+    bool valid = false, ok = false, gather_ok = false, store_ok = false;
+    CUtensorMap tq, tk, tv, tq2, tk2, tv2, to;
+    longlong3 rq, rk, rv;
+  } maps;
   // diagnostics: device event-trace buffer of the coarse kernel (CTA 0)
   unsigned long long* trace = nullptr;
   int32_t trace_cap = 0;
@@ -443,9 +451,26 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
     }
   }
   if (!h.items.empty()) {
-    CUtensorMap tq, tk, tv;
-    if (!encode_map(&tq, Q) || !encode_map(&tk, K) || !encode_map(&tv, V))
+    mg_plan_s::Maps& mp = p->maps;
+    if (!mp.valid || std::memcmp(&mp.q, Q, sizeof(mg_tensor)) || std::memcmp(&mp.k, K, sizeof(mg_tensor)) ||
+        std::memcmp(&mp.v, V, sizeof(mg_tensor)) || std::memcmp(&mp.o, O, sizeof(mg_tensor))) {
+      mp.q = *Q;
+      mp.k = *K;
+      mp.v = *V;
+      mp.o = *O;
+      mp.ok = encode_map(&mp.tq, Q) && encode_map(&mp.tk, K) && encode_map(&mp.tv, V);
+      std::memset(&mp.tq2, 0, sizeof(CUtensorMap));
+      std::memset(&mp.tk2, 0, sizeof(CUtensorMap));
+      std::memset(&mp.tv2, 0, sizeof(CUtensorMap));
+      std::memset(&mp.to, 0, sizeof(CUtensorMap));
+      mp.gather_ok = encode_map2d(&mp.tq2, Q, &mp.rq) && encode_map2d(&mp.tk2, K, &mp.rk) &&
+                     encode_map2d(&mp.tv2, V, &mp.rv);
+      mp.store_ok = encode_map(&mp.to, O);
+      mp.valid = true;
+    }
+    if (!mp.ok)
       return fail(MG_ERR_CUDA, "cuTensorMapEncodeTiled failed (driver entry point unavailable or bad layout)");
+    const CUtensorMap &tq = mp.tq, &tk = mp.tk, &tv = mp.tv;
     mg::CoarseParams cp{};
     cp.items = use_split ? p->d_items_split : p->d_items;
     cp.trefs = p->d_trefs;
@@ -492,18 +517,15 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
       if ((e = mg::launch_coarse(cp, tq, tk, tv, bf16, std::min(sms, cp.total_units), stream)) != cudaSuccess)
         return cuda_fail(e, "coarse kernel launch");
     } else {
-      CUtensorMap tq2, tk2, tv2;
-      std::memset(&tq2, 0, sizeof(tq2));
-      std::memset(&tk2, 0, sizeof(tk2));
-      std::memset(&tv2, 0, sizeof(tv2));
       static const bool no_tma_gather = std::getenv("MG_NO_TMA_GATHER") != nullptr;   // A/B diagnostics
-      cp.gather_tma = !no_tma_gather && encode_map2d(&tq2, Q, &cp.rq) && encode_map2d(&tk2, K, &cp.rk) &&
-                      encode_map2d(&tv2, V, &cp.rv);
-      CUtensorMap to;
-      std::memset(&to, 0, sizeof(to));
+      cp.gather_tma = !no_tma_gather && mp.gather_ok;
+      cp.rq = mp.rq;
+      cp.rk = mp.rk;
+      cp.rv = mp.rv;
       static const bool no_tma_store = std::getenv("MG_NO_TMA_STORE") != nullptr;   // A/B diagnostics
-      cp.tma_store = !no_tma_store && encode_map(&to, O);
-      if ((e = mg::launch_coarse_pp(cp, tq, tk, tv, tq2, tk2, tv2, to, bf16, use_split, std::min(2 * sms, cp.total_units),
+      cp.tma_store = !no_tma_store && mp.store_ok;
+      if ((e = mg::launch_coarse_pp(cp, tq, tk, tv, mp.tq2, mp.tk2, mp.tv2, mp.to, bf16, use_split,
+                                    std::min(2 * sms, cp.total_units),
                                     stream)) != cudaSuccess)
         return cuda_fail(e, "coarse kernel launch");
     }
