@@ -26,7 +26,7 @@ VARIANTS = {"watchdog": ["-DMG_WATCHDOG"], "timeline": ["-DMG_TIMELINE"], "trace
             "pre0": ["-DMG_PRE_CHUNKS=0"], "pre1": ["-DMG_PRE_CHUNKS=1"], "pre2": ["-DMG_PRE_CHUNKS=2"],
             # fine tensor-core kernel: cp.async ring stages per warp (default 2), min blocks per SM
             "fs3": ["-DMG_FINE_STAGES=3"], "fb4": ["-DMG_FINE_MINB=4"], "fb6": ["-DMG_FINE_MINB=6"],
-            "fb8": ["-DMG_FINE_MINB=8"],
+            "fb8": ["-DMG_FINE_MINB=8"], "fp2": ["-DMG_FINE_PAIRS=2"], "fp2b3": ["-DMG_FINE_PAIRS=2", "-DMG_FINE_MINB=3"],
             # skeleton cost: no exponentials / no MMAs / no loads (results are garbage)
             "dbg1": ["-DMG_DBG=1"], "dbg3": ["-DMG_DBG=3"], "dbg7": ["-DMG_DBG=7"]}
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")

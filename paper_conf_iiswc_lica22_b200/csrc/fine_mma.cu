@@ -79,9 +79,14 @@ __device__ __forceinline__ void ldsm_x4_t(uint32_t (&r)[4], uint32_t addr) {
 #ifndef MG_FINE_MINB
 #define MG_FINE_MINB 5
 #endif
+#ifndef MG_FINE_PAIRS
+#define MG_FINE_PAIRS 1
+#endif
 constexpr int kWarps = 4;                   // warps per block, one (row, b*h) each
+constexpr int kP = MG_FINE_PAIRS;           // 16-nnz pairs of 8-nnz chunks per step (1 or 2)
+constexpr int kS = 16 * kP;                 // nnz per step
 constexpr int kStages = MG_FINE_STAGES;     // smem ring stages per warp (kStages - 1 steps in flight)
-constexpr int kStageBytes = 32 * 128;       // 16 K rows + 16 V rows of 128 bytes
+constexpr int kStageBytes = 2 * kS * 128;  // kS K rows + kS V rows of 128 bytes
 constexpr int kSmemBytes = kWarps * kStages * kStageBytes;
 
 }  // namespace
@@ -110,9 +115,9 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(con
   const uint32_t ring = (uint32_t)__cvta_generic_to_shared(fsm) + (threadIdx.x >> 5) * (kStages * kStageBytes);
   // row strides fit 32 bits (checked by the forward's validation: (L - 1) * stride_l < 2^32)
   const uint32_t ksl = (uint32_t)p.k.sl, vsl = (uint32_t)p.v.sl;
-  uint32_t doff[4];   // swizzled destination of this lane's chunk in rows R_i = (lane >> 3) + 4 i
+  uint32_t doff[4 * kP];   // swizzled destination of this lane's chunk in rows R_i = (lane >> 3) + 4 i
 #pragma unroll
-  for (int i = 0; i < 4; ++i) {
+  for (int i = 0; i < 4 * kP; ++i) {
     const int R = (lane >> 3) + 4 * i;
     doff[i] = R * 128 + (((lane & 7) ^ (R & 7)) << 4);
   }
@@ -137,17 +142,17 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(con
   // the row's end they are -1 and read row 0 (masked scores, p = 0).
   auto issue_step = [&](uint32_t stg) {
     if (gi < nrows) {   // warp-uniform
-      const int nb0 = ibeg + 16 * is;
-      if ((is & 1) == 0) icol = nb0 + lane < iend ? __ldg(p.cols + nb0 + lane) : -1;
-      const int off = (is & 1) * 16 + (lane >> 3);
+      const int nb0 = ibeg + kS * is;
+      if (kP == 2 || (is & 1) == 0) icol = nb0 + lane < iend ? __ldg(p.cols + nb0 + lane) : -1;
+      const int off = (kP == 2 ? 0 : (is & 1) * 16) + (lane >> 3);
       const uint32_t st = ring + stg * kStageBytes;
 #pragma unroll
-      for (int i = 0; i < 4; ++i) {
+      for (int i = 0; i < 4 * kP; ++i) {
         const uint32_t cc = (uint32_t)max(__shfl_sync(0xffffffffu, icol, off + 4 * i), 0);
         cp_async16(st + doff[i], iK + cc * ksl);
-        cp_async16(st + doff[i] + 2048, iV + cc * vsl);
+        cp_async16(st + doff[i] + kS * 128, iV + cc * vsl);
       }
-      if (nb0 + 16 < iend) {
+      if (nb0 + kS < iend) {
         ++is;
       } else {
         gi += W;
@@ -192,7 +197,7 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(con
 #pragma unroll
       for (int e = 0; e < 4; ++e) acc[j][e] = 0.f;
 
-    for (int base = beg; base < end; base += 16) {
+    for (int base = beg; base < end; base += kS) {
       issue_step(istage);
       istage = istage == kStages - 1 ? 0 : istage + 1;
       cp_async_wait<kStages - 1>();
@@ -200,33 +205,41 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(con
       const uint32_t st = ring + stage * kStageBytes;
       stage = stage == kStages - 1 ? 0 : stage + 1;
 
-      // ---- SDDMM: chunk A (rows 0-7) -> sa, chunk B (rows 8-15) -> sb; lane holds nnz 2t, 2t+1 of
-      // each; two independent accumulators per chunk (dims 0-31, 32-63) shorten the MMA chains
-      float sa[2][4] = {{0.f, 0.f, 0.f, 0.f}, {0.f, 0.f, 0.f, 0.f}};
-      float sb[2][4] = {{0.f, 0.f, 0.f, 0.f}, {0.f, 0.f, 0.f, 0.f}};
+      // ---- SDDMM per pair: chunk A (rows 16pr + 0-7) and chunk B (rows 16pr + 8-15); lane holds
+      // nnz 2t, 2t+1 of each chunk; two independent accumulators per chunk (dims 0-31, 32-63)
+      float s[kP][4];
 #pragma unroll
-      for (int h = 0; h < 2; ++h) {   // dims 32h .. 32h + 31 = k16 steps 2h, 2h + 1
-        uint32_t ka[4], kb[4];
-        const uint32_t sw = ((uint32_t)(((lane >> 3) + 4 * h) ^ (lane & 7))) << 4;
-        ldsm_x4(ka, st + a_row + sw);
-        ldsm_x4(kb, st + b_row + sw);
-        mma16816<kBF16>(sa[h], qa[2 * h], qa[2 * h], qb[2 * h], qb[2 * h], ka[0], ka[1]);
-        mma16816<kBF16>(sb[h], qa[2 * h], qa[2 * h], qb[2 * h], qb[2 * h], kb[0], kb[1]);
-        mma16816<kBF16>(sa[h], qa[2 * h + 1], qa[2 * h + 1], qb[2 * h + 1], qb[2 * h + 1], ka[2], ka[3]);
-        mma16816<kBF16>(sb[h], qa[2 * h + 1], qa[2 * h + 1], qb[2 * h + 1], qb[2 * h + 1], kb[2], kb[3]);
-      }
-      // this lane's score positions: nnz base + 2t, + 2t+1 (chunk A), + 8 + 2t, + 9 + 2t (chunk B)
-      const int rem = end - base - 2 * t;
-      float s[4] = {rem > 0 ? sa[0][0] + sa[1][0] : -INFINITY, rem > 1 ? sa[0][1] + sa[1][1] : -INFINITY,
-                    rem > 8 ? sb[0][0] + sb[1][0] : -INFINITY, rem > 9 ? sb[0][1] + sb[1][1] : -INFINITY};
-      if (kPad) {   // padding: mask the columns at or beyond n_b (index loads hit L1)
-        const int o4[4] = {0, 1, 8, 9};
+      for (int pr = 0; pr < kP; ++pr) {
+        float sa[2][4] = {{0.f, 0.f, 0.f, 0.f}, {0.f, 0.f, 0.f, 0.f}};
+        float sb[2][4] = {{0.f, 0.f, 0.f, 0.f}, {0.f, 0.f, 0.f, 0.f}};
 #pragma unroll
-        for (int i = 0; i < 4; ++i)
-          if (rem > o4[i] && __ldg(p.cols + base + 2 * t + o4[i]) >= nvalid) s[i] = -INFINITY;
+        for (int h = 0; h < 2; ++h) {   // dims 32h .. 32h + 31 = k16 steps 2h, 2h + 1
+          uint32_t ka[4], kb[4];
+          const uint32_t sw = ((uint32_t)(((lane >> 3) + 4 * h) ^ (lane & 7))) << 4;
+          ldsm_x4(ka, st + pr * 2048 + a_row + sw);
+          ldsm_x4(kb, st + pr * 2048 + b_row + sw);
+          mma16816<kBF16>(sa[h], qa[2 * h], qa[2 * h], qb[2 * h], qb[2 * h], ka[0], ka[1]);
+          mma16816<kBF16>(sb[h], qa[2 * h], qa[2 * h], qb[2 * h], qb[2 * h], kb[0], kb[1]);
+          mma16816<kBF16>(sa[h], qa[2 * h + 1], qa[2 * h + 1], qb[2 * h + 1], qb[2 * h + 1], ka[2], ka[3]);
+          mma16816<kBF16>(sb[h], qa[2 * h + 1], qa[2 * h + 1], qb[2 * h + 1], qb[2 * h + 1], kb[2], kb[3]);
+        }
+        // this lane's positions: nnz base + 16pr + {2t, 2t+1} (chunk A), + {8 + 2t, 9 + 2t} (chunk B)
+        const int rem = end - base - 16 * pr - 2 * t;
+        s[pr][0] = rem > 0 ? sa[0][0] + sa[1][0] : -INFINITY;
+        s[pr][1] = rem > 1 ? sa[0][1] + sa[1][1] : -INFINITY;
+        s[pr][2] = rem > 8 ? sb[0][0] + sb[1][0] : -INFINITY;
+        s[pr][3] = rem > 9 ? sb[0][1] + sb[1][1] : -INFINITY;
+        if (kPad) {   // padding: mask the columns at or beyond n_b (index loads hit L1)
+          const int o4[4] = {0, 1, 8, 9};
+#pragma unroll
+          for (int i = 0; i < 4; ++i)
+            if (rem > o4[i] && __ldg(p.cols + base + 16 * pr + 2 * t + o4[i]) >= nvalid) s[pr][i] = -INFINITY;
+        }
       }
       // ---- online softmax over the step (warp-uniform max: lanes with equal t hold equal values)
-      float mx = fmaxf(fmaxf(s[0], s[1]), fmaxf(s[2], s[3]));
+      float mx = -INFINITY;
+#pragma unroll
+      for (int pr = 0; pr < kP; ++pr) mx = fmaxf(mx, fmaxf(fmaxf(s[pr][0], s[pr][1]), fmaxf(s[pr][2], s[pr][3])));
       mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, 1));
       mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, 2));
       // (mx = -inf only when padding masked the whole step: nothing to add)
@@ -240,20 +253,24 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(con
         m = mx;
       }
       const float nbias = m == -INFINITY ? 0.f : -m * c;   // (all-masked steps: every p is 0)
-      float pr[4];
 #pragma unroll
-      for (int i = 0; i < 4; ++i) {
-        pr[i] = ex2(fmaf(s[i], c, nbias));
-        l += pr[i];
-      }
-      const uint32_t pb0 = pack2<kBF16>(pr[0], pr[1]), pb1 = pack2<kBF16>(pr[2], pr[3]);
-      // ---- SpMM: O^T[dims 16j + g, 16j + g + 8] += V^T . p (A = V^T from ldmatrix.trans)
+      for (int pr = 0; pr < kP; ++pr) {
+        float pv[4];
 #pragma unroll
-      for (int j = 0; j < 4; ++j) {
-        uint32_t a[4];
-        const uint32_t ch = 2 * j + ((lane >> 3) & 1);
-        ldsm_x4_t(a, st + 2048 + vr * 128 + ((ch ^ (vr & 7)) << 4));
-        mma16816<kBF16>(acc[j], a[0], a[1], a[2], a[3], pb0, pb1);
+        for (int i = 0; i < 4; ++i) {
+          pv[i] = ex2(fmaf(s[pr][i], c, nbias));
+          l += pv[i];
+        }
+        const uint32_t pb0 = pack2<kBF16>(pv[0], pv[1]), pb1 = pack2<kBF16>(pv[2], pv[3]);
+        // ---- SpMM: O^T[dims 16j + g, 16j + g + 8] += V^T . p (A = V^T from ldmatrix.trans)
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          uint32_t a[4];
+          const uint32_t ch = 2 * j + ((lane >> 3) & 1);
+          const uint32_t row = vr + 16 * pr;
+          ldsm_x4_t(a, st + kS * 128 + row * 128 + ((ch ^ (row & 7)) << 4));
+          mma16816<kBF16>(acc[j], a[0], a[1], a[2], a[3], pb0, pb1);
+        }
       }
       __syncwarp();   // every lane has read this stage before it is refilled
     }
