@@ -128,6 +128,21 @@ MG_API mg_status mg_plan_create_ex(int64_t L, int32_t heads, int32_t d, int32_t 
                             const int32_t* extra_idx, int64_t n_extra,
                             const mg_plan_opts* opts, mg_plan_t* plan_out);
 
+/* Batched plan with per-sample special-token positions ("their locations are highly dependent on
+ * the input sequence"; the metadata is generated per input): sample b has global tokens
+ * global_idx[global_ptr[b] .. global_ptr[b+1]) and extra pairs extra_idx[extra_ptr[b] ..
+ * extra_ptr[b+1]) (COO (row, col), int32 [*][2]); the pattern of sample b is the single-plan pattern
+ * with those lists (A2-A7). All samples are merged into one work list, so one forward launch
+ * covers the whole batch. The forward's Q/K/V/O batch must equal `batch`. Not supported with a
+ * batched plan: mg_plan_export and the staged entry points (UNSUPPORTED); mg_plan_info_get returns
+ * counts summed over the samples. opts as for mg_plan_create_ex (block must be 128; dense-row items
+ * are not split). Errors: as mg_plan_create, plus INVALID_ARG for batch <= 0, null or decreasing
+ * offset arrays, global_ptr[0] or extra_ptr[0] != 0. */
+MG_API mg_status mg_plan_create_batched(int64_t L, int32_t heads, int32_t d, int32_t window, int64_t batch,
+                                        const int64_t* global_ptr, const int32_t* global_idx,
+                                        const int64_t* extra_ptr, const int32_t* extra_idx,
+                                        const mg_plan_opts* opts, mg_plan_t* plan_out);
+
 /* Frees host and device memory of the plan. Must not race with in-flight forwards that use
  * it (synchronize their streams first). Null is accepted (no-op). */
 MG_API mg_status mg_plan_destroy(mg_plan_t plan);

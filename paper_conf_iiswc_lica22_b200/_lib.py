@@ -15,7 +15,7 @@ STATUS_NAMES = {0: "OK", 1: "INVALID_ARG", 2: "UNSUPPORTED", 3: "OUT_OF_MEMORY",
 
 # Every symbol include/mg.h declares (checked by tests/test_abi.py).
 EXPORTED = [
-    "mg_plan_create", "mg_plan_create_ex", "mg_plan_destroy", "mg_last_error", "mg_plan_info_get",
+    "mg_plan_create", "mg_plan_create_ex", "mg_plan_create_batched", "mg_plan_destroy", "mg_last_error", "mg_plan_info_get",
     "mg_plan_export", "mg_sparse_attention_fwd", "mg_sparse_attention_fwd_host", "mg_selftest_umma",
     "mg_abi_version", "mg_plan_set_profiling", "mg_plan_get_profile", "mg_plan_set_trace",
     "mg_sparse_attention_fwd_padded", "mg_staged_get_sizes", "mg_staged_sddmm", "mg_staged_softmax", "mg_staged_spmm", "mg_sparse_attention_fwd_staged",
@@ -71,6 +71,9 @@ def load() -> C.CDLL:
                                    C.POINTER(P)]
     lib.mg_plan_create_ex.argtypes = [C.c_int64, C.c_int32, C.c_int32, C.c_int32, i32p, C.c_int64, i32p,
                                       C.c_int64, C.POINTER(mg_plan_opts), C.POINTER(P)]
+    lib.mg_plan_create_batched.argtypes = [C.c_int64, C.c_int32, C.c_int32, C.c_int32, C.c_int64,
+                                           C.POINTER(C.c_int64), i32p, C.POINTER(C.c_int64), i32p,
+                                           C.POINTER(mg_plan_opts), C.POINTER(P)]
     lib.mg_plan_destroy.argtypes = [P]
     lib.mg_last_error.restype = C.c_char_p
     lib.mg_last_error.argtypes = []

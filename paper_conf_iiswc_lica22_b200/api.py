@@ -104,6 +104,36 @@ class Plan:
             pass
 
 
+class BatchedPlan(Plan):
+    """mg_plan_create_batched: one plan for a batch whose samples have their own global tokens and
+    extra pairs (lists of arrays, one per sample). Same options as Plan."""
+
+    def __init__(self, L: int, heads: int, d: int, window: int, global_idx_per_sample, extra_idx_per_sample=None,
+                 **opts):
+        lib = load()
+        B = len(global_idx_per_sample)
+        extras = extra_idx_per_sample if extra_idx_per_sample is not None else [None] * B
+        if len(extras) != B:
+            raise ValueError("one extra_idx array per sample")
+        gl = [_i32(np.asarray(g, dtype=np.int64)).reshape(-1) for g in global_idx_per_sample]
+        ex = [_i32(np.zeros((0, 2)) if e is None else e).reshape(-1, 2) for e in extras]
+        gptr = np.zeros(B + 1, np.int64)
+        eptr = np.zeros(B + 1, np.int64)
+        gptr[1:] = np.cumsum([g.size for g in gl])
+        eptr[1:] = np.cumsum([e.shape[0] for e in ex])
+        g_all = _i32(np.concatenate(gl) if B else np.zeros(0))
+        e_all = _i32(np.concatenate(ex) if B else np.zeros((0, 2))).reshape(-1, 2)
+        self._handle = C.c_void_p()
+        self._lib = lib
+        o = mg_plan_opts(opts.get("block", 0), int(opts.get("force_all_fine", False)), opts.get("strip_max_cols", 0),
+                         opts.get("num_sms", 0), opts.get("fine_kernel", 0), opts.get("concurrency", 0),
+                         opts.get("tau", 0.0), opts.get("dense_chunk", 0))
+        i64p = lambda a: a.ctypes.data_as(C.POINTER(C.c_int64))
+        check(lib.mg_plan_create_batched(L, heads, d, window, B, i64p(gptr), _ptr_i32(g_all), i64p(eptr),
+                                         _ptr_i32(e_all), C.byref(o), C.byref(self._handle)))
+        self.L, self.heads, self.d, self.window, self.batch = L, heads, d, window, B
+
+
 def tensor_desc(t) -> mg_tensor:
     """mg_tensor for a torch tensor viewed as [B, H, L, d] (any strides with a unit d-stride)."""
     import torch

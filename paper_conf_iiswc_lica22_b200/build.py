@@ -18,7 +18,8 @@ CSRC = os.path.join(PKG, "csrc")
 BUILD = os.path.join(ROOT, "build", "mg")
 LIB = os.path.join(PKG, "libmg.so")
 # diagnostics variants: libmg_<name>.so with the matching -D flags, loaded via MG_LIB_VARIANT=<name>
-VARIANTS = {"watchdog": ["-DMG_WATCHDOG"], "timeline": ["-DMG_TIMELINE"], "trace": ["-DMG_TRACE"],
+VARIANTS = {"base": [],   # (a plain build under another name: A/B against a stashed source tree)
+            "watchdog": ["-DMG_WATCHDOG"], "timeline": ["-DMG_TIMELINE"], "trace": ["-DMG_TRACE"],
             # A/B of the share of exponentials emulated on the FMA pipe (pairs of 16 per chunk)
             "e0": ["-DMG_EXP_EMU=0"], "e4": ["-DMG_EXP_EMU=4"], "e8": ["-DMG_EXP_EMU=8"],
             "maxpass": ["-DMG_SKIP_MAX=0"],

@@ -55,6 +55,7 @@ struct mg_plan_s {
   std::vector<void*> allocs;
   mg::Item* d_items = nullptr;
   mg::Item* d_items_split = nullptr;   // dense items split into column chunks (chosen per forward)
+  int32_t* d_fine_sample = nullptr;    // batched plans: sample of each fine row
   mg::TileRef* d_trefs = nullptr;
   uint64_t* d_masks = nullptr;
   int32_t* d_strip_cols = nullptr;
@@ -149,6 +150,7 @@ mg_status upload(mg_plan_s* p) {
   const mg::HostPlan& h = p->hp;
   if ((e = upload_vec(p, &p->d_items, h.items)) != cudaSuccess ||
       (e = upload_vec(p, &p->d_items_split, h.items_split)) != cudaSuccess ||
+      (e = upload_vec(p, &p->d_fine_sample, h.fine_sample)) != cudaSuccess ||
       (e = upload_vec(p, &p->d_trefs, h.trefs)) != cudaSuccess ||
       (e = upload_vec(p, &p->d_masks, h.dev_masks)) != cudaSuccess ||
       (e = upload_vec(p, &p->d_strip_cols, h.strip_cols)) != cudaSuccess ||
@@ -166,7 +168,8 @@ mg_status upload(mg_plan_s* p) {
 
 mg_status create_impl(int64_t L, int32_t heads, int32_t d, int32_t window, const int32_t* global_idx,
                       int64_t n_global, const int32_t* extra_idx, int64_t n_extra, const mg_plan_opts* opts,
-                      mg_plan_t* plan_out) {
+                      mg_plan_t* plan_out, int64_t batch = 0, const int64_t* global_ptr = nullptr,
+                      const int64_t* extra_ptr = nullptr) {
   if (!plan_out) return fail(MG_ERR_INVALID_ARG, "plan_out is null");
   *plan_out = nullptr;
   mg::PlanOptions po;
@@ -196,7 +199,11 @@ mg_status create_impl(int64_t L, int32_t heads, int32_t d, int32_t window, const
   bool unsupported = false;
   std::string err;
   try {
-    err = mg::build_plan(p->hp, L, heads, d, window, global_idx, n_global, extra_idx, n_extra, po, &unsupported);
+    if (batch > 0)
+      err = mg::build_batched_plan(p->hp, L, heads, d, window, batch, global_ptr, global_idx, extra_ptr, extra_idx, po,
+                                   &unsupported);
+    else
+      err = mg::build_plan(p->hp, L, heads, d, window, global_idx, n_global, extra_idx, n_extra, po, &unsupported);
   } catch (const std::bad_alloc&) {
     delete p;
     return fail(MG_ERR_OUT_OF_MEMORY, "host allocation failed while building the plan");
@@ -260,6 +267,8 @@ mg_status check_all(const mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, 
     return fail(MG_ERR_INVALID_ARG, "Q/K/V/O batch sizes differ");
   if (K->dtype != Q->dtype || V->dtype != Q->dtype || O->dtype != Q->dtype)
     return fail(MG_ERR_UNSUPPORTED, "Q/K/V/O dtypes differ");
+  if (p->hp.batch > 0 && Q->batch != p->hp.batch)
+    return fail(MG_ERR_INVALID_ARG, "batch size differs from the batched plan's number of samples");
   if (!p->hp.kernel_ready) return fail(MG_ERR_UNSUPPORTED, "the forward requires block == 128");
   if ((int64_t)Q->batch * p->hp.heads >=
       (int64_t(1) << 31) / std::max<int64_t>(1, (int64_t)std::max(p->hp.items.size(), p->hp.items_split.size())))
@@ -334,7 +343,9 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
   if (dev != p->device) return fail(MG_ERR_INVALID_ARG, "the plan was uploaded to another device");
   const mg::HostPlan& h = p->hp;
   const bool bf16 = Q->dtype == MG_BF16;
-  const int BH = (int)(Q->batch * h.heads);
+  // work units per item (and per fine row): every (b, h) of the batch, or for a batched plan (whose
+  // items each belong to one sample) every head
+  const int BH = (int)(h.batch > 0 ? h.heads : Q->batch * h.heads);
   const int nf = (int)h.fine_rows.size();
   const float scale_log2 = (float)(1.4426950408889634 / std::sqrt((double)h.d));
   cudaError_t e;
@@ -433,13 +444,15 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
     fp.part_ml = part_ml;
     fp.q = view(Q); fp.k = view(K); fp.v = view(V); fp.o = view(O);
     fp.H = h.heads; fp.BH = BH; fp.n_fine_rows = nf;
+    fp.fine_sample = h.batch > 0 ? p->d_fine_sample : nullptr;
     fp.scale_log2 = scale_log2;
     fp.concurrent = concurrent;
     fp.valid_len = valid_len;
     fp.part_c_acc = part_c_acc;
     fp.part_c_ml = part_c_ml;
     fp.part_flags = part_flags;
-    e = p->fine_kernel == 1 ? mg::launch_fine(fp, bf16, fstream) : mg::launch_fine_mma(fp, bf16, fstream);
+    // (the CUDA-core variant has no padding support: a padded forward always uses the MMA kernel)
+    e = p->fine_kernel == 1 && !valid_len ? mg::launch_fine(fp, bf16, fstream) : mg::launch_fine_mma(fp, bf16, fstream);
     if (e != cudaSuccess) return cuda_fail(e, "fine kernel launch");
   }
   if (p->profiling && has_f) {
@@ -485,6 +498,7 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
     cp.L = h.L;
     cp.H = h.heads;
     cp.BH = BH;
+    cp.batched = h.batch > 0;
     cp.n_items = (int)(use_split ? h.items_split.size() : h.items.size());
     cp.n_dense_items = use_split ? h.n_dense_items_split : h.n_dense_items;
     cp.n_global = (int)h.global_rows.size();
@@ -509,11 +523,11 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
     cp.trace_cap = p->trace_cap;
     // the paired-pipeline kernel resets its work counter itself (last CTA to exit); the v13 kernel
     // needs it zeroed before the launch
-    if (v13 && (e = cudaMemsetAsync(p->d_counter, 0, sizeof(int32_t), stream)) != cudaSuccess)
+    if (v13 && h.batch == 0 && (e = cudaMemsetAsync(p->d_counter, 0, sizeof(int32_t), stream)) != cudaSuccess)
       return cuda_fail(e, "cudaMemsetAsync");
     const int sms = p->num_sms_override > 0 ? std::min(p->num_sms_override, p->num_sms) : p->num_sms;
     // MG_COARSE=v13 selects the previous single-CTA-per-SM kernel (A/B measurements only)
-    if (v13) {
+    if (v13 && h.batch == 0) {
       if ((e = mg::launch_coarse(cp, tq, tk, tv, bf16, std::min(sms, cp.total_units), stream)) != cudaSuccess)
         return cuda_fail(e, "coarse kernel launch");
     } else {
@@ -609,6 +623,7 @@ mg_status staged_check(mg_plan_s* p, const mg_tensor* t, const char* name) {
   mg_status s = check_tensor(t, name, p, false);
   if (s != MG_OK) return s;
   if (!p->hp.kernel_ready) return fail(MG_ERR_UNSUPPORTED, "the staged forward requires block == 128");
+  if (p->hp.batch > 0) return fail(MG_ERR_UNSUPPORTED, "the staged forward does not take batched plans");
   if ((int64_t)t->batch * p->hp.heads >= 65536) return fail(MG_ERR_UNSUPPORTED, "batch * heads must be < 65536");
   return staged_upload(p);
 }
@@ -679,6 +694,15 @@ mg_status mg_plan_create_ex(int64_t L, int32_t heads, int32_t d, int32_t window,
   return create_impl(L, heads, d, window, global_idx, n_global, extra_idx, n_extra, opts, plan_out);
 }
 
+mg_status mg_plan_create_batched(int64_t L, int32_t heads, int32_t d, int32_t window, int64_t batch,
+                                 const int64_t* global_ptr, const int32_t* global_idx, const int64_t* extra_ptr,
+                                 const int32_t* extra_idx, const mg_plan_opts* opts, mg_plan_t* plan_out) {
+  g_err.clear();
+  if (batch <= 0) return fail(MG_ERR_INVALID_ARG, "batch must be > 0");
+  if (!global_ptr || !extra_ptr) return fail(MG_ERR_INVALID_ARG, "global_ptr / extra_ptr is null");
+  return create_impl(L, heads, d, window, global_idx, 0, extra_idx, 0, opts, plan_out, batch, global_ptr, extra_ptr);
+}
+
 mg_status mg_plan_destroy(mg_plan_t plan) {
   g_err.clear();
   delete plan;
@@ -717,6 +741,7 @@ mg_status mg_plan_export(mg_plan_t plan, int32_t* bsr_row_ptr, int32_t* bsr_col,
   g_err.clear();
   if (!plan) return fail(MG_ERR_INVALID_ARG, "plan is null");
   const mg::HostPlan& h = plan->hp;
+  if (h.batch > 0) return fail(MG_ERR_UNSUPPORTED, "mg_plan_export: batched plans have one partition per sample");
   auto cp = [](auto* dst, const auto& v) {
     if (dst && !v.empty()) std::memcpy(dst, v.data(), v.size() * sizeof(v[0]));
   };
@@ -809,6 +834,7 @@ mg_status mg_staged_softmax(mg_plan_t plan, int64_t batch, mg_dtype dtype, const
   if (batch <= 0) return fail(MG_ERR_INVALID_ARG, "batch must be > 0");
   if (dtype != MG_BF16 && dtype != MG_FP16) return fail(MG_ERR_INVALID_ARG, "dtype is not bf16/fp16");
   if (!plan->hp.kernel_ready) return fail(MG_ERR_UNSUPPORTED, "the staged forward requires block == 128");
+  if (plan->hp.batch > 0) return fail(MG_ERR_UNSUPPORTED, "the staged forward does not take batched plans");
   mg_status s;
   if ((s = staged_upload(plan)) != MG_OK) return s;
   if ((s = staged_buffers_ok(plan, S_tiles, S_csr, S_global)) != MG_OK ||

@@ -388,12 +388,16 @@ __device__ __forceinline__ void softmax_tile(const TileCtx& x, float& m, float& 
 
 }  // namespace
 
-template <bool kBF16, bool kSplit, bool kPad>
+template <bool kBF16, int kMode, bool kPad>
 __global__ void __launch_bounds__(kThreads, 2)
     coarse_pp_kernel(const __grid_constant__ CUtensorMap tmq, const __grid_constant__ CUtensorMap tmk,
                      const __grid_constant__ CUtensorMap tmv, const __grid_constant__ CUtensorMap tmq2,
                      const __grid_constant__ CUtensorMap tmk2, const __grid_constant__ CUtensorMap tmv2,
                      const __grid_constant__ CUtensorMap tmo, const CoarseParams p) {
+  // kMode: 0 = single plan, 1 = single plan with split dense-row items, 2 = batched plan (the mode
+  // paths are compiled only into the instantiations that need them: their code costs the common
+  // path registers and time, measured)
+  constexpr bool kSplit = kMode == 1, kBatched = kMode == 2;
   extern __shared__ uint8_t smem_raw[];
   const uint32_t sbase = (smem_u32(smem_raw) + 1023u) & ~1023u;
   const uint32_t sQ = sbase;
@@ -597,8 +601,9 @@ __global__ void __launch_bounds__(kThreads, 2)
         if (u < p.total_units) {
           const UnitInfo ui = decode_unit(p, u);
           sl.item = p.items[ui.item];
-          sl.bh = ui.bh;
-          if (sl.item.kind == 0) tma_prefetch_4d(&tmq, 0, sl.item.rowA, ui.bh % p.H, ui.bh / p.H);
+          // batched plans: the unit's second index is the head, the sample comes with the item
+          sl.bh = kBatched ? (int)sl.item.useB * p.H + ui.bh : ui.bh;
+          if (sl.item.kind == 0) tma_prefetch_4d(&tmq, 0, sl.item.rowA, sl.bh % p.H, sl.bh / p.H);
         }
         ctl->slot[slot] = sl;
         mbar_arrive(bar(ctl->item_full[slot]));
@@ -705,7 +710,8 @@ __global__ void __launch_bounds__(kThreads, 2)
       int r_out = -1, slot_f = -1;
       if (t < item.nrowsA) {
         r_out = item.kind == 0 ? item.rowA + t : __ldg(p.global_rows + item.rowA + t);
-        if (item.kind == 0) slot_f = __ldg(p.fine_slot + item.rowA + t);
+        if (item.kind == 0)
+          slot_f = __ldg(p.fine_slot + (kBatched ? (int64_t)item.useB * p.L : 0) + item.rowA + t);
       }
       float m = -INFINITY, l = 0.f;
       for (int j = 0; j < item.ntiles; ++j, ++n) {
@@ -729,7 +735,7 @@ __global__ void __launch_bounds__(kThreads, 2)
       // ---------------------------------------------------------------- epilogue (a-8)
       float mf = -INFINITY, lf = 0.f;
       const float4* accf = nullptr;
-      const size_t fidx = (size_t)ubh * p.n_fine_rows + slot_f;
+      const size_t fidx = (size_t)(kBatched ? ubh % p.H : ubh) * p.n_fine_rows + slot_f;
       if (slot_f >= 0 && !p.concurrent) {
         const float2 ml = p.part_ml[fidx];
         mf = ml.x;
@@ -925,11 +931,14 @@ cudaError_t launch_coarse_pp(const CoarseParams& p, const CUtensorMap& tmq, cons
   // that need them (their code costs the common path registers)
   using K = void (*)(const CUtensorMap, const CUtensorMap, const CUtensorMap, const CUtensorMap, const CUtensorMap,
                      const CUtensorMap, const CUtensorMap, const CoarseParams);
-  static const K table[8] = {coarse_pp_kernel<false, false, false>, coarse_pp_kernel<false, false, true>,
-                             coarse_pp_kernel<false, true, false>,  coarse_pp_kernel<false, true, true>,
-                             coarse_pp_kernel<true, false, false>,  coarse_pp_kernel<true, false, true>,
-                             coarse_pp_kernel<true, true, false>,   coarse_pp_kernel<true, true, true>};
-  const K kern = table[(bf16 ? 4 : 0) + (split_dense ? 2 : 0) + (p.valid_len ? 1 : 0)];
+  static const K table[12] = {coarse_pp_kernel<false, 0, false>, coarse_pp_kernel<false, 0, true>,
+                              coarse_pp_kernel<false, 1, false>, coarse_pp_kernel<false, 1, true>,
+                              coarse_pp_kernel<false, 2, false>, coarse_pp_kernel<false, 2, true>,
+                              coarse_pp_kernel<true, 0, false>,  coarse_pp_kernel<true, 0, true>,
+                              coarse_pp_kernel<true, 1, false>,  coarse_pp_kernel<true, 1, true>,
+                              coarse_pp_kernel<true, 2, false>,  coarse_pp_kernel<true, 2, true>};
+  const int mode = p.batched ? 2 : (split_dense ? 1 : 0);
+  const K kern = table[(bf16 ? 6 : 0) + 2 * mode + (p.valid_len ? 1 : 0)];
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBytes);
   if (e != cudaSuccess) return e;
   kern<<<grid, kThreads, kSmemBytes, stream>>>(tmq, tmk, tmv, tmq2, tmk2, tmv2, tmo, p);

@@ -128,7 +128,8 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(con
   const uint16_t *iK = nullptr, *iV = nullptr;
   auto open_issue_row = [&]() {
     if (gi < nrows) {
-      const int bh = (int)(gi / p.n_fine_rows), fi = (int)(gi % p.n_fine_rows);
+      const int u0 = (int)(gi / p.n_fine_rows), fi = (int)(gi % p.n_fine_rows);
+      const int bh = p.fine_sample ? __ldg(p.fine_sample + fi) * p.H + u0 : u0;
       ibeg = __ldg(p.row_ptr + fi);
       iend = __ldg(p.row_ptr + fi + 1);
       const int bb = bh / p.H, hh = bh % p.H;
@@ -170,8 +171,9 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(con
   const uint32_t vr = (lane & 7) + 8 * (lane >> 4);
 
   for (int64_t gw = w0; gw < nrows; gw += W) {
-    const int bh = (int)(gw / p.n_fine_rows);
+    const int u0 = (int)(gw / p.n_fine_rows);
     const int fi = (int)(gw % p.n_fine_rows);
+    const int bh = p.fine_sample ? __ldg(p.fine_sample + fi) * p.H + u0 : u0;   // (batched plans)
     const int enc = __ldg(p.fine_rows + fi);
     const int r = enc & 0x7fffffff;
     const bool final_out = enc < 0;
@@ -289,7 +291,7 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(con
     float inv = l > 0.f ? 1.f / l : 0.f;
     bool write_o = final_out;
     if (!final_out) {
-      const size_t idx = (size_t)bh * p.n_fine_rows + fi;
+      const size_t idx = (size_t)u0 * p.n_fine_rows + fi;
       __stcg(p.part_acc + idx * 64 + d0, v0);
       __stcg(p.part_acc + idx * 64 + d1, v1);
       if (lane == 0) __stcg(p.part_ml + idx, make_float2(m, l));

@@ -51,8 +51,9 @@ __global__ void __launch_bounds__(256, 2) fine_rows_kernel(const FineParams p) {
   const int lane = threadIdx.x & 31;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   if (gw >= (int64_t)p.BH * p.n_fine_rows) return;
-  const int bh = (int)(gw / p.n_fine_rows);
+  const int u0 = (int)(gw / p.n_fine_rows);
   const int fi = (int)(gw % p.n_fine_rows);
+  const int bh = p.fine_sample ? __ldg(p.fine_sample + fi) * p.H + u0 : u0;   // (batched plans)
   const int enc = __ldg(p.fine_rows + fi);
   const int r = enc & 0x7fffffff;
   const bool final_out = enc < 0;
@@ -146,7 +147,7 @@ __global__ void __launch_bounds__(256, 2) fine_rows_kernel(const FineParams p) {
     o4.w = pack2<kBF16>(acc[6] * inv, acc[7] * inv);
     *reinterpret_cast<uint4*>(p.o.data + bb * p.o.sb + hh * p.o.sh + (int64_t)r * p.o.sl + q8 * 8) = o4;
   } else {
-    const size_t idx = (size_t)bh * p.n_fine_rows + fi;
+    const size_t idx = (size_t)u0 * p.n_fine_rows + fi;
     float4* dst = reinterpret_cast<float4*>(p.part_acc + idx * 64 + q8 * 8);
     dst[0] = make_float4(acc[0], acc[1], acc[2], acc[3]);
     dst[1] = make_float4(acc[4], acc[5], acc[6], acc[7]);

@@ -30,8 +30,9 @@ struct CoarseParams {
   TensorView q, k, v, o;
   int64_t L;
   int32_t H, BH;
-  int32_t n_items, n_dense_items;
+  int32_t n_items, n_dense_items;   // (BH = units per item: B*H, or H for a batched plan)
   int32_t n_global, n_fine_rows;
+  int32_t batched;            // batched plan: Item::useB = sample, unit -> (item, head), fine_slot [B][L]
   int32_t total_units;
   float scale_log2;           // (1/sqrt(d)) * log2(e)
   unsigned long long* trace;  // diagnostics: event trace of CTA 0 (null = off)
@@ -68,7 +69,8 @@ struct FineParams {
   float* part_acc;
   float2* part_ml;
   TensorView q, k, v, o;
-  int32_t H, BH, n_fine_rows;
+  int32_t H, BH, n_fine_rows;   // (BH = row units per fine row: B*H, or H for a batched plan)
+  const int32_t* fine_sample;   // batched plan: sample of each fine row (else null)
   float scale_log2;
   int32_t concurrent;         // see CoarseParams::concurrent
   const int32_t* valid_len;   // see CoarseParams::valid_len

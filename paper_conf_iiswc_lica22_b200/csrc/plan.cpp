@@ -312,4 +312,88 @@ std::string build_plan(HostPlan& p, int64_t L, int32_t heads, int32_t d, int32_t
   return "";
 }
 
+std::string build_batched_plan(HostPlan& out, int64_t L, int32_t heads, int32_t d, int32_t window, int64_t batch,
+                               const int64_t* global_ptr, const int32_t* global_idx, const int64_t* extra_ptr,
+                               const int32_t* extra_idx, const PlanOptions& opts, bool* unsupported) {
+  *unsupported = false;
+  if (batch <= 0) return "batch must be > 0";
+  if (!global_ptr || !extra_ptr) return "global_ptr / extra_ptr is null";
+  if (global_ptr[0] != 0 || extra_ptr[0] != 0) return "global_ptr[0] and extra_ptr[0] must be 0";
+  for (int64_t b = 0; b < batch; ++b)
+    if (global_ptr[b + 1] < global_ptr[b] || extra_ptr[b + 1] < extra_ptr[b]) return "offsets must be non-decreasing";
+  if (opts.block != 128) { *unsupported = true; return "batched plans require block == 128"; }
+  PlanOptions po = opts;
+  po.dense_split = 1;   // the split dense-row list is not built for batched plans
+  std::vector<HostPlan> ps(batch);
+  for (int64_t b = 0; b < batch; ++b) {
+    const int64_t ng = global_ptr[b + 1] - global_ptr[b], ne = extra_ptr[b + 1] - extra_ptr[b];
+    std::string e = build_plan(ps[b], L, heads, d, window, global_idx ? global_idx + global_ptr[b] : nullptr, ng,
+                               extra_idx ? extra_idx + 2 * extra_ptr[b] : nullptr, ne, po, unsupported);
+    if (!e.empty()) return "sample " + std::to_string(b) + ": " + e;
+  }
+  out = HostPlan();
+  out.L = L; out.heads = heads; out.d = d; out.window = window; out.block = 128; out.opts = po;
+  out.kernel_ready = true;
+  out.batch = batch;
+  out.fine_slot.assign((size_t)batch * L, -1);
+  out.fine_row_ptr.assign(1, 0);
+  // dense items of every sample first (longest first, as in a single plan), then the band items
+  std::vector<int32_t> tref_off(batch), mask_off(batch), strip_off(batch), grow_off(batch), fine_off(batch);
+  for (int64_t b = 0; b < batch; ++b) {
+    const HostPlan& h = ps[b];
+    tref_off[b] = (int32_t)out.trefs.size();
+    mask_off[b] = (int32_t)(out.dev_masks.size() / 256);
+    strip_off[b] = (int32_t)out.strip_cols.size();
+    grow_off[b] = (int32_t)out.global_rows.size();
+    fine_off[b] = (int32_t)out.fine_rows.size();
+    for (TileRef tr : h.trefs) {
+      if (tr.maskA >= 0) tr.maskA += mask_off[b];
+      if (tr.kind == 1) tr.arg += strip_off[b];
+      out.trefs.push_back(tr);
+    }
+    out.dev_masks.insert(out.dev_masks.end(), h.dev_masks.begin(), h.dev_masks.end());
+    out.strip_cols.insert(out.strip_cols.end(), h.strip_cols.begin(), h.strip_cols.end());
+    out.global_rows.insert(out.global_rows.end(), h.global_rows.begin(), h.global_rows.end());
+    for (size_t i = 0; i < h.fine_rows.size(); ++i) {
+      out.fine_rows.push_back(h.fine_rows[i]);
+      out.fine_sample.push_back((int32_t)b);
+      const int32_t* cb = h.fine_col.data() + h.fine_row_ptr[i];
+      const int32_t* ce = h.fine_col.data() + h.fine_row_ptr[i + 1];
+      out.fine_col.insert(out.fine_col.end(), cb, ce);
+      out.fine_row_ptr.push_back((int32_t)out.fine_col.size());
+    }
+    for (int64_t r = 0; r < L; ++r)
+      if (h.fine_slot[r] >= 0) out.fine_slot[(size_t)b * L + r] = h.fine_slot[r] + fine_off[b];
+    out.nnz_coarse += h.nnz_coarse;
+    out.n_full_tiles += h.n_full_tiles;
+    out.nnz_fine_strip += h.nnz_fine_strip;
+    out.n_strip_tiles += h.n_strip_tiles;
+    out.computed_scores += h.computed_scores;
+    out.softmax_tiles += h.softmax_tiles;
+    out.nnz_total_sum += h.nnz_coarse + (int64_t)h.csr_col.size() + (int64_t)h.global_rows.size() * L;
+    out.csr_col.resize(out.csr_col.size() + h.csr_col.size());   // (counts only; not exported)
+    out.bsr_col.resize(out.bsr_col.size() + h.bsr_col.size());
+  }
+  for (int pass = 0; pass < 2; ++pass) {
+    for (int64_t b = 0; b < batch; ++b) {
+      const HostPlan& h = ps[b];
+      for (int32_t i = 0; i < (int32_t)h.items.size(); ++i) {
+        const bool dense = i < h.n_dense_items;
+        if (dense != (pass == 0)) continue;
+        Item it = h.items[i];
+        it.tref_begin += tref_off[b];
+        if (it.kind == 1) it.rowA += grow_off[b];
+        it.useB = (uint64_t)b;
+        out.items.push_back(it);
+      }
+    }
+    if (pass == 0) out.n_dense_items = (int32_t)out.items.size();
+  }
+  out.items_split = out.items;
+  out.n_dense_items_split = out.n_dense_items;
+  out.dense_nsplit = 1;
+  if (out.csr_col.size() >= (size_t(1) << 31)) { *unsupported = true; return "CSR nnz >= 2^31"; }
+  return "";
+}
+
 }  // namespace mg

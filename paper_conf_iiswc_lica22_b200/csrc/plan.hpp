@@ -58,6 +58,11 @@ struct HostPlan {
   std::vector<Item> items;           // dense items first, then band items in row-block order
   int32_t n_dense_items = 0;
   int32_t n_dense_groups = 0, dense_nsplit = 1;
+  // batched plan (per-sample global / extra positions): batch > 0 samples merged into one
+  // work list; Item::useB = sample; fine_slot is [batch][L]; fine_sample[i] = sample of fine row i
+  int64_t batch = 0;
+  std::vector<int32_t> fine_sample;
+  int64_t nnz_total_sum = 0;
   // alternative work list with the dense items split into chunks (same band items after them)
   std::vector<Item> items_split;
   int32_t n_dense_items_split = 0;
@@ -72,6 +77,11 @@ struct HostPlan {
   int64_t nb() const { return (L + block - 1) / block; }
   int wpr() const { return (block + 63) / 64; }
 };
+
+// Per-sample plans merged into one batched work list (see HostPlan::batch). Returns "" or an error.
+std::string build_batched_plan(HostPlan& out, int64_t L, int32_t heads, int32_t d, int32_t window, int64_t batch,
+                               const int64_t* global_ptr, const int32_t* global_idx, const int64_t* extra_ptr,
+                               const int32_t* extra_idx, const PlanOptions& opts, bool* unsupported);
 
 // Returns "" on success, else an error message; *unsupported is set for UNSUPPORTED errors.
 std::string build_plan(HostPlan& p, int64_t L, int32_t heads, int32_t d, int32_t window,

@@ -189,3 +189,22 @@ def test_tau_plan_export_matches_oracle_configs(cfg, tau):
     if cfg == "F9-RBR":
         # the 64 x 64 random blocks (25% of a 128-tile) become coarse at tau = 0.2
         assert inf["nnz_coarse"] > 64 * 64 * 64
+
+
+# ---------------------------------------------------------------- batched plans (per-sample positions)
+def test_batched_plan_counts_sum_samples_and_validation():
+    L, H, w = 1024, 2, 128
+    Gs = [np.array([0, 5], np.int32), np.array([300], np.int32), np.zeros(0, np.int32)]
+    Es = [None, np.array([[1, 900], [900, 1]], np.int32), random_small_config(np.random.default_rng(2), 64)[3]]
+    bp = mg.BatchedPlan(L, H, 64, w, Gs, Es)
+    infos = [mg.Plan(L, H, 64, w, g, e).info() for g, e in zip(Gs, Es)]
+    bi = bp.info()
+    for key in ("n_tiles", "nnz_coarse", "nnz_fine", "n_global", "nnz_total", "nnz_fine_strip", "n_items"):
+        assert bi[key] == sum(i[key] for i in infos), key
+    with pytest.raises(mg.MGError) as ei:
+        bp.export()
+    assert ei.value.status == _lib.MG_ERR_UNSUPPORTED
+    with pytest.raises(mg.MGError):                 # out-of-range position in one sample
+        mg.BatchedPlan(L, H, 64, w, [[0], [L]])
+    with pytest.raises(mg.MGError):
+        mg.BatchedPlan(L, H, 64, w, [])

@@ -302,3 +302,29 @@ def test_padded_batch(case):
             # adversarial inputs: bf16 output rounding grows with |O| (as for the peaky case)
             assert mx <= TOL_MAX * max(1.0, np.abs(ref).max() / 4) and mean <= TOL_MEAN, (case, b, h, mx, mean)
             assert (got[b, h, lens[b]:] == 0).all()
+
+
+# ------------------------------------------------------------------ batched plans (per-sample positions)
+@pytest.mark.parametrize("kw", [{}, dict(strip_max_cols=-1), dict(strip_max_cols=-1, concurrency=2),
+                                dict(fine_kernel=1, strip_max_cols=-1)])
+def test_batched_plan_per_sample_positions(kw):
+    """One launch over a batch whose samples have different global tokens and residuals (P:66,
+    P:94), against the oracle per sample; padded too."""
+    L, H, w = 1024, 2, 128
+    rng = np.random.default_rng(51)
+    Gs = [np.array([0, 5, 700], np.int32), np.array([300], np.int32), np.zeros(0, np.int32),
+          np.arange(0, 40, dtype=np.int32)]
+    Es = [random_residual(L, w, int(rng.integers(0, 6)), seed=60 + b) for b in range(4)]
+    plan = mg.BatchedPlan(L, H, 64, w, Gs, Es, **kw)
+    q, k, v = make_qkv(4, H, L, 64, seed=52)
+    got = run_gpu(plan, q, k, v)
+    lens = np.array([L, 333, 1000, 129], np.int32)
+    Q, K, V = (to_device(x) for x in (q, k, v))
+    gotp = from_device(mg.sparse_attention_fwd_padded(plan, Q, K, V, torch.from_numpy(lens).cuda()))
+    for b in range(4):
+        for h in range(H):
+            Qh, Kh, Vh = head_inputs_f64(q, k, v, b, h)
+            check(got[b, h], dense_masked_attention(Qh, Kh, Vh, w, Gs[b], Es[b]))
+            check(gotp[b, h], dense_masked_attention(Qh, Kh, Vh, w, Gs[b], Es[b], valid_len=int(lens[b])))
+    with pytest.raises(mg.MGError):                 # batch must match the plan's samples
+        run_gpu(plan, q[:2], k[:2], v[:2])
