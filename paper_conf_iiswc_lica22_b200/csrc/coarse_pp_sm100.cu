@@ -394,10 +394,11 @@ __global__ void __launch_bounds__(kThreads, 2)
                      const __grid_constant__ CUtensorMap tmv, const __grid_constant__ CUtensorMap tmq2,
                      const __grid_constant__ CUtensorMap tmk2, const __grid_constant__ CUtensorMap tmv2,
                      const __grid_constant__ CUtensorMap tmo, const CoarseParams p) {
-  // kMode: 0 = single plan, 1 = single plan with split dense-row items, 2 = batched plan (the mode
-  // paths are compiled only into the instantiations that need them: their code costs the common
-  // path registers and time, measured)
-  constexpr bool kSplit = kMode == 1, kBatched = kMode == 2;
+  // kMode: 0 = single plan, 1 = single plan with split dense-row items, 2 = batched plan, 3 = single
+  // plan without CUDA-core CSR rows (no partial to merge). The mode paths are compiled only into
+  // the instantiations that need them: their code costs the common path registers and time
+  // (measured: 5% on C2 for the batched branches).
+  constexpr bool kSplit = kMode == 1, kBatched = kMode == 2, kNoFine = kMode == 3;
   extern __shared__ uint8_t smem_raw[];
   const uint32_t sbase = (smem_u32(smem_raw) + 1023u) & ~1023u;
   const uint32_t sQ = sbase;
@@ -710,7 +711,7 @@ __global__ void __launch_bounds__(kThreads, 2)
       int r_out = -1, slot_f = -1;
       if (t < item.nrowsA) {
         r_out = item.kind == 0 ? item.rowA + t : __ldg(p.global_rows + item.rowA + t);
-        if (item.kind == 0)
+        if (!kNoFine && item.kind == 0)
           slot_f = __ldg(p.fine_slot + (kBatched ? (int64_t)item.useB * p.L : 0) + item.rowA + t);
       }
       float m = -INFINITY, l = 0.f;
@@ -931,14 +932,16 @@ cudaError_t launch_coarse_pp(const CoarseParams& p, const CUtensorMap& tmq, cons
   // that need them (their code costs the common path registers)
   using K = void (*)(const CUtensorMap, const CUtensorMap, const CUtensorMap, const CUtensorMap, const CUtensorMap,
                      const CUtensorMap, const CUtensorMap, const CoarseParams);
-  static const K table[12] = {coarse_pp_kernel<false, 0, false>, coarse_pp_kernel<false, 0, true>,
+  static const K table[16] = {coarse_pp_kernel<false, 0, false>, coarse_pp_kernel<false, 0, true>,
                               coarse_pp_kernel<false, 1, false>, coarse_pp_kernel<false, 1, true>,
                               coarse_pp_kernel<false, 2, false>, coarse_pp_kernel<false, 2, true>,
+                              coarse_pp_kernel<false, 3, false>, coarse_pp_kernel<false, 3, true>,
                               coarse_pp_kernel<true, 0, false>,  coarse_pp_kernel<true, 0, true>,
                               coarse_pp_kernel<true, 1, false>,  coarse_pp_kernel<true, 1, true>,
-                              coarse_pp_kernel<true, 2, false>,  coarse_pp_kernel<true, 2, true>};
-  const int mode = p.batched ? 2 : (split_dense ? 1 : 0);
-  const K kern = table[(bf16 ? 6 : 0) + 2 * mode + (p.valid_len ? 1 : 0)];
+                              coarse_pp_kernel<true, 2, false>,  coarse_pp_kernel<true, 2, true>,
+                              coarse_pp_kernel<true, 3, false>,  coarse_pp_kernel<true, 3, true>};
+  const int mode = p.batched ? 2 : (split_dense ? 1 : (p.n_fine_rows == 0 ? 3 : 0));
+  const K kern = table[(bf16 ? 8 : 0) + 2 * mode + (p.valid_len ? 1 : 0)];
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBytes);
   if (e != cudaSuccess) return e;
   kern<<<grid, kThreads, kSmemBytes, stream>>>(tmq, tmk, tmv, tmq2, tmk2, tmv2, tmo, p);
