@@ -207,10 +207,12 @@ MG_API mg_status mg_sparse_attention_fwd_padded(mg_plan_t plan, const mg_tensor*
                                          const mg_tensor* V, mg_tensor* O, const int32_t* valid_len,
                                          void* stream);
 
-/* Same computation with HOST tensors: copies Q/K/V host->device into plan-owned staging
- * buffers on `stream`, runs the forward, copies O device->host, all stream-ordered and
- * asynchronous (host buffers should be pinned for the copies to overlap; the caller
- * synchronises `stream` before reading O). Same errors as mg_sparse_attention_fwd. */
+/* Same computation with HOST tensors (dense [B,H,L,d] or [B,L,H,d]): copies Q/K/V host->device
+ * into plan-owned staging buffers, runs the forward, copies O device->host. The batch is processed
+ * in up to 8 chunks on plan-owned copy streams forked from and joined back to `stream`, so the
+ * H2D copies of chunk c+1 and the D2H copy of chunk c-1 overlap the forward of chunk c (batched
+ * plans: one chunk). Asynchronous with respect to the host (host buffers should be pinned; the
+ * caller synchronises `stream` before reading O). Same errors as mg_sparse_attention_fwd. */
 MG_API mg_status mg_sparse_attention_fwd_host(mg_plan_t plan, const mg_tensor* Q, const mg_tensor* K,
                                        const mg_tensor* V, mg_tensor* O, void* stream);
 

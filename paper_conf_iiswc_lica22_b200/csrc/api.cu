@@ -51,6 +51,18 @@ struct mg_plan_s {
   int fine_kernel = 0;   // 0: mma.sync kernel (fine_mma.cu), 1: CUDA-core kernel (fine_rows.cu)
   int concurrency = 0;   // 0 default, 1 serial, 2 concurrent streams (see mg_plan_opts)
   cudaStream_t side = nullptr;              // second stream of the concurrent mode
+  // host-buffer forward: copy streams and per-chunk events (H2D of chunk c+1 and D2H of chunk c-1
+  // overlap the forward of chunk c)
+  cudaStream_t h2d = nullptr, d2h = nullptr;
+  std::vector<cudaEvent_t> host_ev;
+  cudaEvent_t host_event(size_t i) {
+    while (host_ev.size() <= i) {
+      cudaEvent_t e = nullptr;
+      if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) return nullptr;
+      host_ev.push_back(e);
+    }
+    return host_ev[i];
+  }
   cudaEvent_t fork_ev = nullptr, join_ev = nullptr;
   std::vector<void*> allocs;
   mg::Item* d_items = nullptr;
@@ -117,6 +129,9 @@ struct mg_plan_s {
     if (fork_ev) cudaEventDestroy(fork_ev);
     if (join_ev) cudaEventDestroy(join_ev);
     if (side) cudaStreamDestroy(side);
+    for (cudaEvent_t e : host_ev) cudaEventDestroy(e);
+    if (h2d) cudaStreamDestroy(h2d);
+    if (d2h) cudaStreamDestroy(d2h);
     for (void* p : allocs) cudaFree(p);
     if (d_part) cudaFree(d_part);
     if (d_stage) cudaFree(d_stage);
@@ -793,18 +808,50 @@ mg_status mg_sparse_attention_fwd_host(mg_plan_t plan, const mg_tensor* Q, const
                                             : cuda_fail(e, "cudaMallocAsync");
     plan->stage_cap = 4 * bytes;
   }
-  mg_tensor dq = *Q, dk = *K, dv = *V, dO = *O;
-  dq.data = plan->d_stage;
-  dk.data = plan->d_stage + bytes;
-  dv.data = plan->d_stage + 2 * bytes;
-  dO.data = plan->d_stage + 3 * bytes;
-  if ((e = cudaMemcpyAsync(dq.data, Q->data, bytes, cudaMemcpyHostToDevice, stream)) != cudaSuccess ||
-      (e = cudaMemcpyAsync(dk.data, K->data, bytes, cudaMemcpyHostToDevice, stream)) != cudaSuccess ||
-      (e = cudaMemcpyAsync(dv.data, V->data, bytes, cudaMemcpyHostToDevice, stream)) != cudaSuccess)
-    return cuda_fail(e, "H2D copy");
-  if ((s = fwd_impl(plan, &dq, &dk, &dv, &dO, stream)) != MG_OK) return s;
-  if ((e = cudaMemcpyAsync(O->data, dO.data, bytes, cudaMemcpyDeviceToHost, stream)) != cudaSuccess)
-    return cuda_fail(e, "D2H copy");
+  // Pipelined over batch chunks: the H2D copies of chunk c+1 (h2d stream) and the D2H copy of chunk
+  // c-1 (d2h stream) overlap the forward of chunk c (`stream`); host tensors are dense, so a batch
+  // chunk is one contiguous range of each. Batched plans (one pattern per sample) run as one chunk.
+  const int64_t B = Q->batch;
+  const int64_t nchunk = plan->hp.batch > 0 ? 1 : std::min<int64_t>(B, 8);
+  const size_t per_b = bytes / (size_t)B;
+  uint8_t* dst[4] = {plan->d_stage, plan->d_stage + bytes, plan->d_stage + 2 * bytes, plan->d_stage + 3 * bytes};
+  const uint8_t* src[3] = {static_cast<const uint8_t*>(Q->data), static_cast<const uint8_t*>(K->data),
+                           static_cast<const uint8_t*>(V->data)};
+  if (!plan->h2d) {
+    if ((e = cudaStreamCreateWithFlags(&plan->h2d, cudaStreamNonBlocking)) != cudaSuccess ||
+        (e = cudaStreamCreateWithFlags(&plan->d2h, cudaStreamNonBlocking)) != cudaSuccess)
+      return cuda_fail(e, "stream creation");
+  }
+  cudaEvent_t ev_start = plan->host_event(0), ev_end = plan->host_event(1);
+  if (!ev_start || !ev_end || !plan->host_event(2 + 2 * nchunk)) return fail(MG_ERR_CUDA, "event creation failed");
+  if ((e = cudaEventRecord(ev_start, stream)) != cudaSuccess ||
+      (e = cudaStreamWaitEvent(plan->h2d, ev_start, 0)) != cudaSuccess ||
+      (e = cudaStreamWaitEvent(plan->d2h, ev_start, 0)) != cudaSuccess)
+    return cuda_fail(e, "stream fork");
+  for (int64_t c = 0; c < nchunk; ++c) {
+    const int64_t b0 = B * c / nchunk, b1 = B * (c + 1) / nchunk;
+    const size_t off = (size_t)b0 * per_b, len = (size_t)(b1 - b0) * per_b;
+    cudaEvent_t ev_in = plan->host_event(2 + 2 * c), ev_done = plan->host_event(3 + 2 * c);
+    for (int i = 0; i < 3; ++i)
+      if ((e = cudaMemcpyAsync(dst[i] + off, src[i] + off, len, cudaMemcpyHostToDevice, plan->h2d)) != cudaSuccess)
+        return cuda_fail(e, "H2D copy");
+    if ((e = cudaEventRecord(ev_in, plan->h2d)) != cudaSuccess || (e = cudaStreamWaitEvent(stream, ev_in, 0)) != cudaSuccess)
+      return cuda_fail(e, "event");
+    mg_tensor dq = *Q, dk = *K, dv = *V, dO = *O;
+    dq.data = dst[0] + off;
+    dk.data = dst[1] + off;
+    dv.data = dst[2] + off;
+    dO.data = dst[3] + off;
+    dq.batch = dk.batch = dv.batch = dO.batch = b1 - b0;
+    if ((s = fwd_impl(plan, &dq, &dk, &dv, &dO, stream)) != MG_OK) return s;
+    if ((e = cudaEventRecord(ev_done, stream)) != cudaSuccess || (e = cudaStreamWaitEvent(plan->d2h, ev_done, 0)) != cudaSuccess)
+      return cuda_fail(e, "event");
+    if ((e = cudaMemcpyAsync(static_cast<uint8_t*>(O->data) + off, dst[3] + off, len, cudaMemcpyDeviceToHost,
+                             plan->d2h)) != cudaSuccess)
+      return cuda_fail(e, "D2H copy");
+  }
+  if ((e = cudaEventRecord(ev_end, plan->d2h)) != cudaSuccess || (e = cudaStreamWaitEvent(stream, ev_end, 0)) != cudaSuccess)
+    return cuda_fail(e, "stream join");
   return MG_OK;
 }
 
