@@ -242,9 +242,11 @@ def main():
     dev = torch.device("cuda", local)
 
     cfg = get_config(args.workload)
+    t_plan = time.perf_counter()
     plan = mg.Plan(cfg.L, cfg.H, cfg.d, cfg.window, cfg.global_idx, cfg.extra_idx,
                    strip_max_cols=args.strip_max_cols, fine_kernel=args.fine_kernel,
                    concurrency=args.concurrency, tau=args.tau, dense_chunk=args.dense_chunk)
+    plan_build_ms = 1e3 * (time.perf_counter() - t_plan)   # host, once per pattern (before inference)
     info = plan.info()
     BH = cfg.B * cfg.H
     useful = 4.0 * info["nnz_total"] * cfg.d * BH
@@ -293,6 +295,15 @@ def main():
     total_ms = float(t_ms.item())
     ms_per_step = total_ms / args.steps
     value = world * useful / (ms_per_step * 1e-3) / 1e12
+
+    # ---------------- warm-L2 figure (no flush between steps; reported beside the flushed value)
+    plan.set_profiling(True)
+    for _ in range(min(args.steps, 100)):
+        fwd()
+    torch.cuda.synchronize()
+    pw = plan.get_profile()
+    plan.set_profiling(False)
+    warm_ms = pw["total_ms"] / max(1, pw["calls"])
 
     # ---------------- e2e: host buffers through the C ABI (H2D + fwd + D2H every step)
     hq, hk, hv = (h.pin_memory() for h in host)
@@ -371,6 +382,8 @@ def main():
         "vs_baseline": None, "dtype": "bf16", "data": "synthetic", "config": workload_config(cfg, world),
         "fwd_ms": {"mean": ms_per_step, "timing": "library CUDA events on the launch stream, first to last kernel"},
         "useful_gflop_per_gpu": useful / 1e9,
+        "fwd_ms_warm_l2": warm_ms,
+        "plan_build_ms": plan_build_ms,
         "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": 3 * nbytes, "d2h_bytes_per_step": nbytes,
                 "ms_per_step": float(e2e_ms.item()),
                 "path": "mg_sparse_attention_fwd_host (pinned host Q/K/V/O, copies inside the timed region)"},
