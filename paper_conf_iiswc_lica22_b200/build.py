@@ -28,6 +28,8 @@ VARIANTS = {"base": [],   # (a plain build under another name: A/B against a sta
             # fine tensor-core kernel: cp.async ring stages per warp (default 2), min blocks per SM
             "fs3": ["-DMG_FINE_STAGES=3"], "fb4": ["-DMG_FINE_MINB=4"], "fb6": ["-DMG_FINE_MINB=6"],
             "fb8": ["-DMG_FINE_MINB=8"], "fp2": ["-DMG_FINE_PAIRS=2"], "fp2b3": ["-DMG_FINE_PAIRS=2", "-DMG_FINE_MINB=3"],
+            "fw8": ["-DMG_FINE_WARPS=8", "-DMG_FINE_MINB=3"], "fw2": ["-DMG_FINE_WARPS=2", "-DMG_FINE_MINB=10"],
+            "fw1": ["-DMG_FINE_WARPS=1", "-DMG_FINE_MINB=20"],
             # skeleton cost: no exponentials / no MMAs / no loads (results are garbage)
             "dbg1": ["-DMG_DBG=1"], "dbg3": ["-DMG_DBG=3"], "dbg7": ["-DMG_DBG=7"]}
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")

@@ -82,7 +82,10 @@ __device__ __forceinline__ void ldsm_x4_t(uint32_t (&r)[4], uint32_t addr) {
 #ifndef MG_FINE_PAIRS
 #define MG_FINE_PAIRS 1
 #endif
-constexpr int kWarps = 4;                   // warps per block, one (row, b*h) each
+#ifndef MG_FINE_WARPS
+#define MG_FINE_WARPS 4
+#endif
+constexpr int kWarps = MG_FINE_WARPS;       // warps per block, each a persistent row sequence
 constexpr int kP = MG_FINE_PAIRS;           // 16-nnz pairs of 8-nnz chunks per step (1 or 2)
 constexpr int kS = 16 * kP;                 // nnz per step
 constexpr int kStages = MG_FINE_STAGES;     // smem ring stages per warp (kStages - 1 steps in flight)
