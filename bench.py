@@ -367,6 +367,9 @@ def main():
                 "unit": "GB/s", "frac": achieved / peak, "avg_launch_ms": fine_avg,
                 "algorithmic_per_launch": nbytes_f,
                 "algorithmic_rule": "per nnz: K row + V row (2*d*2 B) + 4 B index; per row: Q read + partial write",
+                "note": "the gathered K/V rows of a head (4 MB) are served by L2, so the algorithmic rate can exceed "
+                        "the HBM peak the north_star measures against (frac > 1); `traffic` (ncu DRAM bytes) is "
+                        "what reached HBM; the L2-gather ceiling is ~22 TB/s (tools/microbench/gather_bw.cu)",
                 "peak_source": peak_src, "traffic": None}
     tr_path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(tr_path):
