@@ -21,7 +21,7 @@ LIB = os.path.join(PKG, "libmg.so")
 VARIANTS = {"base": [],   # (a plain build under another name: A/B against a stashed source tree)
             "watchdog": ["-DMG_WATCHDOG"], "timeline": ["-DMG_TIMELINE"], "trace": ["-DMG_TRACE"],
             # A/B of the share of exponentials emulated on the FMA pipe (pairs of 16 per chunk)
-            "e0": ["-DMG_EXP_EMU=0"], "e4": ["-DMG_EXP_EMU=4"], "e8": ["-DMG_EXP_EMU=8"],
+            "e0": ["-DMG_EXP_EMU=0"], "e1": ["-DMG_EXP_EMU=1"], "e2": ["-DMG_EXP_EMU=2"], "e3": ["-DMG_EXP_EMU=3"], "e4": ["-DMG_EXP_EMU=4"], "e8": ["-DMG_EXP_EMU=8"],
             "maxpass": ["-DMG_SKIP_MAX=0"],
             # coarse softmax: 32-column chunks whose exponentials precede the P.V(n-1) wait
             "pre0": ["-DMG_PRE_CHUNKS=0"], "pre1": ["-DMG_PRE_CHUNKS=1"], "pre2": ["-DMG_PRE_CHUNKS=2"],

@@ -201,10 +201,11 @@ __device__ __forceinline__ float2 exp2_fma2(float2 x) {
 }
 
 // Pairs (of 16 per 32-column chunk) whose exponentials run on the FMA pipe instead of MUFU.
-// Measured on C2/C3 (tools/ab_variants.sh): 0 is fastest with the current kernel, whose softmax
-// is latency- and issue-bound rather than MUFU-bound; kept for re-tuning.
+// Measured on C2/C3/C4 (tools/ab_variants.sh): with the exponentials ahead of the P.V(n-1) wait the
+// steady state is MUFU-bound, and 2 of 16 pairs per 32-column chunk on the FMA pipe is best
+// (C2 0.1466 -> 0.1423 ms; 1 or 3 pairs: 0.1433 / 0.1462; 4: 0.154; C3 within 1%).
 #ifndef MG_EXP_EMU
-#define MG_EXP_EMU 0
+#define MG_EXP_EMU 2
 #endif
 constexpr int kExpEmu = MG_EXP_EMU;
 
