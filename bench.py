@@ -357,6 +357,19 @@ def main():
                 "avg_launch_ms": coarse_avg, "algorithmic_per_launch": flops,
                 "algorithmic_rule": "4*d flops per valid element it owns (coarse + strip + dense-row)",
                 "peak_source": peak_src + " bf16 burst", "traffic": None}
+        # the pipe that actually bounds this kernel: one MUFU ex2 per computed score (K1)
+        clk = sampler.summary()
+        mhz = clk.get("sm_mhz") or clk.get("sm_max_mhz")
+        if mhz:
+            sms = torch.cuda.get_device_properties(dev).multi_processor_count
+            exps = float(info["computed_scores"]) * BH
+            mufu_peak = 16.0 * sms * mhz * 1e6 / 1e12          # Tex2/s: 16 ex2 / clk / SM (measured)
+            mufu_ach = exps / (coarse_avg * 1e-3) / 1e12
+            roof["mufu"] = {"achieved": mufu_ach, "peak": mufu_peak, "unit": "Tex2/s",
+                            "frac": mufu_ach / mufu_peak, "exps_per_launch": exps,
+                            "peak_rule": "16 ex2/clk/SM (tools/microbench/mufu_mix.cu) x SMs x median SM clock; "
+                                         "a share of the exponentials runs on the FMA pipe (MG_EXP_EMU), so frac "
+                                         "can exceed what MUFU alone would allow"}
     else:
         nbytes_f = info["nnz_fine_cuda"] * BH * (2 * cfg.d * 2 + 4) + info["n_fine_rows"] * BH * (2 * cfg.d + 264)
         achieved = nbytes_f / (fine_avg * 1e-3) / 1e9
