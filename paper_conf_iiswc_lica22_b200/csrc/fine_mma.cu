@@ -111,6 +111,19 @@ constexpr int kSmemBytes = kWarps * kStages * kStageBytes;
 // warps in the grid; neighbouring warps stay on neighbouring rows of the same head, so the head's
 // K/V stay in L2), and the gather pointer runs ahead across row boundaries, so a row's first gathers
 // are in flight while the previous row is computed (one row is only ~11 steps).
+// (b*h, CSR row) of a global row index: 32-bit division whenever the row space fits 32 bits (a
+// 64-bit division is a ~100-instruction software routine, run twice per row)
+__device__ __forceinline__ void split_row(int64_t g, int n, bool r32, int& u0, int& fi) {
+  if (r32) {
+    const uint32_t g32 = (uint32_t)g, q = g32 / (uint32_t)n;
+    u0 = (int)q;
+    fi = (int)(g32 - q * (uint32_t)n);
+  } else {
+    u0 = (int)(g / n);
+    fi = (int)(g % n);
+  }
+}
+
 template <bool kBF16, bool kPad>
 __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(const FineParams p) {
   extern __shared__ __align__(128) uint8_t fsm[];
@@ -119,6 +132,7 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(con
   const float c = p.scale_log2;
   const float thresh = 8.f / c;
   const int64_t nrows = (int64_t)p.BH * p.n_fine_rows;
+  const bool r32 = nrows <= (int64_t)0xffffffffLL;   // (split_row is only called with an index < nrows)
   const int64_t W = (int64_t)gridDim.x * kWarps;
   const int64_t w0 = (int64_t)blockIdx.x * kWarps + (threadIdx.x >> 5);
   const uint32_t ring = (uint32_t)__cvta_generic_to_shared(fsm) + (threadIdx.x >> 5) * (kStages * kStageBytes);
@@ -143,7 +157,8 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(con
   auto row_ref = [&](int64_t gr) {
     RowRef rr{0, 0, 0};
     if (gr < nrows) {
-      const int u0 = (int)(gr / p.n_fine_rows), fi = (int)(gr % p.n_fine_rows);
+      int u0, fi;
+      split_row(gr, p.n_fine_rows, r32, u0, fi);
       rr.bh = p.fine_sample ? __ldg(p.fine_sample + fi) * p.H + u0 : u0;
       rr.beg = __ldg(p.row_ptr + fi);
       rr.end = __ldg(p.row_ptr + fi + 1);
@@ -207,7 +222,8 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(con
   const uint16_t *iK = nullptr, *iV = nullptr;
   auto open_issue_row = [&]() {
     if (gi < nrows) {
-      const int u0 = (int)(gi / p.n_fine_rows), fi = (int)(gi % p.n_fine_rows);
+      int u0, fi;
+      split_row(gi, p.n_fine_rows, r32, u0, fi);
       const int bh = p.fine_sample ? __ldg(p.fine_sample + fi) * p.H + u0 : u0;
       ibeg = __ldg(p.row_ptr + fi);
       iend = __ldg(p.row_ptr + fi + 1);
@@ -253,8 +269,8 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(con
   const uint32_t vr = (lane & 7) + 8 * (lane >> 4);
 
   for (int64_t gw = w0; gw < nrows; gw += W) {
-    const int u0 = (int)(gw / p.n_fine_rows);
-    const int fi = (int)(gw % p.n_fine_rows);
+    int u0, fi;
+    split_row(gw, p.n_fine_rows, r32, u0, fi);
     const int bh = p.fine_sample ? __ldg(p.fine_sample + fi) * p.H + u0 : u0;   // (batched plans)
     const int enc = __ldg(p.fine_rows + fi);
     const int r = enc & 0x7fffffff;
