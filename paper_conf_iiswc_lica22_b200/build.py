@@ -26,7 +26,7 @@ VARIANTS = {"base": [],   # (a plain build under another name: A/B against a sta
             # coarse softmax: 32-column chunks whose exponentials precede the P.V(n-1) wait
             "pre0": ["-DMG_PRE_CHUNKS=0"], "pre1": ["-DMG_PRE_CHUNKS=1"], "pre2": ["-DMG_PRE_CHUNKS=2"],
             # fine tensor-core kernel: cp.async ring stages per warp (default 2), min blocks per SM
-            "fs3": ["-DMG_FINE_STAGES=3"], "pf1": ["-DMG_FINE_PREF=1"], "pf1b4": ["-DMG_FINE_PREF=1", "-DMG_FINE_MINB=4"], "fs4": ["-DMG_FINE_STAGES=4"], "fs3b4": ["-DMG_FINE_STAGES=3", "-DMG_FINE_MINB=4"], "fs3b6": ["-DMG_FINE_STAGES=3", "-DMG_FINE_MINB=6"], "fb4": ["-DMG_FINE_MINB=4"], "fb6": ["-DMG_FINE_MINB=6"],
+            "fs3": ["-DMG_FINE_STAGES=3"], "fs4": ["-DMG_FINE_STAGES=4"], "fs3b4": ["-DMG_FINE_STAGES=3", "-DMG_FINE_MINB=4"], "fs3b6": ["-DMG_FINE_STAGES=3", "-DMG_FINE_MINB=6"], "fb4": ["-DMG_FINE_MINB=4"], "fb6": ["-DMG_FINE_MINB=6"],
             "fb8": ["-DMG_FINE_MINB=8"], "fp2": ["-DMG_FINE_PAIRS=2"], "fp2b3": ["-DMG_FINE_PAIRS=2", "-DMG_FINE_MINB=3"],
             "fw8": ["-DMG_FINE_WARPS=8", "-DMG_FINE_MINB=3"], "fw2": ["-DMG_FINE_WARPS=2", "-DMG_FINE_MINB=10"],
             "fw1": ["-DMG_FINE_WARPS=1", "-DMG_FINE_MINB=20"],

@@ -82,12 +82,6 @@ __device__ __forceinline__ void ldsm_x4_t(uint32_t (&r)[4], uint32_t addr) {
 #ifndef MG_FINE_PAIRS
 #define MG_FINE_PAIRS 1
 #endif
-// MG_FINE_PREF=1: column indices loaded one 32-nnz window ahead and row bounds one row ahead of
-// the gather pointer. Measured slower on C4 (2.59 / 2.48 ms at 5 / 4 blocks per SM vs 2.44 ms):
-// the extra registers cost more than the index-load latency they hide. Kept off for the record.
-#ifndef MG_FINE_PREF
-#define MG_FINE_PREF 0
-#endif
 #ifndef MG_FINE_WARPS
 #define MG_FINE_WARPS 4
 #endif
@@ -95,7 +89,8 @@ constexpr int kWarps = MG_FINE_WARPS;       // warps per block, each a persisten
 constexpr int kP = MG_FINE_PAIRS;           // 16-nnz pairs of 8-nnz chunks per step (1 or 2)
 constexpr int kS = 16 * kP;                 // nnz per step
 constexpr int kStages = MG_FINE_STAGES;     // smem ring stages per warp (kStages - 1 steps in flight)
-constexpr int kStageBytes = 2 * kS * 128;  // kS K rows + kS V rows of 128 bytes
+constexpr int kQOff = 2 * kS * 128;        // the q row of a row's first step follows its K and V rows
+constexpr int kStageBytes = kQOff + 128;   // kS K rows + kS V rows + q, 128 bytes each
 constexpr int kSmemBytes = kWarps * kStages * kStageBytes;
 
 }  // namespace
@@ -145,81 +140,10 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(con
     doff[i] = R * 128 + (((lane & 7) ^ (R & 7)) << 4);
   }
 
-#if MG_FINE_PREF
-  // ---- gather pointer with its column indices one 32-nnz window ahead. The issue sequence is the
-  // warp's rows gi = w0, w0 + W, ... each as windows of 32 nnz (kS-nnz steps); `icol` holds the
-  // current window's indices (lane i: index iwb + i), `ncol` the next window's, loaded one window
-  // before use, and the bounds of the row after the next window's row are loaded one row ahead, so
-  // no step waits on an index or row-pointer load.
-  struct RowRef {
-    int beg, end, bh;
-  };
-  auto row_ref = [&](int64_t gr) {
-    RowRef rr{0, 0, 0};
-    if (gr < nrows) {
-      int u0, fi;
-      split_row(gr, p.n_fine_rows, r32, u0, fi);
-      rr.bh = p.fine_sample ? __ldg(p.fine_sample + fi) * p.H + u0 : u0;
-      rr.beg = __ldg(p.row_ptr + fi);
-      rr.end = __ldg(p.row_ptr + fi + 1);
-    }
-    return rr;
-  };
-  const uint16_t *iK = nullptr, *iV = nullptr;
-  auto set_kv = [&](int bh) {
-    const int bb = bh / p.H, hh = bh % p.H;
-    iK = p.k.data + bb * p.k.sb + hh * p.k.sh + (lane & 7) * 8;
-    iV = p.v.data + bb * p.v.sb + hh * p.v.sh + (lane & 7) * 8;
-  };
-  int64_t gi = w0, ngi = w0;
-  RowRef nrow = row_ref(w0), prow;
-  int iend = nrow.end, iwb = nrow.beg, nwb = nrow.beg, isub = 0;
-  int icol = w0 < nrows && iwb + lane < iend ? __ldg(p.cols + iwb + lane) : -1, ncol = -1;
-  set_kv(nrow.bh);
-  // next window after (ngi, nwb): same row if it has one, else the first window of row ngi + W
-  auto next_window = [&]() {
-    if (nwb + 32 < nrow.end) {
-      nwb += 32;
-    } else {
-      ngi += W;
-      nrow = prow;
-      nwb = nrow.beg;
-      prow = row_ref(ngi + W);
-    }
-    ncol = ngi < nrows && nwb + lane < nrow.end ? __ldg(p.cols + nwb + lane) : -1;
-  };
-  prow = row_ref(w0 + W);
-  next_window();
-  auto issue_step = [&](uint32_t stg) {
-    if (gi < nrows) {   // warp-uniform
-      const int nb0 = iwb + kS * isub;
-      const int off = kS * isub + (lane >> 3);
-      const uint32_t st = ring + stg * kStageBytes;
-#pragma unroll
-      for (int i = 0; i < 4 * kP; ++i) {
-        const uint32_t cc = (uint32_t)max(__shfl_sync(0xffffffffu, icol, off + 4 * i), 0);
-        cp_async16(st + doff[i], iK + cc * ksl);
-        cp_async16(st + doff[i] + kS * 128, iV + cc * vsl);
-      }
-      if (nb0 + kS < iend && isub + 1 < 32 / kS) {
-        ++isub;
-      } else {   // advance to the prefetched window
-        if (ngi != gi) set_kv(nrow.bh);
-        gi = ngi;
-        iend = nrow.end;
-        iwb = nwb;
-        icol = ncol;
-        isub = 0;
-        next_window();
-      }
-    }
-    cp_async_commit();   // (an empty group past the end keeps the wait count uniform)
-  };
-#else
   // ---- gather pointer: row gi (global work index), step is of [ibeg, iend)
   int64_t gi = w0;
   int ibeg = 0, iend = 0, is = 0, icol = -1;
-  const uint16_t *iK = nullptr, *iV = nullptr;
+  const uint16_t *iK = nullptr, *iV = nullptr, *iQ = nullptr;
   auto open_issue_row = [&]() {
     if (gi < nrows) {
       int u0, fi;
@@ -230,6 +154,8 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(con
       const int bb = bh / p.H, hh = bh % p.H;
       iK = p.k.data + bb * p.k.sb + hh * p.k.sh + (lane & 7) * 8;
       iV = p.v.data + bb * p.v.sb + hh * p.v.sh + (lane & 7) * 8;
+      const int rq = __ldg(p.fine_rows + fi) & 0x7fffffff;
+      iQ = p.q.data + bb * p.q.sb + hh * p.q.sh + (int64_t)rq * p.q.sl + (lane & 7) * 8;
     }
     is = 0;
   };
@@ -242,6 +168,9 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(con
       if (kP == 2 || (is & 1) == 0) icol = nb0 + lane < iend ? __ldg(p.cols + nb0 + lane) : -1;
       const int off = (kP == 2 ? 0 : (is & 1) * 16) + (lane >> 3);
       const uint32_t st = ring + stg * kStageBytes;
+      // a row's first step also carries its q row (lanes 0-7, 16 B each), so the computing side
+      // never waits on a dependent q load at a row start
+      if (is == 0 && lane < 8) cp_async16(st + kQOff + (lane << 4), iQ);
 #pragma unroll
       for (int i = 0; i < 4 * kP; ++i) {
         const uint32_t cc = (uint32_t)max(__shfl_sync(0xffffffffu, icol, off + 4 * i), 0);
@@ -258,10 +187,7 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(con
     cp_async_commit();   // (an empty group past the end keeps the wait count uniform)
   };
 
-#endif
-#if !MG_FINE_PREF
   open_issue_row();
-#endif
 #pragma unroll
   for (int s = 0; s < kStages - 1; ++s) issue_step(s);
   uint32_t stage = 0, istage = kStages - 1;
@@ -276,14 +202,9 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(con
     const int r = enc & 0x7fffffff;
     const bool final_out = enc < 0;
     const int bb = bh / p.H, hh = bh % p.H;
-    // q as the SDDMM's A operand (every row = q): k16 step j uses dims 16j + 2t (+1), 16j + 8 + 2t (+1)
-    const uint16_t* qrow = p.q.data + bb * p.q.sb + hh * p.q.sh + (int64_t)r * p.q.sl;
-    uint32_t qa[4], qb[4];
-#pragma unroll
-    for (int j = 0; j < 4; ++j) {
-      qa[j] = __ldg(reinterpret_cast<const uint32_t*>(qrow + 16 * j + 2 * t));
-      qb[j] = __ldg(reinterpret_cast<const uint32_t*>(qrow + 16 * j + 8 + 2 * t));
-    }
+    // q as the SDDMM's A operand (every row = q): k16 step j uses dims 16j + 2t (+1), 16j + 8 + 2t (+1);
+    // read from the q slot of the row's first ring stage
+    uint32_t qa[4] = {0u, 0u, 0u, 0u}, qb[4] = {0u, 0u, 0u, 0u};
     const int beg = __ldg(p.row_ptr + fi), end = __ldg(p.row_ptr + fi + 1);
     // padding (A18): columns >= n_b are masked; a row >= n_b is written as 0 if it is final (a row
     // with a coarse part is zeroed by the coarse kernel)
@@ -304,6 +225,13 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(con
       __syncwarp();
       const uint32_t st = ring + stage * kStageBytes;
       stage = stage == kStages - 1 ? 0 : stage + 1;
+      if (base == beg) {
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          asm volatile("ld.shared.u32 %0, [%1];" : "=r"(qa[j]) : "r"(st + kQOff + 32 * j + 4 * t));
+          asm volatile("ld.shared.u32 %0, [%1];" : "=r"(qb[j]) : "r"(st + kQOff + 32 * j + 16 + 4 * t));
+        }
+      }
 
       // ---- SDDMM per pair: chunk A (rows 16pr + 0-7) and chunk B (rows 16pr + 8-15); lane holds
       // nnz 2t, 2t+1 of each chunk; two independent accumulators per chunk (dims 0-31, 32-63)
