@@ -34,7 +34,7 @@ VARIANTS = {"base": [],   # (a plain build under another name: A/B against a sta
             "dbg1": ["-DMG_DBG=1"], "dbg3": ["-DMG_DBG=3"], "dbg7": ["-DMG_DBG=7"]}
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 
-SOURCES = ["plan.cpp", "api.cu", "coarse_sm100.cu", "coarse_pp_sm100.cu", "fine_rows.cu", "fine_mma.cu", "staged.cu", "selftest_umma.cu"]
+SOURCES = ["plan.cpp", "api.cu", "coarse_pp_sm100.cu", "fine_rows.cu", "fine_mma.cu", "staged.cu", "selftest_umma.cu"]
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 COMMON = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC,-fvisibility=hidden",
           "-I", os.path.join(ROOT, "include"), "-I", CSRC]

@@ -1,6 +1,6 @@
 // C ABI of the Multigrain forward (include/mg.h). Host-side: validation, plan lifetime,
 // device upload, TMA descriptors, workspace, launches. Every step of the attention runs in the
-// kernels of coarse_sm100.cu and fine_rows.cu; there is no CPU fallback.
+// kernels of coarse_pp_sm100.cu, fine_mma.cu / fine_rows.cu and staged.cu; there is no CPU fallback.
 #include <cudaTypedefs.h>
 
 #include <algorithm>
@@ -163,6 +163,10 @@ mg_status upload(mg_plan_s* p) {
   cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, p->device);
   if (major != 10) return fail(MG_ERR_UNSUPPORTED, "this library is built for sm_100a (B200) only");
   const mg::HostPlan& h = p->hp;
+  // the fine kernels' gather pointer issues one ring step per row start (fine_mma.cu issue_step):
+  // every fine row must hold at least one entry (plan.cpp never lists an empty CSR row)
+  for (size_t i = 0; i + 1 < h.fine_row_ptr.size(); ++i)
+    if (h.fine_row_ptr[i + 1] <= h.fine_row_ptr[i]) return fail(MG_ERR_INTERNAL, "plan lists an empty fine row");
   if ((e = upload_vec(p, &p->d_items, h.items)) != cudaSuccess ||
       (e = upload_vec(p, &p->d_items_split, h.items_split)) != cudaSuccess ||
       (e = upload_vec(p, &p->d_fine_sample, h.fine_sample)) != cudaSuccess ||
@@ -366,11 +370,7 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
   cudaError_t e;
   // Concurrent coarse || fine (north_star item 5): chosen by measurement, only with
   // the tensor-core fine kernel and the paired-pipeline coarse kernel.
-  static const bool v13 = [] {
-    const char* e = std::getenv("MG_COARSE");
-    return e && std::strcmp(e, "v13") == 0;
-  }();
-  const bool concurrent = nf > 0 && !h.items.empty() && p->fine_kernel == 0 && !v13 &&
+  const bool concurrent = nf > 0 && !h.items.empty() && p->fine_kernel == 0 &&
                           (p->concurrency == 2 || (p->concurrency == 0 && kConcurrentDefault));
   // fp32 partials of the CUDA-core CSR rows (fine -> coarse; and coarse -> fine plus one counter
   // per row when concurrent). Layout by capacity: [fine acc 64][fine ml 2][coarse acc 64][coarse ml 2]
@@ -396,7 +396,7 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
   int32_t* part_flags = reinterpret_cast<int32_t*>(p->d_part + cap * 132);
   // split dense-row items (a work list with the global rows' column tiles in chunks): chosen when
   // the unsplit dense items would be few against the SMs (each would be a long serial chain), or
-  // forced by the plan option; per (b*h, row group) chunk partials + monotone counters
+  // forced by the plan option; per (b*h, row group) chunk partials + chunk counters
   const bool use_split = h.dense_nsplit > 1 && h.n_dense_groups > 0 &&
                          (h.opts.dense_split == 2 ||
                           (h.opts.dense_split == 0 && (int64_t)h.n_dense_groups * BH * 2 <= p->num_sms));
@@ -467,7 +467,9 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
     fp.part_c_ml = part_c_ml;
     fp.part_flags = part_flags;
     // (the CUDA-core variant has no padding support: a padded forward always uses the MMA kernel)
-    e = p->fine_kernel == 1 && !valid_len ? mg::launch_fine(fp, bf16, fstream) : mg::launch_fine_mma(fp, bf16, fstream);
+    const int fsms = p->num_sms_override > 0 ? std::min(p->num_sms_override, p->num_sms) : p->num_sms;
+    e = p->fine_kernel == 1 && !valid_len ? mg::launch_fine(fp, bf16, fstream)
+                                          : mg::launch_fine_mma(fp, bf16, fsms, fstream);
     if (e != cudaSuccess) return cuda_fail(e, "fine kernel launch");
   }
   if (p->profiling && has_f) {
@@ -536,16 +538,9 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
     cp.debug_flags = dbg;
     cp.trace = p->trace;
     cp.trace_cap = p->trace_cap;
-    // the paired-pipeline kernel resets its work counter itself (last CTA to exit); the v13 kernel
-    // needs it zeroed before the launch
-    if (v13 && h.batch == 0 && (e = cudaMemsetAsync(p->d_counter, 0, sizeof(int32_t), stream)) != cudaSuccess)
-      return cuda_fail(e, "cudaMemsetAsync");
+    // (the kernel resets its work counter itself: the last CTA to exit zeroes it)
     const int sms = p->num_sms_override > 0 ? std::min(p->num_sms_override, p->num_sms) : p->num_sms;
-    // MG_COARSE=v13 selects the previous single-CTA-per-SM kernel (A/B measurements only)
-    if (v13 && h.batch == 0) {
-      if ((e = mg::launch_coarse(cp, tq, tk, tv, bf16, std::min(sms, cp.total_units), stream)) != cudaSuccess)
-        return cuda_fail(e, "coarse kernel launch");
-    } else {
+    {
       static const bool no_tma_gather = std::getenv("MG_NO_TMA_GATHER") != nullptr;   // A/B diagnostics
       cp.gather_tma = !no_tma_gather && mp.gather_ok;
       cp.rq = mp.rq;
@@ -812,7 +807,12 @@ mg_status mg_sparse_attention_fwd_host(mg_plan_t plan, const mg_tensor* Q, const
   // c-1 (d2h stream) overlap the forward of chunk c (`stream`); host tensors are dense, so a batch
   // chunk is one contiguous range of each. Batched plans (one pattern per sample) run as one chunk.
   const int64_t B = Q->batch;
-  const int64_t nchunk = plan->hp.batch > 0 ? 1 : std::min<int64_t>(B, 8);
+  // a batch chunk is one contiguous byte range of every tensor only when the batch is the outermost
+  // dimension of each (dense [B,H,L,d] or [B,L,H,d]); any other dense layout moves as one span
+  bool batch_outer = true;
+  for (const mg_tensor* t : {Q, K, V, static_cast<const mg_tensor*>(O)})
+    batch_outer = batch_outer && t->stride_b == t->heads * t->seq_len * t->head_dim;
+  const int64_t nchunk = (plan->hp.batch > 0 || !batch_outer) ? 1 : std::min<int64_t>(B, 8);
   const size_t per_b = bytes / (size_t)B;
   uint8_t* dst[4] = {plan->d_stage, plan->d_stage + bytes, plan->d_stage + 2 * bytes, plan->d_stage + 3 * bytes};
   const uint8_t* src[3] = {static_cast<const uint8_t*>(Q->data), static_cast<const uint8_t*>(K->data),
@@ -828,29 +828,44 @@ mg_status mg_sparse_attention_fwd_host(mg_plan_t plan, const mg_tensor* Q, const
       (e = cudaStreamWaitEvent(plan->h2d, ev_start, 0)) != cudaSuccess ||
       (e = cudaStreamWaitEvent(plan->d2h, ev_start, 0)) != cudaSuccess)
     return cuda_fail(e, "stream fork");
+  // every return after the fork joins the copy streams back into `stream` first, so that a caller
+  // who synchronises `stream` after an error may free the pinned buffers the copies read
+  auto join = [&]() {
+    cudaEventRecord(ev_end, plan->h2d);
+    cudaStreamWaitEvent(stream, ev_end, 0);
+    cudaEventRecord(ev_end, plan->d2h);
+    cudaStreamWaitEvent(stream, ev_end, 0);
+  };
+  auto fail_joined = [&](mg_status st) {
+    const std::string msg = g_err;
+    join();
+    g_err = msg;
+    return st;
+  };
   for (int64_t c = 0; c < nchunk; ++c) {
     const int64_t b0 = B * c / nchunk, b1 = B * (c + 1) / nchunk;
     const size_t off = (size_t)b0 * per_b, len = (size_t)(b1 - b0) * per_b;
     cudaEvent_t ev_in = plan->host_event(2 + 2 * c), ev_done = plan->host_event(3 + 2 * c);
     for (int i = 0; i < 3; ++i)
       if ((e = cudaMemcpyAsync(dst[i] + off, src[i] + off, len, cudaMemcpyHostToDevice, plan->h2d)) != cudaSuccess)
-        return cuda_fail(e, "H2D copy");
+        return fail_joined(cuda_fail(e, "H2D copy"));
     if ((e = cudaEventRecord(ev_in, plan->h2d)) != cudaSuccess || (e = cudaStreamWaitEvent(stream, ev_in, 0)) != cudaSuccess)
-      return cuda_fail(e, "event");
+      return fail_joined(cuda_fail(e, "event"));
     mg_tensor dq = *Q, dk = *K, dv = *V, dO = *O;
     dq.data = dst[0] + off;
     dk.data = dst[1] + off;
     dv.data = dst[2] + off;
     dO.data = dst[3] + off;
     dq.batch = dk.batch = dv.batch = dO.batch = b1 - b0;
-    if ((s = fwd_impl(plan, &dq, &dk, &dv, &dO, stream)) != MG_OK) return s;
+    if ((s = fwd_impl(plan, &dq, &dk, &dv, &dO, stream)) != MG_OK) return fail_joined(s);
     if ((e = cudaEventRecord(ev_done, stream)) != cudaSuccess || (e = cudaStreamWaitEvent(plan->d2h, ev_done, 0)) != cudaSuccess)
-      return cuda_fail(e, "event");
+      return fail_joined(cuda_fail(e, "event"));
     if ((e = cudaMemcpyAsync(static_cast<uint8_t*>(O->data) + off, dst[3] + off, len, cudaMemcpyDeviceToHost,
                              plan->d2h)) != cudaSuccess)
-      return cuda_fail(e, "D2H copy");
+      return fail_joined(cuda_fail(e, "D2H copy"));
   }
-  if ((e = cudaEventRecord(ev_end, plan->d2h)) != cudaSuccess || (e = cudaStreamWaitEvent(stream, ev_end, 0)) != cudaSuccess)
+  if ((e = cudaEventRecord(ev_end, plan->h2d)) != cudaSuccess || (e = cudaStreamWaitEvent(stream, ev_end, 0)) != cudaSuccess ||
+      (e = cudaEventRecord(ev_end, plan->d2h)) != cudaSuccess || (e = cudaStreamWaitEvent(stream, ev_end, 0)) != cudaSuccess)
     return cuda_fail(e, "stream join");
   return MG_OK;
 }

@@ -770,8 +770,11 @@ __global__ void __launch_bounds__(kThreads, 2)
         }
         __threadfence();
         named_bar_sync(1, 128);
+        // per-group chunk counter in [0, nrowsB): atomicInc wraps it back to 0 on the last chunk, so it
+        // is ready for the next forward and never overflows
         if (threadIdx.x == 0)
-          ctl->dense_last = (atomicAdd(p.dense_ctr + gidx, 1) % item.nrowsB) == item.nrowsB - 1;
+          ctl->dense_last = atomicInc(reinterpret_cast<unsigned*>(p.dense_ctr) + gidx, (unsigned)item.nrowsB - 1u) ==
+                            (unsigned)item.nrowsB - 1u;
         named_bar_sync(1, 128);
         skip = !ctl->dense_last;
         if (!skip && t < item.nrowsA) {

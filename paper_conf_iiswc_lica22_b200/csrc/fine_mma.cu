@@ -8,7 +8,7 @@
 //
 // A step handles 16 nnz of the row, as two chunks A and B of 8. Lane = 4g + t.
 //   SDDMM  s^T = q . K_c^T as mma(M=16 x N=8 x K=16) x 4 per chunk (64 dims): A = q broadcast to
-//          all 16 rows (lane registers straight from global memory), B column n = gathered K row
+//          all 16 rows (lane registers from the q slot of the row's first ring stage), B column n = gathered K row
 //          of chunk nnz n (ldmatrix from the swizzled stage). D: lane (g,t) gets the scores of
 //          chunk nnz 2t and 2t+1.
 //   SpMM   O^T = V_c^T . p as mma(M=16 dims x N=8 x K=16 nnz) x 4 (64 dims): k = nnz (chunk A
@@ -19,6 +19,9 @@
 // running max/sum and O accumulate in fp32. Lazy rescaling: the exponent keeps a stale max until
 // a step's max exceeds it by 8/c (p <= 256), warp-uniform because all lanes see the same max.
 #include <algorithm>
+#include <map>
+#include <mutex>
+#include <utility>
 
 #include <cuda_bf16.h>
 #include <cuda_fp16.h>
@@ -159,7 +162,9 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(con
     }
     is = 0;
   };
-  // issue the gathers of the pointer's step into ring stage `stg` and advance the pointer. Indices
+  // issue the gathers of the pointer's step into ring stage `stg` and advance the pointer. Every
+  // fine row has at least one entry (checked at plan upload, api.cu), so each row start issues
+  // exactly the ceil(nnz / kS) steps the computing side consumes, the first carrying q. Indices
   // come from `icol` (lane i holds index ibeg + 32 w + i of window w; steps 2w, 2w + 1 use it); past
   // the row's end they are -1 and read row 0 (masked scores, p = 0).
   auto issue_step = [&](uint32_t stg) {
@@ -356,25 +361,32 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(con
   cp_async_wait<0>();
 }
 
-cudaError_t launch_fine_mma(const FineParams& p, bool bf16, cudaStream_t stream) {
+cudaError_t launch_fine_mma(const FineParams& p, bool bf16, int sms, cudaStream_t stream) {
   const int64_t warps = (int64_t)p.BH * p.n_fine_rows;
   if (warps == 0) return cudaSuccess;
   auto kern = bf16 ? (p.valid_len ? fine_mma_kernel<true, true> : fine_mma_kernel<true, false>)
                    : (p.valid_len ? fine_mma_kernel<false, true> : fine_mma_kernel<false, false>);
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytes);
   if (e != cudaSuccess) return e;
-  // persistent grid: every resident block slot of every SM, or fewer if the rows are few
-  static int per_sm[4] = {0, 0, 0, 0}, sms = 0;   // per kernel variant
+  // persistent grid: every resident block slot of `sms` SMs (the plan's SM count, or its num_sms
+  // test override), or fewer if the rows are few. Resident blocks per SM of each variant, per
+  // device, computed once under a lock (launches may come from several host threads).
+  static std::mutex mu;
+  static std::map<std::pair<int, int>, int> per_sm;
   const int vi = (bf16 ? 2 : 0) + (p.valid_len ? 1 : 0);
-  if (per_sm[vi] == 0) {
-    int dev = 0, n = 0;
-    if ((e = cudaGetDevice(&dev)) != cudaSuccess ||
-        (e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev)) != cudaSuccess ||
-        (e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kern, kWarps * 32, kSmemBytes)) != cudaSuccess)
-      return e;
-    per_sm[vi] = std::max(n, 1);
+  int dev = 0, n = 0;
+  if ((e = cudaGetDevice(&dev)) != cudaSuccess) return e;
+  {
+    std::lock_guard<std::mutex> lk(mu);
+    auto it = per_sm.find({dev, vi});
+    if (it == per_sm.end()) {
+      if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kern, kWarps * 32, kSmemBytes)) != cudaSuccess)
+        return e;
+      it = per_sm.emplace(std::make_pair(dev, vi), std::max(n, 1)).first;
+    }
+    n = it->second;
   }
-  const int64_t blocks = std::min<int64_t>((warps + kWarps - 1) / kWarps, (int64_t)per_sm[vi] * sms);
+  const int64_t blocks = std::min<int64_t>((warps + kWarps - 1) / kWarps, (int64_t)n * std::max(sms, 1));
   kern<<<(unsigned)blocks, kWarps * 32, kSmemBytes, stream>>>(p);
   return cudaGetLastError();
 }

@@ -16,7 +16,7 @@ struct TensorView {
 };
 
 // Coarse / dense-row / strip kernel: tcgen05 SDDMM -> online SpSoftmax -> tcgen05 SpMM,
-// persistent over (item, batch*head) units. See coarse_sm100.cu.
+// persistent over (item, batch*head) units. See coarse_pp_sm100.cu.
 struct CoarseParams {
   const Item* items;
   const TileRef* trefs;
@@ -52,7 +52,7 @@ struct CoarseParams {
   const int32_t* valid_len;
   // split dense-row items (Item::nrowsB > 1): per (b*h, row group) chunk partials and counters
   float* dense_part;          // [BH][n_dense_groups][dense_nsplit][128][68]: acc[64], m, l, pad (16-B rows)
-  int32_t* dense_ctr;         // [BH][n_dense_groups], +1 per finished chunk (monotone, mod nsplit)
+  int32_t* dense_ctr;         // [BH][n_dense_groups], finished chunks of the current forward (wraps to 0)
   int32_t n_dense_groups, dense_nsplit;
   // band items whose rows are all theirs to write (Item::useA) store O by TMA from shared memory
   // (the item's Q buffer) instead of per-thread row stores
@@ -106,8 +106,6 @@ cudaError_t launch_staged_sddmm(const StagedParams& p, bool bf16, cudaStream_t s
 cudaError_t launch_staged_softmax(const StagedParams& p, bool bf16, cudaStream_t stream);
 cudaError_t launch_staged_spmm(const StagedParams& p, bool bf16, cudaStream_t stream);
 
-cudaError_t launch_coarse(const CoarseParams& p, const CUtensorMap& tmq, const CUtensorMap& tmk,
-                          const CUtensorMap& tmv, bool bf16, int grid, cudaStream_t stream);
 // Paired-pipeline variant: two CTAs per SM (grid = 2 x SMs), see coarse_pp_sm100.cu.
 cudaError_t launch_coarse_pp(const CoarseParams& p, const CUtensorMap& tmq, const CUtensorMap& tmk,
                              const CUtensorMap& tmv, const CUtensorMap& tmq2, const CUtensorMap& tmk2,
@@ -115,7 +113,7 @@ cudaError_t launch_coarse_pp(const CoarseParams& p, const CUtensorMap& tmq, cons
                              cudaStream_t stream);
 cudaError_t launch_fine(const FineParams& p, bool bf16, cudaStream_t stream);
 // Warp-level tensor-core variant (mma.sync m16n8k16), the default; see fine_mma.cu.
-cudaError_t launch_fine_mma(const FineParams& p, bool bf16, cudaStream_t stream);
+cudaError_t launch_fine_mma(const FineParams& p, bool bf16, int sms, cudaStream_t stream);
 cudaError_t launch_selftest_umma(int mode, const void* A, const void* B, float* D, cudaStream_t stream);
 
 }  // namespace mg
