@@ -1,18 +1,23 @@
 """Benchmark of the Multigrain compound sparse attention forward on B200 (BASELINE.json metric).
 
-    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload C2] [--impl mine|reference]
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload C2|C5|...] [--impl mine|reference]
 
 One "step" = one mg_sparse_attention_fwd over one batch of the workload (every hot-path step:
 plan already built, SDDMM -> merged SpSoftmax -> SpMM over the coarse, fine and dense-row parts).
-N=1 workload: C2 (Longformer-base L=4096, H=12, B=8, w=512, 32 global tokens) — BASELINE.json
-configs[1], the config its metric is quoted on. N>1 (torchrun, one process per GPU): every rank
-runs its own C2 batch (weak scaling over batch x heads; no data-path collective — the parts are
-independent), then an NCCL all_gather of O is timed separately (north_star: gather outputs only).
+N=1 default workload: C2 (Longformer-base L=4096, H=12, B=8, w=512, 32 global tokens) —
+BASELINE.json configs[1], the config its metric is quoted on. N>1 default (torchrun, one process
+per GPU): C5, BASELINE.json configs[4] — the C2 pattern at a global batch of 64 sharded over the
+ranks in contiguous batch slices (dist.shard_range, B/n per rank; strong scaling). The (b, h)
+units are independent, so there is no data-path collective; an NCCL all_gather of O
+(north_star: gather outputs in the scaling bench) is timed separately. `--workload C5 --gpus 1`
+gives the single-GPU time T1 of the sweep; efficiency T1 / (n Tn) is left to the driver. Any other
+workload at N>1 runs weak (each rank its own seeded batch).
 
 Timing: W untimed warm-up steps; the K timed steps are bracketed by barrier + synchronize; each
-step is preceded by a 256 MB L2 flush (outside its CUDA-event pair) and timed with CUDA events on
-the launching stream; max over ranks. value = useful TFLOP/s of the whole job,
-useful flops = 4 * nnz(M) * d * B * H.
+step is preceded by a 256 MB L2 flush (outside its CUDA-event pair) and timed by the library's
+CUDA events on the launching stream (mg_plan_get_profile_calls: mean, median, min per step);
+max over ranks. value = useful TFLOP/s of the whole job, useful flops = 4 * nnz(M) * d * B * H
+(SURVEY.md §8(d)).
 """
 from __future__ import annotations
 
@@ -30,6 +35,9 @@ sys.path.insert(0, ROOT)
 METRIC = "sparse-attn fwd ms and useful TFLOP/s per B200 (Longformer L=4096), 1/2/4/8 GPU"
 UNIT = "TFLOP/s"
 FALLBACK_PEAKS = {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0}
+# L2 -> SM gather ceiling measured on B200 (tools/microbench/gather_bw.cu: 8 lanes per 128-B row,
+# 16-B register loads, no arithmetic), the honest roofline of the L2-served fine kernel
+L2_GATHER_GBS = 22200.0
 
 
 def parse():
@@ -37,8 +45,9 @@ def parse():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=1000)
     ap.add_argument("--warmup", type=int, default=20)
-    ap.add_argument("--workload", default="C2",
-                    choices=["C1", "C2", "C3", "C4", "QDS-LS", "F9-LS", "F9-LSG", "F9-LBR", "F9-RBR"])
+    ap.add_argument("--workload", default=None,
+                    choices=["C1", "C2", "C3", "C4", "C5", "QDS-LS", "F9-LS", "F9-LSG", "F9-LBR", "F9-RBR"],
+                    help="default: C2 at N=1, C5 (strong scaling, global batch 64) at N>1")
     ap.add_argument("--impl", default="mine", choices=["mine", "reference"])
     ap.add_argument("--e2e-steps", type=int, default=30)
     ap.add_argument("--cpu-seconds", type=float, default=12.0, help="CPU oracle sample budget")
@@ -64,15 +73,55 @@ def load_peaks():
     return dict(FALLBACK_PEAKS), "fallback (B200_PROFILING.md)"
 
 
-def workload_config(cfg, n_gpus):
+def resolve_workload(args, world):
+    return args.workload or ("C2" if world == 1 else "C5")
+
+
+# ------------------------------------------------------------------ sharding (host logic; gloo-tested)
+def shard_for_rank(cfg, world: int, rank: int, strong: bool):
+    """Batch rows [lo, hi) of the global batch this rank computes. Strong scaling (C5): the global
+    batch cfg.B is split into contiguous slices (dist.shard_range: the (b, h) units are
+    independent). Weak scaling: every rank computes its own batch of cfg.B."""
+    from paper_conf_iiswc_lica22_b200.dist import shard_range
+    if strong:
+        return shard_range(cfg.B, world, rank)
+    return 0, cfg.B
+
+
+def batch_inputs(cfg, lo: int, hi: int, rank: int, strong: bool):
+    """Q, K, V bit patterns [hi - lo, H, L, d] of the rank's slice. Strong scaling draws every batch
+    element from its own seed (cfg.seed + 1000 b), so a slice does not depend on the world size and
+    the gathered output equals the single-GPU output of the global batch element for element."""
+    import numpy as np
+    from paper_conf_iiswc_lica22_b200.dist import rank_seed
+    from workloads import make_qkv
+    if not strong:
+        return make_qkv(cfg.B, cfg.H, cfg.L, cfg.d, seed=rank_seed(cfg.seed, rank))
+    parts = [make_qkv(1, cfg.H, cfg.L, cfg.d, seed=cfg.seed + 1000 * b) for b in range(lo, hi)]
+    if not parts:
+        z = np.zeros((0, cfg.H, cfg.L, cfg.d), np.uint16)
+        return z, z.copy(), z.copy()
+    return tuple(np.concatenate([p[i] for p in parts]) for i in range(3))
+
+
+def gather_output(O_local, global_batch: int, strong: bool):
+    """The scaling bench's only collective: all_gather of O (strong: reassembled [global_batch, ...]
+    in batch order; weak: [world, B, ...])."""
+    from paper_conf_iiswc_lica22_b200.dist import gather_batches, gather_outputs
+    return gather_batches(O_local, global_batch) if strong else gather_outputs(O_local)
+
+
+def workload_config(cfg, n_gpus, strong, b_local):
     return {
         "workload": f"{cfg.name}: {cfg.note}",
-        "B_per_gpu": cfg.B, "H": cfg.H, "L": cfg.L, "d": cfg.d, "window": cfg.window,
+        "B_per_gpu": b_local, "H": cfg.H, "L": cfg.L, "d": cfg.d, "window": cfg.window,
         "n_global": int(len(cfg.global_idx)), "n_extra": int(len(cfg.extra_idx)),
-        "global_batch": cfg.B * n_gpus,
-        "parallelism": f"{n_gpus} rank(s), batch x heads sharded, no data-path collective",
+        "global_batch": cfg.B if strong else cfg.B * n_gpus,
+        "parallelism": (f"{n_gpus} rank(s), global batch sharded in contiguous slices (strong), no data-path collective"
+                        if strong else f"{n_gpus} rank(s), one batch per rank (weak), no data-path collective"),
         "l2": "256 MB L2 flush written before every timed step (outside the event pair)",
-        "inputs": "Q,K,V ~ N(0,1) -> bf16 (workloads.make_qkv, seed 0 + 1000*rank)",
+        "inputs": ("Q,K,V ~ N(0,1) -> bf16 (workloads.make_qkv, seed 1000*b per batch element)" if strong
+                   else "Q,K,V ~ N(0,1) -> bf16 (workloads.make_qkv, seed 0 + 1000*rank)"),
     }
 
 
@@ -140,35 +189,44 @@ def nvml_index(local: int) -> int:
 
 
 # ------------------------------------------------------------------ CPU oracle baseline
-def blas_threads():
-    try:
-        from threadpoolctl import threadpool_info
-        n = [i.get("num_threads", 1) for i in threadpool_info() if i.get("user_api") == "blas"]
-        return max(n) if n else 1
-    except Exception:  # noqa: BLE001
-        return 1
+def _oracle_unit(args):
+    """One (b, h) unit of the CPU baseline: the oracle's dense masked attention (O-4, fp64)."""
+    from threadpoolctl import threadpool_limits
+    from oracle import dense_masked_attention
+    from workloads import bits_to_f64
+    q, k, v, window, g, e = args
+    with threadpool_limits(1):   # one core per worker process (the pool provides the parallelism)
+        dense_masked_attention(bits_to_f64(q), bits_to_f64(k), bits_to_f64(v), window, g, e)
+    return 1
 
 
-def cpu_oracle_heads(cfg, budget_s: float):
-    """Time the oracle's dense masked attention (O-4, fp64) head by head until the budget is spent."""
-    from oracle import ExtraIndex, dense_masked_attention, global_flags, head_inputs_f64
+def cpu_oracle_pool(cfg, budget_s: float):
+    """The oracle as it stands (never tuned) over the workload's (b, h) units with a process pool of
+    os.cpu_count() single-threaded workers, until every unit is done or the budget is spent."""
+    import multiprocessing as mp
+    from oracle import ExtraIndex, global_flags
     from oracle.mask import mask_row_cols
     from workloads import make_qkv
     g, ex = global_flags(cfg.L, cfg.global_idx), ExtraIndex(cfg.L, cfg.extra_idx)
     nnz = sum(mask_row_cols(r, cfg.L, cfg.window, g, ex).size for r in range(cfg.L))
-    q, k, v = make_qkv(1, min(cfg.H, 12), cfg.L, cfg.d, seed=cfg.seed)
-    done, t0 = 0, time.perf_counter()
-    while done < q.shape[1]:
-        Q, K, V = head_inputs_f64(q, k, v, 0, done)
-        dense_masked_attention(Q, K, V, cfg.window, cfg.global_idx, cfg.extra_idx)
-        done += 1
-        if time.perf_counter() - t0 > budget_s:
-            break
-    dt = time.perf_counter() - t0
-    return {"value": 4.0 * nnz * cfg.d * done / dt / 1e12, "unit": UNIT, "cores": blas_threads(),
-            "kind": "oracle",
-            "sample": f"oracle.dense_masked_attention (fp64 numpy) on {done} of {cfg.B * cfg.H} (b,h) heads of "
-                      f"{cfg.name}, {dt:.1f} s wall; useful flops counted as for the GPU"}
+    q, k, v = make_qkv(cfg.B, cfg.H, cfg.L, cfg.d, seed=cfg.seed)
+    units = [(q[b, h], k[b, h], v[b, h], cfg.window, cfg.global_idx, cfg.extra_idx)
+             for b in range(cfg.B) for h in range(cfg.H)]
+    cores = os.cpu_count() or 1
+    ctx = mp.get_context("spawn")
+    with ctx.Pool(cores) as pool:
+        pool.map(_oracle_unit, units[:cores])          # warm the workers (imports), untimed
+        done, t0 = 0, time.perf_counter()
+        for _ in pool.imap(_oracle_unit, units, chunksize=1):
+            done += 1
+            if time.perf_counter() - t0 > budget_s and done % cores == 0:
+                break
+        dt = time.perf_counter() - t0
+        pool.terminate()
+    return {"value": 4.0 * nnz * cfg.d * done / dt / 1e12, "unit": UNIT, "cores": cores, "kind": "oracle",
+            "sample": f"oracle.dense_masked_attention (fp64 numpy) on {done} of {len(units)} (b,h) units of "
+                      f"{cfg.name} ({'all' if done == len(units) else 'a bounded sample'}), process pool of "
+                      f"{cores} single-threaded workers, {dt:.1f} s wall; useful flops counted as for the GPU"}
 
 
 def run_reference(args):
@@ -180,7 +238,10 @@ def run_reference(args):
     from oracle import ExtraIndex, attention_rows, global_flags, head_inputs_f64
     from oracle.mask import mask_row_cols
     from workloads import get_config, make_qkv
-    cfg = get_config(args.workload)
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    cfg = get_config(resolve_workload(args, max(world, args.gpus)))
+    strong = cfg.name == "C5"
+    lo, hi = shard_for_rank(cfg, max(world, args.gpus), 0, strong)
     q, k, v = make_qkv(1, 1, cfg.L, cfg.d, seed=cfg.seed)
     Q, K, V = head_inputs_f64(q, k, v, 0, 0)
     g = global_flags(cfg.L, cfg.global_idx)
@@ -207,8 +268,8 @@ def run_reference(args):
     line = {
         "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * tot_t / args.steps,
-        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-        "config": workload_config(cfg, args.gpus),
+        "higher_is_better": True, "scaling": "strong" if strong else "weak", "vs_baseline": None, "dtype": "f64",
+        "data": "synthetic", "config": workload_config(cfg, args.gpus, strong, hi - lo),
         "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle",
                          "sample": f"oracle.attention_rows (fp64) on {R} random rows of one (b,h) head of "
                                    f"{cfg.name} per step"},
@@ -228,7 +289,7 @@ def main():
     import torch.distributed as dist
 
     import paper_conf_iiswc_lica22_b200 as mg
-    from workloads import get_config, make_qkv
+    from workloads import get_config
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -241,18 +302,21 @@ def main():
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     dev = torch.device("cuda", local)
 
-    cfg = get_config(args.workload)
+    cfg = get_config(resolve_workload(args, world))
+    strong = cfg.name == "C5"
+    lo, hi = shard_for_rank(cfg, world, rank, strong)
+    b_local = hi - lo
     t_plan = time.perf_counter()
     plan = mg.Plan(cfg.L, cfg.H, cfg.d, cfg.window, cfg.global_idx, cfg.extra_idx,
                    strip_max_cols=args.strip_max_cols, fine_kernel=args.fine_kernel,
                    concurrency=args.concurrency, tau=args.tau, dense_chunk=args.dense_chunk)
     plan_build_ms = 1e3 * (time.perf_counter() - t_plan)   # host, once per pattern (before inference)
     info = plan.info()
-    BH = cfg.B * cfg.H
-    useful = 4.0 * info["nnz_total"] * cfg.d * BH
+    BH = b_local * cfg.H
+    useful = 4.0 * info["nnz_total"] * cfg.d * BH                      # this rank
+    useful_job = 4.0 * info["nnz_total"] * cfg.d * cfg.H * (cfg.B if strong else cfg.B * world)
 
-    from paper_conf_iiswc_lica22_b200.dist import rank_seed
-    q, k, v = make_qkv(cfg.B, cfg.H, cfg.L, cfg.d, seed=rank_seed(cfg.seed, rank))
+    q, k, v = batch_inputs(cfg, lo, hi, rank, strong)
     host = [torch.from_numpy(x.view(np.int16)).view(torch.bfloat16) for x in (q, k, v)]
     Q, K, V = (h.to(dev) for h in host)
     O = torch.empty_like(Q)
@@ -286,15 +350,16 @@ def main():
     if world > 1:
         dist.barrier()
     sampler.stop()
-    prof = plan.get_profile()
+    prof, per_call = plan.get_profile_calls()
     plan.set_profiling(False)
     assert prof["calls"] == args.steps
-    t_ms = torch.tensor([prof["total_ms"]], dtype=torch.float64, device=dev)
+    t_ms = torch.tensor([prof["total_ms"], float(np.median(per_call)), float(np.min(per_call))],
+                        dtype=torch.float64, device=dev)
     if world > 1:
         dist.all_reduce(t_ms, op=dist.ReduceOp.MAX)
-    total_ms = float(t_ms.item())
+    total_ms, med_ms, min_ms = (float(x) for x in t_ms.tolist())
     ms_per_step = total_ms / args.steps
-    value = world * useful / (ms_per_step * 1e-3) / 1e12
+    value = useful_job / (ms_per_step * 1e-3) / 1e12
 
     # ---------------- warm-L2 figure (no flush between steps; reported beside the flushed value)
     plan.set_profiling(True)
@@ -323,20 +388,19 @@ def main():
     e2e_ms = torch.tensor([e0.elapsed_time(e1) / n_e2e], dtype=torch.float64, device=dev)
     if world > 1:
         dist.all_reduce(e2e_ms, op=dist.ReduceOp.MAX)
-    e2e_value = world * useful / (float(e2e_ms.item()) * 1e-3) / 1e12
+    e2e_value = useful_job / (float(e2e_ms.item()) * 1e-3) / 1e12
     nbytes = Q.numel() * 2
 
     # ---------------- N>1: NCCL all_gather of O, timed separately (not part of the fwd)
     gather_ms = None
     if world > 1:
-        from paper_conf_iiswc_lica22_b200.dist import gather_outputs
-        gather_outputs(O)
+        gather_output(O, cfg.B, strong)
         torch.cuda.synchronize()
         dist.barrier()
         g0, g1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         g0.record(stream)
         for _ in range(5):
-            gather_outputs(O)
+            gather_output(O, cfg.B, strong)
         g1.record(stream)
         torch.cuda.synchronize()
         gt = torch.tensor([g0.elapsed_time(g1) / 5], dtype=torch.float64, device=dev)
@@ -347,6 +411,47 @@ def main():
     peaks, peak_src = load_peaks()
     coarse_avg = prof["coarse_ms"] / max(1, prof["calls"])
     fine_avg = prof["fine_ms"] / max(1, prof["calls"])
+    roof = roofline(cfg, info, BH, coarse_avg, fine_avg, peaks, peak_src, sampler.summary(), dev, args)
+
+    line = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
+        "scaling": "strong" if strong else "weak",
+        "vs_baseline": None, "dtype": "bf16", "data": "synthetic",
+        "config": workload_config(cfg, world, strong, b_local),
+        "fwd_ms": {"mean": ms_per_step, "median": med_ms, "min": min_ms, "steps": args.steps,
+                   "timing": "library CUDA events on the launch stream, first to last kernel of each call; "
+                             "max over ranks"},
+        "useful_gflop_per_gpu": useful / 1e9,
+        "fwd_ms_warm_l2": warm_ms,
+        "plan_build_ms": plan_build_ms,
+        "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": 3 * nbytes, "d2h_bytes_per_step": nbytes,
+                "ms_per_step": float(e2e_ms.item()),
+                "path": "mg_sparse_attention_fwd_host (pinned host Q/K/V/O, copies inside the timed region)"},
+        "gpu_launches": int(args.steps * info["kernels_per_fwd"]),
+        "kernels_per_fwd": info["kernels_per_fwd"],
+        "roofline": roof,
+        "clocks": sampler.summary(),
+        "plan": {k_: info[k_] for k_ in ("n_tiles", "n_full_tiles", "nnz_total", "nnz_fine", "nnz_fine_strip",
+                                          "nnz_fine_cuda", "n_items", "computed_scores")},
+        "paper_context": "Multigrain reports 2.07x (Longformer) / 1.55x (QDS) end-to-end over Triton, FP16, "
+                         "A100/RTX 3090 (PAPER.md P:12); no absolute numbers are published",
+    }
+    if gather_ms is not None:
+        line["allgather_O_ms"] = gather_ms
+    if args.ablation:
+        line["staged_ablation"] = staged_ablation(mg, plan, Q, K, V, O, stream, flush, useful, ms_per_step, args)
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        line["cpu_baseline"] = cpu_oracle_pool(cfg, args.cpu_seconds)
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+def roofline(cfg, info, BH, coarse_avg, fine_avg, peaks, peak_src, clk, dev, args):
+    import torch
     if coarse_avg >= fine_avg:
         coarse_nnz = info["nnz_coarse"] + info["nnz_fine_strip"] + info["n_global"] * cfg.L
         flops = 4.0 * coarse_nnz * cfg.d * BH
@@ -358,7 +463,6 @@ def main():
                 "algorithmic_rule": "4*d flops per valid element it owns (coarse + strip + dense-row)",
                 "peak_source": peak_src + " bf16 burst", "traffic": None}
         # the pipe that actually bounds this kernel: one MUFU ex2 per computed score (K1)
-        clk = sampler.summary()
         mhz = clk.get("sm_mhz") or clk.get("sm_max_mhz")
         if mhz:
             sms = torch.cuda.get_device_properties(dev).multi_processor_count
@@ -382,8 +486,13 @@ def main():
                 "algorithmic_rule": "per nnz: K row + V row (2*d*2 B) + 4 B index; per row: Q read + partial write",
                 "note": "the gathered K/V rows of a head (4 MB) are served by L2, so the algorithmic rate can exceed "
                         "the HBM peak the north_star measures against (frac > 1); `traffic` (ncu DRAM bytes) is "
-                        "what reached HBM; the L2-gather ceiling is ~22 TB/s (tools/microbench/gather_bw.cu)",
+                        "what reached HBM; see `l2` for the fraction of the L2 gather ceiling",
                 "peak_source": peak_src, "traffic": None}
+        # the level that actually serves the gathers: L2 (K2)
+        l2_peak = L2_GATHER_GBS
+        roof["l2"] = {"achieved": achieved, "peak": l2_peak, "unit": "GB/s", "frac": achieved / l2_peak,
+                      "peak_rule": "measured L2->SM gather ceiling, 8 lanes per 128-B row, 16-B loads, no arithmetic "
+                                   "(tools/microbench/gather_bw.cu, B200)"}
     tr_path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(tr_path):
         tr = json.load(open(tr_path)).get(cfg.name, {})
@@ -391,35 +500,20 @@ def main():
         if key in tr:
             roof["traffic"] = tr[key].get("dram_bytes_per_launch")
             roof["traffic_source"] = tr[key].get("source")
+            if "lts_bytes_per_launch" in tr[key]:
+                roof["l2_traffic"] = tr[key]["lts_bytes_per_launch"]
+    return roof
 
-    line = {
-        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
-        "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak",
-        "vs_baseline": None, "dtype": "bf16", "data": "synthetic", "config": workload_config(cfg, world),
-        "fwd_ms": {"mean": ms_per_step, "timing": "library CUDA events on the launch stream, first to last kernel"},
-        "useful_gflop_per_gpu": useful / 1e9,
-        "fwd_ms_warm_l2": warm_ms,
-        "plan_build_ms": plan_build_ms,
-        "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": 3 * nbytes, "d2h_bytes_per_step": nbytes,
-                "ms_per_step": float(e2e_ms.item()),
-                "path": "mg_sparse_attention_fwd_host (pinned host Q/K/V/O, copies inside the timed region)"},
-        "gpu_launches": int(args.steps * info["kernels_per_fwd"]),
-        "kernels_per_fwd": info["kernels_per_fwd"],
-        "roofline": roof,
-        "clocks": sampler.summary(),
-        "plan": {k_: info[k_] for k_ in ("n_tiles", "n_full_tiles", "nnz_total", "nnz_fine", "nnz_fine_strip",
-                                          "nnz_fine_cuda", "n_items", "computed_scores")},
-        "paper_context": "Multigrain reports 2.07x (Longformer) / 1.55x (QDS) end-to-end over Triton, FP16, "
-                         "A100/RTX 3090 (PAPER.md P:12); no absolute numbers are published",
-    }
-    if gather_ms is not None:
-        line["allgather_O_ms"] = gather_ms
-    if args.ablation:
-        # the paper's dataflow (S and P materialised, SDDMM -> 3-sweep SpSoftmax -> SpMM kernels),
-        # same inputs, same L2 flush, CUDA events on the same stream
-        Os = mg.sparse_attention_fwd_staged(plan, Q, K, V, None, stream)
+
+def staged_ablation(mg, plan, Q, K, V, O, stream, flush, useful, ms_per_step, args):
+    """The paper's dataflow (S and P materialised, SDDMM -> 3-sweep SpSoftmax -> SpMM kernels), same
+    inputs, same L2 flush, CUDA events on the same stream; serial and multi-stream."""
+    import torch
+    out = {}
+    for name, ms_kw in (("serial", dict(multi_stream=False)), ("multi_stream", dict(multi_stream=True))):
+        Os = mg.sparse_attention_fwd_staged(plan, Q, K, V, None, stream, **ms_kw)
         for _ in range(3):
-            mg.sparse_attention_fwd_staged(plan, Q, K, V, Os, stream)
+            mg.sparse_attention_fwd_staged(plan, Q, K, V, Os, stream, **ms_kw)
         n_ab = max(3, min(50, args.steps))
         ab = []
         for _ in range(n_ab):
@@ -427,23 +521,16 @@ def main():
                 flush.zero_()
             a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             a0.record(stream)
-            mg.sparse_attention_fwd_staged(plan, Q, K, V, Os, stream)
+            mg.sparse_attention_fwd_staged(plan, Q, K, V, Os, stream, **ms_kw)
             a1.record(stream)
             ab.append((a0, a1))
         torch.cuda.synchronize()
         st_ms = sum(a.elapsed_time(b) for a, b in ab) / n_ab
         diff = (Os.float() - O.float()).abs()
-        line["staged_ablation"] = {"ms_per_step": st_ms, "tflops": useful / (st_ms * 1e-3) / 1e12,
-                                   "fused_speedup": st_ms / ms_per_step, "steps": n_ab,
-                                   "max_abs_vs_fused": float(diff.max()),
-                                   "path": "mg_sparse_attention_fwd_staged (S, P in HBM; 5-7 kernels)"}
-    if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        line["cpu_baseline"] = cpu_oracle_heads(cfg, args.cpu_seconds)
-    if rank == 0:
-        print(json.dumps(line), flush=True)
-    if world > 1:
-        dist.destroy_process_group()
-    return 0
+        out[name] = {"ms_per_step": st_ms, "tflops": useful / (st_ms * 1e-3) / 1e12,
+                     "fused_speedup": st_ms / ms_per_step, "steps": n_ab, "max_abs_vs_fused": float(diff.max())}
+    out["path"] = "mg_sparse_attention_fwd_staged (S, P in HBM; SDDMM / SpSoftmax / SpMM kernels)"
+    return out
 
 
 if __name__ == "__main__":

@@ -258,6 +258,16 @@ MG_API mg_status mg_staged_spmm(mg_plan_t plan, const void* P_tiles, const void*
                                 const mg_tensor* V, mg_tensor* O, float* O_csr, void* stream);
 MG_API mg_status mg_sparse_attention_fwd_staged(mg_plan_t plan, const mg_tensor* Q, const mg_tensor* K,
                                                 const mg_tensor* V, mg_tensor* O, void* stream);
+/* mg_sparse_attention_fwd_staged_ex: as mg_sparse_attention_fwd_staged; flags bit 0
+ * (MG_STAGED_MULTI_STREAM) runs the coarse and fine kernels of each step concurrently on a
+ * plan-owned second stream forked from and joined back into `stream` (the paper's multi-stream
+ * execution, P:96 step 3): SDDMM of the BSR tiles and dense rows || SDDMM of the CSR
+ * residual; the compound SpSoftmax (which needs both parts' statistics) after the join; SpMM of
+ * the dense-row chunks || SpMM of the CSR residual, then the BSR row blocks (which add O_csr).
+ * Same results bit for bit as the single-stream call. INVALID_ARG for unknown flag bits. */
+#define MG_STAGED_MULTI_STREAM 1
+MG_API mg_status mg_sparse_attention_fwd_staged_ex(mg_plan_t plan, const mg_tensor* Q, const mg_tensor* K,
+                                                   const mg_tensor* V, mg_tensor* O, int32_t flags, void* stream);
 
 /* ------------------------------------------------------------------------------------
  * Profiling (tracing subsystem). When enabled, every forward records CUDA events on its
@@ -273,6 +283,11 @@ typedef struct {
 
 MG_API mg_status mg_plan_set_profiling(mg_plan_t plan, int32_t enable);
 MG_API mg_status mg_plan_get_profile(mg_plan_t plan, mg_profile* out);
+/* mg_plan_get_profile_calls: as mg_plan_get_profile, and also writes the first-to-last-launch
+ * duration of each recorded call, in call order, to per_call_ms[0 .. min(calls, cap)) (host
+ * buffer owned by the caller; may be null when cap == 0), so that a caller can report the median
+ * and minimum of a timed run. INVALID_ARG: null plan/out, cap < 0, or cap > 0 with a null buffer. */
+MG_API mg_status mg_plan_get_profile_calls(mg_plan_t plan, mg_profile* out, double* per_call_ms, int64_t cap);
 
 /* ------------------------------------------------------------------------------------
  * Diagnostics (used by the GPU tests; not part of the attention path).

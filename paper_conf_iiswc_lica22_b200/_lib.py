@@ -17,8 +17,8 @@ STATUS_NAMES = {0: "OK", 1: "INVALID_ARG", 2: "UNSUPPORTED", 3: "OUT_OF_MEMORY",
 EXPORTED = [
     "mg_plan_create", "mg_plan_create_ex", "mg_plan_create_batched", "mg_plan_destroy", "mg_last_error", "mg_plan_info_get",
     "mg_plan_export", "mg_sparse_attention_fwd", "mg_sparse_attention_fwd_host", "mg_selftest_umma",
-    "mg_abi_version", "mg_plan_set_profiling", "mg_plan_get_profile", "mg_plan_set_trace",
-    "mg_sparse_attention_fwd_padded", "mg_staged_get_sizes", "mg_staged_sddmm", "mg_staged_softmax", "mg_staged_spmm", "mg_sparse_attention_fwd_staged",
+    "mg_abi_version", "mg_plan_set_profiling", "mg_plan_get_profile", "mg_plan_get_profile_calls", "mg_plan_set_trace",
+    "mg_sparse_attention_fwd_padded", "mg_staged_get_sizes", "mg_staged_sddmm", "mg_staged_softmax", "mg_staged_spmm", "mg_sparse_attention_fwd_staged", "mg_sparse_attention_fwd_staged_ex",
 ]
 
 
@@ -86,12 +86,14 @@ def load() -> C.CDLL:
     lib.mg_selftest_umma.argtypes = [C.c_int32, P, P, P, P]
     lib.mg_plan_set_profiling.argtypes = [P, C.c_int32]
     lib.mg_plan_get_profile.argtypes = [P, C.POINTER(mg_profile)]
+    lib.mg_plan_get_profile_calls.argtypes = [P, C.POINTER(mg_profile), C.POINTER(C.c_double), C.c_int64]
     lib.mg_plan_set_trace.argtypes = [P, P, C.c_int64]
     lib.mg_staged_get_sizes.argtypes = [P, C.POINTER(mg_staged_sizes)]
     lib.mg_staged_sddmm.argtypes = [P, tp, tp, P, P, P, P]
     lib.mg_staged_softmax.argtypes = [P, C.c_int64, C.c_int32, P, P, P, P, P, P, P]
     lib.mg_staged_spmm.argtypes = [P, P, P, P, tp, tp, P, P]
     lib.mg_sparse_attention_fwd_staged.argtypes = [P, tp, tp, tp, tp, P]
+    lib.mg_sparse_attention_fwd_staged_ex.argtypes = [P, tp, tp, tp, tp, C.c_int32, P]
     lib.mg_abi_version.restype = C.c_int32
     lib.mg_abi_version.argtypes = []
     for name in EXPORTED:

@@ -84,6 +84,15 @@ class Plan:
         check(self._lib.mg_plan_get_profile(self._handle, C.byref(pr)))
         return {"calls": pr.calls, "fine_ms": pr.fine_ms, "coarse_ms": pr.coarse_ms, "total_ms": pr.total_ms}
 
+    def get_profile_calls(self) -> tuple[dict, list]:
+        """mg_plan_get_profile_calls: as get_profile, plus each call's first-to-last-launch ms."""
+        pr = mg_profile()
+        cap = 1 << 16
+        buf = (C.c_double * cap)()
+        check(self._lib.mg_plan_get_profile_calls(self._handle, C.byref(pr), buf, cap))
+        per = [buf[i] for i in range(min(pr.calls, cap))]
+        return {"calls": pr.calls, "fine_ms": pr.fine_ms, "coarse_ms": pr.coarse_ms, "total_ms": pr.total_ms}, per
+
     def set_trace(self, buf=None) -> None:
         """mg_plan_set_trace: zeroed device int64 tensor of >= 128 elements (MG_TRACE builds add their
         per-role phase counters to it, see tools/trace_coarse.py) or None to stop."""
@@ -242,14 +251,15 @@ def staged_spmm(plan: Plan, V, O, bufs: dict, stream=None):
     return O
 
 
-def sparse_attention_fwd_staged(plan: Plan, Q, K, V, O=None, stream=None):
-    """mg_sparse_attention_fwd_staged: the paper's dataflow (SDDMM -> SpSoftmax -> SpMM kernels)."""
+def sparse_attention_fwd_staged(plan: Plan, Q, K, V, O=None, stream=None, multi_stream: bool = False):
+    """mg_sparse_attention_fwd_staged(_ex): the paper's dataflow (SDDMM -> SpSoftmax -> SpMM kernels);
+    multi_stream=True runs each step's coarse and fine kernels on two streams."""
     import torch
     if O is None:
         O = torch.empty(Q.shape, dtype=Q.dtype, device=Q.device)
     dq, dk, dv, do = tensor_desc(Q), tensor_desc(K), tensor_desc(V), tensor_desc(O)
-    check(plan._lib.mg_sparse_attention_fwd_staged(plan.handle, C.byref(dq), C.byref(dk), C.byref(dv),
-                                                   C.byref(do), _stream_ptr(stream)))
+    check(plan._lib.mg_sparse_attention_fwd_staged_ex(plan.handle, C.byref(dq), C.byref(dk), C.byref(dv),
+                                                      C.byref(do), 1 if multi_stream else 0, _stream_ptr(stream)))
     return O
 
 

@@ -91,6 +91,8 @@ struct mg_plan_s {
   uint64_t* d_tile_masks = nullptr;
   uint8_t* d_row_is_global = nullptr;
   uint8_t* d_staged_ws = nullptr;   // S, P and O_csr buffers of mg_sparse_attention_fwd_staged
+  cudaStream_t staged_side = nullptr;   // second stream of the multi-stream staged forward
+  cudaEvent_t staged_ev = nullptr;
   size_t staged_ws_cap = 0;
   // TMA descriptors of the last forward's Q/K/V/O (re-encoded only when a tensor descriptor changes:
   // cuTensorMapEncodeTiled is host work on every call otherwise)
@@ -137,6 +139,8 @@ struct mg_plan_s {
     if (d_stage) cudaFree(d_stage);
     if (d_dense) cudaFree(d_dense);
     if (d_staged_ws) cudaFree(d_staged_ws);
+    if (staged_side) cudaStreamDestroy(staged_side);
+    if (staged_ev) cudaEventDestroy(staged_ev);
   }
 };
 
@@ -646,14 +650,14 @@ mg_status staged_buffers_ok(const mg_plan_s* p, const void* tiles, const void* c
 }
 
 mg_status staged_sddmm_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, float* St, float* Sf, float* Sg,
-                            cudaStream_t stream) {
+                            cudaStream_t stream, cudaStream_t side) {
   mg::StagedParams sp = staged_params(p, Q->batch);
   sp.q = view(Q);
   sp.k = view(K);
   sp.S_t = St;
   sp.S_f = Sf;
   sp.S_g = Sg;
-  cudaError_t e = mg::launch_staged_sddmm(sp, Q->dtype == MG_BF16, stream);
+  cudaError_t e = mg::launch_staged_sddmm(sp, Q->dtype == MG_BF16, stream, side);
   return e == cudaSuccess ? MG_OK : cuda_fail(e, "staged SDDMM launch");
 }
 
@@ -671,7 +675,7 @@ mg_status staged_softmax_impl(mg_plan_s* p, int64_t batch, mg_dtype dt, const fl
 }
 
 mg_status staged_spmm_impl(mg_plan_s* p, const void* Pt, const void* Pf, const void* Pg, const mg_tensor* V,
-                           mg_tensor* O, float* Of, cudaStream_t stream) {
+                           mg_tensor* O, float* Of, cudaStream_t stream, cudaStream_t side = nullptr) {
   mg::StagedParams sp = staged_params(p, V->batch);
   sp.v = view(V);
   sp.o = view(O);
@@ -679,7 +683,7 @@ mg_status staged_spmm_impl(mg_plan_s* p, const void* Pt, const void* Pf, const v
   sp.P_f = static_cast<uint16_t*>(const_cast<void*>(Pf));
   sp.P_g = static_cast<uint16_t*>(const_cast<void*>(Pg));
   sp.O_f = Of;
-  cudaError_t e = mg::launch_staged_spmm(sp, V->dtype == MG_BF16, stream);
+  cudaError_t e = mg::launch_staged_spmm(sp, V->dtype == MG_BF16, stream, side ? side : stream, p->staged_ev);
   return e == cudaSuccess ? MG_OK : cuda_fail(e, "staged SpMM launch");
 }
 
@@ -886,7 +890,8 @@ mg_status mg_staged_sddmm(mg_plan_t plan, const mg_tensor* Q, const mg_tensor* K
   if ((s = staged_check(plan, Q, "Q")) != MG_OK || (s = staged_check(plan, K, "K")) != MG_OK) return s;
   if (K->batch != Q->batch || K->dtype != Q->dtype) return fail(MG_ERR_INVALID_ARG, "Q/K batch or dtype differ");
   if ((s = staged_buffers_ok(plan, S_tiles, S_csr, S_global)) != MG_OK) return s;
-  return staged_sddmm_impl(plan, Q, K, S_tiles, S_csr, S_global, static_cast<cudaStream_t>(stream));
+  return staged_sddmm_impl(plan, Q, K, S_tiles, S_csr, S_global, static_cast<cudaStream_t>(stream),
+                           static_cast<cudaStream_t>(stream));
 }
 
 mg_status mg_staged_softmax(mg_plan_t plan, int64_t batch, mg_dtype dtype, const float* S_tiles, const float* S_csr,
@@ -918,9 +923,10 @@ mg_status mg_staged_spmm(mg_plan_t plan, const void* P_tiles, const void* P_csr,
   return staged_spmm_impl(plan, P_tiles, P_csr, P_global, V, O, O_csr, static_cast<cudaStream_t>(stream));
 }
 
-mg_status mg_sparse_attention_fwd_staged(mg_plan_t plan, const mg_tensor* Q, const mg_tensor* K, const mg_tensor* V,
-                                         mg_tensor* O, void* stream_) {
+mg_status mg_sparse_attention_fwd_staged_ex(mg_plan_t plan, const mg_tensor* Q, const mg_tensor* K, const mg_tensor* V,
+                                            mg_tensor* O, int32_t flags, void* stream_) {
   g_err.clear();
+  if (flags & ~MG_STAGED_MULTI_STREAM) return fail(MG_ERR_INVALID_ARG, "unknown staged flags");
   if (!plan) return fail(MG_ERR_INVALID_ARG, "plan is null");
   mg_status s = check_all(plan, Q, K, V, O, false);
   if (s != MG_OK) return s;
@@ -952,9 +958,34 @@ mg_status mg_sparse_attention_fwd_staged(mg_plan_t plan, const mg_tensor* Q, con
   void* Pf = w + bt + bf + bg + pt;
   void* Pg = w + bt + bf + bg + pt + pf;
   float* Of = reinterpret_cast<float*>(w + bt + bf + bg + pt + pf + pg);
-  if ((s = staged_sddmm_impl(plan, Q, K, St, Sf, Sg, stream)) != MG_OK) return s;
+  cudaStream_t side = stream;
+  const bool multi = (flags & MG_STAGED_MULTI_STREAM) && !plan->hp.csr_col.empty();
+  if (multi) {
+    if (!plan->staged_side) {
+      if ((e = cudaStreamCreateWithFlags(&plan->staged_side, cudaStreamNonBlocking)) != cudaSuccess)
+        return cuda_fail(e, "stream creation");
+    }
+    side = plan->staged_side;
+  }
+  if (!plan->staged_ev && (e = cudaEventCreateWithFlags(&plan->staged_ev, cudaEventDisableTiming)) != cudaSuccess)
+    return cuda_fail(e, "event creation");
+  // fork: the side stream starts after everything before this call on `stream`
+  auto sync_into = [&](cudaStream_t from, cudaStream_t to) {
+    cudaError_t r = cudaEventRecord(plan->staged_ev, from);
+    return r == cudaSuccess ? cudaStreamWaitEvent(to, plan->staged_ev, 0) : r;
+  };
+  if (multi && (e = sync_into(stream, side)) != cudaSuccess) return cuda_fail(e, "stream fork");
+  if ((s = staged_sddmm_impl(plan, Q, K, St, Sf, Sg, stream, side)) != MG_OK) return s;
+  if (multi && (e = sync_into(side, stream)) != cudaSuccess) return cuda_fail(e, "stream join");
   if ((s = staged_softmax_impl(plan, Q->batch, (mg_dtype)Q->dtype, St, Sf, Sg, Pt, Pf, Pg, stream)) != MG_OK) return s;
-  return staged_spmm_impl(plan, Pt, Pf, Pg, V, O, Of, stream);
+  if (multi && (e = sync_into(stream, side)) != cudaSuccess) return cuda_fail(e, "stream fork");
+  // (launch_staged_spmm joins the side stream back before the row blocks that read O_csr)
+  return staged_spmm_impl(plan, Pt, Pf, Pg, V, O, Of, stream, side);
+}
+
+mg_status mg_sparse_attention_fwd_staged(mg_plan_t plan, const mg_tensor* Q, const mg_tensor* K, const mg_tensor* V,
+                                         mg_tensor* O, void* stream) {
+  return mg_sparse_attention_fwd_staged_ex(plan, Q, K, V, O, 0, stream);
 }
 
 mg_status mg_plan_set_profiling(mg_plan_t plan, int32_t enable) {
@@ -966,26 +997,35 @@ mg_status mg_plan_set_profiling(mg_plan_t plan, int32_t enable) {
   return MG_OK;
 }
 
-mg_status mg_plan_get_profile(mg_plan_t plan, mg_profile* out) {
+mg_status mg_plan_get_profile_calls(mg_plan_t plan, mg_profile* out, double* per_call_ms, int64_t cap) {
   g_err.clear();
   if (!plan || !out) return fail(MG_ERR_INVALID_ARG, "null argument");
+  if (cap < 0 || (cap > 0 && !per_call_ms)) return fail(MG_ERR_INVALID_ARG, "bad per-call buffer");
   std::memset(out, 0, sizeof(*out));
   auto ms = [&](int32_t a, int32_t b) {
     float t = 0.f;
     if (a >= 0 && b >= 0) cudaEventElapsedTime(&t, plan->prof_events[a], plan->prof_events[b]);
     return (double)t;
   };
+  int64_t i = 0;
   for (const auto& c : plan->prof_calls) {
     cudaError_t e = cudaEventSynchronize(plan->prof_events[c.last]);
     if (e != cudaSuccess) return cuda_fail(e, "cudaEventSynchronize");
     out->fine_ms += ms(c.fb, c.fe);
     out->coarse_ms += ms(c.cb, c.ce);
-    out->total_ms += ms(c.first, c.last);
+    const double tot = ms(c.first, c.last);
+    out->total_ms += tot;
+    if (i < cap) per_call_ms[i] = tot;
+    ++i;
   }
   out->calls = (int64_t)plan->prof_calls.size();
   plan->prof_used = 0;
   plan->prof_calls.clear();
   return MG_OK;
+}
+
+mg_status mg_plan_get_profile(mg_plan_t plan, mg_profile* out) {
+  return mg_plan_get_profile_calls(plan, out, nullptr, 0);
 }
 
 mg_status mg_plan_set_trace(mg_plan_t plan, void* device_buffer, int64_t capacity_events) {

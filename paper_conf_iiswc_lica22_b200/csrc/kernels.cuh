@@ -98,13 +98,18 @@ struct StagedParams {
   uint16_t* P_g;
   float* O_f;
   int64_t L, nnz_csr, Lpad;
+  int32_t blk0;                 // staged_spmm_tiles: first block index of this launch (split launches)
   int32_t H, BH, nb, n_tiles, n_global;
   float sf;                     // 1 / sqrt(d)
 };
 
-cudaError_t launch_staged_sddmm(const StagedParams& p, bool bf16, cudaStream_t stream);
+// `side`: stream of the CSR kernels (== stream: single-stream order). With a separate side stream
+// the caller forks it from `stream` before and joins it after; launch_staged_spmm makes `stream`
+// wait for the CSR SpMM (event `ev`) before the BSR row blocks that add O_csr.
+cudaError_t launch_staged_sddmm(const StagedParams& p, bool bf16, cudaStream_t stream, cudaStream_t side);
 cudaError_t launch_staged_softmax(const StagedParams& p, bool bf16, cudaStream_t stream);
-cudaError_t launch_staged_spmm(const StagedParams& p, bool bf16, cudaStream_t stream);
+cudaError_t launch_staged_spmm(const StagedParams& p, bool bf16, cudaStream_t stream, cudaStream_t side,
+                               cudaEvent_t ev);
 
 // Paired-pipeline variant: two CTAs per SM (grid = 2 x SMs), see coarse_pp_sm100.cu.
 cudaError_t launch_coarse_pp(const CoarseParams& p, const CUtensorMap& tmq, const CUtensorMap& tmk,

@@ -346,7 +346,7 @@ __global__ void __launch_bounds__(256) staged_spmm_tiles(const StagedParams p) {
   __shared__ __align__(128) uint8_t sm[kT * 256 + kT * 128];
   const uint32_t sP = smem_u32(sm), sV = sP + kT * 256;
   const int bh = blockIdx.y, bb = bh / p.H, hh = bh % p.H;
-  const int x = blockIdx.x;
+  const int x = blockIdx.x + p.blk0;
   const bool dense = x >= p.nb;
   const int gchunk = dense ? x - p.nb : -1;
   const int nrows = dense ? min(kT, p.n_global - gchunk * kT) : kT;
@@ -418,18 +418,18 @@ __global__ void __launch_bounds__(256) staged_spmm_tiles(const StagedParams p) {
   }
 }
 
-cudaError_t launch_staged_sddmm(const StagedParams& p, bool bf16, cudaStream_t stream) {
+cudaError_t launch_staged_sddmm(const StagedParams& p, bool bf16, cudaStream_t stream, cudaStream_t side) {
   const int gtiles = ((p.n_global + kT - 1) / kT) * p.nb;
-  if (p.n_tiles + gtiles > 0) {
+  if (p.nnz_csr > 0) {   // fine part (side stream when concurrent)
+    const int64_t warps = (int64_t)p.BH * p.L;
+    staged_sddmm_csr<<<(unsigned)((warps + 7) / 8), 256, 0, side>>>(p, bf16);
+  }
+  if (p.n_tiles + gtiles > 0) {   // coarse tiles and dense-row tiles
     dim3 grid(p.n_tiles + gtiles, p.BH);
     if (bf16)
       staged_sddmm_tiles<true><<<grid, 256, 0, stream>>>(p);
     else
       staged_sddmm_tiles<false><<<grid, 256, 0, stream>>>(p);
-  }
-  if (p.nnz_csr > 0) {
-    const int64_t warps = (int64_t)p.BH * p.L;
-    staged_sddmm_csr<<<(unsigned)((warps + 7) / 8), 256, 0, stream>>>(p, bf16);
   }
   return cudaGetLastError();
 }
@@ -444,17 +444,33 @@ cudaError_t launch_staged_softmax(const StagedParams& p, bool bf16, cudaStream_t
   return cudaGetLastError();
 }
 
-cudaError_t launch_staged_spmm(const StagedParams& p, bool bf16, cudaStream_t stream) {
+cudaError_t launch_staged_spmm(const StagedParams& p, bool bf16, cudaStream_t stream, cudaStream_t side,
+                               cudaEvent_t ev) {
+  auto tiles = [&](int blk0, int nblk) {
+    if (nblk <= 0) return;
+    StagedParams q = p;
+    q.blk0 = blk0;
+    dim3 grid(nblk, p.BH);
+    if (bf16)
+      staged_spmm_tiles<true><<<grid, 256, 0, stream>>>(q);
+    else
+      staged_spmm_tiles<false><<<grid, 256, 0, stream>>>(q);
+  };
+  const int gchunks = (p.n_global + kT - 1) / kT;
   if (p.nnz_csr > 0) {
     const int64_t warps = (int64_t)p.BH * p.L;
-    staged_spmm_csr<<<(unsigned)((warps + 7) / 8), 256, 0, stream>>>(p, bf16);
+    staged_spmm_csr<<<(unsigned)((warps + 7) / 8), 256, 0, side>>>(p, bf16);
   }
-  const int blocks = p.nb + (p.n_global + kT - 1) / kT;
-  dim3 grid(blocks, p.BH);
-  if (bf16)
-    staged_spmm_tiles<true><<<grid, 256, 0, stream>>>(p);
-  else
-    staged_spmm_tiles<false><<<grid, 256, 0, stream>>>(p);
+  if (side != stream && p.nnz_csr > 0) {
+    // dense-row chunks need no O_csr: they run beside the CSR SpMM; the row blocks wait for it
+    tiles(p.nb, gchunks);
+    cudaError_t e = cudaEventRecord(ev, side);
+    if (e == cudaSuccess) e = cudaStreamWaitEvent(stream, ev, 0);
+    if (e != cudaSuccess) return e;
+    tiles(0, p.nb);
+  } else {
+    tiles(0, p.nb + gchunks);
+  }
   return cudaGetLastError();
 }
 

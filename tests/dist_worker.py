@@ -1,8 +1,9 @@
 """Worker for tests/test_dist_gloo.py, launched with torch.distributed.run (2 ranks, gloo, CPU).
 
-Per rank: shard the batch (strong scaling) or draw its own seeded batch (weak scaling), run the
-fp64 oracle as the stand-in forward, gather with the bench's gather helpers; rank 0 saves the
-gathered arrays to argv[1].
+Drives bench.py's own multi-GPU host logic (shard_for_rank, batch_inputs, gather_output) with the
+fp64 oracle as the stand-in forward: strong scaling (a global batch sharded in contiguous slices,
+as for C5) and weak scaling (each rank its own seeded batch). Rank 0 saves the gathered arrays to
+argv[1].
 """
 import os
 import sys
@@ -14,11 +15,13 @@ import numpy as np  # noqa: E402
 import torch  # noqa: E402
 import torch.distributed as dist  # noqa: E402
 
+import bench  # noqa: E402
 from oracle import dense_masked_attention, head_inputs_f64  # noqa: E402
-from paper_conf_iiswc_lica22_b200.dist import gather_batches, gather_outputs, rank_seed, shard_range  # noqa: E402
-from workloads import make_qkv  # noqa: E402
+from workloads import Config  # noqa: E402
 
-L, H, D, WINDOW, G = 64, 2, 64, 8, [0, 5]
+L, H, D, WINDOW = 64, 2, 64, 8
+G = np.array([0, 5], np.int32)
+CFG = Config("T5", 5, H, L, D, WINDOW, G, np.zeros((0, 2), np.int32), 3, "tiny strong-scaling batch")
 
 
 def oracle_fwd(q, k, v):
@@ -33,14 +36,15 @@ def oracle_fwd(q, k, v):
 def main():
     dist.init_process_group("gloo")
     rank, world = dist.get_rank(), dist.get_world_size()
-    Bg = 5
-    q, k, v = make_qkv(Bg, H, L, D, seed=3)
-    lo, hi = shard_range(Bg, world, rank)
-    full = gather_batches(torch.from_numpy(oracle_fwd(q[lo:hi], k[lo:hi], v[lo:hi])), Bg)
-    qw, kw, vw = make_qkv(2, H, L, D, seed=rank_seed(0, rank))
-    allw = gather_outputs(torch.from_numpy(oracle_fwd(qw, kw, vw)))
+    lo, hi = bench.shard_for_rank(CFG, world, rank, strong=True)
+    q, k, v = bench.batch_inputs(CFG, lo, hi, rank, strong=True)
+    full = bench.gather_output(torch.from_numpy(oracle_fwd(q, k, v)), CFG.B, strong=True)
+    lo, hi = bench.shard_for_rank(CFG, world, rank, strong=False)
+    qw, kw, vw = bench.batch_inputs(CFG, lo, hi, rank, strong=False)
+    allw = bench.gather_output(torch.from_numpy(oracle_fwd(qw, kw, vw)), CFG.B, strong=False)
     if rank == 0:
-        np.savez(sys.argv[1], full=full.numpy(), weak=allw.numpy())
+        np.savez(sys.argv[1], full=full.numpy(), weak=allw.numpy(), spans=np.array(
+            [bench.shard_for_rank(CFG, world, r, strong=True) for r in range(world)]))
     dist.barrier()
     dist.destroy_process_group()
 

@@ -33,12 +33,13 @@ def _free_port():
 
 
 def test_gloo_world2_shard_and_gather(tmp_path):
-    """torch.distributed.run --nproc-per-node 2 (gloo): sharded oracle forward + gather equals the
-    single-process result over the global batch; weak-scaling ranks draw distinct seeded batches."""
+    """torch.distributed.run --nproc-per-node 2 (gloo) over bench.py's own shard / input / gather
+    functions: the sharded oracle forward + gather equals the single-process result over the global
+    batch element for element (strong scaling, C5's scheme); weak-scaling ranks draw distinct batches."""
     import subprocess
     import sys
-    from workloads import make_qkv
     sys.path.insert(0, os.path.dirname(__file__))
+    import bench
     import dist_worker as dw
     out = tmp_path / "gathered.npz"
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
@@ -47,8 +48,30 @@ def test_gloo_world2_shard_and_gather(tmp_path):
     r = subprocess.run(cmd, capture_output=True, text=True, timeout=600)
     assert r.returncode == 0, r.stderr[-2000:]
     res = np.load(out)
-    q, k, v = make_qkv(5, dw.H, dw.L, dw.D, seed=3)
+    assert res["spans"].tolist() == [[0, 3], [3, 5]]
+    q, k, v = bench.batch_inputs(dw.CFG, 0, dw.CFG.B, 0, strong=True)
     assert np.array_equal(res["full"], dw.oracle_fwd(q, k, v))
     for rank in range(2):
-        qw, kw, vw = make_qkv(2, dw.H, dw.L, dw.D, seed=rank_seed(0, rank))
+        qw, kw, vw = bench.batch_inputs(dw.CFG, 0, dw.CFG.B, rank, strong=False)
         assert np.array_equal(res["weak"][rank], dw.oracle_fwd(qw, kw, vw))
+    assert not np.array_equal(res["weak"][0], res["weak"][1])
+
+
+def test_bench_torchrun_world2_c5_line():
+    """torchrun --nproc-per-node 2 bench.py --gpus 2 (the driver's N>1 launch) defaults to C5, the
+    global batch of 64 sharded over the ranks: its reference arm runs on CPU (rank 0 prints one
+    line, rank 1 exits 0) and carries scaling "strong" and the sharded config."""
+    import json
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
+           "--master-addr=127.0.0.1", f"--master-port={_free_port()}", os.path.join(root, "bench.py"),
+           "--gpus", "2", "--impl", "reference", "--steps", "3", "--warmup", "3"]
+    r = subprocess.run(cmd, capture_output=True, text=True, timeout=600, cwd=root)
+    assert r.returncode == 0, r.stderr[-2000:]
+    lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1
+    d = json.loads(lines[0])
+    assert d["scaling"] == "strong" and d["config"]["global_batch"] == 64 and d["config"]["B_per_gpu"] == 32
+    assert d["config"]["workload"].startswith("C5")

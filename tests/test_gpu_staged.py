@@ -119,3 +119,26 @@ def test_staged_rejects_null_buffers():
     bufs["S_tiles"] = None
     with pytest.raises(mg.MGError):
         mg.staged_sddmm(plan, Q, Q, bufs)
+
+
+@pytest.mark.parametrize("kw", [dict(strip_max_cols=-1), {}, dict(force_all_fine=True)])
+def test_staged_multi_stream_bit_identical(kw):
+    """MG_STAGED_MULTI_STREAM (coarse || fine kernels of each step on two streams):
+    bit-identical to the single-stream staged forward and within the bar of the oracle; repeated
+    calls reuse the plan's side stream and event."""
+    L, H, B, w = 1024, 2, 2, 128
+    G = np.array([0, 3, 600], np.int32)
+    E = random_residual(L, w, 5, seed=8)
+    q, k, v = make_qkv(B, H, L, 64, seed=19, dist="adversarial", global_idx=G)
+    plan = mg.Plan(L, H, 64, w, G, E, **kw)
+    Q, K, V = (to_device(x) for x in (q, k, v))
+    one = from_device(mg.sparse_attention_fwd_staged(plan, Q, K, V))
+    for _ in range(3):
+        two = from_device(mg.sparse_attention_fwd_staged(plan, Q, K, V, multi_stream=True))
+        assert np.array_equal(one, two)
+    for b in range(B):
+        for h in range(H):
+            Qh, Kh, Vh = head_inputs_f64(q, k, v, b, h)
+            ref = dense_masked_attention(Qh, Kh, Vh, w, G, E)
+            mx, mean = err_stats(two[b, h], ref)
+            assert mx <= TOL_MAX * max(1.0, np.abs(ref).max() / 4) and mean <= TOL_MEAN, (b, h, mx, mean)
