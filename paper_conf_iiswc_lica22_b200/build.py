@@ -31,7 +31,10 @@ VARIANTS = {"base": [],   # (a plain build under another name: A/B against a sta
             "fw8": ["-DMG_FINE_WARPS=8", "-DMG_FINE_MINB=3"], "fw2": ["-DMG_FINE_WARPS=2", "-DMG_FINE_MINB=10"],
             "fw1": ["-DMG_FINE_WARPS=1", "-DMG_FINE_MINB=20"],
             # skeleton cost: no exponentials / no MMAs / no loads (results are garbage)
-            "dbg1": ["-DMG_DBG=1"], "dbg3": ["-DMG_DBG=3"], "dbg7": ["-DMG_DBG=7"]}
+            "dbg1": ["-DMG_DBG=1"], "dbg2": ["-DMG_DBG=2"], "dbg3": ["-DMG_DBG=3"], "dbg7": ["-DMG_DBG=7"],
+            "dbg8": ["-DMG_DBG=8"], "dbg16": ["-DMG_DBG=16"], "dbg24": ["-DMG_DBG=24"], "dbg25": ["-DMG_DBG=25"],
+            "dbg31": ["-DMG_DBG=31"], "tl7": ["-DMG_TIMELINE", "-DMG_DBG=7"], "tl1": ["-DMG_TIMELINE", "-DMG_DBG=1"],
+            "iq1": ["-DMG_IDLE_QUARTERS=1"]}
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 
 SOURCES = ["plan.cpp", "api.cu", "coarse_pp_sm100.cu", "fine_rows.cu", "fine_mma.cu", "staged.cu", "selftest_umma.cu"]

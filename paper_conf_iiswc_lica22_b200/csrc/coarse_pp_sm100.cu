@@ -227,7 +227,9 @@ __device__ __forceinline__ void chunk_exp(const uint32_t (&r)[32], float2 c2, fl
   for (int i = 0; i < 32; i += 2) {
     const float2 x = __ffma2_rn(make_float2(__uint_as_float(r[i]), __uint_as_float(r[i + 1])), c2, nb2);
     float2 pp;
-    if ((i >> 1) < kExpEmu) {
+    if (kDbgNoExp) {
+      pp = x;
+    } else if ((i >> 1) < kExpEmu) {
       pp = exp2_fma2(x);
     } else {
       pp.x = ex2(x.x);
@@ -286,6 +288,13 @@ __device__ __forceinline__ void tl_item(const CoarseParams& p, uint32_t it, int 
                                              field] = (uint32_t)clock64();
 #endif
 }
+
+// lane quarters without valid rows skip the softmax: measured slower (C2 0.1525 vs 0.1428 ms, C3
+// 0.0819 vs 0.0779, same box, r02), so off by default (MG_IDLE_QUARTERS=1 builds it)
+#ifndef MG_IDLE_QUARTERS
+#define MG_IDLE_QUARTERS 0
+#endif
+constexpr bool kIdleQuarters = MG_IDLE_QUARTERS;
 
 #ifndef MG_PRE_CHUNKS
 #define MG_PRE_CHUNKS 4
@@ -716,7 +725,22 @@ __global__ void __launch_bounds__(kThreads, 2)
           slot_f = __ldg(p.fine_slot + (kBatched ? (int64_t)item.useB * p.L : 0) + item.rowA + t);
       }
       float m = -INFINITY, l = 0.f;
+      // a lane quarter without a valid row (a gathered global-row item with <= 96 rows, e.g. C2's 32
+      // global rows) does no softmax work: its S is not read and its P rows are left as they are
+      // (P.V computes garbage O rows that are never stored, and the next item's first P.V
+      // overwrites O). It still takes part in the per-tile barriers, in order (s_free(n), then
+      // p_full(n) only after P.V(n-1): a p_full arrival may not run ahead into the next phase).
+      const bool idle = kIdleQuarters && warp * 32 >= item.nrowsA;
       for (int j = 0; j < item.ntiles; ++j, ++n) {
+        if (idle) {
+          mbar_wait(bar(ctl->s_full), n & 1);
+          __syncwarp();
+          if (lane == 0) mbar_arrive(bar(ctl->s_free));
+          if (n > 0) mbar_wait(bar(ctl->pv_done), (n - 1) & 1);
+          __syncwarp();
+          if (lane == 0) mbar_arrive(bar(ctl->p_full));
+          continue;
+        }
         const uint32_t st = n % kSt;
         mbar_wait(bar(ctl->s_full), n & 1);
         // the tile's descriptor and bitmask travel with its V stage (freed only after P.V(n))
