@@ -46,7 +46,7 @@ def parse():
     ap.add_argument("--steps", type=int, default=1000)
     ap.add_argument("--warmup", type=int, default=20)
     ap.add_argument("--workload", default=None,
-                    choices=["C1", "C2", "C3", "C4", "C5", "QDS-LS", "F9-LS", "F9-LSG", "F9-LBR", "F9-RBR"],
+                    choices=["C1", "C2", "C3", "C4", "C5", "QDS-LS", "F9-LS", "F9-LSG", "F9-LBR", "F9-RBR", "DIL-LD"],
                     help="default: C2 at N=1, C5 (strong scaling, global batch 64) at N>1")
     ap.add_argument("--impl", default="mine", choices=["mine", "reference"])
     ap.add_argument("--e2e-steps", type=int, default=30)
@@ -59,6 +59,7 @@ def parse():
     ap.add_argument("--concurrency", type=int, default=0, choices=[0, 1, 2],
                     help="coarse vs CSR kernels: 0 = library default, 1 = serial, 2 = concurrent streams")
     ap.add_argument("--tau", type=float, default=0.0, help="tile density threshold (0 = band rule)")
+    ap.add_argument("--block", type=int, default=0, choices=[0, 64, 128], help="plan block size (0 = 128)")
     ap.add_argument("--dense-chunk", type=int, default=0, help="column tiles per dense-row item (-1: no split)")
     ap.add_argument("--fine-kernel", type=int, default=0, choices=[0, 1],
                     help="CSR rows: 0 = warp-level tensor-core kernel, 1 = CUDA-core kernel (A/B)")
@@ -309,7 +310,7 @@ def main():
     t_plan = time.perf_counter()
     plan = mg.Plan(cfg.L, cfg.H, cfg.d, cfg.window, cfg.global_idx, cfg.extra_idx,
                    strip_max_cols=args.strip_max_cols, fine_kernel=args.fine_kernel,
-                   concurrency=args.concurrency, tau=args.tau, dense_chunk=args.dense_chunk)
+                   concurrency=args.concurrency, tau=args.tau, dense_chunk=args.dense_chunk, block=args.block)
     plan_build_ms = 1e3 * (time.perf_counter() - t_plan)   # host, once per pattern (before inference)
     info = plan.info()
     BH = b_local * cfg.H

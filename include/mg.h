@@ -48,7 +48,7 @@ typedef struct mg_plan_s* mg_plan_t;
 typedef enum {
   MG_OK = 0,
   MG_ERR_INVALID_ARG = 1,   /* bad sizes, indices out of range, null pointers, layout mismatch */
-  MG_ERR_UNSUPPORTED = 2,   /* valid but not implemented in v1 (d != 64, block != 128 on fwd, ...) */
+  MG_ERR_UNSUPPORTED = 2,   /* valid but not implemented (head_dim other than 64/128, block other than 64/128 on fwd, ...) */
   MG_ERR_OUT_OF_MEMORY = 3, /* host or device allocation failed */
   MG_ERR_CUDA = 4,          /* a CUDA runtime/driver error; message in mg_last_error() */
   MG_ERR_INTERNAL = 5
@@ -106,7 +106,10 @@ MG_API mg_status mg_plan_create(int64_t L, int32_t heads, int32_t d, int32_t win
 /* Test/ablation options. Zero-initialised means "default". */
 typedef struct {
   int32_t block;          /* tile size b; 0 -> 128. Any b <= 64 or multiple of 64 builds a plan
-                             (for export tests); the forward requires b == 128. */
+                             (for export tests); the forward takes b = 128 or b = 64 (the paper's
+                             block: its 64 x 64 BSR tiles run as the quadrants of
+                             128 x 128 tcgen05 tiles, non-member quadrants masked, so the forward
+                             executes exactly the b = 64 coarse/fine partition). */
   int32_t force_all_fine; /* 1: no coarse tiles; every non-global element goes to the CSR part */
   int32_t strip_max_cols; /* max gathered columns per row block for the tensor-core strip path of
                              the CSR residual; 0 -> default (128); -1 disables the strip path */
@@ -135,7 +138,7 @@ MG_API mg_status mg_plan_create_ex(int64_t L, int32_t heads, int32_t d, int32_t 
  * with those lists (A2-A7). All samples are merged into one work list, so one forward launch
  * covers the whole batch. The forward's Q/K/V/O batch must equal `batch`. Not supported with a
  * batched plan: mg_plan_export and the staged entry points (UNSUPPORTED); mg_plan_info_get returns
- * counts summed over the samples. opts as for mg_plan_create_ex (block must be 128; dense-row items
+ * counts summed over the samples. opts as for mg_plan_create_ex (block 64 or 128; dense-row items
  * are not split). Errors: as mg_plan_create, plus INVALID_ARG for batch <= 0, null or decreasing
  * offset arrays, global_ptr[0] or extra_ptr[0] != 0. */
 MG_API mg_status mg_plan_create_batched(int64_t L, int32_t heads, int32_t d, int32_t window, int64_t batch,
@@ -192,7 +195,7 @@ MG_API mg_status mg_plan_export(mg_plan_t plan, int32_t* bsr_row_ptr, int32_t* b
  * partial statistics of the CSR part) is plan-owned and grown stream-ordered on `stream`,
  * so one plan must not be used by two concurrent forwards on different streams.
  * Errors: INVALID_ARG (null, shape/dtype mismatch with the plan or between tensors,
- * head_dim stride != 1, misaligned data or strides), UNSUPPORTED (block != 128,
+ * head_dim stride != 1, misaligned data or strides), UNSUPPORTED (block not 64 or 128,
  * dtypes that differ, (L - 1) * stride_l of K or V >= 2^32 elements), CUDA.
  * ---------------------------------------------------------------------------------- */
 MG_API mg_status mg_sparse_attention_fwd(mg_plan_t plan, const mg_tensor* Q, const mg_tensor* K,
@@ -288,6 +291,22 @@ MG_API mg_status mg_plan_get_profile(mg_plan_t plan, mg_profile* out);
  * buffer owned by the caller; may be null when cap == 0), so that a caller can report the median
  * and minimum of a timed run. INVALID_ARG: null plan/out, cap < 0, or cap > 0 with a null buffer. */
 MG_API mg_status mg_plan_get_profile_calls(mg_plan_t plan, mg_profile* out, double* per_call_ms, int64_t cap);
+
+/* ------------------------------------------------------------------------------------
+ * Per-pattern choice of the coarse/fine split by measured cost ("the more low-sparsity
+ * sparse blocks there are, the more benefits the fine-grained kernel has"; blocked
+ * patterns). mg_plan_autotune builds one plan per candidate (block b in {128, 64} x density
+ * threshold tau in {0, 0.1, 0.25, 0.5}, A17), times each candidate's forward on the caller's
+ * device tensors (2 warm-up + 5 timed calls, CUDA events on `stream`, median) and returns the
+ * fastest plan; *chosen (may be null) receives its options and *best_ms its median time. The
+ * patterns are as for mg_plan_create; O is overwritten (scratch). Synchronous (it waits for the
+ * timing events). Errors: as mg_plan_create and mg_sparse_attention_fwd; the candidates' plans are
+ * destroyed on every path.
+ * ---------------------------------------------------------------------------------- */
+MG_API mg_status mg_plan_autotune(int64_t L, int32_t heads, int32_t d, int32_t window, const int32_t* global_idx,
+                                  int64_t n_global, const int32_t* extra_idx, int64_t n_extra, const mg_tensor* Q,
+                                  const mg_tensor* K, const mg_tensor* V, mg_tensor* O, void* stream,
+                                  mg_plan_t* plan_out, mg_plan_opts* chosen, double* best_ms);
 
 /* ------------------------------------------------------------------------------------
  * Diagnostics (used by the GPU tests; not part of the attention path).

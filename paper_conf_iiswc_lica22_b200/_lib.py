@@ -18,7 +18,7 @@ EXPORTED = [
     "mg_plan_create", "mg_plan_create_ex", "mg_plan_create_batched", "mg_plan_destroy", "mg_last_error", "mg_plan_info_get",
     "mg_plan_export", "mg_sparse_attention_fwd", "mg_sparse_attention_fwd_host", "mg_selftest_umma",
     "mg_abi_version", "mg_plan_set_profiling", "mg_plan_get_profile", "mg_plan_get_profile_calls", "mg_plan_set_trace",
-    "mg_sparse_attention_fwd_padded", "mg_staged_get_sizes", "mg_staged_sddmm", "mg_staged_softmax", "mg_staged_spmm", "mg_sparse_attention_fwd_staged", "mg_sparse_attention_fwd_staged_ex",
+    "mg_sparse_attention_fwd_padded", "mg_staged_get_sizes", "mg_staged_sddmm", "mg_staged_softmax", "mg_staged_spmm", "mg_sparse_attention_fwd_staged", "mg_sparse_attention_fwd_staged_ex", "mg_plan_autotune",
 ]
 
 
@@ -94,6 +94,8 @@ def load() -> C.CDLL:
     lib.mg_staged_spmm.argtypes = [P, P, P, P, tp, tp, P, P]
     lib.mg_sparse_attention_fwd_staged.argtypes = [P, tp, tp, tp, tp, P]
     lib.mg_sparse_attention_fwd_staged_ex.argtypes = [P, tp, tp, tp, tp, C.c_int32, P]
+    lib.mg_plan_autotune.argtypes = [C.c_int64, C.c_int32, C.c_int32, C.c_int32, i32p, C.c_int64, i32p, C.c_int64,
+                                     tp, tp, tp, tp, P, C.POINTER(P), C.POINTER(mg_plan_opts), C.POINTER(C.c_double)]
     lib.mg_abi_version.restype = C.c_int32
     lib.mg_abi_version.argtypes = []
     for name in EXPORTED:

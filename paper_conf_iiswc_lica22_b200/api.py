@@ -113,6 +113,28 @@ class Plan:
             pass
 
 
+def autotune_plan(L: int, heads: int, d: int, window: int, global_idx, extra_idx, Q, K, V, O=None, stream=None):
+    """mg_plan_autotune: the fastest of the block {128, 64} x tau {0, 0.1, 0.25, 0.5} plans of this
+    pattern, timed on the given device tensors (O is scratch). Returns (plan, chosen options, ms)."""
+    import torch
+    lib = load()
+    g = _i32(list(global_idx) if not isinstance(global_idx, np.ndarray) else global_idx).reshape(-1)
+    e = _i32(np.zeros((0, 2)) if extra_idx is None else extra_idx).reshape(-1, 2)
+    if O is None:
+        O = torch.empty(Q.shape, dtype=Q.dtype, device=Q.device)
+    dq, dk, dv, do = tensor_desc(Q), tensor_desc(K), tensor_desc(V), tensor_desc(O)
+    h = C.c_void_p()
+    chosen = mg_plan_opts()
+    ms = C.c_double()
+    check(lib.mg_plan_autotune(L, heads, d, window, _ptr_i32(g), g.size, _ptr_i32(e), e.shape[0], C.byref(dq),
+                               C.byref(dk), C.byref(dv), C.byref(do), _stream_ptr(stream), C.byref(h),
+                               C.byref(chosen), C.byref(ms)))
+    plan = Plan.__new__(Plan)
+    plan._handle, plan._lib = h, lib
+    plan.L, plan.heads, plan.d, plan.window = L, heads, d, window
+    return plan, {"block": chosen.block, "tau": chosen.tau}, ms.value
+
+
 class BatchedPlan(Plan):
     """mg_plan_create_batched: one plan for a batch whose samples have their own global tokens and
     extra pairs (lists of arrays, one per sample). Same options as Plan."""

@@ -158,7 +158,7 @@ cudaError_t upload_vec(mg_plan_s* p, T** dst, const std::vector<T>& v) {
 
 mg_status upload(mg_plan_s* p) {
   if (p->uploaded) return MG_OK;
-  if (!p->hp.kernel_ready) return fail(MG_ERR_UNSUPPORTED, "the forward requires block == 128");
+  if (!p->hp.kernel_ready) return fail(MG_ERR_UNSUPPORTED, "the forward requires block 64 or 128");
   cudaError_t e = cudaGetDevice(&p->device);
   if (e != cudaSuccess) return cuda_fail(e, "cudaGetDevice");
   e = cudaDeviceGetAttribute(&p->num_sms, cudaDevAttrMultiProcessorCount, p->device);
@@ -292,7 +292,7 @@ mg_status check_all(const mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, 
     return fail(MG_ERR_UNSUPPORTED, "Q/K/V/O dtypes differ");
   if (p->hp.batch > 0 && Q->batch != p->hp.batch)
     return fail(MG_ERR_INVALID_ARG, "batch size differs from the batched plan's number of samples");
-  if (!p->hp.kernel_ready) return fail(MG_ERR_UNSUPPORTED, "the forward requires block == 128");
+  if (!p->hp.kernel_ready) return fail(MG_ERR_UNSUPPORTED, "the forward requires block 64 or 128");
   if ((int64_t)Q->batch * p->hp.heads >=
       (int64_t(1) << 31) / std::max<int64_t>(1, (int64_t)std::max(p->hp.items.size(), p->hp.items_split.size())))
     return fail(MG_ERR_UNSUPPORTED, "batch * heads * work items exceeds int32");
@@ -636,7 +636,7 @@ mg::StagedParams staged_params(const mg_plan_s* p, int64_t batch) {
 mg_status staged_check(mg_plan_s* p, const mg_tensor* t, const char* name) {
   mg_status s = check_tensor(t, name, p, false);
   if (s != MG_OK) return s;
-  if (!p->hp.kernel_ready) return fail(MG_ERR_UNSUPPORTED, "the staged forward requires block == 128");
+  if (!p->hp.kernel_ready || p->hp.block != 128) return fail(MG_ERR_UNSUPPORTED, "the staged forward requires block == 128");
   if (p->hp.batch > 0) return fail(MG_ERR_UNSUPPORTED, "the staged forward does not take batched plans");
   if ((int64_t)t->batch * p->hp.heads >= 65536) return fail(MG_ERR_UNSUPPORTED, "batch * heads must be < 65536");
   return staged_upload(p);
@@ -900,7 +900,7 @@ mg_status mg_staged_softmax(mg_plan_t plan, int64_t batch, mg_dtype dtype, const
   if (!plan) return fail(MG_ERR_INVALID_ARG, "plan is null");
   if (batch <= 0) return fail(MG_ERR_INVALID_ARG, "batch must be > 0");
   if (dtype != MG_BF16 && dtype != MG_FP16) return fail(MG_ERR_INVALID_ARG, "dtype is not bf16/fp16");
-  if (!plan->hp.kernel_ready) return fail(MG_ERR_UNSUPPORTED, "the staged forward requires block == 128");
+  if (!plan->hp.kernel_ready || plan->hp.block != 128) return fail(MG_ERR_UNSUPPORTED, "the staged forward requires block == 128");
   if (plan->hp.batch > 0) return fail(MG_ERR_UNSUPPORTED, "the staged forward does not take batched plans");
   mg_status s;
   if ((s = staged_upload(plan)) != MG_OK) return s;
@@ -986,6 +986,75 @@ mg_status mg_sparse_attention_fwd_staged_ex(mg_plan_t plan, const mg_tensor* Q, 
 mg_status mg_sparse_attention_fwd_staged(mg_plan_t plan, const mg_tensor* Q, const mg_tensor* K, const mg_tensor* V,
                                          mg_tensor* O, void* stream) {
   return mg_sparse_attention_fwd_staged_ex(plan, Q, K, V, O, 0, stream);
+}
+
+mg_status mg_plan_autotune(int64_t L, int32_t heads, int32_t d, int32_t window, const int32_t* global_idx,
+                           int64_t n_global, const int32_t* extra_idx, int64_t n_extra, const mg_tensor* Q,
+                           const mg_tensor* K, const mg_tensor* V, mg_tensor* O, void* stream_, mg_plan_t* plan_out,
+                           mg_plan_opts* chosen, double* best_ms) {
+  g_err.clear();
+  if (!plan_out) return fail(MG_ERR_INVALID_ARG, "plan_out is null");
+  *plan_out = nullptr;
+  cudaStream_t stream = static_cast<cudaStream_t>(stream_);
+  cudaEvent_t ev[2] = {nullptr, nullptr};
+  cudaError_t e;
+  if ((e = cudaEventCreate(&ev[0])) != cudaSuccess || (e = cudaEventCreate(&ev[1])) != cudaSuccess) {
+    if (ev[0]) cudaEventDestroy(ev[0]);
+    return cuda_fail(e, "cudaEventCreate");
+  }
+  mg_plan_t best = nullptr;
+  mg_plan_opts best_opts{};
+  double best_t = 0.0;
+  mg_status status = MG_OK;
+  const int32_t blocks[2] = {128, 64};
+  const float taus[4] = {0.f, 0.1f, 0.25f, 0.5f};
+  for (int32_t b : blocks) {
+    for (float tau : taus) {
+      mg_plan_opts o{};
+      o.block = b;
+      o.tau = tau;
+      mg_plan_t cand = nullptr;
+      mg_status s = create_impl(L, heads, d, window, global_idx, n_global, extra_idx, n_extra, &o, &cand);
+      if (s == MG_OK) s = check_all(cand, Q, K, V, O, false);
+      std::vector<float> ts;
+      for (int i = 0; i < 7 && s == MG_OK; ++i) {
+        if (cudaEventRecord(ev[0], stream) != cudaSuccess) s = fail(MG_ERR_CUDA, "cudaEventRecord");
+        if (s == MG_OK) s = fwd_impl(cand, Q, K, V, O, stream);
+        if (s == MG_OK && (e = cudaEventRecord(ev[1], stream)) != cudaSuccess) s = cuda_fail(e, "cudaEventRecord");
+        if (s == MG_OK && (e = cudaEventSynchronize(ev[1])) != cudaSuccess) s = cuda_fail(e, "cudaEventSynchronize");
+        float ms = 0.f;
+        if (s == MG_OK && i >= 2) {
+          cudaEventElapsedTime(&ms, ev[0], ev[1]);
+          ts.push_back(ms);
+        }
+      }
+      if (s != MG_OK) {
+        delete cand;
+        if (best) delete best;
+        best = nullptr;
+        status = s;
+        break;
+      }
+      std::sort(ts.begin(), ts.end());
+      const double med = ts[ts.size() / 2];
+      if (!best || med < best_t) {
+        if (best) delete best;
+        best = cand;
+        best_t = med;
+        best_opts = o;
+      } else {
+        delete cand;
+      }
+    }
+    if (status != MG_OK) break;
+  }
+  cudaEventDestroy(ev[0]);
+  cudaEventDestroy(ev[1]);
+  if (status != MG_OK) return status;
+  *plan_out = best;
+  if (chosen) *chosen = best_opts;
+  if (best_ms) *best_ms = best_t;
+  return MG_OK;
 }
 
 mg_status mg_plan_set_profiling(mg_plan_t plan, int32_t enable) {

@@ -152,15 +152,50 @@ std::string build_plan(HostPlan& p, int64_t L, int32_t heads, int32_t d, int32_t
     if (pc == (int64_t)b * b) p.n_full_tiles++;
   }
 
-  // ---- kernel-side structures (tcgen05 path needs b == 128)
-  if (b != 128) return "";
+  // ---- kernel-side structures: the tcgen05 kernel computes 128 x 128 tiles (M = 128). With b = 128
+  // the kernel tiles are the BSR tiles. With b = 64 (the paper's block size) each
+  // kernel tile groups the 2 x 2 block of 64-tiles it covers: its bitmask is the union of the member
+  // 64-tiles' masks, non-member quadrants are all zero (their union elements are in the b = 64 CSR
+  // residual), so the forward executes exactly the b = 64 partition.
+  if (b != 128 && b != 64) return "";
   p.kernel_ready = true;
   const int64_t B = 128;
-  p.dev_masks.assign(p.tile_masks.begin(), p.tile_masks.end());  // 256 words per tile
-  std::vector<uint8_t> tile_full(nt, 0);
-  for (int64_t t = 0; t < nt; ++t) {
+  const int64_t nbk = (L + B - 1) / B;
+  std::vector<int32_t> k_row_ptr, k_col;
+  if (b == 128) {
+    k_row_ptr = p.bsr_row_ptr;
+    k_col = p.bsr_col;
+    p.dev_masks.assign(p.tile_masks.begin(), p.tile_masks.end());  // 256 words per tile
+  } else {
+    k_row_ptr.push_back(0);
+    std::vector<int32_t> slot(nbk, -1);
+    for (int64_t I = 0; I < nbk; ++I) {
+      const int64_t first = (int64_t)k_col.size();
+      for (int64_t a = 0; a < 2 && 2 * I + a < nb; ++a)
+        for (int32_t t = p.bsr_row_ptr[2 * I + a]; t < p.bsr_row_ptr[2 * I + a + 1]; ++t) {
+          const int32_t Jk = p.bsr_col[t] / 2;
+          if (slot[Jk] < 0) {
+            slot[Jk] = 0;
+            k_col.push_back(Jk);
+          }
+        }
+      std::sort(k_col.begin() + first, k_col.end());
+      for (int64_t i = first; i < (int64_t)k_col.size(); ++i) slot[k_col[i]] = (int32_t)i;
+      p.dev_masks.resize(k_col.size() * 256, 0ull);
+      for (int64_t a = 0; a < 2 && 2 * I + a < nb; ++a)
+        for (int32_t t = p.bsr_row_ptr[2 * I + a]; t < p.bsr_row_ptr[2 * I + a + 1]; ++t) {
+          const int32_t kt = slot[p.bsr_col[t] / 2], q = p.bsr_col[t] & 1;
+          for (int r = 0; r < 64; ++r) p.dev_masks[(size_t)kt * 256 + (a * 64 + r) * 2 + q] = p.tile_masks[(size_t)t * 64 + r];
+        }
+      for (int64_t i = first; i < (int64_t)k_col.size(); ++i) slot[k_col[i]] = -1;
+      k_row_ptr.push_back((int32_t)k_col.size());
+    }
+  }
+  const int64_t nkt = (int64_t)k_col.size();
+  std::vector<uint8_t> tile_full(nkt, 0);
+  for (int64_t t = 0; t < nkt; ++t) {
     bool full = true;
-    for (int w = 0; w < 256 && full; ++w) full = p.tile_masks[t * 256 + w] == ~0ull;
+    for (int w = 0; w < 256 && full; ++w) full = p.dev_masks[t * 256 + w] == ~0ull;
     tile_full[t] = full;
   }
   auto new_mask = [&]() -> int32_t {
@@ -178,7 +213,7 @@ std::string build_plan(HostPlan& p, int64_t L, int32_t heads, int32_t d, int32_t
   int32_t ragged_mask = kMaskFull;
   if (L % B) {
     ragged_mask = new_mask();
-    const int64_t valid = L - (nb - 1) * B;
+    const int64_t valid = L - (nbk - 1) * B;
     for (int a = 0; a < 128; ++a)
       for (int64_t c = 0; c < valid; ++c) p.dev_masks[(size_t)ragged_mask * 256 + a * 2 + c / 64] |= 1ull << (c % 64);
   }
@@ -186,9 +221,9 @@ std::string build_plan(HostPlan& p, int64_t L, int32_t heads, int32_t d, int32_t
   const int64_t G = (int64_t)p.global_rows.size();
   for (int64_t k = 0; k < G; k += 128) {
     const int32_t nr = (int32_t)std::min<int64_t>(128, G - k);
-    Item it{1, (int32_t)k, (int32_t)(k / 128), (int32_t)nb, (int32_t)p.trefs.size(), nr, 1, 0, 0ull, 0ull};
-    for (int64_t J = 0; J < nb; ++J) {
-      const int32_t m = (J == nb - 1) ? ragged_mask : kMaskFull;
+    Item it{1, (int32_t)k, (int32_t)(k / 128), (int32_t)nbk, (int32_t)p.trefs.size(), nr, 1, 0, 0ull, 0ull};
+    for (int64_t J = 0; J < nbk; ++J) {
+      const int32_t m = (J == nbk - 1) ? ragged_mask : kMaskFull;
       p.trefs.push_back(TileRef{(int32_t)(J * B), 0, 128, m, kMaskSkip, 0, 0, 0});
       count(m, 128, nr);
     }
@@ -198,12 +233,12 @@ std::string build_plan(HostPlan& p, int64_t L, int32_t heads, int32_t d, int32_t
   // the same rows split into chunks of <= dense_chunk column tiles (a separate work list, chosen
   // per forward when the dense items would be too few to spread over the SMs); the chunks' fp32
   // partials are merged by the last chunk to finish. The chunks reuse the unsplit items' tile refs.
-  const int64_t chunk = std::max<int64_t>(1, std::min<int64_t>(opts.dense_chunk, nb));
-  const int32_t nsplit = (int32_t)((nb + chunk - 1) / chunk);
+  const int64_t chunk = std::max<int64_t>(1, std::min<int64_t>(opts.dense_chunk, nbk));
+  const int32_t nsplit = (int32_t)((nbk + chunk - 1) / chunk);
   p.dense_nsplit = nsplit;
   for (const Item& d : p.items) {
     for (int32_t sc = 0; sc < nsplit; ++sc) {
-      const int64_t J0 = sc * chunk, J1 = std::min<int64_t>(nb, J0 + chunk);
+      const int64_t J0 = sc * chunk, J1 = std::min<int64_t>(nbk, J0 + chunk);
       p.items_split.push_back(Item{1, d.rowA, d.rowB, (int32_t)(J1 - J0), d.tref_begin + (int32_t)J0, d.nrowsA,
                                    nsplit, sc, 0ull, 0ull});
     }
@@ -212,8 +247,8 @@ std::string build_plan(HostPlan& p, int64_t L, int32_t heads, int32_t d, int32_t
   p.n_dense_items = (int32_t)p.items.size();
 
   // distinct CSR columns of each row block
-  std::vector<std::vector<int32_t>> blk_cols(nb);
-  for (int64_t I = 0; I < nb; ++I) {
+  std::vector<std::vector<int32_t>> blk_cols(nbk);
+  for (int64_t I = 0; I < nbk; ++I) {
     const int64_t r0 = I * B, r1 = std::min<int64_t>(L, r0 + B);
     auto& cols = blk_cols[I];
     for (int64_t r = r0; r < r1; ++r)
@@ -222,7 +257,7 @@ std::string build_plan(HostPlan& p, int64_t L, int32_t heads, int32_t d, int32_t
     cols.erase(std::unique(cols.begin(), cols.end()), cols.end());
   }
   const int strip_max = opts.strip_max_cols;
-  std::vector<uint8_t> blk_strip(nb, 0);  // CSR residual of the block carried by a strip tile
+  std::vector<uint8_t> blk_strip(nbk, 0);  // CSR residual of the block carried by a strip tile
   // strip tile over `cols` with the bitmask of row block I (kMaskSkip if I < 0)
   auto strip_mask = [&](int64_t I, const std::vector<int32_t>& cols, int ncols) -> int32_t {
     if (I < 0) return kMaskSkip;
@@ -258,13 +293,13 @@ std::string build_plan(HostPlan& p, int64_t L, int32_t heads, int32_t d, int32_t
   };
 
   // band items: one per row block with coarse tiles (its BSR tiles, then its strip if any)
-  for (int64_t I = 0; I < nb; ++I) {
-    if (p.bsr_row_ptr[I + 1] == p.bsr_row_ptr[I]) continue;
+  for (int64_t I = 0; I < nbk; ++I) {
+    if (k_row_ptr[I + 1] == k_row_ptr[I]) continue;
     const int32_t nr = (int32_t)std::min<int64_t>(B, L - I * B);
     Item it{0, (int32_t)(I * B), 0, 0, (int32_t)p.trefs.size(), nr, 0, 0, 0ull, 0ull};
-    for (int32_t t = p.bsr_row_ptr[I]; t < p.bsr_row_ptr[I + 1]; ++t) {
+    for (int32_t t = k_row_ptr[I]; t < k_row_ptr[I + 1]; ++t) {
       const int32_t m = tile_full[t] ? kMaskFull : t;
-      p.trefs.push_back(TileRef{p.bsr_col[t] * (int32_t)B, 0, 128, m, kMaskSkip, 0, 0, 0});
+      p.trefs.push_back(TileRef{k_col[t] * (int32_t)B, 0, 128, m, kMaskSkip, 0, 0, 0});
       count(m, 128, nr);
     }
     // CSR residual as a tensor-core strip where the block's distinct columns are few
@@ -280,9 +315,9 @@ std::string build_plan(HostPlan& p, int64_t L, int32_t heads, int32_t d, int32_t
 
   // CSR rows left to the CUDA-core fine kernel
   p.fine_slot.assign(L, -1);
-  for (int64_t I = 0; I < nb; ++I) {
+  for (int64_t I = 0; I < nbk; ++I) {
     if (blk_strip[I]) continue;
-    const bool has_tiles = p.bsr_row_ptr[I + 1] > p.bsr_row_ptr[I];
+    const bool has_tiles = k_row_ptr[I + 1] > k_row_ptr[I];
     const int64_t r0 = I * B, r1 = std::min<int64_t>(L, r0 + B);
     for (int64_t r = r0; r < r1; ++r) {
       if (p.csr_row_ptr[r + 1] == p.csr_row_ptr[r]) continue;
@@ -321,7 +356,7 @@ std::string build_batched_plan(HostPlan& out, int64_t L, int32_t heads, int32_t 
   if (global_ptr[0] != 0 || extra_ptr[0] != 0) return "global_ptr[0] and extra_ptr[0] must be 0";
   for (int64_t b = 0; b < batch; ++b)
     if (global_ptr[b + 1] < global_ptr[b] || extra_ptr[b + 1] < extra_ptr[b]) return "offsets must be non-decreasing";
-  if (opts.block != 128) { *unsupported = true; return "batched plans require block == 128"; }
+  if (opts.block != 128 && opts.block != 64) { *unsupported = true; return "batched plans require block 64 or 128"; }
   PlanOptions po = opts;
   po.dense_split = 1;   // the split dense-row list is not built for batched plans
   std::vector<HostPlan> ps(batch);

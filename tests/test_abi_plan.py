@@ -208,3 +208,35 @@ def test_batched_plan_counts_sum_samples_and_validation():
         mg.BatchedPlan(L, H, 64, w, [[0], [L]])
     with pytest.raises(mg.MGError):
         mg.BatchedPlan(L, H, 64, w, [])
+
+
+@pytest.mark.parametrize("cfg", ["C1", "C2", "C3", "DIL-LD"])
+def test_block64_kernel_tiles_group_the_64_tiles(cfg):
+    """b = 64 runs on 128 x 128 tcgen05 tiles grouping 2 x 2 blocks of 64-tiles: the
+    band part computes 128^2 scores per distinct group of the exported b = 64 BSR, and the forward
+    accepts the plan (kernel structures built); the exported partition stays the b = 64 one."""
+    c = get_config(cfg)
+    p64 = mg.Plan(c.L, c.H, c.d, c.window, c.global_idx, c.extra_idx, block=64)
+    e = p64.export()
+    groups = set()
+    for I in range(len(e["bsr_row_ptr"]) - 1):
+        for t in range(e["bsr_row_ptr"][I], e["bsr_row_ptr"][I + 1]):
+            groups.add((I // 2, int(e["bsr_col"][t]) // 2))
+    # band-only reference: the same pattern without global rows / extras / strips
+    pb = mg.Plan(c.L, c.H, c.d, c.window, [], None, block=64)
+    eb = pb.export()
+    gb = {(I // 2, int(eb["bsr_col"][t]) // 2) for I in range(len(eb["bsr_row_ptr"]) - 1)
+          for t in range(eb["bsr_row_ptr"][I], eb["bsr_row_ptr"][I + 1])}
+    assert pb.info()["computed_scores"] == 128 * 128 * len(gb)
+    inf = p64.info()
+    assert inf["n_items"] > 0 and inf["computed_scores"] >= 128 * 128 * len(groups)
+    assert inf["nnz_total"] == mg.Plan(c.L, c.H, c.d, c.window, c.global_idx, c.extra_idx).info()["nnz_total"]
+
+
+def test_block64_batched_plan_accepted():
+    L, H, w = 1024, 2, 128
+    bp = mg.BatchedPlan(L, H, 64, w, [np.array([0, 5], np.int32), np.array([300], np.int32)], None, block=64)
+    assert bp.info()["n_items"] > 0
+    with pytest.raises(mg.MGError) as ei:
+        mg.BatchedPlan(L, H, 64, w, [[0], [1]], None, block=32)
+    assert ei.value.status == _lib.MG_ERR_UNSUPPORTED

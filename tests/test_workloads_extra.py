@@ -45,10 +45,23 @@ def test_qds_ls_selected_columns_all_to_one():
     assert 1.7 <= (p.n_tiles - full) / full <= 2.3
 
 
+@pytest.mark.parametrize("b", [128, 64])
 @pytest.mark.parametrize("name", EXTRA_WORKLOADS)
-def test_extra_workload_plan_bit_exact(name):
+def test_extra_workload_plan_bit_exact(name, b):
     c = get_config(name)
-    ref = canonical_plan(c.L, c.window, c.global_idx, c.extra_idx, 128)
-    got = mg.Plan(c.L, c.H, c.d, c.window, c.global_idx, c.extra_idx).export()
+    ref = canonical_plan(c.L, c.window, c.global_idx, c.extra_idx, b)
+    got = mg.Plan(c.L, c.H, c.d, c.window, c.global_idx, c.extra_idx, block=b).export()
     for f in ("bsr_row_ptr", "bsr_col", "tile_masks", "csr_row_ptr", "csr_col", "global_rows"):
         assert np.array_equal(got[f], getattr(ref, f)), f
+
+
+def test_dilated_pattern_strides():
+    """Dilated local pattern: row r attends r +- k * stride (k = 1..taps) besides its window."""
+    c = get_config("DIL-LD")
+    g, ex = global_flags(c.L, c.global_idx), ExtraIndex(c.L, c.extra_idx)
+    w1 = c.window // 2
+    for r in (0, 1, 700, 2048, c.L - 1):
+        cols = set(mask_row_cols(r, c.L, c.window, g, ex).tolist())
+        band = {x for x in range(max(0, r - w1), min(c.L, r + w1 + 1))}
+        dil = {r + s * k * 16 for k in range(1, 33) for s in (1, -1) if 0 <= r + s * k * 16 < c.L}
+        assert cols == band | dil

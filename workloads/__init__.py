@@ -145,6 +145,27 @@ def uniform_random_pairs(L: int, per_row: int, seed: int) -> np.ndarray:
     return out
 
 
+def dilated_pairs(L: int, stride: int, taps: int) -> np.ndarray:
+    """Dilated pattern ("tokens located at a constant stride distance", used "as a dilated
+    local pattern combined with a local pattern"): every row r attends to r + k * stride for
+    k = +-1 .. +-taps (inside [0, L)). Entries that fall inside a local window are absorbed by the
+    plan's set semantics. Returns int32 [n, 2] (row, col) pairs."""
+    r = np.arange(L, dtype=np.int64)
+    out = []
+    for k in range(1, taps + 1):
+        for sgn in (1, -1):
+            c = r + sgn * k * stride
+            ok = (c >= 0) & (c < L)
+            out.append(np.stack([r[ok], c[ok]], axis=1))
+    return np.concatenate(out).astype(np.int32) if out else np.zeros((0, 2), np.int32)
+
+
+def _dil() -> "Config":
+    L = 4096
+    return Config("DIL-LD", 1, 4, L, 64, 256, np.zeros(0, np.int32), dilated_pairs(L, 16, 32), 0,
+                  "local w=256 + dilated local (stride 16, 32 taps each side, P:68)")
+
+
 def _f9(name: str) -> "Config":
     L, rng = 4096, np.random.default_rng(9)
     if name == "F9-LS":
@@ -174,7 +195,7 @@ def _qds_ls() -> "Config":
                   "QDS-Transformer as L+S: w=128, 64 special tokens as column-only selected tokens, B=8")
 
 
-EXTRA_WORKLOADS = ("QDS-LS", "F9-LS", "F9-LSG", "F9-LBR", "F9-RBR")
+EXTRA_WORKLOADS = ("QDS-LS", "F9-LS", "F9-LSG", "F9-LBR", "F9-RBR", "DIL-LD")
 
 
 def _build_configs():
@@ -199,7 +220,7 @@ def get_config(name: str) -> Config:
     C4's residual is generated on first use (~1 s)."""
     if name in EXTRA_WORKLOADS:
         if name not in _C4_CACHE:
-            _C4_CACHE[name] = _qds_ls() if name == "QDS-LS" else _f9(name)
+            _C4_CACHE[name] = _qds_ls() if name == "QDS-LS" else (_dil() if name == "DIL-LD" else _f9(name))
         return _C4_CACHE[name]
     if name == "C4":
         if "C4" not in _C4_CACHE:
