@@ -60,6 +60,8 @@ def parse():
                     help="coarse vs CSR kernels: 0 = library default, 1 = serial, 2 = concurrent streams")
     ap.add_argument("--tau", type=float, default=0.0, help="tile density threshold (0 = band rule)")
     ap.add_argument("--block", type=int, default=0, choices=[0, 64, 128], help="plan block size (0 = 128)")
+    ap.add_argument("--head-dim", type=int, default=0, choices=[0, 64, 128],
+                    help="head dimension override (0 = the workload's, 64); 128 for the d = 128 line")
     ap.add_argument("--dense-chunk", type=int, default=0, help="column tiles per dense-row item (-1: no split)")
     ap.add_argument("--fine-kernel", type=int, default=0, choices=[0, 1],
                     help="CSR rows: 0 = warp-level tensor-core kernel, 1 = CUDA-core kernel (A/B)")
@@ -241,6 +243,9 @@ def run_reference(args):
     from workloads import get_config, make_qkv
     world = int(os.environ.get("WORLD_SIZE", "1"))
     cfg = get_config(resolve_workload(args, max(world, args.gpus)))
+    if args.head_dim:
+        import dataclasses
+        cfg = dataclasses.replace(cfg, d=args.head_dim)
     strong = cfg.name == "C5"
     lo, hi = shard_for_rank(cfg, max(world, args.gpus), 0, strong)
     q, k, v = make_qkv(1, 1, cfg.L, cfg.d, seed=cfg.seed)
@@ -304,6 +309,9 @@ def main():
     dev = torch.device("cuda", local)
 
     cfg = get_config(resolve_workload(args, world))
+    if args.head_dim:
+        import dataclasses
+        cfg = dataclasses.replace(cfg, d=args.head_dim)
     strong = cfg.name == "C5"
     lo, hi = shard_for_rank(cfg, world, rank, strong)
     b_local = hi - lo

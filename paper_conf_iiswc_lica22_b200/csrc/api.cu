@@ -320,9 +320,9 @@ bool encode_map(CUtensorMap* m, const mg_tensor* t) {
   return r == CUDA_SUCCESS;
 }
 
-// 2-D [rows, 64] view of a strided [B, H, L, 64] tensor for TMA row gathers (tile::gather4, box
-// 64 x 1): the row stride is the gcd of the element strides, which must be a multiple of 64
-// (true for dense [B,H,L,d] and [B,L,H,d]); row(b, h, l) = b * r.x + h * r.y + l * r.z.
+// 2-D [rows, 64] view of a strided [B, H, L, d] tensor for TMA row gathers (tile::gather4, box
+// 64 x 1) with a row stride of 64 elements; row(b, h, l) = b * r.x + h * r.y + l * r.z (+ 1 for the
+// second 64 columns of a d = 128 row).
 bool encode_map2d(CUtensorMap* m, const mg_tensor* t, longlong3* r) {
   auto fn = tensor_map_encoder();
   if (!fn) return false;
@@ -330,11 +330,14 @@ bool encode_map2d(CUtensorMap* m, const mg_tensor* t, longlong3* r) {
     while (b) { const int64_t c = a % b; a = b; b = c; }
     return a;
   };
+  // rows of 64 elements (a d = 128 row is two consecutive view rows): every stride must be a
+  // multiple of 64 elements (true for dense [B,H,L,d] and [B,L,H,d])
   int64_t rs = 0;
   for (int64_t s : {t->stride_b, t->stride_h, t->stride_l})
     if (s > 0) rs = gcd(rs, s);
   if (rs <= 0 || rs % 64) return false;
-  const int64_t span = (t->batch - 1) * t->stride_b + (t->heads - 1) * t->stride_h + (t->seq_len - 1) * t->stride_l + 64;
+  rs = 64;
+  const int64_t span = (t->batch - 1) * t->stride_b + (t->heads - 1) * t->stride_h + (t->seq_len - 1) * t->stride_l + t->head_dim;
   const int64_t rows = (span + rs - 1) / rs;
   if (rows >= (int64_t(1) << 31)) return false;
   cuuint64_t dims[2] = {64, (cuuint64_t)rows};
@@ -377,27 +380,29 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
   const bool concurrent = nf > 0 && !h.items.empty() && p->fine_kernel == 0 &&
                           (p->concurrency == 2 || (p->concurrency == 0 && kConcurrentDefault));
   // fp32 partials of the CUDA-core CSR rows (fine -> coarse; and coarse -> fine plus one counter
-  // per row when concurrent). Layout by capacity: [fine acc 64][fine ml 2][coarse acc 64][coarse ml 2]
+  // per row when concurrent). Layout by capacity: [fine acc d][fine ml 2][coarse acc d][coarse ml 2]
   // floats per slot, then one int32 counter per slot (zeroed at allocation; even between forwards).
+  const int D = h.d;
   const size_t need = ((size_t)BH * nf + 3) & ~size_t(3);   // multiple of 4: 16-byte aligned sections
   if (need > p->part_cap) {
     if (p->d_part) {
       if ((e = cudaFreeAsync(p->d_part, stream)) != cudaSuccess) return cuda_fail(e, "cudaFreeAsync");
       p->d_part = nullptr;
     }
-    if ((e = cudaMallocAsync(reinterpret_cast<void**>(&p->d_part), need * 133 * sizeof(float), stream)) != cudaSuccess)
+    if ((e = cudaMallocAsync(reinterpret_cast<void**>(&p->d_part), need * (2 * D + 5) * sizeof(float), stream)) !=
+        cudaSuccess)
       return e == cudaErrorMemoryAllocation ? fail(MG_ERR_OUT_OF_MEMORY, "workspace allocation failed")
                                             : cuda_fail(e, "cudaMallocAsync");
-    if ((e = cudaMemsetAsync(p->d_part + need * 132, 0, need * sizeof(int32_t), stream)) != cudaSuccess)
+    if ((e = cudaMemsetAsync(p->d_part + need * (2 * D + 4), 0, need * sizeof(int32_t), stream)) != cudaSuccess)
       return cuda_fail(e, "cudaMemsetAsync");
     p->part_cap = need;
   }
   const size_t cap = p->part_cap;
   float* part_acc = p->d_part;
-  float2* part_ml = reinterpret_cast<float2*>(p->d_part + cap * 64);
-  float* part_c_acc = p->d_part + cap * 66;
-  float2* part_c_ml = reinterpret_cast<float2*>(p->d_part + cap * 130);
-  int32_t* part_flags = reinterpret_cast<int32_t*>(p->d_part + cap * 132);
+  float2* part_ml = reinterpret_cast<float2*>(p->d_part + cap * D);
+  float* part_c_acc = p->d_part + cap * (D + 2);
+  float2* part_c_ml = reinterpret_cast<float2*>(p->d_part + cap * (2 * D + 2));
+  int32_t* part_flags = reinterpret_cast<int32_t*>(p->d_part + cap * (2 * D + 4));
   // split dense-row items (a work list with the global rows' column tiles in chunks): chosen when
   // the unsplit dense items would be few against the SMs (each would be a long serial chain), or
   // forced by the plan option; per (b*h, row group) chunk partials + chunk counters
@@ -407,7 +412,7 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
   float* dense_part = nullptr;
   int32_t* dense_ctr = nullptr;
   if (use_split) {
-    const size_t per_bh_part = (size_t)h.n_dense_groups * h.dense_nsplit * 128 * 68 * sizeof(float);
+    const size_t per_bh_part = (size_t)h.n_dense_groups * h.dense_nsplit * 128 * (D + 4) * sizeof(float);
     const size_t per_bh_ctr = (size_t)h.n_dense_groups * sizeof(int32_t);
     if ((size_t)BH > p->dense_cap) {
       if (p->d_dense) {
@@ -463,6 +468,7 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
     fp.part_ml = part_ml;
     fp.q = view(Q); fp.k = view(K); fp.v = view(V); fp.o = view(O);
     fp.H = h.heads; fp.BH = BH; fp.n_fine_rows = nf;
+    fp.d = D;
     fp.fine_sample = h.batch > 0 ? p->d_fine_sample : nullptr;
     fp.scale_log2 = scale_log2;
     fp.concurrent = concurrent;
@@ -472,7 +478,8 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
     fp.part_flags = part_flags;
     // (the CUDA-core variant has no padding support: a padded forward always uses the MMA kernel)
     const int fsms = p->num_sms_override > 0 ? std::min(p->num_sms_override, p->num_sms) : p->num_sms;
-    e = p->fine_kernel == 1 && !valid_len ? mg::launch_fine(fp, bf16, fstream)
+    // (the CUDA-core variant takes d = 64 only: other forwards use the MMA kernel)
+    e = p->fine_kernel == 1 && !valid_len && D == 64 ? mg::launch_fine(fp, bf16, fstream)
                                           : mg::launch_fine_mma(fp, bf16, fsms, fstream);
     if (e != cudaSuccess) return cuda_fail(e, "fine kernel launch");
   }
@@ -519,6 +526,7 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
     cp.L = h.L;
     cp.H = h.heads;
     cp.BH = BH;
+    cp.d = D;
     cp.batched = h.batch > 0;
     cp.n_items = (int)(use_split ? h.items_split.size() : h.items.size());
     cp.n_dense_items = use_split ? h.n_dense_items_split : h.n_dense_items;
@@ -553,7 +561,7 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
       static const bool no_tma_store = std::getenv("MG_NO_TMA_STORE") != nullptr;   // A/B diagnostics
       cp.tma_store = !no_tma_store && mp.store_ok;
       if ((e = mg::launch_coarse_pp(cp, tq, tk, tv, mp.tq2, mp.tk2, mp.tv2, mp.to, bf16, use_split,
-                                    std::min(2 * sms, cp.total_units),
+                                    std::min(mg::coarse_pp_ctas_per_sm(D) * sms, cp.total_units),
                                     stream)) != cudaSuccess)
         return cuda_fail(e, "coarse kernel launch");
     }
@@ -637,6 +645,7 @@ mg_status staged_check(mg_plan_s* p, const mg_tensor* t, const char* name) {
   mg_status s = check_tensor(t, name, p, false);
   if (s != MG_OK) return s;
   if (!p->hp.kernel_ready || p->hp.block != 128) return fail(MG_ERR_UNSUPPORTED, "the staged forward requires block == 128");
+  if (p->hp.d != 64) return fail(MG_ERR_UNSUPPORTED, "the staged forward requires head_dim == 64");
   if (p->hp.batch > 0) return fail(MG_ERR_UNSUPPORTED, "the staged forward does not take batched plans");
   if ((int64_t)t->batch * p->hp.heads >= 65536) return fail(MG_ERR_UNSUPPORTED, "batch * heads must be < 65536");
   return staged_upload(p);
@@ -901,6 +910,7 @@ mg_status mg_staged_softmax(mg_plan_t plan, int64_t batch, mg_dtype dtype, const
   if (batch <= 0) return fail(MG_ERR_INVALID_ARG, "batch must be > 0");
   if (dtype != MG_BF16 && dtype != MG_FP16) return fail(MG_ERR_INVALID_ARG, "dtype is not bf16/fp16");
   if (!plan->hp.kernel_ready || plan->hp.block != 128) return fail(MG_ERR_UNSUPPORTED, "the staged forward requires block == 128");
+  if (plan->hp.d != 64) return fail(MG_ERR_UNSUPPORTED, "the staged forward requires head_dim == 64");
   if (plan->hp.batch > 0) return fail(MG_ERR_UNSUPPORTED, "the staged forward does not take batched plans");
   mg_status s;
   if ((s = staged_upload(plan)) != MG_OK) return s;

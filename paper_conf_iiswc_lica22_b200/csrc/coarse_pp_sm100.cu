@@ -45,10 +45,21 @@ namespace {
 constexpr int kThreads = 256;
 constexpr int kSt = 2;                       // K ring and V ring depth
 constexpr int kItems = 4;                    // work-item ring depth
-constexpr uint32_t kTileBytes = 128 * 128;   // 128 rows x 64 x 16-bit
+constexpr uint32_t kSub = 128 * 128;         // one SWIZZLE_128B sub-tile: 128 rows x 64 x 16-bit
 constexpr uint32_t kMaskBytes = 128 * 16;    // 128 rows x 128 validity bits
-constexpr uint32_t kTmemCols = 256;
-constexpr uint32_t kTS = 0, kTP = 128, kTO = 192;
+constexpr uint32_t kTS = 0, kTP = 128;       // TMEM columns of S (fp32) and P (packed 16-bit pairs)
+
+// Head dimension kD = 64 or 128 (D_h). A Q/K/V/O tile is kD / 64 sub-tiles of 64 columns
+// (one TMA box / one 128-byte swizzle row each). d = 64: two CTAs per SM (TMEM 256 columns: S, P,
+// O [192, 256)); d = 128: one CTA per SM (TMEM 512: S, P, O [256, 384); shared memory 6 x 32 KB).
+template <int kD>
+struct DCfg {
+  static constexpr uint32_t kTileBytes = 128 * kD * 2;
+  static constexpr int kNSub = kD / 64;
+  static constexpr uint32_t kTmemCols = kD == 64 ? 256 : 512;
+  static constexpr uint32_t kTO = kD == 64 ? 192 : 256;
+  static constexpr int kMinBlocks = kD == 64 ? 2 : 1;
+};
 
 struct __align__(16) Slot {
   Item item;
@@ -68,10 +79,14 @@ struct __align__(16) Ctl {
   int32_t dense_last;                         // split dense item: this chunk finished its row group last
 };
 
-constexpr size_t kSmemBytes = 1024 + 6 * kTileBytes + kSt * kMaskBytes + sizeof(Ctl);
-static_assert(kSmemBytes <= 113 * 1024, "two CTAs per SM");
+template <int kD>
+constexpr size_t smem_bytes() {
+  return 1024 + 6 * DCfg<kD>::kTileBytes + kSt * kMaskBytes + sizeof(Ctl);
+}
+static_assert(smem_bytes<64>() <= 113 * 1024, "two CTAs per SM at d = 64");
+static_assert(smem_bytes<128>() <= 227 * 1024, "one CTA per SM at d = 128");
 // setmaxnreg applies per warpgroup: warps 0-3 (softmax) grow, warps 4-7 (control) shrink. The
-// pool of one CTA is (65536 / 2 / kThreads) x kThreads registers.
+// pool of one CTA is (65536 / CTAs per SM / kThreads) x kThreads registers.
 constexpr int kRegsCtl = 64, kRegsSoftmax = 192;
 static_assert(128 * kRegsCtl + 128 * kRegsSoftmax <= (65536 / 2 / kThreads & ~7) * kThreads, "register pool");
 
@@ -88,29 +103,31 @@ __device__ __forceinline__ UnitInfo decode_unit(const CoarseParams& p, int u) {
   return {p.n_dense_items + v % nband, v / nband};
 }
 
-// Copy rows idx[0..nvalid) (idx < 0 -> zeros) of a [*, 64] 16-bit matrix into a K-major
-// SWIZZLE_128B tile (row r at r*128 B, 16-byte chunk c at (c ^ (r & 7)) * 16); rows
-// [nvalid, nfill) are zero-filled. One warp; each lane keeps kBatch 16-byte loads in flight.
+// Copy rows idx[0..nvalid) (idx < 0 -> zeros) of a [*, kD] 16-bit matrix into a K-major
+// SWIZZLE_128B tile of kD / 64 sub-tiles (64-column sub-tile s at dst + s * kSub; row r at r*128 B,
+// 16-byte chunk c at (c ^ (r & 7)) * 16); rows [nvalid, nfill) are zero-filled. One warp; each lane
+// keeps kBatch 16-byte loads in flight.
+template <int kD>
 __device__ __forceinline__ void gather_rows(uint32_t dst, const uint16_t* base, int64_t sl, const int32_t* idx,
                                             int nvalid, int nfill, int lane) {
-  constexpr int kBatch = 4;
-  const int total = nfill * 8;
+  constexpr int kBatch = 4, kCh = kD / 8;   // 16-byte chunks per row
+  const int total = nfill * kCh;
   for (int e0 = 0; e0 < total; e0 += 32 * kBatch) {
     int4 val[kBatch];
 #pragma unroll
     for (int k = 0; k < kBatch; ++k) {
-      const int e = e0 + k * 32 + lane, r = e >> 3;
+      const int e = e0 + k * 32 + lane, r = e / kCh;
       val[k] = make_int4(0, 0, 0, 0);
       if (e < total && r < nvalid) {
         const int src = __ldg(idx + r);
-        if (src >= 0) val[k] = ld_nc_v4(base + (int64_t)src * sl + (e & 7) * 8);
+        if (src >= 0) val[k] = ld_nc_v4(base + (int64_t)src * sl + (e % kCh) * 8);
       }
     }
 #pragma unroll
     for (int k = 0; k < kBatch; ++k) {
-      const int e = e0 + k * 32 + lane, r = e >> 3;
+      const int e = e0 + k * 32 + lane, r = e / kCh, ch = e % kCh;
       if (e < total) {
-        const uint32_t a = dst + r * 128 + (((e & 7) ^ (r & 7)) << 4);
+        const uint32_t a = dst + (ch >> 3) * kSub + r * 128 + (((ch & 7) ^ (r & 7)) << 4);
         asm volatile("st.shared.v4.s32 [%0], {%1, %2, %3, %4};" ::"r"(a), "r"(val[k].x), "r"(val[k].y),
                      "r"(val[k].z), "r"(val[k].w)
                      : "memory");
@@ -316,8 +333,9 @@ struct TileCtx {
 // One tile of the online SpSoftmax for this thread's row (NQ x 32 columns): read S(n) from TMEM
 // and release it, mask, row max, lazy rescale decision, then (after P.V(n-1)) rescale O if the
 // max moved and store P(n) = 2^(s*c - m*c) as packed 16-bit pairs, chunk by chunk.
-template <int NQ, bool kBF16>
+template <int NQ, bool kBF16, int kD>
 __device__ __forceinline__ void softmax_tile(const TileCtx& x, float& m, float& l) {
+  constexpr uint32_t kTO = DCfg<kD>::kTO;
   const uint32_t lane = threadIdx.x & 31;
   uint32_t r[NQ][32];
 #pragma unroll
@@ -369,7 +387,7 @@ __device__ __forceinline__ void softmax_tile(const TileCtx& x, float& m, float& 
   tc_fence_after();
   if (x.j > 0 && __any_sync(0xffffffffu, need && alpha != 1.f)) {
 #pragma unroll 1
-    for (int h = 0; h < 4; ++h) {
+    for (int h = 0; h < kD / 16; ++h) {
       uint32_t o[16];
       tmem_ld16(x.tl + kTO + h * 16, o);
       tmem_wait_ld();
@@ -398,8 +416,8 @@ __device__ __forceinline__ void softmax_tile(const TileCtx& x, float& m, float& 
 
 }  // namespace
 
-template <bool kBF16, int kMode, bool kPad>
-__global__ void __launch_bounds__(kThreads, 2)
+template <bool kBF16, int kMode, bool kPad, int kD>
+__global__ void __launch_bounds__(kThreads, DCfg<kD>::kMinBlocks)
     coarse_pp_kernel(const __grid_constant__ CUtensorMap tmq, const __grid_constant__ CUtensorMap tmk,
                      const __grid_constant__ CUtensorMap tmv, const __grid_constant__ CUtensorMap tmq2,
                      const __grid_constant__ CUtensorMap tmk2, const __grid_constant__ CUtensorMap tmv2,
@@ -409,6 +427,8 @@ __global__ void __launch_bounds__(kThreads, 2)
   // the instantiations that need them: their code costs the common path registers and time
   // (measured: 5% on C2 for the batched branches).
   constexpr bool kSplit = kMode == 1, kBatched = kMode == 2, kNoFine = kMode == 3;
+  constexpr uint32_t kTileBytes = DCfg<kD>::kTileBytes, kTmemCols = DCfg<kD>::kTmemCols, kTO = DCfg<kD>::kTO;
+  constexpr int kNSub = DCfg<kD>::kNSub;
   extern __shared__ uint8_t smem_raw[];
   const uint32_t sbase = (smem_u32(smem_raw) + 1023u) & ~1023u;
   const uint32_t sQ = sbase;
@@ -486,16 +506,20 @@ __global__ void __launch_bounds__(kThreads, 2)
       if (item.kind == 0) {
         if (lane == 0) {
           mbar_arrive_expect_tx(qf, kTileBytes);
-          tma_load_4d(dQ, &tmq, qf, 0, item.rowA, hh, bb, pol_q);
+#pragma unroll
+          for (int sb = 0; sb < kNSub; ++sb) tma_load_4d(dQ + sb * kSub, &tmq, qf, 64 * sb, item.rowA, hh, bb, pol_q);
         }
       } else if (p.gather_tma) {
         if (lane == 0) mbar_arrive_expect_tx(qf, kTileBytes);
         __syncwarp();
         const int4 ix = load_idx4(p.global_rows + item.rowA, 4 * lane, item.nrowsA);
-        gather4(dQ + lane * 512, &tmq2, qf, row_coords(ix, bb * p.rq.x + hh * p.rq.y, p.rq.z), pol_q);
+#pragma unroll
+        for (int sb = 0; sb < kNSub; ++sb)
+          gather4(dQ + sb * kSub + lane * 512, &tmq2, qf, row_coords(ix, bb * p.rq.x + hh * p.rq.y + sb, p.rq.z),
+                  pol_q);
       } else {
-        gather_rows(dQ, p.q.data + bb * p.q.sb + hh * p.q.sh, p.q.sl, p.global_rows + item.rowA, item.nrowsA, 128,
-                    lane);
+        gather_rows<kD>(dQ, p.q.data + bb * p.q.sb + hh * p.q.sh, p.q.sl, p.global_rows + item.rowA, item.nrowsA,
+                        128, lane);
         fence_proxy_async_smem();
         __syncwarp();
         if (lane == 0) mbar_arrive(qf);
@@ -525,14 +549,21 @@ __global__ void __launch_bounds__(kThreads, 2)
           if (kind == 0) {
             if (lane == 0) {
               mbar_arrive_expect_tx(kf, kDbgNoLoads ? 0 : kTileBytes);
-              if (!kDbgNoLoads) tma_load_4d(dK, &tmk, kf, 0, arg, hh, bb, pol_kv);
+              if (!kDbgNoLoads) {
+#pragma unroll
+                for (int sb = 0; sb < kNSub; ++sb) tma_load_4d(dK + sb * kSub, &tmk, kf, 64 * sb, arg, hh, bb, pol_kv);
+              }
             }
           } else if (p.gather_tma) {
-            if (lane == 0) mbar_arrive_expect_tx(kf, ncols * 128);
+            if (lane == 0) mbar_arrive_expect_tx(kf, ncols * 2 * kD);
             __syncwarp();
-            if (4 * lane < ncols) gather4(dK + lane * 512, &tmk2, kf, row_coords(six, krow0, p.rk.z), pol_kv);
+            if (4 * lane < ncols) {
+#pragma unroll
+              for (int sb = 0; sb < kNSub; ++sb)
+                gather4(dK + sb * kSub + lane * 512, &tmk2, kf, row_coords(six, krow0 + sb, p.rk.z), pol_kv);
+            }
           } else {
-            gather_rows(dK, p.k.data + bb * p.k.sb + hh * p.k.sh, p.k.sl, p.strip_cols + arg, ncols, ncols, lane);
+            gather_rows<kD>(dK, p.k.data + bb * p.k.sb + hh * p.k.sh, p.k.sl, p.strip_cols + arg, ncols, ncols, lane);
             fence_proxy_async_smem();
             __syncwarp();
             if (lane == 0) mbar_arrive(kf);
@@ -579,14 +610,21 @@ __global__ void __launch_bounds__(kThreads, 2)
           if (kind == 0) {
             if (lane == 0) {
               mbar_arrive_expect_tx(vf, (kDbgNoLoads ? 0 : kTileBytes) + mbytes);
-              if (!kDbgNoLoads) tma_load_4d(dV, &tmv, vf, 0, arg, hh, bb, pol_kv);
+              if (!kDbgNoLoads) {
+#pragma unroll
+                for (int sb = 0; sb < kNSub; ++sb) tma_load_4d(dV + sb * kSub, &tmv, vf, 64 * sb, arg, hh, bb, pol_kv);
+              }
             }
           } else if (p.gather_tma) {
-            if (lane == 0) mbar_arrive_expect_tx(vf, ncols * 128 + mbytes);
+            if (lane == 0) mbar_arrive_expect_tx(vf, ncols * 2 * kD + mbytes);
             __syncwarp();
-            if (4 * lane < ncols) gather4(dV + lane * 512, &tmv2, vf, row_coords(six, vrow0, p.rv.z), pol_kv);
+            if (4 * lane < ncols) {
+#pragma unroll
+              for (int sb = 0; sb < kNSub; ++sb)
+                gather4(dV + sb * kSub + lane * 512, &tmv2, vf, row_coords(six, vrow0 + sb, p.rv.z), pol_kv);
+            }
           } else {
-            gather_rows(dV, p.v.data + bb * p.v.sb + hh * p.v.sh, p.v.sl, p.strip_cols + arg, ncols, ncols, lane);
+            gather_rows<kD>(dV, p.v.data + bb * p.v.sb + hh * p.v.sh, p.v.sl, p.strip_cols + arg, ncols, ncols, lane);
             fence_proxy_async_smem();
             __syncwarp();
             if (lane == 0) mbar_arrive_expect_tx(vf, mbytes);
@@ -645,10 +683,13 @@ __global__ void __launch_bounds__(kThreads, 2)
         tl_rec(p, e.n, 7);
         tc_fence_after();
         const uint32_t vA = sV + e.st * kTileBytes;
-        // chunk c (16 keys): P at columns [kTP + 8c, kTP + 8c + 8) (packed pairs), V rows [16c, 16c + 16)
-        for (int c = 0; c < (kDbgNoMma ? 0 : e.ncols >> 4); ++c)
-          mma_ts(tmem + kTO, tmem + kTP + c * 8, smem_desc_sw128(vA + c * 2048, 8192, 1024), idesc_pv,
-                 (e.first && c == 0) ? 0u : 1u);
+        // chunk c (16 keys): P at columns [kTP + 8c, kTP + 8c + 8) (packed pairs), V rows [16c, 16c + 16);
+        // one N = 64 MMA per 64-column V sub-tile (O columns [kTO + 64 sb, kTO + 64 sb + 64))
+#pragma unroll
+        for (int sb = 0; sb < kNSub; ++sb)
+          for (int c = 0; c < (kDbgNoMma ? 0 : e.ncols >> 4); ++c)
+            mma_ts(tmem + kTO + 64 * sb, tmem + kTP + c * 8, smem_desc_sw128(vA + sb * kSub + c * 2048, 8192, 1024),
+                   idesc_pv, (e.first && c == 0) ? 0u : 1u);
         tl_rec(p, e.n, 4);
         mma_commit(bar(ctl->pv_done));
         mma_commit(bar(ctl->v_empty[e.st]));
@@ -681,9 +722,11 @@ __global__ void __launch_bounds__(kThreads, 2)
           const uint32_t idesc_s = idesc_f16(kBF16, 128, ncols, false, false);
           const uint32_t kA = sK + st * kTileBytes;
 #pragma unroll
-          for (int kk = 0; kk < (kDbgNoMma ? 0 : 4); ++kk)
-            mma_ss(tmem + kTS, smem_desc_sw128(qa + kk * 32, 16, 1024), smem_desc_sw128(kA + kk * 32, 16, 1024),
-                   idesc_s, kk > 0);
+          for (int kk = 0; kk < (kDbgNoMma ? 0 : kD / 16); ++kk) {
+            const uint32_t ko = (kk >> 2) * kSub + (kk & 3) * 32;   // K step kk: sub-tile kk / 4, 32 B each
+            mma_ss(tmem + kTS, smem_desc_sw128(qa + ko, 16, 1024), smem_desc_sw128(kA + ko, 16, 1024), idesc_s,
+                   kk > 0);
+          }
           mma_commit(bar(ctl->s_full));
           mma_commit(bar(ctl->k_empty[st]));
           // (q_empty is arrived by the softmax epilogue: the Q buffer also stages the item's O tile)
@@ -752,13 +795,14 @@ __global__ void __launch_bounds__(kThreads, 2)
                          bar(ctl->pv_done), bar(ctl->p_full), c, thresh, &p};
         if (threadIdx.x == 0) tl_rec(p, n, 0);
         switch (desc.x >> 5) {                            // 32-column chunks of the tile
-          case 4: softmax_tile<4, kBF16>(tc, m, l); break;
-          case 3: softmax_tile<3, kBF16>(tc, m, l); break;
-          case 2: softmax_tile<2, kBF16>(tc, m, l); break;
-          default: softmax_tile<1, kBF16>(tc, m, l); break;
+          case 4: softmax_tile<4, kBF16, kD>(tc, m, l); break;
+          case 3: softmax_tile<3, kBF16, kD>(tc, m, l); break;
+          case 2: softmax_tile<2, kBF16, kD>(tc, m, l); break;
+          default: softmax_tile<1, kBF16, kD>(tc, m, l); break;
         }
       }
       // ---------------------------------------------------------------- epilogue (a-8)
+      // O is processed in kD / 64 halves of 64 columns (d = 64: one, read once up front)
       float mf = -INFINITY, lf = 0.f;
       const float4* accf = nullptr;
       const size_t fidx = (size_t)(kBatched ? ubh % p.H : ubh) * p.n_fine_rows + slot_f;
@@ -766,32 +810,44 @@ __global__ void __launch_bounds__(kThreads, 2)
         const float2 ml = p.part_ml[fidx];
         mf = ml.x;
         lf = ml.y;
-        accf = reinterpret_cast<const float4*>(p.part_acc + fidx * 64);
+        accf = reinterpret_cast<const float4*>(p.part_acc + fidx * kD);
       }
       if (threadIdx.x == 0) tl_rec(p, n - 1, 11);
       mbar_wait(bar(ctl->pv_done), (n - 1) & 1);          // the item's last P.V
       tc_fence_after();
       uint32_t o[2][32];
-      tmem_ld32(tl + kTO, o[0]);
-      tmem_ld32(tl + kTO + 32, o[1]);
-      tmem_wait_ld();
-      tc_fence_before();
+      auto load_o = [&](int sb) {
+        tmem_ld32(tl + kTO + 64 * sb, o[0]);
+        tmem_ld32(tl + kTO + 64 * sb + 32, o[1]);
+        tmem_wait_ld();
+      };
+      if (kNSub == 1) load_o(0);
       if (threadIdx.x == 0) tl_rec(p, n - 1, 12);
       bool skip = false;
+      // split dense-row item whose chunk finishes its group last: O is merged from the chunk partials
+      bool merge_chunks = false;
+      const float* chunk_base = nullptr;
+      float mu0 = 0.f;
+      constexpr int kPartStride = kD + 4;                 // acc[kD], m, l, pad (16-byte rows)
       if (kSplit && item.kind == 1 && item.nrowsB > 1) {
         // split dense-row item: publish this chunk's (m, l, acc) per row; the chunk that finishes
         // its row group last merges all chunks by log-sum-exp and writes O (a-4 over column chunks)
         const size_t gidx = (size_t)ubh * p.n_dense_groups + item.rowB;
-        float* part = p.dense_part + ((gidx * p.dense_nsplit + item.turns) * 128 + t) * 68;
-        if (t < item.nrowsA) {
-          float4* dst = reinterpret_cast<float4*>(part);
+        float* part = p.dense_part + ((gidx * p.dense_nsplit + item.turns) * 128 + t) * kPartStride;
+        // (tcgen05.ld is warp-collective: every lane loads, only valid rows store)
 #pragma unroll
-          for (int i = 0; i < 16; ++i)
-            __stcg(dst + i, make_float4(__uint_as_float(o[i >> 3][(i & 7) * 4]), __uint_as_float(o[i >> 3][(i & 7) * 4 + 1]),
-                                        __uint_as_float(o[i >> 3][(i & 7) * 4 + 2]),
-                                        __uint_as_float(o[i >> 3][(i & 7) * 4 + 3])));
-          __stcg(reinterpret_cast<float2*>(part + 64), make_float2(m, l));
+        for (int sb = 0; sb < kNSub; ++sb) {
+          if (kNSub > 1) load_o(sb);
+          if (t < item.nrowsA) {
+            float4* dst = reinterpret_cast<float4*>(part + 64 * sb);
+#pragma unroll
+            for (int i = 0; i < 16; ++i)
+              __stcg(dst + i, make_float4(__uint_as_float(o[i >> 3][(i & 7) * 4]), __uint_as_float(o[i >> 3][(i & 7) * 4 + 1]),
+                                          __uint_as_float(o[i >> 3][(i & 7) * 4 + 2]),
+                                          __uint_as_float(o[i >> 3][(i & 7) * 4 + 3])));
+          }
         }
+        if (t < item.nrowsA) __stcg(reinterpret_cast<float2*>(part + kD), make_float2(m, l));
         __threadfence();
         named_bar_sync(1, 128);
         // per-group chunk counter in [0, nrowsB): atomicInc wraps it back to 0 on the last chunk, so it
@@ -803,20 +859,86 @@ __global__ void __launch_bounds__(kThreads, 2)
         skip = !ctl->dense_last;
         if (!skip && t < item.nrowsA) {
           __threadfence();
-          const float* base = p.dense_part + (gidx * p.dense_nsplit * 128 + t) * 68;
+          chunk_base = p.dense_part + (gidx * p.dense_nsplit * 128 + t) * kPartStride;
           float mm = -INFINITY;
-          for (int k = 0; k < item.nrowsB; ++k) mm = fmaxf(mm, __ldcg(base + (size_t)k * 128 * 68 + 64));
-          const float mu0 = mm == -INFINITY ? 0.f : mm;
-          // merged row accumulated in place of this chunk's O registers
+          for (int k = 0; k < item.nrowsB; ++k) mm = fmaxf(mm, __ldcg(chunk_base + (size_t)k * 128 * kPartStride + kD));
+          mu0 = mm == -INFINITY ? 0.f : mm;
+          float den0 = 0.f;
+          for (int k = 0; k < item.nrowsB; ++k)
+            den0 += __ldcg(chunk_base + (size_t)k * 128 * kPartStride + kD + 1) *
+                    ex2((__ldcg(chunk_base + (size_t)k * 128 * kPartStride + kD) - mu0) * c);
+          // the merged row goes through the common store below: O = merged (scale 1), l = den0, m = mm
+          merge_chunks = true;
+          m = mm;
+          l = den0;
+        }
+      }
+      if (kNSub > 1 && p.concurrent) {
+        // (tcgen05.ld is warp-collective: the d = 128 halves are loaded by every lane, stored below
+        // by the rows with a CUDA-core CSR part)
+#pragma unroll
+        for (int sb = 0; sb < kNSub; ++sb) {
+          load_o(sb);
+          if (slot_f >= 0) {
+            float4* dst = reinterpret_cast<float4*>(p.part_c_acc + fidx * kD + 64 * sb);
+#pragma unroll
+            for (int i = 0; i < 16; ++i)
+              __stcg(dst + i, make_float4(__uint_as_float(o[i >> 3][(i & 7) * 4]), __uint_as_float(o[i >> 3][(i & 7) * 4 + 1]),
+                                          __uint_as_float(o[i >> 3][(i & 7) * 4 + 2]), __uint_as_float(o[i >> 3][(i & 7) * 4 + 3])));
+          }
+        }
+      }
+      if (slot_f >= 0 && p.concurrent) {
+        // publish this row's coarse partial; the side that finishes the row second merges both
+        if (kNSub == 1) {
+          float4* dst = reinterpret_cast<float4*>(p.part_c_acc + fidx * kD);
+#pragma unroll
+          for (int i = 0; i < 16; ++i)
+            __stcg(dst + i, make_float4(__uint_as_float(o[i >> 3][(i & 7) * 4]), __uint_as_float(o[i >> 3][(i & 7) * 4 + 1]),
+                                        __uint_as_float(o[i >> 3][(i & 7) * 4 + 2]), __uint_as_float(o[i >> 3][(i & 7) * 4 + 3])));
+        }
+        __stcg(p.part_c_ml + fidx, make_float2(m, l));
+        __threadfence();
+        const int old = atomicAdd(p.part_flags + fidx, 1);
+        if (old & 1) {
+          __threadfence();
+          const float2 ml = __ldcg(p.part_ml + fidx);
+          mf = ml.x;
+          lf = ml.y;
+          accf = reinterpret_cast<const float4*>(p.part_acc + fidx * kD);
+        } else {
+          skip = true;
+        }
+      }
+      const float mt = fmaxf(m, mf);
+      const float mu = mt == -INFINITY ? 0.f : mt;
+      const float ac = ex2((m - mu) * c), af = ex2((mf - mu) * c);
+      const float den = l * ac + lf * af;
+      // normalised row -> 16-bit, 8 x 16-byte stores per 64 columns of this thread's row. A row with
+      // no valid element in this item (a global row inside a band row block: it is owned by the
+      // dense-row part, A5) is not written. (Staging the tile through shared memory for 4-rows-per-
+      // instruction stores measured 10% slower: tools/experiments/.)
+      // padding (A18): rows at or beyond the batch element's valid length are written as 0 by
+      // every item that holds them (whatever the merge protocol decided)
+      const bool pad_row = kPad && r_out >= 0 &&
+                           r_out >= min(max(__ldg(p.valid_len + ubh / p.H), 0), (int)p.L);
+      // (only blocks without global rows and without CUDA-core CSR rows: no other writer, no partial
+      // to merge; measured: merging partials in this path costs C2 3% and gains nothing on C4)
+      const bool tma_out = !kPad && p.tma_store && item.kind == 0 && (item.useA & 3) == 3;   // uniform per item
+      const bool write_row = !tma_out && !pad_row && r_out >= 0 && mt != -INFINITY && !skip;
+      const int bb = ubh / p.H, hh = ubh % p.H;
+      uint16_t* orow = p.o.data + bb * p.o.sb + hh * p.o.sh + (int64_t)max(r_out, 0) * p.o.sl;
+      const uint32_t sO = sQ + (it & 1) * kTileBytes;
+#pragma unroll
+      for (int sb = 0; sb < kNSub; ++sb) {
+        if (kNSub > 1) load_o(sb);   // (warp-collective: every lane, before any per-row choice)
+        if (merge_chunks) {
 #pragma unroll
           for (int i = 0; i < 64; ++i) o[i >> 5][i & 31] = 0u;
-          float den0 = 0.f;
           for (int k = 0; k < item.nrowsB; ++k) {
-            const float* pk = base + (size_t)k * 128 * 68;
-            const float2 ml = __ldcg(reinterpret_cast<const float2*>(pk + 64));
-            const float a = ex2((ml.x - mu0) * c);
-            den0 += ml.y * a;
-            const float4* src = reinterpret_cast<const float4*>(pk);
+            const float* pk = chunk_base + (size_t)k * 128 * kPartStride;
+            const float a = ex2((__ldcg(pk + kD) - mu0) * c);
+            const float4* src = reinterpret_cast<const float4*>(pk + 64 * sb);
 #pragma unroll
             for (int i = 0; i < 16; ++i) {
               const float4 v = __ldcg(src + i);
@@ -827,108 +949,70 @@ __global__ void __launch_bounds__(kThreads, 2)
               q4[3] = __float_as_uint(fmaf(v.w, a, __uint_as_float(q4[3])));
             }
           }
-          // hand the merged row to the common store below: O = o (scale 1), l = den0, m = mm
-          m = mm;
-          l = den0;
         }
-      }
-      if (slot_f >= 0 && p.concurrent) {
-        // publish this row's coarse partial; the side that finishes the row second merges both
-        float4* dst = reinterpret_cast<float4*>(p.part_c_acc + fidx * 64);
+        if (tma_out) {
+          // normalised rows into the item's Q buffer (SWIZZLE_128B layout of the O tensor map), then one
+          // TMA store per 128 x 64 sub-tile (rows beyond L are clipped by the map)
+          const float inv = (r_out >= 0 && mt != -INFINITY) ? __frcp_rn(den) : 0.f;
 #pragma unroll
-        for (int i = 0; i < 16; ++i)
-          __stcg(dst + i, make_float4(__uint_as_float(o[i >> 3][(i & 7) * 4]), __uint_as_float(o[i >> 3][(i & 7) * 4 + 1]),
-                                      __uint_as_float(o[i >> 3][(i & 7) * 4 + 2]), __uint_as_float(o[i >> 3][(i & 7) * 4 + 3])));
-        __stcg(p.part_c_ml + fidx, make_float2(m, l));
-        __threadfence();
-        const int old = atomicAdd(p.part_flags + fidx, 1);
-        if (old & 1) {
-          __threadfence();
-          const float2 ml = __ldcg(p.part_ml + fidx);
-          mf = ml.x;
-          lf = ml.y;
-          accf = reinterpret_cast<const float4*>(p.part_acc + fidx * 64);
-        } else {
-          skip = true;
-        }
-      }
-      const float mt = fmaxf(m, mf);
-      const float mu = mt == -INFINITY ? 0.f : mt;
-      const float ac = ex2((m - mu) * c), af = ex2((mf - mu) * c);
-      const float den = l * ac + lf * af;
-      // normalised row -> 16-bit, 8 x 16-byte stores of this thread's row. A row with no valid
-      // element in this item (a global row inside a band row block: it is owned by the dense-row
-      // part, A5) is not written. (Staging the tile through shared memory for 4-rows-per-
-      // instruction stores measured 10% slower: tools/experiments/.)
-      // padding (A18): rows at or beyond the batch element's valid length are written as 0 by
-      // every item that holds them (whatever the merge protocol decided)
-      const bool pad_row = kPad && r_out >= 0 &&
-                           r_out >= min(max(__ldg(p.valid_len + ubh / p.H), 0), (int)p.L);
-      // (only blocks without global rows and without CUDA-core CSR rows: no other writer, no partial
-      // to merge; measured: merging partials in this path costs C2 3% and gains nothing on C4)
-      const bool tma_out = !kPad && p.tma_store && item.kind == 0 && (item.useA & 3) == 3;   // uniform per item
-      if (tma_out) {
-        // normalised rows into the item's Q buffer (SWIZZLE_128B layout of the O tensor map), then one
-        // TMA store of the 128 x 64 tile (rows beyond L are clipped by the map)
-        const uint32_t sO = sQ + (it & 1) * kTileBytes;
-        const float inv = (r_out >= 0 && mt != -INFINITY) ? __frcp_rn(den) : 0.f;
+          for (int h = 0; h < 2; ++h) {
 #pragma unroll
-        for (int h = 0; h < 2; ++h) {
+            for (int q8 = 0; q8 < 4; ++q8) {
+              float a[8];
 #pragma unroll
-          for (int q8 = 0; q8 < 4; ++q8) {
-            float a[8];
+              for (int i = 0; i < 8; ++i) a[i] = __uint_as_float(o[h][q8 * 8 + i]) * (ac * inv);
+              const int ch = h * 4 + q8;
+              asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(sO + sb * kSub + t * 128 + ((ch ^ (t & 7)) << 4)),
+                           "r"(pack2<kBF16>(a[0], a[1])), "r"(pack2<kBF16>(a[2], a[3])), "r"(pack2<kBF16>(a[4], a[5])),
+                           "r"(pack2<kBF16>(a[6], a[7]))
+                           : "memory");
+            }
+          }
+        } else if (pad_row) {
+          uint4* o16 = reinterpret_cast<uint4*>(orow + 64 * sb);
 #pragma unroll
-            for (int i = 0; i < 8; ++i) a[i] = __uint_as_float(o[h][q8 * 8 + i]) * (ac * inv);
-            const int ch = h * 4 + q8;
-            asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(sO + t * 128 + ((ch ^ (t & 7)) << 4)),
-                         "r"(pack2<kBF16>(a[0], a[1])), "r"(pack2<kBF16>(a[2], a[3])), "r"(pack2<kBF16>(a[4], a[5])),
-                         "r"(pack2<kBF16>(a[6], a[7]))
-                         : "memory");
+          for (int i = 0; i < 8; ++i) o16[i] = make_uint4(0u, 0u, 0u, 0u);
+        } else if (write_row) {
+          const float inv = __frcp_rn(den);
+#pragma unroll
+          for (int h = 0; h < 2; ++h) {
+#pragma unroll
+            for (int q8 = 0; q8 < 4; ++q8) {
+              float a[8];
+#pragma unroll
+              for (int i = 0; i < 8; ++i) a[i] = __uint_as_float(o[h][q8 * 8 + i]) * ac;
+              if (accf) {
+                const float4 f0 = __ldcg(accf + 16 * sb + h * 8 + q8 * 2), f1 = __ldcg(accf + 16 * sb + h * 8 + q8 * 2 + 1);
+                a[0] = fmaf(f0.x, af, a[0]);
+                a[1] = fmaf(f0.y, af, a[1]);
+                a[2] = fmaf(f0.z, af, a[2]);
+                a[3] = fmaf(f0.w, af, a[3]);
+                a[4] = fmaf(f1.x, af, a[4]);
+                a[5] = fmaf(f1.y, af, a[5]);
+                a[6] = fmaf(f1.z, af, a[6]);
+                a[7] = fmaf(f1.w, af, a[7]);
+              }
+              uint4 o4;
+              o4.x = pack2<kBF16>(a[0] * inv, a[1] * inv);
+              o4.y = pack2<kBF16>(a[2] * inv, a[3] * inv);
+              o4.z = pack2<kBF16>(a[4] * inv, a[5] * inv);
+              o4.w = pack2<kBF16>(a[6] * inv, a[7] * inv);
+              *reinterpret_cast<uint4*>(orow + 64 * sb + h * 32 + q8 * 8) = o4;
+            }
           }
         }
+      }
+      if (tma_out) {
         fence_proxy_async_smem();
         named_bar_sync(1, 128);
         if (threadIdx.x == 0) {
-          tma_store_4d(&tmo, sO, 0, item.rowA, ubh % p.H, ubh / p.H);
+#pragma unroll
+          for (int sb = 0; sb < kNSub; ++sb) tma_store_4d(&tmo, sO + sb * kSub, 64 * sb, item.rowA, hh, bb);
           bulk_commit_group();
           bulk_wait_group_read0();   // the buffer is reloaded with a later item's Q after q_empty
         }
-      } else if (pad_row) {
-        const int bb = ubh / p.H, hh = ubh % p.H;
-        uint4* orow = reinterpret_cast<uint4*>(p.o.data + bb * p.o.sb + hh * p.o.sh + (int64_t)r_out * p.o.sl);
-#pragma unroll
-        for (int i = 0; i < 8; ++i) orow[i] = make_uint4(0u, 0u, 0u, 0u);
-      } else if (r_out >= 0 && mt != -INFINITY && !skip) {
-        const float inv = __frcp_rn(den);
-        const int bb = ubh / p.H, hh = ubh % p.H;
-        uint16_t* orow = p.o.data + bb * p.o.sb + hh * p.o.sh + (int64_t)r_out * p.o.sl;
-#pragma unroll
-        for (int h = 0; h < 2; ++h) {
-#pragma unroll
-          for (int q8 = 0; q8 < 4; ++q8) {
-            float a[8];
-#pragma unroll
-            for (int i = 0; i < 8; ++i) a[i] = __uint_as_float(o[h][q8 * 8 + i]) * ac;
-            if (accf) {
-              const float4 f0 = __ldcg(accf + h * 8 + q8 * 2), f1 = __ldcg(accf + h * 8 + q8 * 2 + 1);
-              a[0] = fmaf(f0.x, af, a[0]);
-              a[1] = fmaf(f0.y, af, a[1]);
-              a[2] = fmaf(f0.z, af, a[2]);
-              a[3] = fmaf(f0.w, af, a[3]);
-              a[4] = fmaf(f1.x, af, a[4]);
-              a[5] = fmaf(f1.y, af, a[5]);
-              a[6] = fmaf(f1.z, af, a[6]);
-              a[7] = fmaf(f1.w, af, a[7]);
-            }
-            uint4 o4;
-            o4.x = pack2<kBF16>(a[0] * inv, a[1] * inv);
-            o4.y = pack2<kBF16>(a[2] * inv, a[3] * inv);
-            o4.z = pack2<kBF16>(a[4] * inv, a[5] * inv);
-            o4.w = pack2<kBF16>(a[6] * inv, a[7] * inv);
-            *reinterpret_cast<uint4*>(orow + h * 32 + q8 * 8) = o4;
-          }
-        }
       }
+      tc_fence_before();
       // the item's Q buffer is free (its last S MMA has completed: pv_done above; its O tile, if
       // staged there, has been read by the TMA store)
       if (threadIdx.x == 0) {
@@ -960,20 +1044,26 @@ cudaError_t launch_coarse_pp(const CoarseParams& p, const CUtensorMap& tmq, cons
   // that need them (their code costs the common path registers)
   using K = void (*)(const CUtensorMap, const CUtensorMap, const CUtensorMap, const CUtensorMap, const CUtensorMap,
                      const CUtensorMap, const CUtensorMap, const CoarseParams);
-  static const K table[16] = {coarse_pp_kernel<false, 0, false>, coarse_pp_kernel<false, 0, true>,
-                              coarse_pp_kernel<false, 1, false>, coarse_pp_kernel<false, 1, true>,
-                              coarse_pp_kernel<false, 2, false>, coarse_pp_kernel<false, 2, true>,
-                              coarse_pp_kernel<false, 3, false>, coarse_pp_kernel<false, 3, true>,
-                              coarse_pp_kernel<true, 0, false>,  coarse_pp_kernel<true, 0, true>,
-                              coarse_pp_kernel<true, 1, false>,  coarse_pp_kernel<true, 1, true>,
-                              coarse_pp_kernel<true, 2, false>,  coarse_pp_kernel<true, 2, true>,
-                              coarse_pp_kernel<true, 3, false>,  coarse_pp_kernel<true, 3, true>};
+#define MG_PP_ROW(D)                                                                                            \
+  coarse_pp_kernel<false, 0, false, D>, coarse_pp_kernel<false, 0, true, D>, coarse_pp_kernel<false, 1, false, D>, \
+      coarse_pp_kernel<false, 1, true, D>, coarse_pp_kernel<false, 2, false, D>, coarse_pp_kernel<false, 2, true, D>, \
+      coarse_pp_kernel<false, 3, false, D>, coarse_pp_kernel<false, 3, true, D>, coarse_pp_kernel<true, 0, false, D>, \
+      coarse_pp_kernel<true, 0, true, D>, coarse_pp_kernel<true, 1, false, D>, coarse_pp_kernel<true, 1, true, D>,    \
+      coarse_pp_kernel<true, 2, false, D>, coarse_pp_kernel<true, 2, true, D>, coarse_pp_kernel<true, 3, false, D>,   \
+      coarse_pp_kernel<true, 3, true, D>
+  static const K table[32] = {MG_PP_ROW(64), MG_PP_ROW(128)};
+#undef MG_PP_ROW
+  if (p.d != 64 && p.d != 128) return cudaErrorInvalidValue;
   const int mode = p.batched ? 2 : (split_dense ? 1 : (p.n_fine_rows == 0 ? 3 : 0));
-  const K kern = table[(bf16 ? 8 : 0) + 2 * mode + (p.valid_len ? 1 : 0)];
-  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBytes);
+  const K kern = table[(p.d == 128 ? 16 : 0) + (bf16 ? 8 : 0) + 2 * mode + (p.valid_len ? 1 : 0)];
+  const int smem = (int)(p.d == 128 ? smem_bytes<128>() : smem_bytes<64>());
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (e != cudaSuccess) return e;
-  kern<<<grid, kThreads, kSmemBytes, stream>>>(tmq, tmk, tmv, tmq2, tmk2, tmv2, tmo, p);
+  kern<<<grid, kThreads, smem, stream>>>(tmq, tmk, tmv, tmq2, tmk2, tmv2, tmo, p);
   return cudaGetLastError();
 }
+
+// CTAs per SM of the persistent grid for head dimension d
+int coarse_pp_ctas_per_sm(int d) { return d == 128 ? DCfg<128>::kMinBlocks : DCfg<64>::kMinBlocks; }
 
 }  // namespace mg

@@ -92,9 +92,18 @@ constexpr int kWarps = MG_FINE_WARPS;       // warps per block, each a persisten
 constexpr int kP = MG_FINE_PAIRS;           // 16-nnz pairs of 8-nnz chunks per step (1 or 2)
 constexpr int kS = 16 * kP;                 // nnz per step
 constexpr int kStages = MG_FINE_STAGES;     // smem ring stages per warp (kStages - 1 steps in flight)
-constexpr int kQOff = 2 * kS * 128;        // the q row of a row's first step follows its K and V rows
-constexpr int kStageBytes = kQOff + 128;   // kS K rows + kS V rows + q, 128 bytes each
-constexpr int kSmemBytes = kWarps * kStages * kStageBytes;
+// Head dimension kD = 64 or 128: a gathered row is kD * 2 bytes, copied by kD / 8 lanes
+// (16 B each), 32 / (kD / 8) rows per cp.async instruction.
+template <int kD>
+struct FCfg {
+  static constexpr int kRowBytes = kD * 2;
+  static constexpr int kLPR = kD / 8;                   // lanes per gathered row
+  static constexpr int kRPI = 32 / kLPR;                // rows per cp.async instruction
+  static constexpr int kQOff = 2 * kS * kRowBytes;      // the q row of a row's first step follows its K and V rows
+  static constexpr int kStageBytes = kQOff + kRowBytes; // kS K rows + kS V rows + q
+  static constexpr int kSmemBytes = kWarps * kStages * kStageBytes;
+  static constexpr int kMinB = kD == 64 ? MG_FINE_MINB : 3;
+};
 
 }  // namespace
 
@@ -122,8 +131,12 @@ __device__ __forceinline__ void split_row(int64_t g, int n, bool r32, int& u0, i
   }
 }
 
-template <bool kBF16, bool kPad>
-__global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(const FineParams p) {
+template <bool kBF16, bool kPad, int kD>
+__global__ void __launch_bounds__(kWarps * 32, FCfg<kD>::kMinB) fine_mma_kernel(const FineParams p) {
+  using F = FCfg<kD>;
+  constexpr int kRowBytes = F::kRowBytes, kLPR = F::kLPR, kRPI = F::kRPI, kQOff = F::kQOff;
+  constexpr int kStageBytes = F::kStageBytes;
+  constexpr int kJ = kD / 16;                           // k16 steps of the SDDMM = m16 blocks of the SpMM
   extern __shared__ __align__(128) uint8_t fsm[];
   const int lane = threadIdx.x & 31;
   const int g = lane >> 2, t = lane & 3;
@@ -136,11 +149,12 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(con
   const uint32_t ring = (uint32_t)__cvta_generic_to_shared(fsm) + (threadIdx.x >> 5) * (kStages * kStageBytes);
   // row strides fit 32 bits (checked by the forward's validation: (L - 1) * stride_l < 2^32)
   const uint32_t ksl = (uint32_t)p.k.sl, vsl = (uint32_t)p.v.sl;
-  uint32_t doff[4 * kP];   // swizzled destination of this lane's chunk in rows R_i = (lane >> 3) + 4 i
+  constexpr int kIters = kS / kRPI;   // cp.async instructions per lane per step (each of K and V)
+  uint32_t doff[kIters];   // swizzled destination of this lane's chunk in rows R_i = lane / kLPR + kRPI i
 #pragma unroll
-  for (int i = 0; i < 4 * kP; ++i) {
-    const int R = (lane >> 3) + 4 * i;
-    doff[i] = R * 128 + (((lane & 7) ^ (R & 7)) << 4);
+  for (int i = 0; i < kIters; ++i) {
+    const int R = lane / kLPR + kRPI * i;
+    doff[i] = R * kRowBytes + (((lane % kLPR) ^ (R & 7)) << 4);
   }
 
   // ---- gather pointer: row gi (global work index), step is of [ibeg, iend)
@@ -155,10 +169,10 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(con
       ibeg = __ldg(p.row_ptr + fi);
       iend = __ldg(p.row_ptr + fi + 1);
       const int bb = bh / p.H, hh = bh % p.H;
-      iK = p.k.data + bb * p.k.sb + hh * p.k.sh + (lane & 7) * 8;
-      iV = p.v.data + bb * p.v.sb + hh * p.v.sh + (lane & 7) * 8;
+      iK = p.k.data + bb * p.k.sb + hh * p.k.sh + (lane % kLPR) * 8;
+      iV = p.v.data + bb * p.v.sb + hh * p.v.sh + (lane % kLPR) * 8;
       const int rq = __ldg(p.fine_rows + fi) & 0x7fffffff;
-      iQ = p.q.data + bb * p.q.sb + hh * p.q.sh + (int64_t)rq * p.q.sl + (lane & 7) * 8;
+      iQ = p.q.data + bb * p.q.sb + hh * p.q.sh + (int64_t)rq * p.q.sl + (lane % kLPR) * 8;
     }
     is = 0;
   };
@@ -171,16 +185,16 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(con
     if (gi < nrows) {   // warp-uniform
       const int nb0 = ibeg + kS * is;
       if (kP == 2 || (is & 1) == 0) icol = nb0 + lane < iend ? __ldg(p.cols + nb0 + lane) : -1;
-      const int off = (kP == 2 ? 0 : (is & 1) * 16) + (lane >> 3);
+      const int off = (kP == 2 ? 0 : (is & 1) * 16) + lane / kLPR;
       const uint32_t st = ring + stg * kStageBytes;
-      // a row's first step also carries its q row (lanes 0-7, 16 B each), so the computing side
-      // never waits on a dependent q load at a row start
-      if (is == 0 && lane < 8) cp_async16(st + kQOff + (lane << 4), iQ);
+      // a row's first step also carries its q row (lanes 0 .. kLPR-1, 16 B each), so the computing
+      // side never waits on a dependent q load at a row start
+      if (is == 0 && lane < kLPR) cp_async16(st + kQOff + (lane << 4), iQ);
 #pragma unroll
-      for (int i = 0; i < 4 * kP; ++i) {
-        const uint32_t cc = (uint32_t)max(__shfl_sync(0xffffffffu, icol, off + 4 * i), 0);
+      for (int i = 0; i < kIters; ++i) {
+        const uint32_t cc = (uint32_t)max(__shfl_sync(0xffffffffu, icol, off + kRPI * i), 0);
         cp_async16(st + doff[i], iK + cc * ksl);
-        cp_async16(st + doff[i] + kS * 128, iV + cc * vsl);
+        cp_async16(st + doff[i] + kS * kRowBytes, iV + cc * vsl);
       }
       if (nb0 + kS < iend) {
         ++is;
@@ -196,7 +210,7 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(con
 #pragma unroll
   for (int s = 0; s < kStages - 1; ++s) issue_step(s);
   uint32_t stage = 0, istage = kStages - 1;
-  const uint32_t a_row = (lane & 7) * 128, b_row = a_row + 8 * 128;
+  const uint32_t a_row = (lane & 7) * kRowBytes, b_row = a_row + 8 * kRowBytes;
   const uint32_t vr = (lane & 7) + 8 * (lane >> 4);
 
   for (int64_t gw = w0; gw < nrows; gw += W) {
@@ -209,7 +223,7 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(con
     const int bb = bh / p.H, hh = bh % p.H;
     // q as the SDDMM's A operand (every row = q): k16 step j uses dims 16j + 2t (+1), 16j + 8 + 2t (+1);
     // read from the q slot of the row's first ring stage
-    uint32_t qa[4] = {0u, 0u, 0u, 0u}, qb[4] = {0u, 0u, 0u, 0u};
+    uint32_t qa[kJ], qb[kJ];
     const int beg = __ldg(p.row_ptr + fi), end = __ldg(p.row_ptr + fi + 1);
     // padding (A18): columns >= n_b are masked; a row >= n_b is written as 0 if it is final (a row
     // with a coarse part is zeroed by the coarse kernel)
@@ -217,9 +231,9 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(con
     const bool pad_row = kPad && r >= nvalid;
 
     float m = -INFINITY, l = 0.f;
-    float acc[4][4];
+    float acc[kJ][4];
 #pragma unroll
-    for (int j = 0; j < 4; ++j)
+    for (int j = 0; j < kJ; ++j)
 #pragma unroll
       for (int e = 0; e < 4; ++e) acc[j][e] = 0.f;
 
@@ -232,7 +246,7 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(con
       stage = stage == kStages - 1 ? 0 : stage + 1;
       if (base == beg) {
 #pragma unroll
-        for (int j = 0; j < 4; ++j) {
+        for (int j = 0; j < kJ; ++j) {
           asm volatile("ld.shared.u32 %0, [%1];" : "=r"(qa[j]) : "r"(st + kQOff + 32 * j + 4 * t));
           asm volatile("ld.shared.u32 %0, [%1];" : "=r"(qb[j]) : "r"(st + kQOff + 32 * j + 16 + 4 * t));
         }
@@ -246,15 +260,15 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(con
         float sa[2][4] = {{0.f, 0.f, 0.f, 0.f}, {0.f, 0.f, 0.f, 0.f}};
         float sb[2][4] = {{0.f, 0.f, 0.f, 0.f}, {0.f, 0.f, 0.f, 0.f}};
 #pragma unroll
-        for (int h = 0; h < 2; ++h) {   // dims 32h .. 32h + 31 = k16 steps 2h, 2h + 1
+        for (int h = 0; h < kD / 32; ++h) {   // dims 32h .. 32h + 31 = k16 steps 2h, 2h + 1
           uint32_t ka[4], kb[4];
           const uint32_t sw = ((uint32_t)(((lane >> 3) + 4 * h) ^ (lane & 7))) << 4;
-          ldsm_x4(ka, st + pr * 2048 + a_row + sw);
-          ldsm_x4(kb, st + pr * 2048 + b_row + sw);
-          mma16816<kBF16>(sa[h], qa[2 * h], qa[2 * h], qb[2 * h], qb[2 * h], ka[0], ka[1]);
-          mma16816<kBF16>(sb[h], qa[2 * h], qa[2 * h], qb[2 * h], qb[2 * h], kb[0], kb[1]);
-          mma16816<kBF16>(sa[h], qa[2 * h + 1], qa[2 * h + 1], qb[2 * h + 1], qb[2 * h + 1], ka[2], ka[3]);
-          mma16816<kBF16>(sb[h], qa[2 * h + 1], qa[2 * h + 1], qb[2 * h + 1], qb[2 * h + 1], kb[2], kb[3]);
+          ldsm_x4(ka, st + pr * 16 * kRowBytes + a_row + sw);
+          ldsm_x4(kb, st + pr * 16 * kRowBytes + b_row + sw);
+          mma16816<kBF16>(sa[h & 1], qa[2 * h], qa[2 * h], qb[2 * h], qb[2 * h], ka[0], ka[1]);
+          mma16816<kBF16>(sb[h & 1], qa[2 * h], qa[2 * h], qb[2 * h], qb[2 * h], kb[0], kb[1]);
+          mma16816<kBF16>(sa[h & 1], qa[2 * h + 1], qa[2 * h + 1], qb[2 * h + 1], qb[2 * h + 1], ka[2], ka[3]);
+          mma16816<kBF16>(sb[h & 1], qa[2 * h + 1], qa[2 * h + 1], qb[2 * h + 1], qb[2 * h + 1], kb[2], kb[3]);
         }
         // this lane's positions: nnz base + 16pr + {2t, 2t+1} (chunk A), + {8 + 2t, 9 + 2t} (chunk B)
         const int rem = end - base - 16 * pr - 2 * t;
@@ -280,7 +294,7 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(con
         const float alpha = ex2((m - mx) * c);
         l *= alpha;
 #pragma unroll
-        for (int j = 0; j < 4; ++j)
+        for (int j = 0; j < kJ; ++j)
 #pragma unroll
           for (int e = 0; e < 4; ++e) acc[j][e] *= alpha;
         m = mx;
@@ -297,11 +311,11 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(con
         const uint32_t pb0 = pack2<kBF16>(pv[0], pv[1]), pb1 = pack2<kBF16>(pv[2], pv[3]);
         // ---- SpMM: O^T[dims 16j + g, 16j + g + 8] += V^T . p (A = V^T from ldmatrix.trans)
 #pragma unroll
-        for (int j = 0; j < 4; ++j) {
+        for (int j = 0; j < kJ; ++j) {
           uint32_t a[4];
           const uint32_t ch = 2 * j + ((lane >> 3) & 1);
           const uint32_t row = vr + 16 * pr;
-          ldsm_x4_t(a, st + kS * 128 + row * 128 + ((ch ^ (row & 7)) << 4));
+          ldsm_x4_t(a, st + kS * kRowBytes + row * kRowBytes + ((ch ^ (row & 7)) << 4));
           mma16816<kBF16>(acc[j], a[0], a[1], a[2], a[3], pb0, pb1);
         }
       }
@@ -310,21 +324,32 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(con
     // ---- row epilogue. Row sum: lanes with the same g hold disjoint nnz subsets (t).
     l += __shfl_xor_sync(0xffffffffu, l, 1);
     l += __shfl_xor_sync(0xffffffffu, l, 2);
-    // lane (g, t) owns output dims d0 = 16t + g and d1 = d0 + 8: acc[t][0] and acc[t][2]
-    float v0 = acc[0][0], v1 = acc[0][2];
+    // lane (g, t) owns output dims 16j + g and 16j + g + 8 of the blocks j = t (+ 4 at d = 128):
+    // acc[j][0] and acc[j][2]
+    constexpr int kOwn = kJ / 4;
+    float v[kOwn][2];
+    int dd[kOwn];
 #pragma unroll
-    for (int j = 1; j < 4; ++j)
-      if (t == j) {
-        v0 = acc[j][0];
-        v1 = acc[j][2];
-      }
-    const int d0 = 16 * t + g, d1 = d0 + 8;
+    for (int w = 0; w < kOwn; ++w) {
+      v[w][0] = acc[4 * w][0];
+      v[w][1] = acc[4 * w][2];
+#pragma unroll
+      for (int j = 1; j < 4; ++j)
+        if (t == j) {
+          v[w][0] = acc[4 * w + j][0];
+          v[w][1] = acc[4 * w + j][2];
+        }
+      dd[w] = 16 * (4 * w + t) + g;
+    }
     float inv = l > 0.f ? 1.f / l : 0.f;
     bool write_o = final_out;
     if (!final_out) {
       const size_t idx = (size_t)u0 * p.n_fine_rows + fi;
-      __stcg(p.part_acc + idx * 64 + d0, v0);
-      __stcg(p.part_acc + idx * 64 + d1, v1);
+#pragma unroll
+      for (int w = 0; w < kOwn; ++w) {
+        __stcg(p.part_acc + idx * kD + dd[w], v[w][0]);
+        __stcg(p.part_acc + idx * kD + dd[w] + 8, v[w][1]);
+      }
       if (lane == 0) __stcg(p.part_ml + idx, make_float2(m, l));
       if (p.concurrent) {
         // concurrent coarse || fine: the side that finishes the row second merges (a-8)
@@ -341,21 +366,28 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(con
           const float af = ex2((m - mu) * c), ac = ex2((mlc.x - mu) * c);
           const float den = l * af + mlc.y * ac;
           inv = den > 0.f ? 1.f / den : 0.f;
-          v0 = v0 * af + __ldcg(p.part_c_acc + idx * 64 + d0) * ac;
-          v1 = v1 * af + __ldcg(p.part_c_acc + idx * 64 + d1) * ac;
+#pragma unroll
+          for (int w = 0; w < kOwn; ++w) {
+            v[w][0] = v[w][0] * af + __ldcg(p.part_c_acc + idx * kD + dd[w]) * ac;
+            v[w][1] = v[w][1] * af + __ldcg(p.part_c_acc + idx * kD + dd[w] + 8) * ac;
+          }
           write_o = true;
         }
       }
     }
     if (pad_row) {
       write_o = final_out;   // rows with a coarse part are zeroed by the coarse kernel
-      v0 = v1 = 0.f;
+#pragma unroll
+      for (int w = 0; w < kOwn; ++w) v[w][0] = v[w][1] = 0.f;
     }
     if (write_o) {
       uint16_t* orow = p.o.data + bb * p.o.sb + hh * p.o.sh + (int64_t)r * p.o.sl;
-      const uint32_t pk = pack2<kBF16>(v0 * inv, v1 * inv);
-      orow[d0] = (uint16_t)(pk & 0xffffu);
-      orow[d1] = (uint16_t)(pk >> 16);
+#pragma unroll
+      for (int w = 0; w < kOwn; ++w) {
+        const uint32_t pk = pack2<kBF16>(v[w][0] * inv, v[w][1] * inv);
+        orow[dd[w]] = (uint16_t)(pk & 0xffffu);
+        orow[dd[w] + 8] = (uint16_t)(pk >> 16);
+      }
     }
   }
   cp_async_wait<0>();
@@ -364,8 +396,15 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB) fine_mma_kernel(con
 cudaError_t launch_fine_mma(const FineParams& p, bool bf16, int sms, cudaStream_t stream) {
   const int64_t warps = (int64_t)p.BH * p.n_fine_rows;
   if (warps == 0) return cudaSuccess;
-  auto kern = bf16 ? (p.valid_len ? fine_mma_kernel<true, true> : fine_mma_kernel<true, false>)
-                   : (p.valid_len ? fine_mma_kernel<false, true> : fine_mma_kernel<false, false>);
+  using K = void (*)(const FineParams);
+  static const K table[8] = {fine_mma_kernel<false, false, 64>, fine_mma_kernel<false, true, 64>,
+                             fine_mma_kernel<true, false, 64>,  fine_mma_kernel<true, true, 64>,
+                             fine_mma_kernel<false, false, 128>, fine_mma_kernel<false, true, 128>,
+                             fine_mma_kernel<true, false, 128>,  fine_mma_kernel<true, true, 128>};
+  if (p.d != 64 && p.d != 128) return cudaErrorInvalidValue;
+  const int vi = (p.d == 128 ? 4 : 0) + (bf16 ? 2 : 0) + (p.valid_len ? 1 : 0);
+  const K kern = table[vi];
+  const int kSmemBytes = p.d == 128 ? FCfg<128>::kSmemBytes : FCfg<64>::kSmemBytes;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytes);
   if (e != cudaSuccess) return e;
   // persistent grid: every resident block slot of `sms` SMs (the plan's SM count, or its num_sms
@@ -373,7 +412,6 @@ cudaError_t launch_fine_mma(const FineParams& p, bool bf16, int sms, cudaStream_
   // device, computed once under a lock (launches may come from several host threads).
   static std::mutex mu;
   static std::map<std::pair<int, int>, int> per_sm;
-  const int vi = (bf16 ? 2 : 0) + (p.valid_len ? 1 : 0);
   int dev = 0, n = 0;
   if ((e = cudaGetDevice(&dev)) != cudaSuccess) return e;
   {

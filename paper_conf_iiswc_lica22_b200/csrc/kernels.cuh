@@ -30,6 +30,7 @@ struct CoarseParams {
   TensorView q, k, v, o;
   int64_t L;
   int32_t H, BH;
+  int32_t d;                  // head dimension (64 or 128)
   int32_t n_items, n_dense_items;   // (BH = units per item: B*H, or H for a batched plan)
   int32_t n_global, n_fine_rows;
   int32_t batched;            // batched plan: Item::useB = sample, unit -> (item, head), fine_slot [B][L]
@@ -70,6 +71,7 @@ struct FineParams {
   float2* part_ml;
   TensorView q, k, v, o;
   int32_t H, BH, n_fine_rows;   // (BH = row units per fine row: B*H, or H for a batched plan)
+  int32_t d;                    // head dimension (64 or 128; the CUDA-core kernel takes 64 only)
   const int32_t* fine_sample;   // batched plan: sample of each fine row (else null)
   float scale_log2;
   int32_t concurrent;         // see CoarseParams::concurrent
@@ -116,6 +118,7 @@ cudaError_t launch_coarse_pp(const CoarseParams& p, const CUtensorMap& tmq, cons
                              const CUtensorMap& tmv, const CUtensorMap& tmq2, const CUtensorMap& tmk2,
                              const CUtensorMap& tmv2, const CUtensorMap& tmo, bool bf16, bool split_dense, int grid,
                              cudaStream_t stream);
+int coarse_pp_ctas_per_sm(int d);
 cudaError_t launch_fine(const FineParams& p, bool bf16, cudaStream_t stream);
 // Warp-level tensor-core variant (mma.sync m16n8k16), the default; see fine_mma.cu.
 cudaError_t launch_fine_mma(const FineParams& p, bool bf16, int sms, cudaStream_t stream);

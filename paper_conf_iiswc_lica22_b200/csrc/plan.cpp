@@ -35,7 +35,7 @@ std::string build_plan(HostPlan& p, int64_t L, int32_t heads, int32_t d, int32_t
   const int b = opts.block;
   if (b < 1 || (b > 64 && b % 64) || b > 1024) return "block must be <= 64 or a multiple of 64 (<= 1024)";
   if (!(opts.tau >= 0.0 && opts.tau <= 1.0)) return "tau must be in [0, 1]";
-  if (d != 64) { *unsupported = true; return "v1 supports head_dim == 64 only"; }
+  if (d != 64 && d != 128) { *unsupported = true; return "head_dim must be 64 or 128"; }
   for (int64_t i = 0; i < n_global; ++i)
     if (global_idx[i] < 0 || global_idx[i] >= L) return "global index out of range";
   for (int64_t i = 0; i < 2 * n_extra; ++i)

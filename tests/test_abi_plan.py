@@ -131,7 +131,8 @@ def status_of(fn):
     (dict(L=64, heads=1, d=64, window=2, global_idx=[-1]), _lib.MG_ERR_INVALID_ARG),
     (dict(L=64, heads=1, d=64, window=2, extra_idx=[[0, 64]]), _lib.MG_ERR_INVALID_ARG),
     (dict(L=64, heads=1, d=64, window=2, extra_idx=[[-3, 1]]), _lib.MG_ERR_INVALID_ARG),
-    (dict(L=64, heads=1, d=128, window=2), _lib.MG_ERR_UNSUPPORTED),
+    (dict(L=64, heads=1, d=96, window=2), _lib.MG_ERR_UNSUPPORTED),
+    (dict(L=64, heads=1, d=256, window=2), _lib.MG_ERR_UNSUPPORTED),
     (dict(L=64, heads=1, d=64, window=2, block=96), _lib.MG_ERR_INVALID_ARG),
     (dict(L=64, heads=1, d=64, window=2, strip_max_cols=256), _lib.MG_ERR_INVALID_ARG),
     (dict(L=64, heads=1, d=64, window=2, tau=1.5), _lib.MG_ERR_INVALID_ARG),
