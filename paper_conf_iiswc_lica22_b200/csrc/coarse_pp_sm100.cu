@@ -802,187 +802,161 @@ __global__ void __launch_bounds__(kThreads, DCfg<kD>::kMinBlocks)
         }
       }
       // ---------------------------------------------------------------- epilogue (a-8)
-      // O is processed in kD / 64 halves of 64 columns (d = 64: one, read once up front)
-      float mf = -INFINITY, lf = 0.f;
-      const float4* accf = nullptr;
-      const size_t fidx = (size_t)(kBatched ? ubh % p.H : ubh) * p.n_fine_rows + slot_f;
-      if (slot_f >= 0 && !p.concurrent) {
-        const float2 ml = p.part_ml[fidx];
-        mf = ml.x;
-        lf = ml.y;
-        accf = reinterpret_cast<const float4*>(p.part_acc + fidx * kD);
-      }
-      if (threadIdx.x == 0) tl_rec(p, n - 1, 11);
-      mbar_wait(bar(ctl->pv_done), (n - 1) & 1);          // the item's last P.V
-      tc_fence_after();
-      uint32_t o[2][32];
-      auto load_o = [&](int sb) {
-        tmem_ld32(tl + kTO + 64 * sb, o[0]);
-        tmem_ld32(tl + kTO + 64 * sb + 32, o[1]);
+      // (d = 64 keeps its single-pass epilogue: the per-half form below measured 3% slower on C2)
+      bool tma_out;
+      if constexpr (kNSub == 1) {
+        float mf = -INFINITY, lf = 0.f;
+        const float4* accf = nullptr;
+        const size_t fidx = (size_t)(kBatched ? ubh % p.H : ubh) * p.n_fine_rows + slot_f;
+        if (slot_f >= 0 && !p.concurrent) {
+          const float2 ml = p.part_ml[fidx];
+          mf = ml.x;
+          lf = ml.y;
+          accf = reinterpret_cast<const float4*>(p.part_acc + fidx * 64);
+        }
+        if (threadIdx.x == 0) tl_rec(p, n - 1, 11);
+        mbar_wait(bar(ctl->pv_done), (n - 1) & 1);          // the item's last P.V
+        tc_fence_after();
+        uint32_t o[2][32];
+        tmem_ld32(tl + kTO, o[0]);
+        tmem_ld32(tl + kTO + 32, o[1]);
         tmem_wait_ld();
-      };
-      if (kNSub == 1) load_o(0);
-      if (threadIdx.x == 0) tl_rec(p, n - 1, 12);
-      bool skip = false;
-      // split dense-row item whose chunk finishes its group last: O is merged from the chunk partials
-      bool merge_chunks = false;
-      const float* chunk_base = nullptr;
-      float mu0 = 0.f;
-      constexpr int kPartStride = kD + 4;                 // acc[kD], m, l, pad (16-byte rows)
-      if (kSplit && item.kind == 1 && item.nrowsB > 1) {
-        // split dense-row item: publish this chunk's (m, l, acc) per row; the chunk that finishes
-        // its row group last merges all chunks by log-sum-exp and writes O (a-4 over column chunks)
-        const size_t gidx = (size_t)ubh * p.n_dense_groups + item.rowB;
-        float* part = p.dense_part + ((gidx * p.dense_nsplit + item.turns) * 128 + t) * kPartStride;
-        // (tcgen05.ld is warp-collective: every lane loads, only valid rows store)
-#pragma unroll
-        for (int sb = 0; sb < kNSub; ++sb) {
-          if (kNSub > 1) load_o(sb);
+        tc_fence_before();
+        if (threadIdx.x == 0) tl_rec(p, n - 1, 12);
+        bool skip = false;
+        if (kSplit && item.kind == 1 && item.nrowsB > 1) {
+          // split dense-row item: publish this chunk's (m, l, acc) per row; the chunk that finishes
+          // its row group last merges all chunks by log-sum-exp and writes O (a-4 over column chunks)
+          const size_t gidx = (size_t)ubh * p.n_dense_groups + item.rowB;
+          float* part = p.dense_part + ((gidx * p.dense_nsplit + item.turns) * 128 + t) * 68;
           if (t < item.nrowsA) {
-            float4* dst = reinterpret_cast<float4*>(part + 64 * sb);
-#pragma unroll
+            float4* dst = reinterpret_cast<float4*>(part);
+  #pragma unroll
             for (int i = 0; i < 16; ++i)
               __stcg(dst + i, make_float4(__uint_as_float(o[i >> 3][(i & 7) * 4]), __uint_as_float(o[i >> 3][(i & 7) * 4 + 1]),
                                           __uint_as_float(o[i >> 3][(i & 7) * 4 + 2]),
                                           __uint_as_float(o[i >> 3][(i & 7) * 4 + 3])));
+            __stcg(reinterpret_cast<float2*>(part + 64), make_float2(m, l));
           }
-        }
-        if (t < item.nrowsA) __stcg(reinterpret_cast<float2*>(part + kD), make_float2(m, l));
-        __threadfence();
-        named_bar_sync(1, 128);
-        // per-group chunk counter in [0, nrowsB): atomicInc wraps it back to 0 on the last chunk, so it
-        // is ready for the next forward and never overflows
-        if (threadIdx.x == 0)
-          ctl->dense_last = atomicInc(reinterpret_cast<unsigned*>(p.dense_ctr) + gidx, (unsigned)item.nrowsB - 1u) ==
-                            (unsigned)item.nrowsB - 1u;
-        named_bar_sync(1, 128);
-        skip = !ctl->dense_last;
-        if (!skip && t < item.nrowsA) {
           __threadfence();
-          chunk_base = p.dense_part + (gidx * p.dense_nsplit * 128 + t) * kPartStride;
-          float mm = -INFINITY;
-          for (int k = 0; k < item.nrowsB; ++k) mm = fmaxf(mm, __ldcg(chunk_base + (size_t)k * 128 * kPartStride + kD));
-          mu0 = mm == -INFINITY ? 0.f : mm;
-          float den0 = 0.f;
-          for (int k = 0; k < item.nrowsB; ++k)
-            den0 += __ldcg(chunk_base + (size_t)k * 128 * kPartStride + kD + 1) *
-                    ex2((__ldcg(chunk_base + (size_t)k * 128 * kPartStride + kD) - mu0) * c);
-          // the merged row goes through the common store below: O = merged (scale 1), l = den0, m = mm
-          merge_chunks = true;
-          m = mm;
-          l = den0;
-        }
-      }
-      if (kNSub > 1 && p.concurrent) {
-        // (tcgen05.ld is warp-collective: the d = 128 halves are loaded by every lane, stored below
-        // by the rows with a CUDA-core CSR part)
-#pragma unroll
-        for (int sb = 0; sb < kNSub; ++sb) {
-          load_o(sb);
-          if (slot_f >= 0) {
-            float4* dst = reinterpret_cast<float4*>(p.part_c_acc + fidx * kD + 64 * sb);
-#pragma unroll
-            for (int i = 0; i < 16; ++i)
-              __stcg(dst + i, make_float4(__uint_as_float(o[i >> 3][(i & 7) * 4]), __uint_as_float(o[i >> 3][(i & 7) * 4 + 1]),
-                                          __uint_as_float(o[i >> 3][(i & 7) * 4 + 2]), __uint_as_float(o[i >> 3][(i & 7) * 4 + 3])));
+          named_bar_sync(1, 128);
+          // per-group chunk counter in [0, nrowsB): atomicInc wraps it back to 0 on the last chunk, so it
+          // is ready for the next forward and never overflows
+          if (threadIdx.x == 0)
+            ctl->dense_last = atomicInc(reinterpret_cast<unsigned*>(p.dense_ctr) + gidx, (unsigned)item.nrowsB - 1u) ==
+                              (unsigned)item.nrowsB - 1u;
+          named_bar_sync(1, 128);
+          skip = !ctl->dense_last;
+          if (!skip && t < item.nrowsA) {
+            __threadfence();
+            const float* base = p.dense_part + (gidx * p.dense_nsplit * 128 + t) * 68;
+            float mm = -INFINITY;
+            for (int k = 0; k < item.nrowsB; ++k) mm = fmaxf(mm, __ldcg(base + (size_t)k * 128 * 68 + 64));
+            const float mu0 = mm == -INFINITY ? 0.f : mm;
+            // merged row accumulated in place of this chunk's O registers
+  #pragma unroll
+            for (int i = 0; i < 64; ++i) o[i >> 5][i & 31] = 0u;
+            float den0 = 0.f;
+            for (int k = 0; k < item.nrowsB; ++k) {
+              const float* pk = base + (size_t)k * 128 * 68;
+              const float2 ml = __ldcg(reinterpret_cast<const float2*>(pk + 64));
+              const float a = ex2((ml.x - mu0) * c);
+              den0 += ml.y * a;
+              const float4* src = reinterpret_cast<const float4*>(pk);
+  #pragma unroll
+              for (int i = 0; i < 16; ++i) {
+                const float4 v = __ldcg(src + i);
+                uint32_t* q4 = &o[i >> 3][(i & 7) * 4];
+                q4[0] = __float_as_uint(fmaf(v.x, a, __uint_as_float(q4[0])));
+                q4[1] = __float_as_uint(fmaf(v.y, a, __uint_as_float(q4[1])));
+                q4[2] = __float_as_uint(fmaf(v.z, a, __uint_as_float(q4[2])));
+                q4[3] = __float_as_uint(fmaf(v.w, a, __uint_as_float(q4[3])));
+              }
+            }
+            // hand the merged row to the common store below: O = o (scale 1), l = den0, m = mm
+            m = mm;
+            l = den0;
           }
         }
-      }
-      if (slot_f >= 0 && p.concurrent) {
-        // publish this row's coarse partial; the side that finishes the row second merges both
-        if (kNSub == 1) {
-          float4* dst = reinterpret_cast<float4*>(p.part_c_acc + fidx * kD);
-#pragma unroll
+        if (slot_f >= 0 && p.concurrent) {
+          // publish this row's coarse partial; the side that finishes the row second merges both
+          float4* dst = reinterpret_cast<float4*>(p.part_c_acc + fidx * 64);
+  #pragma unroll
           for (int i = 0; i < 16; ++i)
             __stcg(dst + i, make_float4(__uint_as_float(o[i >> 3][(i & 7) * 4]), __uint_as_float(o[i >> 3][(i & 7) * 4 + 1]),
                                         __uint_as_float(o[i >> 3][(i & 7) * 4 + 2]), __uint_as_float(o[i >> 3][(i & 7) * 4 + 3])));
-        }
-        __stcg(p.part_c_ml + fidx, make_float2(m, l));
-        __threadfence();
-        const int old = atomicAdd(p.part_flags + fidx, 1);
-        if (old & 1) {
+          __stcg(p.part_c_ml + fidx, make_float2(m, l));
           __threadfence();
-          const float2 ml = __ldcg(p.part_ml + fidx);
-          mf = ml.x;
-          lf = ml.y;
-          accf = reinterpret_cast<const float4*>(p.part_acc + fidx * kD);
-        } else {
-          skip = true;
-        }
-      }
-      const float mt = fmaxf(m, mf);
-      const float mu = mt == -INFINITY ? 0.f : mt;
-      const float ac = ex2((m - mu) * c), af = ex2((mf - mu) * c);
-      const float den = l * ac + lf * af;
-      // normalised row -> 16-bit, 8 x 16-byte stores per 64 columns of this thread's row. A row with
-      // no valid element in this item (a global row inside a band row block: it is owned by the
-      // dense-row part, A5) is not written. (Staging the tile through shared memory for 4-rows-per-
-      // instruction stores measured 10% slower: tools/experiments/.)
-      // padding (A18): rows at or beyond the batch element's valid length are written as 0 by
-      // every item that holds them (whatever the merge protocol decided)
-      const bool pad_row = kPad && r_out >= 0 &&
-                           r_out >= min(max(__ldg(p.valid_len + ubh / p.H), 0), (int)p.L);
-      // (only blocks without global rows and without CUDA-core CSR rows: no other writer, no partial
-      // to merge; measured: merging partials in this path costs C2 3% and gains nothing on C4)
-      const bool tma_out = !kPad && p.tma_store && item.kind == 0 && (item.useA & 3) == 3;   // uniform per item
-      const bool write_row = !tma_out && !pad_row && r_out >= 0 && mt != -INFINITY && !skip;
-      const int bb = ubh / p.H, hh = ubh % p.H;
-      uint16_t* orow = p.o.data + bb * p.o.sb + hh * p.o.sh + (int64_t)max(r_out, 0) * p.o.sl;
-      const uint32_t sO = sQ + (it & 1) * kTileBytes;
-#pragma unroll
-      for (int sb = 0; sb < kNSub; ++sb) {
-        if (kNSub > 1) load_o(sb);   // (warp-collective: every lane, before any per-row choice)
-        if (merge_chunks) {
-#pragma unroll
-          for (int i = 0; i < 64; ++i) o[i >> 5][i & 31] = 0u;
-          for (int k = 0; k < item.nrowsB; ++k) {
-            const float* pk = chunk_base + (size_t)k * 128 * kPartStride;
-            const float a = ex2((__ldcg(pk + kD) - mu0) * c);
-            const float4* src = reinterpret_cast<const float4*>(pk + 64 * sb);
-#pragma unroll
-            for (int i = 0; i < 16; ++i) {
-              const float4 v = __ldcg(src + i);
-              uint32_t* q4 = &o[i >> 3][(i & 7) * 4];
-              q4[0] = __float_as_uint(fmaf(v.x, a, __uint_as_float(q4[0])));
-              q4[1] = __float_as_uint(fmaf(v.y, a, __uint_as_float(q4[1])));
-              q4[2] = __float_as_uint(fmaf(v.z, a, __uint_as_float(q4[2])));
-              q4[3] = __float_as_uint(fmaf(v.w, a, __uint_as_float(q4[3])));
-            }
+          const int old = atomicAdd(p.part_flags + fidx, 1);
+          if (old & 1) {
+            __threadfence();
+            const float2 ml = __ldcg(p.part_ml + fidx);
+            mf = ml.x;
+            lf = ml.y;
+            accf = reinterpret_cast<const float4*>(p.part_acc + fidx * 64);
+          } else {
+            skip = true;
           }
         }
+        const float mt = fmaxf(m, mf);
+        const float mu = mt == -INFINITY ? 0.f : mt;
+        const float ac = ex2((m - mu) * c), af = ex2((mf - mu) * c);
+        const float den = l * ac + lf * af;
+        // normalised row -> 16-bit, 8 x 16-byte stores of this thread's row. A row with no valid
+        // element in this item (a global row inside a band row block: it is owned by the dense-row
+        // part, A5) is not written. (Staging the tile through shared memory for 4-rows-per-
+        // instruction stores measured 10% slower: tools/experiments/.)
+        // padding (A18): rows at or beyond the batch element's valid length are written as 0 by
+        // every item that holds them (whatever the merge protocol decided)
+        const bool pad_row = kPad && r_out >= 0 &&
+                             r_out >= min(max(__ldg(p.valid_len + ubh / p.H), 0), (int)p.L);
+        // (only blocks without global rows and without CUDA-core CSR rows: no other writer, no partial
+        // to merge; measured: merging partials in this path costs C2 3% and gains nothing on C4)
+        tma_out = !kPad && p.tma_store && item.kind == 0 && (item.useA & 3) == 3;   // uniform per item
         if (tma_out) {
           // normalised rows into the item's Q buffer (SWIZZLE_128B layout of the O tensor map), then one
-          // TMA store per 128 x 64 sub-tile (rows beyond L are clipped by the map)
+          // TMA store of the 128 x 64 tile (rows beyond L are clipped by the map)
+          const uint32_t sO = sQ + (it & 1) * kTileBytes;
           const float inv = (r_out >= 0 && mt != -INFINITY) ? __frcp_rn(den) : 0.f;
-#pragma unroll
+  #pragma unroll
           for (int h = 0; h < 2; ++h) {
-#pragma unroll
+  #pragma unroll
             for (int q8 = 0; q8 < 4; ++q8) {
               float a[8];
-#pragma unroll
+  #pragma unroll
               for (int i = 0; i < 8; ++i) a[i] = __uint_as_float(o[h][q8 * 8 + i]) * (ac * inv);
               const int ch = h * 4 + q8;
-              asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(sO + sb * kSub + t * 128 + ((ch ^ (t & 7)) << 4)),
+              asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(sO + t * 128 + ((ch ^ (t & 7)) << 4)),
                            "r"(pack2<kBF16>(a[0], a[1])), "r"(pack2<kBF16>(a[2], a[3])), "r"(pack2<kBF16>(a[4], a[5])),
                            "r"(pack2<kBF16>(a[6], a[7]))
                            : "memory");
             }
           }
+          fence_proxy_async_smem();
+          named_bar_sync(1, 128);
+          if (threadIdx.x == 0) {
+            tma_store_4d(&tmo, sO, 0, item.rowA, ubh % p.H, ubh / p.H);
+            bulk_commit_group();
+            bulk_wait_group_read0();   // the buffer is reloaded with a later item's Q after q_empty
+          }
         } else if (pad_row) {
-          uint4* o16 = reinterpret_cast<uint4*>(orow + 64 * sb);
-#pragma unroll
-          for (int i = 0; i < 8; ++i) o16[i] = make_uint4(0u, 0u, 0u, 0u);
-        } else if (write_row) {
+          const int bb = ubh / p.H, hh = ubh % p.H;
+          uint4* orow = reinterpret_cast<uint4*>(p.o.data + bb * p.o.sb + hh * p.o.sh + (int64_t)r_out * p.o.sl);
+  #pragma unroll
+          for (int i = 0; i < 8; ++i) orow[i] = make_uint4(0u, 0u, 0u, 0u);
+        } else if (r_out >= 0 && mt != -INFINITY && !skip) {
           const float inv = __frcp_rn(den);
-#pragma unroll
+          const int bb = ubh / p.H, hh = ubh % p.H;
+          uint16_t* orow = p.o.data + bb * p.o.sb + hh * p.o.sh + (int64_t)r_out * p.o.sl;
+  #pragma unroll
           for (int h = 0; h < 2; ++h) {
-#pragma unroll
+  #pragma unroll
             for (int q8 = 0; q8 < 4; ++q8) {
               float a[8];
-#pragma unroll
+  #pragma unroll
               for (int i = 0; i < 8; ++i) a[i] = __uint_as_float(o[h][q8 * 8 + i]) * ac;
               if (accf) {
-                const float4 f0 = __ldcg(accf + 16 * sb + h * 8 + q8 * 2), f1 = __ldcg(accf + 16 * sb + h * 8 + q8 * 2 + 1);
+                const float4 f0 = __ldcg(accf + h * 8 + q8 * 2), f1 = __ldcg(accf + h * 8 + q8 * 2 + 1);
                 a[0] = fmaf(f0.x, af, a[0]);
                 a[1] = fmaf(f0.y, af, a[1]);
                 a[2] = fmaf(f0.z, af, a[2]);
@@ -997,22 +971,223 @@ __global__ void __launch_bounds__(kThreads, DCfg<kD>::kMinBlocks)
               o4.y = pack2<kBF16>(a[2] * inv, a[3] * inv);
               o4.z = pack2<kBF16>(a[4] * inv, a[5] * inv);
               o4.w = pack2<kBF16>(a[6] * inv, a[7] * inv);
-              *reinterpret_cast<uint4*>(orow + 64 * sb + h * 32 + q8 * 8) = o4;
+              *reinterpret_cast<uint4*>(orow + h * 32 + q8 * 8) = o4;
             }
           }
         }
-      }
-      if (tma_out) {
-        fence_proxy_async_smem();
-        named_bar_sync(1, 128);
-        if (threadIdx.x == 0) {
-#pragma unroll
-          for (int sb = 0; sb < kNSub; ++sb) tma_store_4d(&tmo, sO + sb * kSub, 64 * sb, item.rowA, hh, bb);
-          bulk_commit_group();
-          bulk_wait_group_read0();   // the buffer is reloaded with a later item's Q after q_empty
+      } else {
+        // O is processed in kD / 64 halves of 64 columns (d = 64: one, read once up front)
+        float mf = -INFINITY, lf = 0.f;
+        const float4* accf = nullptr;
+        const size_t fidx = (size_t)(kBatched ? ubh % p.H : ubh) * p.n_fine_rows + slot_f;
+        if (slot_f >= 0 && !p.concurrent) {
+          const float2 ml = p.part_ml[fidx];
+          mf = ml.x;
+          lf = ml.y;
+          accf = reinterpret_cast<const float4*>(p.part_acc + fidx * kD);
         }
+        if (threadIdx.x == 0) tl_rec(p, n - 1, 11);
+        mbar_wait(bar(ctl->pv_done), (n - 1) & 1);          // the item's last P.V
+        tc_fence_after();
+        uint32_t o[2][32];
+        auto load_o = [&](int sb) {
+          tmem_ld32(tl + kTO + 64 * sb, o[0]);
+          tmem_ld32(tl + kTO + 64 * sb + 32, o[1]);
+          tmem_wait_ld();
+        };
+        if (kNSub == 1) load_o(0);
+        if (threadIdx.x == 0) tl_rec(p, n - 1, 12);
+        bool skip = false;
+        // split dense-row item whose chunk finishes its group last: O is merged from the chunk partials
+        bool merge_chunks = false;
+        const float* chunk_base = nullptr;
+        float mu0 = 0.f;
+        constexpr int kPartStride = kD + 4;                 // acc[kD], m, l, pad (16-byte rows)
+        if (kSplit && item.kind == 1 && item.nrowsB > 1) {
+          // split dense-row item: publish this chunk's (m, l, acc) per row; the chunk that finishes
+          // its row group last merges all chunks by log-sum-exp and writes O (a-4 over column chunks)
+          const size_t gidx = (size_t)ubh * p.n_dense_groups + item.rowB;
+          float* part = p.dense_part + ((gidx * p.dense_nsplit + item.turns) * 128 + t) * kPartStride;
+          // (tcgen05.ld is warp-collective: every lane loads, only valid rows store)
+  #pragma unroll
+          for (int sb = 0; sb < kNSub; ++sb) {
+            if (kNSub > 1) load_o(sb);
+            if (t < item.nrowsA) {
+              float4* dst = reinterpret_cast<float4*>(part + 64 * sb);
+  #pragma unroll
+              for (int i = 0; i < 16; ++i)
+                __stcg(dst + i, make_float4(__uint_as_float(o[i >> 3][(i & 7) * 4]), __uint_as_float(o[i >> 3][(i & 7) * 4 + 1]),
+                                            __uint_as_float(o[i >> 3][(i & 7) * 4 + 2]),
+                                            __uint_as_float(o[i >> 3][(i & 7) * 4 + 3])));
+            }
+          }
+          if (t < item.nrowsA) __stcg(reinterpret_cast<float2*>(part + kD), make_float2(m, l));
+          __threadfence();
+          named_bar_sync(1, 128);
+          // per-group chunk counter in [0, nrowsB): atomicInc wraps it back to 0 on the last chunk, so it
+          // is ready for the next forward and never overflows
+          if (threadIdx.x == 0)
+            ctl->dense_last = atomicInc(reinterpret_cast<unsigned*>(p.dense_ctr) + gidx, (unsigned)item.nrowsB - 1u) ==
+                              (unsigned)item.nrowsB - 1u;
+          named_bar_sync(1, 128);
+          skip = !ctl->dense_last;
+          if (!skip && t < item.nrowsA) {
+            __threadfence();
+            chunk_base = p.dense_part + (gidx * p.dense_nsplit * 128 + t) * kPartStride;
+            float mm = -INFINITY;
+            for (int k = 0; k < item.nrowsB; ++k) mm = fmaxf(mm, __ldcg(chunk_base + (size_t)k * 128 * kPartStride + kD));
+            mu0 = mm == -INFINITY ? 0.f : mm;
+            float den0 = 0.f;
+            for (int k = 0; k < item.nrowsB; ++k)
+              den0 += __ldcg(chunk_base + (size_t)k * 128 * kPartStride + kD + 1) *
+                      ex2((__ldcg(chunk_base + (size_t)k * 128 * kPartStride + kD) - mu0) * c);
+            // the merged row goes through the common store below: O = merged (scale 1), l = den0, m = mm
+            merge_chunks = true;
+            m = mm;
+            l = den0;
+          }
+        }
+        if (kNSub > 1 && p.concurrent) {
+          // (tcgen05.ld is warp-collective: the d = 128 halves are loaded by every lane, stored below
+          // by the rows with a CUDA-core CSR part)
+  #pragma unroll
+          for (int sb = 0; sb < kNSub; ++sb) {
+            load_o(sb);
+            if (slot_f >= 0) {
+              float4* dst = reinterpret_cast<float4*>(p.part_c_acc + fidx * kD + 64 * sb);
+  #pragma unroll
+              for (int i = 0; i < 16; ++i)
+                __stcg(dst + i, make_float4(__uint_as_float(o[i >> 3][(i & 7) * 4]), __uint_as_float(o[i >> 3][(i & 7) * 4 + 1]),
+                                            __uint_as_float(o[i >> 3][(i & 7) * 4 + 2]), __uint_as_float(o[i >> 3][(i & 7) * 4 + 3])));
+            }
+          }
+        }
+        if (slot_f >= 0 && p.concurrent) {
+          // publish this row's coarse partial; the side that finishes the row second merges both
+          if (kNSub == 1) {
+            float4* dst = reinterpret_cast<float4*>(p.part_c_acc + fidx * kD);
+  #pragma unroll
+            for (int i = 0; i < 16; ++i)
+              __stcg(dst + i, make_float4(__uint_as_float(o[i >> 3][(i & 7) * 4]), __uint_as_float(o[i >> 3][(i & 7) * 4 + 1]),
+                                          __uint_as_float(o[i >> 3][(i & 7) * 4 + 2]), __uint_as_float(o[i >> 3][(i & 7) * 4 + 3])));
+          }
+          __stcg(p.part_c_ml + fidx, make_float2(m, l));
+          __threadfence();
+          const int old = atomicAdd(p.part_flags + fidx, 1);
+          if (old & 1) {
+            __threadfence();
+            const float2 ml = __ldcg(p.part_ml + fidx);
+            mf = ml.x;
+            lf = ml.y;
+            accf = reinterpret_cast<const float4*>(p.part_acc + fidx * kD);
+          } else {
+            skip = true;
+          }
+        }
+        const float mt = fmaxf(m, mf);
+        const float mu = mt == -INFINITY ? 0.f : mt;
+        const float ac = ex2((m - mu) * c), af = ex2((mf - mu) * c);
+        const float den = l * ac + lf * af;
+        // normalised row -> 16-bit, 8 x 16-byte stores per 64 columns of this thread's row. A row with
+        // no valid element in this item (a global row inside a band row block: it is owned by the
+        // dense-row part, A5) is not written. (Staging the tile through shared memory for 4-rows-per-
+        // instruction stores measured 10% slower: tools/experiments/.)
+        // padding (A18): rows at or beyond the batch element's valid length are written as 0 by
+        // every item that holds them (whatever the merge protocol decided)
+        const bool pad_row = kPad && r_out >= 0 &&
+                             r_out >= min(max(__ldg(p.valid_len + ubh / p.H), 0), (int)p.L);
+        // (only blocks without global rows and without CUDA-core CSR rows: no other writer, no partial
+        // to merge; measured: merging partials in this path costs C2 3% and gains nothing on C4)
+        tma_out = !kPad && p.tma_store && item.kind == 0 && (item.useA & 3) == 3;   // uniform per item
+        const bool write_row = !tma_out && !pad_row && r_out >= 0 && mt != -INFINITY && !skip;
+        const int bb = ubh / p.H, hh = ubh % p.H;
+        uint16_t* orow = p.o.data + bb * p.o.sb + hh * p.o.sh + (int64_t)max(r_out, 0) * p.o.sl;
+        const uint32_t sO = sQ + (it & 1) * kTileBytes;
+  #pragma unroll
+        for (int sb = 0; sb < kNSub; ++sb) {
+          if (kNSub > 1) load_o(sb);   // (warp-collective: every lane, before any per-row choice)
+          if (merge_chunks) {
+  #pragma unroll
+            for (int i = 0; i < 64; ++i) o[i >> 5][i & 31] = 0u;
+            for (int k = 0; k < item.nrowsB; ++k) {
+              const float* pk = chunk_base + (size_t)k * 128 * kPartStride;
+              const float a = ex2((__ldcg(pk + kD) - mu0) * c);
+              const float4* src = reinterpret_cast<const float4*>(pk + 64 * sb);
+  #pragma unroll
+              for (int i = 0; i < 16; ++i) {
+                const float4 v = __ldcg(src + i);
+                uint32_t* q4 = &o[i >> 3][(i & 7) * 4];
+                q4[0] = __float_as_uint(fmaf(v.x, a, __uint_as_float(q4[0])));
+                q4[1] = __float_as_uint(fmaf(v.y, a, __uint_as_float(q4[1])));
+                q4[2] = __float_as_uint(fmaf(v.z, a, __uint_as_float(q4[2])));
+                q4[3] = __float_as_uint(fmaf(v.w, a, __uint_as_float(q4[3])));
+              }
+            }
+          }
+          if (tma_out) {
+            // normalised rows into the item's Q buffer (SWIZZLE_128B layout of the O tensor map), then one
+            // TMA store per 128 x 64 sub-tile (rows beyond L are clipped by the map)
+            const float inv = (r_out >= 0 && mt != -INFINITY) ? __frcp_rn(den) : 0.f;
+  #pragma unroll
+            for (int h = 0; h < 2; ++h) {
+  #pragma unroll
+              for (int q8 = 0; q8 < 4; ++q8) {
+                float a[8];
+  #pragma unroll
+                for (int i = 0; i < 8; ++i) a[i] = __uint_as_float(o[h][q8 * 8 + i]) * (ac * inv);
+                const int ch = h * 4 + q8;
+                asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(sO + sb * kSub + t * 128 + ((ch ^ (t & 7)) << 4)),
+                             "r"(pack2<kBF16>(a[0], a[1])), "r"(pack2<kBF16>(a[2], a[3])), "r"(pack2<kBF16>(a[4], a[5])),
+                             "r"(pack2<kBF16>(a[6], a[7]))
+                             : "memory");
+              }
+            }
+          } else if (pad_row) {
+            uint4* o16 = reinterpret_cast<uint4*>(orow + 64 * sb);
+  #pragma unroll
+            for (int i = 0; i < 8; ++i) o16[i] = make_uint4(0u, 0u, 0u, 0u);
+          } else if (write_row) {
+            const float inv = __frcp_rn(den);
+  #pragma unroll
+            for (int h = 0; h < 2; ++h) {
+  #pragma unroll
+              for (int q8 = 0; q8 < 4; ++q8) {
+                float a[8];
+  #pragma unroll
+                for (int i = 0; i < 8; ++i) a[i] = __uint_as_float(o[h][q8 * 8 + i]) * ac;
+                if (accf) {
+                  const float4 f0 = __ldcg(accf + 16 * sb + h * 8 + q8 * 2), f1 = __ldcg(accf + 16 * sb + h * 8 + q8 * 2 + 1);
+                  a[0] = fmaf(f0.x, af, a[0]);
+                  a[1] = fmaf(f0.y, af, a[1]);
+                  a[2] = fmaf(f0.z, af, a[2]);
+                  a[3] = fmaf(f0.w, af, a[3]);
+                  a[4] = fmaf(f1.x, af, a[4]);
+                  a[5] = fmaf(f1.y, af, a[5]);
+                  a[6] = fmaf(f1.z, af, a[6]);
+                  a[7] = fmaf(f1.w, af, a[7]);
+                }
+                uint4 o4;
+                o4.x = pack2<kBF16>(a[0] * inv, a[1] * inv);
+                o4.y = pack2<kBF16>(a[2] * inv, a[3] * inv);
+                o4.z = pack2<kBF16>(a[4] * inv, a[5] * inv);
+                o4.w = pack2<kBF16>(a[6] * inv, a[7] * inv);
+                *reinterpret_cast<uint4*>(orow + 64 * sb + h * 32 + q8 * 8) = o4;
+              }
+            }
+          }
+        }
+        if (tma_out) {
+          fence_proxy_async_smem();
+          named_bar_sync(1, 128);
+          if (threadIdx.x == 0) {
+  #pragma unroll
+            for (int sb = 0; sb < kNSub; ++sb) tma_store_4d(&tmo, sO + sb * kSub, 64 * sb, item.rowA, hh, bb);
+            bulk_commit_group();
+            bulk_wait_group_read0();   // the buffer is reloaded with a later item's Q after q_empty
+          }
+        }
+        tc_fence_before();
       }
-      tc_fence_before();
       // the item's Q buffer is free (its last S MMA has completed: pv_done above; its O tile, if
       // staged there, has been read by the TMA store)
       if (threadIdx.x == 0) {
