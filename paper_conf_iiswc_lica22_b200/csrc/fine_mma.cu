@@ -88,6 +88,10 @@ __device__ __forceinline__ void ldsm_x4_t(uint32_t (&r)[4], uint32_t addr) {
 #ifndef MG_FINE_WARPS
 #define MG_FINE_WARPS 4
 #endif
+#ifndef MG_FINE_IDX_AHEAD
+#define MG_FINE_IDX_AHEAD 1
+#endif
+constexpr bool kIdxAhead = MG_FINE_IDX_AHEAD;   // column-index window prefetched one step ahead
 constexpr int kWarps = MG_FINE_WARPS;       // warps per block, each a persistent row sequence
 constexpr int kP = MG_FINE_PAIRS;           // 16-nnz pairs of 8-nnz chunks per step (1 or 2)
 constexpr int kS = 16 * kP;                 // nnz per step
@@ -159,7 +163,7 @@ __global__ void __launch_bounds__(kWarps * 32, FCfg<kD>::kMinB) fine_mma_kernel(
 
   // ---- gather pointer: row gi (global work index), step is of [ibeg, iend)
   int64_t gi = w0;
-  int ibeg = 0, iend = 0, is = 0, icol = -1;
+  int ibeg = 0, iend = 0, is = 0, icol = -1, icol_next = -1;
   const uint16_t *iK = nullptr, *iV = nullptr, *iQ = nullptr;
   auto open_issue_row = [&]() {
     if (gi < nrows) {
@@ -184,7 +188,10 @@ __global__ void __launch_bounds__(kWarps * 32, FCfg<kD>::kMinB) fine_mma_kernel(
   auto issue_step = [&](uint32_t stg) {
     if (gi < nrows) {   // warp-uniform
       const int nb0 = ibeg + kS * is;
-      if (kP == 2 || (is & 1) == 0) icol = nb0 + lane < iend ? __ldg(p.cols + nb0 + lane) : -1;
+      // column indices: a row's first window is loaded here; later windows of the row were
+      // prefetched one step earlier (MG_FINE_IDX_AHEAD), so the index load latency overlaps a step
+      if (kP == 2 || (is & 1) == 0)
+        icol = (kIdxAhead && kP == 1 && is > 0) ? icol_next : (nb0 + lane < iend ? __ldg(p.cols + nb0 + lane) : -1);
       const int off = (kP == 2 ? 0 : (is & 1) * 16) + lane / kLPR;
       const uint32_t st = ring + stg * kStageBytes;
       // a row's first step also carries its q row (lanes 0 .. kLPR-1, 16 B each), so the computing
@@ -196,6 +203,8 @@ __global__ void __launch_bounds__(kWarps * 32, FCfg<kD>::kMinB) fine_mma_kernel(
         cp_async16(st + doff[i], iK + cc * ksl);
         cp_async16(st + doff[i] + kS * kRowBytes, iV + cc * vsl);
       }
+      if (kIdxAhead && kP == 1 && (is & 1) == 1 && nb0 + kS < iend)
+        icol_next = nb0 + kS + lane < iend ? __ldg(p.cols + nb0 + kS + lane) : -1;
       if (nb0 + kS < iend) {
         ++is;
       } else {
