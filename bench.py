@@ -232,53 +232,88 @@ def cpu_oracle_pool(cfg, budget_s: float):
                       f"{cores} single-threaded workers, {dt:.1f} s wall; useful flops counted as for the GPU"}
 
 
+_REF = {}
+
+
+def _ref_init(name, head_dim, seed_heads):
+    """Worker initializer of the reference arm: the workload's pattern and a few (b, h) heads of
+    seeded inputs, built once per worker process."""
+    import dataclasses
+    from oracle import ExtraIndex, global_flags, head_inputs_f64
+    from workloads import get_config, make_qkv
+    from threadpoolctl import threadpool_limits
+    threadpool_limits(1)
+    cfg = get_config(name)
+    if head_dim:
+        cfg = dataclasses.replace(cfg, d=head_dim)
+    q, k, v = make_qkv(1, seed_heads, cfg.L, cfg.d, seed=cfg.seed)
+    _REF.update(cfg=cfg, heads=[head_inputs_f64(q, k, v, 0, h) for h in range(seed_heads)],
+                g=global_flags(cfg.L, cfg.global_idx), ex=ExtraIndex(cfg.L, cfg.extra_idx))
+
+
+def _ref_task(args):
+    """One worker's share of a reference step: the oracle (attention_rows, fp64) on R random rows of
+    one head; returns (seconds, useful nnz)."""
+    import numpy as np
+    from oracle import attention_rows
+    from oracle.mask import mask_row_cols
+    seed, R = args
+    cfg = _REF["cfg"]
+    rng = np.random.default_rng(seed)
+    Q, K, V = _REF["heads"][seed % len(_REF["heads"])]
+    rows = rng.choice(cfg.L, R, replace=False)
+    nnz = sum(mask_row_cols(int(r), cfg.L, cfg.window, _REF["g"], _REF["ex"]).size for r in rows)
+    t0 = time.perf_counter()
+    attention_rows(Q, K, V, rows, cfg.window, _REF["g"], _REF["ex"])
+    return time.perf_counter() - t0, nnz
+
+
 def run_reference(args):
-    """--impl reference: the oracle (as it stands) on the host cores, one bounded sample per step."""
+    """--impl reference: the oracle (as it stands) on the host cores, one bounded sample per step:
+    os.cpu_count() single-threaded worker processes each evaluate 32 random rows of one head
+    (oracle.attention_rows, fp64); the step's wall clock is the pool's."""
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return 0
-    import numpy as np
-    from oracle import ExtraIndex, attention_rows, global_flags, head_inputs_f64
-    from oracle.mask import mask_row_cols
-    from workloads import get_config, make_qkv
+    import multiprocessing as mp
+    from workloads import get_config
     world = int(os.environ.get("WORLD_SIZE", "1"))
-    cfg = get_config(resolve_workload(args, max(world, args.gpus)))
+    name = resolve_workload(args, max(world, args.gpus))
+    cfg = get_config(name)
     if args.head_dim:
         import dataclasses
         cfg = dataclasses.replace(cfg, d=args.head_dim)
     strong = cfg.name == "C5"
     lo, hi = shard_for_rank(cfg, max(world, args.gpus), 0, strong)
-    q, k, v = make_qkv(1, 1, cfg.L, cfg.d, seed=cfg.seed)
-    Q, K, V = head_inputs_f64(q, k, v, 0, 0)
-    g = global_flags(cfg.L, cfg.global_idx)
-    ex = ExtraIndex(cfg.L, cfg.extra_idx)
+    cores = os.cpu_count() or 1
     R = 32
-    rng = np.random.default_rng(0)
+    with mp.get_context("spawn").Pool(cores, initializer=_ref_init, initargs=(name, args.head_dim, 2)) as pool:
+        step_no = 0
 
-    def step():
-        rows = rng.choice(cfg.L, R, replace=False)
-        nnz = sum(mask_row_cols(int(r), cfg.L, cfg.window, g, ex).size for r in rows)
-        t0 = time.perf_counter()
-        attention_rows(Q, K, V, rows, cfg.window, g, ex)
-        return time.perf_counter() - t0, nnz
+        def step():
+            nonlocal step_no
+            tasks = [(step_no * cores + i, R) for i in range(cores)]
+            step_no += 1
+            t0 = time.perf_counter()
+            res = pool.map(_ref_task, tasks, chunksize=1)
+            return time.perf_counter() - t0, sum(n for _, n in res)
 
-    for _ in range(args.warmup):
-        step()
-    tot_t, tot_nnz = 0.0, 0
-    for _ in range(args.steps):
-        t, n = step()
-        tot_t += t
-        tot_nnz += n
+        for _ in range(args.warmup):
+            step()
+        tot_t, tot_nnz = 0.0, 0
+        for _ in range(args.steps):
+            t, n = step()
+            tot_t += t
+            tot_nnz += n
     value = 4.0 * tot_nnz * cfg.d / tot_t / 1e12
-    cores = 1  # attention_rows: per-row numpy on one thread (vectors of <= L elements)
     line = {
         "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * tot_t / args.steps,
         "higher_is_better": True, "scaling": "strong" if strong else "weak", "vs_baseline": None, "dtype": "f64",
         "data": "synthetic", "config": workload_config(cfg, args.gpus, strong, hi - lo),
         "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle",
-                         "sample": f"oracle.attention_rows (fp64) on {R} random rows of one (b,h) head of "
-                                   f"{cfg.name} per step"},
+                         "sample": f"oracle.attention_rows (fp64) on {R} random rows of one (b,h) head per worker, "
+                                   f"{cores} single-threaded worker processes per step, {cfg.name}"},
         "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)

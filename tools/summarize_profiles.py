@@ -12,7 +12,9 @@ PROF = os.path.join(ROOT, "profiles")
 tag = sys.argv[1] if len(sys.argv) > 1 else "r01"
 os.makedirs(PROF, exist_ok=True)
 
-WANT = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum", "lts__t_bytes.sum",
+WANT = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum", "lts__t_sectors.sum",
+        "lts__t_sectors.sum.pct_of_peak_sustained_elapsed", "LTS.TriageCompute.lts__throughput.avg.pct_of_peak_sustained_elapsed",
+        "lts__t_sector_hit_rate.pct", "lts__t_requests_srcunit_tex.sum",
         "sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_active",
         "sm__inst_executed_pipe_xu.avg.pct_of_peak_sustained_active",
         "smsp__issue_active.avg.pct_of_peak_sustained_active", "sm__warps_active.avg.per_cycle_active",
@@ -31,7 +33,8 @@ def raw(rep):
 traffic_path = os.path.join(PROF, "ncu_traffic.json")
 traffic = json.load(open(traffic_path)) if os.path.exists(traffic_path) else {}
 for name, cfg, key in [("full_c2_coarse", "C2", "coarse"), ("full_c4_fine", "C4", "fine"),
-                       ("full_c4_coarse", "C4", "coarse")]:
+                       ("full_c4_coarse", "C4", "coarse"), ("full_c3_coarse", "C3", "coarse"),
+                       ("full_c2d128_coarse", "C2-d128", "coarse")]:
     rep = os.path.join(OUT, name + ".ncu-rep")
     if not os.path.exists(rep):
         continue
@@ -45,13 +48,18 @@ for name, cfg, key in [("full_c2_coarse", "C2", "coarse"), ("full_c4_fine", "C4"
         f = float(v.replace(",", ""))
         return f * {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}.get(u, 1)
     rd = tobytes(*m["dram__bytes_read.sum"]); wr = tobytes(*m["dram__bytes_write.sum"])
-    traffic.setdefault(cfg, {})[key] = {"dram_bytes_per_launch": rd + wr, "dram_read": rd, "dram_write": wr,
-                                        "source": f"profiles/{tag}_ncu_{name}.txt"}
+    ent = {"dram_bytes_per_launch": rd + wr, "dram_read": rd, "dram_write": wr,
+           "source": f"profiles/{tag}_ncu_{name}.txt"}
+    if "lts__t_sectors.sum" in m:
+        ent["lts_bytes_per_launch"] = 32.0 * float(m["lts__t_sectors.sum"][1].replace(",", ""))
+        ent["lts_sectors_pct_of_peak"] = float(m["lts__t_sectors.sum.pct_of_peak_sustained_elapsed"][1].replace(",", ""))
+        ent["l2_hit_rate_pct"] = float(m["lts__t_sector_hit_rate.pct"][1].replace(",", ""))
+    traffic.setdefault(cfg, {})[key] = ent
 json.dump(traffic, open(traffic_path, "w"), indent=1)
-for W in ("C2", "C4"):
+for W in ("C2", "C3", "C4", "C2-d128"):
     src = os.path.join(OUT, f"launches_{W}.csv")
     if not os.path.exists(src):
         continue
-    rows = [l for l in open(src) if l.startswith('"ID"') or "mg::" in l or "coarse" in l or "fine_rows" in l]
+    rows = [l for l in open(src) if l.startswith('"ID"') or "mg::" in l or "coarse" in l or "fine_" in l]
     open(os.path.join(PROF, f"{tag}_launches_{W}.csv"), "w").writelines(rows)
 print("written", sorted(os.listdir(PROF)))
