@@ -19,6 +19,7 @@
 // running max/sum and O accumulate in fp32. Lazy rescaling: the exponent keeps a stale max until
 // a step's max exceeds it by 8/c (p <= 256), warp-uniform because all lanes see the same max.
 #include <algorithm>
+#include <cstdlib>
 #include <map>
 #include <mutex>
 #include <utility>
@@ -402,6 +403,264 @@ __global__ void __launch_bounds__(kWarps * 32, FCfg<kD>::kMinB) fine_mma_kernel(
   cp_async_wait<0>();
 }
 
+// ---------------------------------------------------------------------------------------------
+// Two heads per warp (d = 64, even head count): heads 2u and 2u + 1 of one batch element share the
+// CSR row's column indices (the plan is shared across heads, A8), so one index window, one set of
+// shuffles / gather offsets and one row's bookkeeping serve both heads, and each warp runs two
+// independent SDDMM -> softmax -> SpMM chains (instruction-level parallelism for the mma.sync ->
+// softmax -> mma.sync latency chain). Stage layout: [K_h0 kS rows][V_h0 kS rows][K_h1][V_h1][q_h0][q_h1].
+#ifndef MG_FINE_MINB2
+#define MG_FINE_MINB2 3
+#endif
+namespace {
+constexpr int kHB = 2 * kS * 128;                 // K + V rows of one head in a stage
+constexpr int kQOff2 = 2 * kHB;
+constexpr int kStageBytes2 = kQOff2 + 2 * 128;
+constexpr int kSmemBytes2 = kWarps * kStages * kStageBytes2;
+}  // namespace
+
+template <bool kBF16, bool kPad>
+__global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB2) fine_mma2_kernel(const FineParams p) {
+  constexpr int kD = 64, kRowBytes = 128, kLPR = 8, kRPI = 4, kJ = 4;
+  extern __shared__ __align__(128) uint8_t fsm[];
+  const int lane = threadIdx.x & 31;
+  const int g = lane >> 2, t = lane & 3;
+  const float c = p.scale_log2;
+  const float thresh = 8.f / c;
+  const int nhp = p.BH >> 1;                           // head pairs per fine row
+  const int64_t nrows = (int64_t)nhp * p.n_fine_rows;
+  const bool r32 = nrows <= (int64_t)0xffffffffLL;
+  const int64_t W = (int64_t)gridDim.x * kWarps;
+  const int64_t w0 = (int64_t)blockIdx.x * kWarps + (threadIdx.x >> 5);
+  const uint32_t ring = (uint32_t)__cvta_generic_to_shared(fsm) + (threadIdx.x >> 5) * (kStages * kStageBytes2);
+  const uint32_t ksl = (uint32_t)p.k.sl, vsl = (uint32_t)p.v.sl;
+  // head strides fit 32 bits (checked by the launcher)
+  const uint32_t ksh = (uint32_t)p.k.sh, vsh = (uint32_t)p.v.sh, qsh = (uint32_t)p.q.sh;
+  constexpr int kIters = kS / kRPI;
+  uint32_t doff[kIters];
+#pragma unroll
+  for (int i = 0; i < kIters; ++i) {
+    const int R = lane / kLPR + kRPI * i;
+    doff[i] = R * kRowBytes + (((lane % kLPR) ^ (R & 7)) << 4);
+  }
+
+  int64_t gi = w0;
+  int ibeg = 0, iend = 0, is = 0, icol = -1, icol_next = -1;
+  const uint16_t *iK = nullptr, *iV = nullptr, *iQ = nullptr;
+  auto open_issue_row = [&]() {
+    if (gi < nrows) {
+      int u0, fi;
+      split_row(gi, p.n_fine_rows, r32, u0, fi);
+      const int bh = (p.fine_sample ? __ldg(p.fine_sample + fi) * p.H : 0) + 2 * u0;   // first head of the pair
+      ibeg = __ldg(p.row_ptr + fi);
+      iend = __ldg(p.row_ptr + fi + 1);
+      const int bb = bh / p.H, hh = bh % p.H;
+      iK = p.k.data + bb * p.k.sb + hh * p.k.sh + (lane % kLPR) * 8;
+      iV = p.v.data + bb * p.v.sb + hh * p.v.sh + (lane % kLPR) * 8;
+      const int rq = __ldg(p.fine_rows + fi) & 0x7fffffff;
+      // lanes 0-7: q of the first head, lanes 8-15: q of the second
+      iQ = p.q.data + bb * p.q.sb + hh * p.q.sh + (int64_t)rq * p.q.sl + (lane % kLPR) * 8 + ((lane >> 3) & 1) * qsh;
+    }
+    is = 0;
+  };
+  auto issue_step = [&](uint32_t stg) {
+    if (gi < nrows) {
+      const int nb0 = ibeg + kS * is;
+      if ((is & 1) == 0) icol = is > 0 ? icol_next : (nb0 + lane < iend ? __ldg(p.cols + nb0 + lane) : -1);
+      const int off = (is & 1) * 16 + lane / kLPR;
+      const uint32_t st = ring + stg * kStageBytes2;
+      if (is == 0 && lane < 2 * kLPR) cp_async16(st + kQOff2 + (lane << 4), iQ);
+#pragma unroll
+      for (int i = 0; i < kIters; ++i) {
+        const uint32_t cc = (uint32_t)max(__shfl_sync(0xffffffffu, icol, off + kRPI * i), 0);
+        const uint16_t* k0 = iK + cc * ksl;
+        const uint16_t* v0 = iV + cc * vsl;
+        cp_async16(st + doff[i], k0);
+        cp_async16(st + doff[i] + kS * kRowBytes, v0);
+        cp_async16(st + kHB + doff[i], k0 + ksh);
+        cp_async16(st + kHB + doff[i] + kS * kRowBytes, v0 + vsh);
+      }
+      if ((is & 1) == 1 && nb0 + kS < iend) icol_next = nb0 + kS + lane < iend ? __ldg(p.cols + nb0 + kS + lane) : -1;
+      if (nb0 + kS < iend) {
+        ++is;
+      } else {
+        gi += W;
+        open_issue_row();
+      }
+    }
+    cp_async_commit();
+  };
+
+  open_issue_row();
+#pragma unroll
+  for (int s0 = 0; s0 < kStages - 1; ++s0) issue_step(s0);
+  uint32_t stage = 0, istage = kStages - 1;
+  const uint32_t a_row = (lane & 7) * kRowBytes, b_row = a_row + 8 * kRowBytes;
+  const uint32_t vr = (lane & 7) + 8 * (lane >> 4);
+
+  for (int64_t gw = w0; gw < nrows; gw += W) {
+    int u0, fi;
+    split_row(gw, p.n_fine_rows, r32, u0, fi);
+    const int bh = (p.fine_sample ? __ldg(p.fine_sample + fi) * p.H : 0) + 2 * u0;
+    const int enc = __ldg(p.fine_rows + fi);
+    const int r = enc & 0x7fffffff;
+    const bool final_out = enc < 0;
+    const int bb = bh / p.H, hh = bh % p.H;
+    uint32_t qa[2][kJ], qb[2][kJ];
+    const int beg = __ldg(p.row_ptr + fi), end = __ldg(p.row_ptr + fi + 1);
+    const int nvalid = kPad ? max(__ldg(p.valid_len + bb), 0) : 0x7fffffff;
+    const bool pad_row = kPad && r >= nvalid;
+
+    float m[2] = {-INFINITY, -INFINITY}, l[2] = {0.f, 0.f};
+    float acc[2][kJ][4];
+#pragma unroll
+    for (int hd = 0; hd < 2; ++hd)
+#pragma unroll
+      for (int j = 0; j < kJ; ++j)
+#pragma unroll
+        for (int e = 0; e < 4; ++e) acc[hd][j][e] = 0.f;
+
+    for (int base = beg; base < end; base += kS) {
+      issue_step(istage);
+      istage = istage == kStages - 1 ? 0 : istage + 1;
+      cp_async_wait<kStages - 1>();
+      __syncwarp();
+      const uint32_t st = ring + stage * kStageBytes2;
+      stage = stage == kStages - 1 ? 0 : stage + 1;
+      if (base == beg) {
+#pragma unroll
+        for (int hd = 0; hd < 2; ++hd)
+#pragma unroll
+          for (int j = 0; j < kJ; ++j) {
+            asm volatile("ld.shared.u32 %0, [%1];" : "=r"(qa[hd][j]) : "r"(st + kQOff2 + hd * 128 + 32 * j + 4 * t));
+            asm volatile("ld.shared.u32 %0, [%1];" : "=r"(qb[hd][j]) : "r"(st + kQOff2 + hd * 128 + 32 * j + 16 + 4 * t));
+          }
+      }
+      const int rem = end - base - 2 * t;
+      float s[2][4];
+#pragma unroll
+      for (int hd = 0; hd < 2; ++hd) {
+        const uint32_t sk = st + hd * kHB;
+        float sa[2][4] = {{0.f, 0.f, 0.f, 0.f}, {0.f, 0.f, 0.f, 0.f}};
+        float sb[2][4] = {{0.f, 0.f, 0.f, 0.f}, {0.f, 0.f, 0.f, 0.f}};
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          uint32_t ka[4], kb[4];
+          const uint32_t sw = ((uint32_t)(((lane >> 3) + 4 * h) ^ (lane & 7))) << 4;
+          ldsm_x4(ka, sk + a_row + sw);
+          ldsm_x4(kb, sk + b_row + sw);
+          mma16816<kBF16>(sa[h], qa[hd][2 * h], qa[hd][2 * h], qb[hd][2 * h], qb[hd][2 * h], ka[0], ka[1]);
+          mma16816<kBF16>(sb[h], qa[hd][2 * h], qa[hd][2 * h], qb[hd][2 * h], qb[hd][2 * h], kb[0], kb[1]);
+          mma16816<kBF16>(sa[h], qa[hd][2 * h + 1], qa[hd][2 * h + 1], qb[hd][2 * h + 1], qb[hd][2 * h + 1], ka[2], ka[3]);
+          mma16816<kBF16>(sb[h], qa[hd][2 * h + 1], qa[hd][2 * h + 1], qb[hd][2 * h + 1], qb[hd][2 * h + 1], kb[2], kb[3]);
+        }
+        s[hd][0] = rem > 0 ? sa[0][0] + sa[1][0] : -INFINITY;
+        s[hd][1] = rem > 1 ? sa[0][1] + sa[1][1] : -INFINITY;
+        s[hd][2] = rem > 8 ? sb[0][0] + sb[1][0] : -INFINITY;
+        s[hd][3] = rem > 9 ? sb[0][1] + sb[1][1] : -INFINITY;
+      }
+      if (kPad) {   // padding: mask the columns at or beyond n_b (same columns for both heads)
+        const int o4[4] = {0, 1, 8, 9};
+#pragma unroll
+        for (int i = 0; i < 4; ++i)
+          if (rem > o4[i] && __ldg(p.cols + base + 2 * t + o4[i]) >= nvalid) s[0][i] = s[1][i] = -INFINITY;
+      }
+      float mx[2];
+#pragma unroll
+      for (int hd = 0; hd < 2; ++hd) mx[hd] = fmaxf(fmaxf(s[hd][0], s[hd][1]), fmaxf(s[hd][2], s[hd][3]));
+#pragma unroll
+      for (int hd = 0; hd < 2; ++hd) mx[hd] = fmaxf(mx[hd], __shfl_xor_sync(0xffffffffu, mx[hd], 1));
+#pragma unroll
+      for (int hd = 0; hd < 2; ++hd) mx[hd] = fmaxf(mx[hd], __shfl_xor_sync(0xffffffffu, mx[hd], 2));
+#pragma unroll
+      for (int hd = 0; hd < 2; ++hd) {
+        if (mx[hd] > m[hd] + thresh) {
+          const float alpha = ex2((m[hd] - mx[hd]) * c);
+          l[hd] *= alpha;
+#pragma unroll
+          for (int j = 0; j < kJ; ++j)
+#pragma unroll
+            for (int e = 0; e < 4; ++e) acc[hd][j][e] *= alpha;
+          m[hd] = mx[hd];
+        }
+      }
+#pragma unroll
+      for (int hd = 0; hd < 2; ++hd) {
+        const float nbias = m[hd] == -INFINITY ? 0.f : -m[hd] * c;
+        float pv[4];
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          pv[i] = ex2(fmaf(s[hd][i], c, nbias));
+          l[hd] += pv[i];
+        }
+        const uint32_t pb0 = pack2<kBF16>(pv[0], pv[1]), pb1 = pack2<kBF16>(pv[2], pv[3]);
+        const uint32_t sv = st + hd * kHB + kS * kRowBytes;
+#pragma unroll
+        for (int j = 0; j < kJ; ++j) {
+          uint32_t a[4];
+          const uint32_t ch = 2 * j + ((lane >> 3) & 1);
+          ldsm_x4_t(a, sv + vr * kRowBytes + ((ch ^ (vr & 7)) << 4));
+          mma16816<kBF16>(acc[hd][j], a[0], a[1], a[2], a[3], pb0, pb1);
+        }
+      }
+      __syncwarp();
+    }
+    // ---- row epilogue of both heads
+#pragma unroll
+    for (int hd = 0; hd < 2; ++hd) {
+      float lh = l[hd];
+      lh += __shfl_xor_sync(0xffffffffu, lh, 1);
+      lh += __shfl_xor_sync(0xffffffffu, lh, 2);
+      float v0 = acc[hd][0][0], v1 = acc[hd][0][2];
+#pragma unroll
+      for (int j = 1; j < 4; ++j)
+        if (t == j) {
+          v0 = acc[hd][j][0];
+          v1 = acc[hd][j][2];
+        }
+      const int d0 = 16 * t + g;
+      float inv = lh > 0.f ? 1.f / lh : 0.f;
+      bool write_o = final_out;
+      if (!final_out) {
+        const size_t idx = (size_t)(2 * u0 + hd) * p.n_fine_rows + fi;
+        __stcg(p.part_acc + idx * kD + d0, v0);
+        __stcg(p.part_acc + idx * kD + d0 + 8, v1);
+        if (lane == 0) __stcg(p.part_ml + idx, make_float2(m[hd], lh));
+        if (p.concurrent) {
+          __threadfence();
+          __syncwarp();
+          int old = 0;
+          if (lane == 0) old = atomicAdd(p.part_flags + idx, 1);
+          old = __shfl_sync(0xffffffffu, old, 0);
+          if (old & 1) {
+            __threadfence();
+            const float2 mlc = __ldcg(p.part_c_ml + idx);
+            const float mt = fmaxf(m[hd], mlc.x);
+            const float mu = mt == -INFINITY ? 0.f : mt;
+            const float af = ex2((m[hd] - mu) * c), ac = ex2((mlc.x - mu) * c);
+            const float den = lh * af + mlc.y * ac;
+            inv = den > 0.f ? 1.f / den : 0.f;
+            v0 = v0 * af + __ldcg(p.part_c_acc + idx * kD + d0) * ac;
+            v1 = v1 * af + __ldcg(p.part_c_acc + idx * kD + d0 + 8) * ac;
+            write_o = true;
+          }
+        }
+      }
+      if (pad_row) {
+        write_o = final_out;
+        v0 = v1 = 0.f;
+      }
+      if (write_o) {
+        uint16_t* orow = p.o.data + bb * p.o.sb + (hh + hd) * p.o.sh + (int64_t)r * p.o.sl;
+        const uint32_t pk = pack2<kBF16>(v0 * inv, v1 * inv);
+        orow[d0] = (uint16_t)(pk & 0xffffu);
+        orow[d0 + 8] = (uint16_t)(pk >> 16);
+      }
+    }
+  }
+  cp_async_wait<0>();
+}
+
 cudaError_t launch_fine_mma(const FineParams& p, bool bf16, int sms, cudaStream_t stream) {
   const int64_t warps = (int64_t)p.BH * p.n_fine_rows;
   if (warps == 0) return cudaSuccess;
@@ -411,9 +670,19 @@ cudaError_t launch_fine_mma(const FineParams& p, bool bf16, int sms, cudaStream_
                              fine_mma_kernel<false, false, 128>, fine_mma_kernel<false, true, 128>,
                              fine_mma_kernel<true, false, 128>,  fine_mma_kernel<true, true, 128>};
   if (p.d != 64 && p.d != 128) return cudaErrorInvalidValue;
-  const int vi = (p.d == 128 ? 4 : 0) + (bf16 ? 2 : 0) + (p.valid_len ? 1 : 0);
-  const K kern = table[vi];
-  const int kSmemBytes = p.d == 128 ? FCfg<128>::kSmemBytes : FCfg<64>::kSmemBytes;
+  // two heads per warp when the heads pair up within a batch element and the head strides fit the
+  // kernel's 32-bit offsets (MG_FINE_HEADS2=0 in the environment selects one head per warp, A/B)
+  static const bool no_hp2 = [] {
+    const char* e = std::getenv("MG_FINE_HEADS2");
+    return e && e[0] == '0';
+  }();
+  const bool hp2 = !no_hp2 && p.d == 64 && (p.H % 2) == 0 && p.k.sh < (int64_t(1) << 31) &&
+                   p.v.sh < (int64_t(1) << 31) && p.q.sh < (int64_t(1) << 31);
+  static const K table2[4] = {fine_mma2_kernel<false, false>, fine_mma2_kernel<false, true>,
+                              fine_mma2_kernel<true, false>, fine_mma2_kernel<true, true>};
+  const int vi = hp2 ? 8 + (bf16 ? 2 : 0) + (p.valid_len ? 1 : 0) : (p.d == 128 ? 4 : 0) + (bf16 ? 2 : 0) + (p.valid_len ? 1 : 0);
+  const K kern = hp2 ? table2[vi - 8] : table[vi];
+  const int kSmemBytes = hp2 ? kSmemBytes2 : (p.d == 128 ? FCfg<128>::kSmemBytes : FCfg<64>::kSmemBytes);
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytes);
   if (e != cudaSuccess) return e;
   // persistent grid: every resident block slot of `sms` SMs (the plan's SM count, or its num_sms
@@ -433,7 +702,8 @@ cudaError_t launch_fine_mma(const FineParams& p, bool bf16, int sms, cudaStream_
     }
     n = it->second;
   }
-  const int64_t blocks = std::min<int64_t>((warps + kWarps - 1) / kWarps, (int64_t)n * std::max(sms, 1));
+  const int64_t units = hp2 ? warps / 2 : warps;
+  const int64_t blocks = std::min<int64_t>((units + kWarps - 1) / kWarps, (int64_t)n * std::max(sms, 1));
   kern<<<(unsigned)blocks, kWarps * 32, kSmemBytes, stream>>>(p);
   return cudaGetLastError();
 }
