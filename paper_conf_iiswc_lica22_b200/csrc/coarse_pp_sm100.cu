@@ -75,6 +75,7 @@ struct __align__(16) Ctl {
   uint64_t q_full[2], q_empty[2];
   uint64_t k_full[kSt], k_empty[kSt], v_full[kSt], v_empty[kSt];
   uint64_t s_full, s_free, p_full, pv_done;
+  uint64_t mk_full[kSt], mk_empty[kSt];       // late-P.V mode: tile descriptor / bitmask ring
   uint32_t tmem_base;
   int32_t dense_last;                         // split dense item: this chunk finished its row group last
 };
@@ -313,6 +314,23 @@ __device__ __forceinline__ void tl_item(const CoarseParams& p, uint32_t it, int 
 #endif
 constexpr bool kIdleQuarters = MG_IDLE_QUARTERS;
 
+// Mask ring (MG_MASK_RING, default): the tile descriptors and bitmasks travel in their own
+// two-stage ring, released by the softmax warps once read, instead of with the V stage (released
+// only when P.V(n) has completed), so a tile's softmax never waits for its V load (measured C2
+// 0.1426 vs 0.1433 ms, C3 0.0774 vs 0.0782, same box).
+// Late P.V (MG_PV_LATE, off): the MMA warp issues P.V(n-1) after S(n+1) instead of after S(n), so
+// the next S does not queue behind a P.V in the in-order tensor pipe (an item's last P.V, which the
+// epilogue waits on, still goes right after the next S): measured slower (C2 0.168 vs 0.141 ms),
+// the softmax then waits on the later P.V before its P store.
+#ifndef MG_PV_LATE
+#define MG_PV_LATE 0
+#endif
+#ifndef MG_MASK_RING
+#define MG_MASK_RING 1
+#endif
+constexpr bool kLatePV = MG_PV_LATE;
+constexpr bool kLate = MG_MASK_RING || MG_PV_LATE;   // (the mask ring; the late P.V needs it)
+
 #ifndef MG_PRE_CHUNKS
 #define MG_PRE_CHUNKS 4
 #endif
@@ -454,6 +472,8 @@ __global__ void __launch_bounds__(kThreads, DCfg<kD>::kMinBlocks)
       mbar_init(bar(ctl->k_empty[s]), 1);
       mbar_init(bar(ctl->v_full[s]), 1);
       mbar_init(bar(ctl->v_empty[s]), 1);
+      mbar_init(bar(ctl->mk_full[s]), 1);
+      mbar_init(bar(ctl->mk_empty[s]), 4);
     }
     mbar_init(bar(ctl->s_full), 1);
     mbar_init(bar(ctl->s_free), 4);
@@ -568,8 +588,10 @@ __global__ void __launch_bounds__(kThreads, DCfg<kD>::kMinBlocks)
             __syncwarp();
             if (lane == 0) mbar_arrive(kf);
           }
-          mbar_wait(bar(ctl->v_empty[st]), sph);
           const uint32_t mbytes = maskA >= 0 ? kMaskBytes : 0;
+          // the tile's descriptor / bitmask stage: with the V stage, or (late P.V) its own ring
+          if (kLate) mbar_wait(bar(ctl->mk_empty[st]), sph);
+          else mbar_wait(bar(ctl->v_empty[st]), sph);
           if (kPad) {
             // padding: the tile's columns below n_b (published with vdesc by the v_full arrive)
             const int nvalid = min(max(__ldg(p.valid_len + bb), 0), (int)p.L);
@@ -604,19 +626,32 @@ __global__ void __launch_bounds__(kThreads, DCfg<kD>::kMinBlocks)
             }
           }
           if (lane == 0) {
-            ctl->vdesc[st] = make_int2(ncols, maskA);   // published by the v_full arrive
+            ctl->vdesc[st] = make_int2(ncols, maskA);   // published by the v_full (mk_full) arrive
             tl_rec(p, g, 6);
+          }
+          const uint32_t vmb = kLate ? 0u : mbytes;     // mask bytes completing on the V barrier
+          if (kLate) {
+            const uint32_t mf = bar(ctl->mk_full[st]);
+            if (lane == 0) {
+              if (mbytes) {
+                mbar_arrive_expect_tx(mf, mbytes);
+                bulk_load(sMsk + st * kMaskBytes, p.masks + (size_t)maskA * 256, kMaskBytes, mf);
+              } else {
+                mbar_arrive(mf);
+              }
+            }
+            mbar_wait(bar(ctl->v_empty[st]), sph);
           }
           if (kind == 0) {
             if (lane == 0) {
-              mbar_arrive_expect_tx(vf, (kDbgNoLoads ? 0 : kTileBytes) + mbytes);
+              mbar_arrive_expect_tx(vf, (kDbgNoLoads ? 0 : kTileBytes) + vmb);
               if (!kDbgNoLoads) {
 #pragma unroll
                 for (int sb = 0; sb < kNSub; ++sb) tma_load_4d(dV + sb * kSub, &tmv, vf, 64 * sb, arg, hh, bb, pol_kv);
               }
             }
           } else if (p.gather_tma) {
-            if (lane == 0) mbar_arrive_expect_tx(vf, ncols * 2 * kD + mbytes);
+            if (lane == 0) mbar_arrive_expect_tx(vf, ncols * 2 * kD + vmb);
             __syncwarp();
             if (4 * lane < ncols) {
 #pragma unroll
@@ -627,9 +662,9 @@ __global__ void __launch_bounds__(kThreads, DCfg<kD>::kMinBlocks)
             gather_rows<kD>(dV, p.v.data + bb * p.v.sb + hh * p.v.sh, p.v.sl, p.strip_cols + arg, ncols, ncols, lane);
             fence_proxy_async_smem();
             __syncwarp();
-            if (lane == 0) mbar_arrive_expect_tx(vf, mbytes);
+            if (lane == 0) mbar_arrive_expect_tx(vf, vmb);
           }
-          if (lane == 0 && mbytes) bulk_load(sMsk + st * kMaskBytes, p.masks + (size_t)maskA * 256, kMaskBytes, vf);
+          if (!kLate && lane == 0 && mbytes) bulk_load(sMsk + st * kMaskBytes, p.masks + (size_t)maskA * 256, kMaskBytes, vf);
         }
       }
     }
@@ -675,8 +710,11 @@ __global__ void __launch_bounds__(kThreads, DCfg<kD>::kMinBlocks)
       struct Pend {
         uint32_t n, st;
         int ncols;
-        bool first, valid;
-      } pend{0, 0, 0, false, false};
+        bool first, valid, last;
+      } pend{0, 0, 0, false, false, false};
+      // late P.V: up to two pending P.V (tiles n-2, n-1 while S(n) is issued), in tile order
+      Pend fifo[2];
+      int nfifo = 0;
       auto issue_pv = [&](const Pend& e) {
         mbar_wait(bar(ctl->v_full[e.st]), (e.n / kSt) & 1);
         mbar_wait(bar(ctl->p_full), e.n & 1);
@@ -694,6 +732,10 @@ __global__ void __launch_bounds__(kThreads, DCfg<kD>::kMinBlocks)
         mma_commit(bar(ctl->pv_done));
         mma_commit(bar(ctl->v_empty[e.st]));
       };
+      auto flush_fifo = [&]() {
+        for (int i = 0; i < nfifo; ++i) issue_pv(fifo[i]);
+        nfifo = 0;
+      };
       for (uint32_t it = 0;; ++it) {
         const uint32_t slot = it % kItems;
         mbar_wait(bar(ctl->item_full[slot]), (it / kItems) & 1);
@@ -704,7 +746,9 @@ __global__ void __launch_bounds__(kThreads, DCfg<kD>::kMinBlocks)
         if (u >= p.total_units) break;
         const uint32_t qs = it & 1;
         // finish the previous item first unless this item's Q tile is already resident
-        if (pend.valid && !mbar_test_wait(bar(ctl->q_full[qs]), (it >> 1) & 1)) {
+        if (kLatePV) {
+          if (nfifo && !mbar_test_wait(bar(ctl->q_full[qs]), (it >> 1) & 1)) flush_fifo();
+        } else if (pend.valid && !mbar_test_wait(bar(ctl->q_full[qs]), (it >> 1) & 1)) {
           issue_pv(pend);
           pend.valid = false;
         }
@@ -731,10 +775,20 @@ __global__ void __launch_bounds__(kThreads, DCfg<kD>::kMinBlocks)
           mma_commit(bar(ctl->k_empty[st]));
           // (q_empty is arrived by the softmax epilogue: the Q buffer also stages the item's O tile)
           tl_rec(p, n, 3);
-          if (pend.valid) issue_pv(pend);
-          pend = Pend{n, st, ncols, j == 0, true};
+          if (kLatePV) {
+            // due now: P.V(k) for k <= n - 2, and P.V(n - 1) if it is its item's last tile
+            int done = 0;
+            while (done < nfifo && (fifo[done].n + 2 <= n || fifo[done].last)) issue_pv(fifo[done++]);
+            for (int i = done; i < nfifo; ++i) fifo[i - done] = fifo[i];
+            nfifo -= done;
+            fifo[nfifo++] = Pend{n, st, ncols, j == 0, true, j == ntiles - 1};
+          } else {
+            if (pend.valid) issue_pv(pend);
+            pend = Pend{n, st, ncols, j == 0, true, false};
+          }
         }
       }
+      if (kLatePV) flush_fifo();
       if (pend.valid) issue_pv(pend);
     }
     __syncwarp();
@@ -781,13 +835,17 @@ __global__ void __launch_bounds__(kThreads, DCfg<kD>::kMinBlocks)
           if (lane == 0) mbar_arrive(bar(ctl->s_free));
           if (n > 0) mbar_wait(bar(ctl->pv_done), (n - 1) & 1);
           __syncwarp();
-          if (lane == 0) mbar_arrive(bar(ctl->p_full));
+          if (lane == 0) {
+            mbar_arrive(bar(ctl->p_full));
+            if (kLate) mbar_arrive(bar(ctl->mk_empty[n % kSt]));
+          }
           continue;
         }
         const uint32_t st = n % kSt;
         mbar_wait(bar(ctl->s_full), n & 1);
-        // the tile's descriptor and bitmask travel with its V stage (freed only after P.V(n))
-        mbar_wait(bar(ctl->v_full[st]), (n / kSt) & 1);
+        // the tile's descriptor and bitmask travel with its V stage (freed only after P.V(n)), or in
+        // their own ring (late P.V)
+        mbar_wait(bar(kLate ? ctl->mk_full[st] : ctl->v_full[st]), (n / kSt) & 1);
         tc_fence_after();
         const int2 desc = ctl->vdesc[st];                 // {ncols, maskA}
         const TileCtx tc{tl, sMsk + st * kMaskBytes + t * 16, desc.y >= 0, kPad ? ctl->cmask[st] : nullptr,
@@ -799,6 +857,10 @@ __global__ void __launch_bounds__(kThreads, DCfg<kD>::kMinBlocks)
           case 3: softmax_tile<3, kBF16, kD>(tc, m, l); break;
           case 2: softmax_tile<2, kBF16, kD>(tc, m, l); break;
           default: softmax_tile<1, kBF16, kD>(tc, m, l); break;
+        }
+        if (kLate) {   // this tile's descriptor / mask stage may be refilled
+          __syncwarp();
+          if (lane == 0) mbar_arrive(bar(ctl->mk_empty[st]));
         }
       }
       // ---------------------------------------------------------------- epilogue (a-8)
