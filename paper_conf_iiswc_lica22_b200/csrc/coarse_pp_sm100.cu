@@ -42,6 +42,29 @@ using namespace ptx;
 
 namespace {
 
+// Column-split softmax: 8 softmax warps per CTA, two per TMEM lane quarter, each taking 64 of a
+// tile's 128 columns (the pair exchanges its half-tile row maxima through shared memory and a
+// 64-thread named barrier); 384 threads per CTA, control warps 8-11. At d = 128 (one CTA per SM)
+// this gives each SM sub-partition two softmax warps instead of one (MG_CSPLIT128, default on);
+// at d = 64 (two CTAs per SM, MG_CSPLIT) it measured slower (C2 0.1555 vs 0.1427 ms).
+#ifndef MG_CSPLIT
+#define MG_CSPLIT 0
+#endif
+#ifndef MG_CSPLIT128
+#define MG_CSPLIT128 1
+#endif
+template <int kD>
+struct WCfg {
+  static constexpr bool kCS = kD == 64 ? (bool)MG_CSPLIT : (bool)MG_CSPLIT128;
+  static constexpr int kSoftWarps = kCS ? 8 : 4;
+  static constexpr int kThreads = 32 * (kSoftWarps + 4);
+  static constexpr int kWProd = kSoftWarps, kWMma = kSoftWarps + 1, kWSched = kSoftWarps + 2, kWIdle = kSoftWarps + 3;
+  // setmaxnreg per warpgroup: (65536 / CTAs per SM / threads, rounded down to 8) per thread in the pool
+  static constexpr int kRegsCtl = kCS ? (kD == 64 ? 48 : 88) : 64;
+  static constexpr int kRegsSoftmax = kCS ? (kD == 64 ? 96 : 208) : 192;
+};
+static_assert(256 * 96 + 128 * 48 <= (65536 / 2 / 384 & ~7) * 384, "register pool (column split, d = 64)");
+static_assert(256 * 208 + 128 * 88 <= (65536 / 1 / 384 & ~7) * 384, "register pool (column split, d = 128)");
 constexpr int kThreads = 256;
 constexpr int kSt = 2;                       // K ring and V ring depth
 constexpr int kItems = 4;                    // work-item ring depth
@@ -78,6 +101,8 @@ struct __align__(16) Ctl {
   uint64_t mk_full[kSt], mk_empty[kSt];       // late-P.V mode: tile descriptor / bitmask ring
   uint32_t tmem_base;
   int32_t dense_last;                         // split dense item: this chunk finished its row group last
+  float xmax[2][2][128];                      // column split: [tile parity][half][row] half-tile maxima
+  float xsum[128];                            // column split: half 1's row sum for the epilogue
 };
 
 template <int kD>
@@ -432,10 +457,90 @@ __device__ __forceinline__ void softmax_tile(const TileCtx& x, float& m, float& 
   }
 }
 
+// Column-split variant of softmax_tile (d = 64): this warp holds NH (0..2) of the tile's 32-column
+// chunks, chunks [2h, 2h + NH); the half-tile maxima of the two warps sharing the rows are combined
+// before the lazy-rescale decision, so both warps take the same (deterministic) decision and use
+// the same reference max for P. Each warp keeps its own partial row sum; it rescales O columns
+// [32h, 32h + 32) and stores P columns [32h, 32h + 32) (packed pairs).
+template <int NH, bool kBF16, int kD>
+__device__ __forceinline__ void softmax_tile_cs(const TileCtx& x, float& m, float& l, int h, int row,
+                                                uint32_t xbar, float* xmax) {
+  constexpr uint32_t kTO = DCfg<kD>::kTO;
+  const uint32_t lane = threadIdx.x & 31;
+  uint32_t r[NH > 0 ? NH : 1][32];
+#pragma unroll
+  for (int q = 0; q < NH; ++q) tmem_ld32(x.tl + kTS + (2 * h + q) * 32, r[q]);
+  if (NH > 0) tmem_wait_ld();
+  tc_fence_before();
+  __syncwarp();
+  if (lane == 0) mbar_arrive(x.s_free);                 // S may be overwritten by S(n+1)
+  if (NH > 0 && (x.masked || x.cmask)) {
+    uint32_t w2[2] = {~0u, ~0u};
+    if (x.masked) {
+      const int4 mw = ld_shared_v4(x.mask_row);
+      w2[0] = (uint32_t)(h ? mw.z : mw.x);
+      w2[1] = (uint32_t)(h ? mw.w : mw.y);
+    }
+    if (x.cmask) {
+#pragma unroll
+      for (int q = 0; q < NH; ++q) w2[q] &= x.cmask[2 * h + q];
+    }
+#pragma unroll
+    for (int q = 0; q < NH; ++q) apply_mask(r[q], w2[q]);
+  }
+  float tmax = -INFINITY;
+#pragma unroll
+  for (int q = 0; q < NH; ++q) tmax = chunk_max(r[q], tmax);
+  // half-tile maxima of the pair -> tile max (double-buffered by tile parity: a slot is rewritten two
+  // tiles later, after the partner has passed the next tile's pair barrier)
+  float* xm = xmax + (x.n & 1) * 256;
+  xm[h * 128 + row] = tmax;
+  named_bar_sync(xbar, 64);
+  tmax = fmaxf(tmax, xm[(1 - h) * 128 + row]);
+  const bool need = tmax > m + x.thresh || (m == -INFINITY && tmax != -INFINITY);
+  float alpha = 1.f;
+  if (need) {
+    alpha = ex2((m - tmax) * x.c);                      // 0 when m = -inf
+    m = tmax;
+  }
+  l *= alpha;
+  const float mu = (m == -INFINITY) ? 0.f : m;
+  const float2 c2 = make_float2(x.c, x.c);
+  const float2 nb2 = make_float2(-mu * x.c, -mu * x.c);
+  float2 rs[2] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
+  uint32_t pre[NH > 0 ? NH : 1][16];
+#pragma unroll
+  for (int q = 0; q < NH; ++q) chunk_exp<kBF16>(r[q], c2, nb2, rs, pre[q]);
+  if (x.n > 0) mbar_wait(x.pv_done, (x.n - 1) & 1);
+  if (threadIdx.x == 0) tl_rec(*x.prm, x.n, 1);
+  tc_fence_after();
+  if (x.j > 0 && __any_sync(0xffffffffu, need && alpha != 1.f)) {
+#pragma unroll 1
+    for (int k = 0; k < kD / 32; ++k) {   // this half's kD / 2 columns of O
+      uint32_t o[16];
+      tmem_ld16(x.tl + kTO + h * (kD / 2) + k * 16, o);
+      tmem_wait_ld();
+#pragma unroll
+      for (int i = 0; i < 16; ++i) o[i] = __float_as_uint(__uint_as_float(o[i]) * alpha);
+      tmem_st16(x.tl + kTO + h * (kD / 2) + k * 16, o);
+    }
+  }
+#pragma unroll
+  for (int q = 0; q < NH; ++q) tmem_st16(x.tl + kTP + (2 * h + q) * 16, pre[q]);
+  l += (rs[0].x + rs[0].y) + (rs[1].x + rs[1].y);
+  tmem_wait_st();
+  tc_fence_before();
+  __syncwarp();
+  if (lane == 0) {
+    mbar_arrive(x.p_full);
+    tl_rec(*x.prm, x.n, threadIdx.x == 0 ? 2 : 7 + ((threadIdx.x >> 5) & 3));
+  }
+}
+
 }  // namespace
 
 template <bool kBF16, int kMode, bool kPad, int kD>
-__global__ void __launch_bounds__(kThreads, DCfg<kD>::kMinBlocks)
+__global__ void __launch_bounds__(WCfg<kD>::kThreads, DCfg<kD>::kMinBlocks)
     coarse_pp_kernel(const __grid_constant__ CUtensorMap tmq, const __grid_constant__ CUtensorMap tmk,
                      const __grid_constant__ CUtensorMap tmv, const __grid_constant__ CUtensorMap tmq2,
                      const __grid_constant__ CUtensorMap tmk2, const __grid_constant__ CUtensorMap tmv2,
@@ -447,6 +552,10 @@ __global__ void __launch_bounds__(kThreads, DCfg<kD>::kMinBlocks)
   constexpr bool kSplit = kMode == 1, kBatched = kMode == 2, kNoFine = kMode == 3;
   constexpr uint32_t kTileBytes = DCfg<kD>::kTileBytes, kTmemCols = DCfg<kD>::kTmemCols, kTO = DCfg<kD>::kTO;
   constexpr int kNSub = DCfg<kD>::kNSub;
+  using W = WCfg<kD>;
+  constexpr bool kCS = W::kCS;
+  constexpr int kSoftWarps = W::kSoftWarps;
+  constexpr int kRegsCtl = W::kRegsCtl, kRegsSoftmax = W::kRegsSoftmax;
   extern __shared__ uint8_t smem_raw[];
   const uint32_t sbase = (smem_u32(smem_raw) + 1023u) & ~1023u;
   const uint32_t sQ = sbase;
@@ -461,7 +570,7 @@ __global__ void __launch_bounds__(kThreads, DCfg<kD>::kMinBlocks)
   if (threadIdx.x == 0) {
     for (int b = 0; b < kItems; ++b) {
       mbar_init(bar(ctl->item_full[b]), 1);
-      mbar_init(bar(ctl->item_empty[b]), 2 + 4);   // producer + MMA thread + 4 softmax warps
+      mbar_init(bar(ctl->item_empty[b]), 2 + kSoftWarps);   // producer + MMA thread + softmax warps
     }
     for (int b = 0; b < 2; ++b) {
       mbar_init(bar(ctl->q_full[b]), 1);
@@ -473,15 +582,15 @@ __global__ void __launch_bounds__(kThreads, DCfg<kD>::kMinBlocks)
       mbar_init(bar(ctl->v_full[s]), 1);
       mbar_init(bar(ctl->v_empty[s]), 1);
       mbar_init(bar(ctl->mk_full[s]), 1);
-      mbar_init(bar(ctl->mk_empty[s]), 4);
+      mbar_init(bar(ctl->mk_empty[s]), kSoftWarps);
     }
     mbar_init(bar(ctl->s_full), 1);
-    mbar_init(bar(ctl->s_free), 4);
-    mbar_init(bar(ctl->p_full), 4);
+    mbar_init(bar(ctl->s_free), kSoftWarps);
+    mbar_init(bar(ctl->p_full), kSoftWarps);
     mbar_init(bar(ctl->pv_done), 1);
     fence_barrier_init();
   }
-  if (warp == 4 && lane == 0) {
+  if (warp == W::kWProd && lane == 0) {
     prefetch_tmap(&tmq);
     prefetch_tmap(&tmk);
     prefetch_tmap(&tmv);
@@ -491,7 +600,7 @@ __global__ void __launch_bounds__(kThreads, DCfg<kD>::kMinBlocks)
       prefetch_tmap(&tmv2);
     }
   }
-  if (warp == 5) {
+  if (warp == W::kWMma) {
     tmem_alloc(smem_u32(&ctl->tmem_base), kTmemCols);
     tmem_relinquish();
   }
@@ -500,7 +609,7 @@ __global__ void __launch_bounds__(kThreads, DCfg<kD>::kMinBlocks)
   tc_fence_after();
   const uint32_t tmem = ctl->tmem_base;
 
-  if (warp == 4) {
+  if (warp == W::kWProd) {
     // ============================================================ producer
     asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(kRegsCtl) : "memory");
     const uint64_t pol_kv = policy_evict_last();   // K/V tiles are re-read by neighbouring items
@@ -668,7 +777,7 @@ __global__ void __launch_bounds__(kThreads, DCfg<kD>::kMinBlocks)
         }
       }
     }
-  } else if (warp == 6) {
+  } else if (warp == W::kWSched) {
     // ============================================================ scheduler
     asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(kRegsCtl) : "memory");
     // Claims work items (dynamic counter) into a kItems-deep ring, i.e. up to kItems items ahead of
@@ -697,7 +806,7 @@ __global__ void __launch_bounds__(kThreads, DCfg<kD>::kMinBlocks)
       if (u >= p.total_units) break;
       __syncwarp();
     }
-  } else if (warp == 5) {
+  } else if (warp == W::kWMma) {
     // ============================================================ MMA issuer (lane 0)
     asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(kRegsCtl) : "memory");
     if (lane == 0) {
@@ -792,13 +901,16 @@ __global__ void __launch_bounds__(kThreads, DCfg<kD>::kMinBlocks)
       if (pend.valid) issue_pv(pend);
     }
     __syncwarp();
-  } else if (warp == 7) {
+  } else if (warp == W::kWIdle) {
     asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(kRegsCtl) : "memory");
   } else {
     // ============================================================ softmax + epilogue
     asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(kRegsSoftmax) : "memory");
-    const int t = warp * 32 + lane;                       // row of the Q tile = TMEM lane
-    const uint32_t tl = tmem + ((uint32_t)(warp * 32) << 16);
+    // row of the Q tile = TMEM lane (warp w owns lane quarter w % 4); column split: half h = w / 4
+    const int hh_cs = kCS ? warp >> 2 : 0;
+    const int t = kCS ? (warp & 3) * 32 + lane + 128 * hh_cs : warp * 32 + lane;   // (> 127: half-1 warp)
+    const int row = (warp & 3) * 32 + lane;
+    const uint32_t tl = tmem + ((uint32_t)((warp & 3) * 32) << 16);
     const float c = p.scale_log2;
     // lazy rescaling (O accumulates in TMEM): the exponent keeps a stale row max m until a tile's
     // max exceeds it by more than 2^8 in probability, so p <= 256 and O rarely needs a rescale
@@ -848,15 +960,27 @@ __global__ void __launch_bounds__(kThreads, DCfg<kD>::kMinBlocks)
         mbar_wait(bar(kLate ? ctl->mk_full[st] : ctl->v_full[st]), (n / kSt) & 1);
         tc_fence_after();
         const int2 desc = ctl->vdesc[st];                 // {ncols, maskA}
-        const TileCtx tc{tl, sMsk + st * kMaskBytes + t * 16, desc.y >= 0, kPad ? ctl->cmask[st] : nullptr,
+        const TileCtx tc{tl, sMsk + st * kMaskBytes + row * 16, desc.y >= 0, kPad ? ctl->cmask[st] : nullptr,
                          n, j, bar(ctl->s_free),
                          bar(ctl->pv_done), bar(ctl->p_full), c, thresh, &p};
         if (threadIdx.x == 0) tl_rec(p, n, 0);
-        switch (desc.x >> 5) {                            // 32-column chunks of the tile
-          case 4: softmax_tile<4, kBF16, kD>(tc, m, l); break;
-          case 3: softmax_tile<3, kBF16, kD>(tc, m, l); break;
-          case 2: softmax_tile<2, kBF16, kD>(tc, m, l); break;
-          default: softmax_tile<1, kBF16, kD>(tc, m, l); break;
+        if constexpr (kCS) {
+          // this warp's 32-column chunks of the tile: [2h, 2h + nh)
+          const int nh = min(max((desc.x >> 5) - 2 * hh_cs, 0), 2);
+          const uint32_t xbar = 2 + (warp & 3);
+          float* xm = &ctl->xmax[0][0][0];
+          switch (nh) {
+            case 2: softmax_tile_cs<2, kBF16, kD>(tc, m, l, hh_cs, row, xbar, xm); break;
+            case 1: softmax_tile_cs<1, kBF16, kD>(tc, m, l, hh_cs, row, xbar, xm); break;
+            default: softmax_tile_cs<0, kBF16, kD>(tc, m, l, hh_cs, row, xbar, xm); break;
+          }
+        } else {
+          switch (desc.x >> 5) {                          // 32-column chunks of the tile
+            case 4: softmax_tile<4, kBF16, kD>(tc, m, l); break;
+            case 3: softmax_tile<3, kBF16, kD>(tc, m, l); break;
+            case 2: softmax_tile<2, kBF16, kD>(tc, m, l); break;
+            default: softmax_tile<1, kBF16, kD>(tc, m, l); break;
+          }
         }
         if (kLate) {   // this tile's descriptor / mask stage may be refilled
           __syncwarp();
@@ -864,6 +988,13 @@ __global__ void __launch_bounds__(kThreads, DCfg<kD>::kMinBlocks)
         }
       }
       // ---------------------------------------------------------------- epilogue (a-8)
+      if constexpr (kCS) {
+        // column split: the row sum is the two halves' sums; the half-0 warps (0-3) run the epilogue
+        if (hh_cs == 1) ctl->xsum[row] = l;
+        named_bar_sync(2 + (warp & 3), 64);
+        if (hh_cs == 1) continue;
+        l += ctl->xsum[row];
+      }
       // (d = 64 keeps its single-pass epilogue: the per-half form below measured 3% slower on C2)
       bool tma_out;
       if constexpr (kNSub == 1) {
@@ -1261,7 +1392,7 @@ __global__ void __launch_bounds__(kThreads, DCfg<kD>::kMinBlocks)
 
   tc_fence_before();
   __syncthreads();
-  if (warp == 5) tmem_dealloc(tmem, kTmemCols);
+  if (warp == W::kWMma) tmem_dealloc(tmem, kTmemCols);
   // the last CTA to finish resets the work counter for the next launch (every CTA's scheduler has
   // claimed its final, out-of-range unit before its CTA gets here), so no memset precedes a launch
   if (threadIdx.x == 0) {
@@ -1296,7 +1427,8 @@ cudaError_t launch_coarse_pp(const CoarseParams& p, const CUtensorMap& tmq, cons
   const int smem = (int)(p.d == 128 ? smem_bytes<128>() : smem_bytes<64>());
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (e != cudaSuccess) return e;
-  kern<<<grid, kThreads, smem, stream>>>(tmq, tmk, tmv, tmq2, tmk2, tmv2, tmo, p);
+  const int threads = p.d == 128 ? WCfg<128>::kThreads : WCfg<64>::kThreads;
+  kern<<<grid, threads, smem, stream>>>(tmq, tmk, tmv, tmq2, tmk2, tmv2, tmo, p);
   return cudaGetLastError();
 }
 
