@@ -459,6 +459,27 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
     if (has_f) pc.fb = pc.first;
     if (has_c && !has_f) pc.cb = pc.first;
   }
+  // TMA descriptors of Q/K/V/O (re-encoded only when a tensor descriptor changes): the coarse kernel's
+  // tiles and row gathers, the fine kernel's row gathers
+  {
+    mg_plan_s::Maps& mp = p->maps;
+    if (!mp.valid || std::memcmp(&mp.q, Q, sizeof(mg_tensor)) || std::memcmp(&mp.k, K, sizeof(mg_tensor)) ||
+        std::memcmp(&mp.v, V, sizeof(mg_tensor)) || std::memcmp(&mp.o, O, sizeof(mg_tensor))) {
+      mp.q = *Q;
+      mp.k = *K;
+      mp.v = *V;
+      mp.o = *O;
+      mp.ok = encode_map(&mp.tq, Q) && encode_map(&mp.tk, K) && encode_map(&mp.tv, V);
+      std::memset(&mp.tq2, 0, sizeof(CUtensorMap));
+      std::memset(&mp.tk2, 0, sizeof(CUtensorMap));
+      std::memset(&mp.tv2, 0, sizeof(CUtensorMap));
+      std::memset(&mp.to, 0, sizeof(CUtensorMap));
+      mp.gather_ok = encode_map2d(&mp.tq2, Q, &mp.rq) && encode_map2d(&mp.tk2, K, &mp.rk) &&
+                     encode_map2d(&mp.tv2, V, &mp.rv);
+      mp.store_ok = encode_map(&mp.to, O);
+      mp.valid = true;
+    }
+  }
   if (nf > 0) {
     mg::FineParams fp{};
     fp.fine_rows = p->d_fine_rows;
@@ -479,8 +500,27 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
     // (the CUDA-core variant has no padding support: a padded forward always uses the MMA kernel)
     const int fsms = p->num_sms_override > 0 ? std::min(p->num_sms_override, p->num_sms) : p->num_sms;
     // (the CUDA-core variant takes d = 64 only: other forwards use the MMA kernel)
-    e = p->fine_kernel == 1 && !valid_len && D == 64 ? mg::launch_fine(fp, bf16, fstream)
-                                          : mg::launch_fine_mma(fp, bf16, fsms, fstream);
+    // two heads per warp with TMA row gathers (tile::gather4): measured slower than the cp.async
+    // gathers (C4 fine kernel 2.575 vs 1.887 ms), so only on request (MG_FINE_TMA=1, A/B)
+    static const bool no_fine_tma = [] {
+      const char* ev = std::getenv("MG_FINE_TMA");
+      return !(ev && ev[0] == '1');
+    }();
+    const mg_plan_s::Maps& mp = p->maps;
+    static const bool no_heads2 = [] {
+      const char* ev = std::getenv("MG_FINE_HEADS2");
+      return ev && ev[0] == '0';
+    }();
+    const bool fine_tma = !no_fine_tma && !no_heads2 && p->fine_kernel == 0 && D == 64 && (h.heads % 2) == 0 &&
+                          mp.gather_ok;
+    fp.rq = mp.rq;
+    fp.rk = mp.rk;
+    fp.rv = mp.rv;
+    if (fine_tma)
+      e = mg::launch_fine_tma2(fp, mp.tq2, mp.tk2, mp.tv2, bf16, fsms, fstream);
+    else
+      e = p->fine_kernel == 1 && !valid_len && D == 64 ? mg::launch_fine(fp, bf16, fstream)
+                                                       : mg::launch_fine_mma(fp, bf16, fsms, fstream);
     if (e != cudaSuccess) return cuda_fail(e, "fine kernel launch");
   }
   if (p->profiling && has_f) {
@@ -493,22 +533,6 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
   }
   if (!h.items.empty()) {
     mg_plan_s::Maps& mp = p->maps;
-    if (!mp.valid || std::memcmp(&mp.q, Q, sizeof(mg_tensor)) || std::memcmp(&mp.k, K, sizeof(mg_tensor)) ||
-        std::memcmp(&mp.v, V, sizeof(mg_tensor)) || std::memcmp(&mp.o, O, sizeof(mg_tensor))) {
-      mp.q = *Q;
-      mp.k = *K;
-      mp.v = *V;
-      mp.o = *O;
-      mp.ok = encode_map(&mp.tq, Q) && encode_map(&mp.tk, K) && encode_map(&mp.tv, V);
-      std::memset(&mp.tq2, 0, sizeof(CUtensorMap));
-      std::memset(&mp.tk2, 0, sizeof(CUtensorMap));
-      std::memset(&mp.tv2, 0, sizeof(CUtensorMap));
-      std::memset(&mp.to, 0, sizeof(CUtensorMap));
-      mp.gather_ok = encode_map2d(&mp.tq2, Q, &mp.rq) && encode_map2d(&mp.tk2, K, &mp.rk) &&
-                     encode_map2d(&mp.tv2, V, &mp.rv);
-      mp.store_ok = encode_map(&mp.to, O);
-      mp.valid = true;
-    }
     if (!mp.ok)
       return fail(MG_ERR_CUDA, "cuTensorMapEncodeTiled failed (driver entry point unavailable or bad layout)");
     const CUtensorMap &tq = mp.tq, &tk = mp.tk, &tv = mp.tv;

@@ -176,24 +176,6 @@ __device__ __forceinline__ int4 load_idx4(const int32_t* idx, int i0, int n) {
   return v;
 }
 
-// rows of the 2-D [rows, 64] view of a tensor: base + idx * step; idx < 0 -> -1 (out of bounds:
-// the TMA zero-fills the row)
-__device__ __forceinline__ int4 row_coords(int4 ix, int64_t base, int64_t step) {
-  auto f = [&](int i) { return i < 0 ? -1 : (int)(base + (int64_t)i * step); };
-  return make_int4(f(ix.x), f(ix.y), f(ix.z), f(ix.w));
-}
-
-// TMA row gather (tile::gather4): 4 rows of 64 16-bit elements into 4 consecutive 128-byte rows
-// of a SWIZZLE_128B tile at `dst` (the swizzle follows the shared address, as for tiled loads)
-__device__ __forceinline__ void gather4(uint32_t dst, const CUtensorMap* m, uint32_t bar, int4 rows,
-                                        uint64_t policy) {
-  asm volatile(
-      "cp.async.bulk.tensor.2d.shared::cluster.global.tile::gather4.mbarrier::complete_tx::bytes.L2::cache_hint"
-      " [%0], [%1, {%2, %3, %4, %5, %6}], [%7], %8;" ::"r"(dst),
-      "l"(reinterpret_cast<uint64_t>(m)), "r"(0), "r"(rows.x), "r"(rows.y), "r"(rows.z), "r"(rows.w), "r"(bar),
-      "l"(policy)
-      : "memory");
-}
 
 template <bool kBF16>
 __device__ __forceinline__ uint32_t pack2(float lo, float hi) {

@@ -661,6 +661,302 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB2) fine_mma2_kernel(c
   cp_async_wait<0>();
 }
 
+// ---------------------------------------------------------------------------------------------
+// Two heads per warp with TMA row gathers (tile::gather4): per step, lanes 0-15 each issue one
+// gather of 4 rows (K and V of both heads, 16 rows each) and, at a row start, lane 16 gathers the
+// two q rows, all completing on the stage's mbarrier; one warp instruction replaces the 16 cp.async
+// per lane of fine_mma2_kernel. Stage (1024-byte aligned, SWIZZLE_128B = the ring's XOR layout):
+// [K_h0 16 rows][V_h0][K_h1][V_h1][q_h0, q_h1, 2 zero rows] = 8.5 KB, padded to 9 KB.
+namespace {
+constexpr int kStageBytesT = 9216;
+constexpr int kQOffT = 4 * kS * 128;
+constexpr int kSmemBytesT = 1024 + kWarps * kStages * kStageBytesT + kWarps * kStages * 8;
+}  // namespace
+
+template <bool kBF16, bool kPad>
+__global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB2)
+    fine_tma2_kernel(const __grid_constant__ CUtensorMap tmq2, const __grid_constant__ CUtensorMap tmk2,
+                     const __grid_constant__ CUtensorMap tmv2, const FineParams p) {
+  constexpr int kD = 64, kRowBytes = 128, kJ = 4;
+  extern __shared__ __align__(128) uint8_t fsm[];
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const int g = lane >> 2, t = lane & 3;
+  const float c = p.scale_log2;
+  const float thresh = 8.f / c;
+  const int nhp = p.BH >> 1;
+  const int64_t nrows = (int64_t)nhp * p.n_fine_rows;
+  const bool r32 = nrows <= (int64_t)0xffffffffLL;
+  const int64_t W = (int64_t)gridDim.x * kWarps;
+  const int64_t w0 = (int64_t)blockIdx.x * kWarps + wid;
+  const uint32_t base = ((uint32_t)__cvta_generic_to_shared(fsm) + 1023u) & ~1023u;
+  const uint32_t ring = base + wid * (kStages * kStageBytesT);
+  const uint32_t bars = base + kWarps * kStages * kStageBytesT + wid * (kStages * 8);
+  if (lane == 0) {
+    for (int s0 = 0; s0 < kStages; ++s0) mbar_init(bars + 8 * s0, 1);
+    fence_barrier_init();
+  }
+  __syncwarp();
+  if (threadIdx.x == 0) {
+    prefetch_tmap(&tmk2);
+    prefetch_tmap(&tmv2);
+    prefetch_tmap(&tmq2);
+  }
+  const uint64_t pol = policy_evict_last();
+  // lane j < 16 gathers rows 4 (j % 4) .. + 3 of the step into block j / 4: K_h0, V_h0, K_h1, V_h1
+  const int gblk = (lane >> 2) & 3, gq = lane & 3;
+  const CUtensorMap* gmap = (gblk & 1) ? &tmv2 : &tmk2;
+  const int64_t rstep = (gblk & 1) ? p.rv.z : p.rk.z;
+
+  int64_t gi = w0;
+  int ibeg = 0, iend = 0, is = 0, icol = -1, icol_next = -1;
+  int64_t grow0 = 0;          // this lane's gather: row of (b, head of its block, column 0)
+  int qrow0 = 0, qrow1 = 0;   // the row's q rows in the Q view
+  auto open_issue_row = [&]() {
+    if (gi < nrows) {
+      int u0, fi;
+      split_row(gi, p.n_fine_rows, r32, u0, fi);
+      const int bh = (p.fine_sample ? __ldg(p.fine_sample + fi) * p.H : 0) + 2 * u0;
+      ibeg = __ldg(p.row_ptr + fi);
+      iend = __ldg(p.row_ptr + fi + 1);
+      const int bb = bh / p.H, hh = bh % p.H + (gblk >> 1);
+      grow0 = (gblk & 1) ? bb * p.rv.x + hh * p.rv.y : bb * p.rk.x + hh * p.rk.y;
+      const int rq = __ldg(p.fine_rows + fi) & 0x7fffffff;
+      const int hq = bh % p.H;
+      qrow0 = (int)(bb * p.rq.x + hq * p.rq.y + (int64_t)rq * p.rq.z);
+      qrow1 = (int)(qrow0 + p.rq.y);
+    }
+    is = 0;
+  };
+  uint32_t phase = 0;   // bit s: parity of the next completion of stage s
+  auto issue_step = [&](uint32_t stg) {
+    if (gi < nrows) {
+      const int nb0 = ibeg + kS * is;
+      if ((is & 1) == 0) icol = is > 0 ? icol_next : (nb0 + lane < iend ? __ldg(p.cols + nb0 + lane) : -1);
+      const int off = (is & 1) * 16 + 4 * gq;
+      int4 cols;
+      cols.x = __shfl_sync(0xffffffffu, icol, off);
+      cols.y = __shfl_sync(0xffffffffu, icol, off + 1);
+      cols.z = __shfl_sync(0xffffffffu, icol, off + 2);
+      cols.w = __shfl_sync(0xffffffffu, icol, off + 3);
+      const uint32_t st = ring + stg * kStageBytesT, bar = bars + 8 * stg;
+      // (the stage was last read by this warp's ldmatrix: order those generic reads before the
+      // async-proxy writes)
+      fence_proxy_async_smem();
+      if (lane == 0) mbar_arrive_expect_tx(bar, 4 * kS * kRowBytes + (is == 0 ? 512u : 0u));
+      __syncwarp();
+      if (lane < 16) gather4(st + gblk * (kS * kRowBytes) + gq * 512, gmap, bar, row_coords(cols, grow0, rstep), pol);
+      if (is == 0 && lane == 16) gather4(st + kQOffT, &tmq2, bar, make_int4(qrow0, qrow1, -1, -1), pol);
+      if ((is & 1) == 1 && nb0 + kS < iend) icol_next = nb0 + kS + lane < iend ? __ldg(p.cols + nb0 + kS + lane) : -1;
+      if (nb0 + kS < iend) {
+        ++is;
+      } else {
+        gi += W;
+        open_issue_row();
+      }
+    }
+  };
+
+  open_issue_row();
+#pragma unroll
+  for (int s0 = 0; s0 < kStages - 1; ++s0) issue_step(s0);
+  uint32_t stage = 0, istage = kStages - 1;
+  const uint32_t a_row = (lane & 7) * kRowBytes, b_row = a_row + 8 * kRowBytes;
+  const uint32_t vr = (lane & 7) + 8 * (lane >> 4);
+
+  for (int64_t gw = w0; gw < nrows; gw += W) {
+    int u0, fi;
+    split_row(gw, p.n_fine_rows, r32, u0, fi);
+    const int bh = (p.fine_sample ? __ldg(p.fine_sample + fi) * p.H : 0) + 2 * u0;
+    const int enc = __ldg(p.fine_rows + fi);
+    const int r = enc & 0x7fffffff;
+    const bool final_out = enc < 0;
+    const int bb = bh / p.H, hh = bh % p.H;
+    uint32_t qa[2][kJ], qb[2][kJ];
+    const int beg = __ldg(p.row_ptr + fi), end = __ldg(p.row_ptr + fi + 1);
+    const int nvalid = kPad ? max(__ldg(p.valid_len + bb), 0) : 0x7fffffff;
+    const bool pad_row = kPad && r >= nvalid;
+
+    float m[2] = {-INFINITY, -INFINITY}, l[2] = {0.f, 0.f};
+    float acc[2][kJ][4];
+#pragma unroll
+    for (int hd = 0; hd < 2; ++hd)
+#pragma unroll
+      for (int j = 0; j < kJ; ++j)
+#pragma unroll
+        for (int e = 0; e < 4; ++e) acc[hd][j][e] = 0.f;
+
+    for (int base_i = beg; base_i < end; base_i += kS) {
+      issue_step(istage);
+      istage = istage == kStages - 1 ? 0 : istage + 1;
+      mbar_wait(bars + 8 * stage, (phase >> stage) & 1);
+      phase ^= 1u << stage;
+      const uint32_t st = ring + stage * kStageBytesT;
+      stage = stage == kStages - 1 ? 0 : stage + 1;
+      if (base_i == beg) {
+#pragma unroll
+        for (int hd = 0; hd < 2; ++hd)
+#pragma unroll
+          for (int j = 0; j < kJ; ++j) {
+            // the q rows' 16-byte chunks are swizzled like every row of the stage (row 0 / 1)
+            const uint32_t qrow = st + kQOffT + hd * 128;
+            const uint32_t ch0 = (2 * j) ^ hd, ch1 = (2 * j + 1) ^ hd;
+            asm volatile("ld.shared.u32 %0, [%1];" : "=r"(qa[hd][j]) : "r"(qrow + (ch0 << 4) + 4 * t));
+            asm volatile("ld.shared.u32 %0, [%1];" : "=r"(qb[hd][j]) : "r"(qrow + (ch1 << 4) + 4 * t));
+          }
+      }
+      const int rem = end - base_i - 2 * t;
+      float s[2][4];
+#pragma unroll
+      for (int hd = 0; hd < 2; ++hd) {
+        const uint32_t sk = st + hd * kHB;
+        float sa[2][4] = {{0.f, 0.f, 0.f, 0.f}, {0.f, 0.f, 0.f, 0.f}};
+        float sb[2][4] = {{0.f, 0.f, 0.f, 0.f}, {0.f, 0.f, 0.f, 0.f}};
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          uint32_t ka[4], kb[4];
+          const uint32_t sw = ((uint32_t)(((lane >> 3) + 4 * h) ^ (lane & 7))) << 4;
+          ldsm_x4(ka, sk + a_row + sw);
+          ldsm_x4(kb, sk + b_row + sw);
+          mma16816<kBF16>(sa[h], qa[hd][2 * h], qa[hd][2 * h], qb[hd][2 * h], qb[hd][2 * h], ka[0], ka[1]);
+          mma16816<kBF16>(sb[h], qa[hd][2 * h], qa[hd][2 * h], qb[hd][2 * h], qb[hd][2 * h], kb[0], kb[1]);
+          mma16816<kBF16>(sa[h], qa[hd][2 * h + 1], qa[hd][2 * h + 1], qb[hd][2 * h + 1], qb[hd][2 * h + 1], ka[2], ka[3]);
+          mma16816<kBF16>(sb[h], qa[hd][2 * h + 1], qa[hd][2 * h + 1], qb[hd][2 * h + 1], qb[hd][2 * h + 1], kb[2], kb[3]);
+        }
+        s[hd][0] = rem > 0 ? sa[0][0] + sa[1][0] : -INFINITY;
+        s[hd][1] = rem > 1 ? sa[0][1] + sa[1][1] : -INFINITY;
+        s[hd][2] = rem > 8 ? sb[0][0] + sb[1][0] : -INFINITY;
+        s[hd][3] = rem > 9 ? sb[0][1] + sb[1][1] : -INFINITY;
+      }
+      if (kPad) {
+        const int o4[4] = {0, 1, 8, 9};
+#pragma unroll
+        for (int i = 0; i < 4; ++i)
+          if (rem > o4[i] && __ldg(p.cols + base_i + 2 * t + o4[i]) >= nvalid) s[0][i] = s[1][i] = -INFINITY;
+      }
+      float mx[2];
+#pragma unroll
+      for (int hd = 0; hd < 2; ++hd) mx[hd] = fmaxf(fmaxf(s[hd][0], s[hd][1]), fmaxf(s[hd][2], s[hd][3]));
+#pragma unroll
+      for (int hd = 0; hd < 2; ++hd) mx[hd] = fmaxf(mx[hd], __shfl_xor_sync(0xffffffffu, mx[hd], 1));
+#pragma unroll
+      for (int hd = 0; hd < 2; ++hd) mx[hd] = fmaxf(mx[hd], __shfl_xor_sync(0xffffffffu, mx[hd], 2));
+#pragma unroll
+      for (int hd = 0; hd < 2; ++hd) {
+        if (mx[hd] > m[hd] + thresh) {
+          const float alpha = ex2((m[hd] - mx[hd]) * c);
+          l[hd] *= alpha;
+#pragma unroll
+          for (int j = 0; j < kJ; ++j)
+#pragma unroll
+            for (int e = 0; e < 4; ++e) acc[hd][j][e] *= alpha;
+          m[hd] = mx[hd];
+        }
+      }
+#pragma unroll
+      for (int hd = 0; hd < 2; ++hd) {
+        const float nbias = m[hd] == -INFINITY ? 0.f : -m[hd] * c;
+        float pv[4];
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          pv[i] = ex2(fmaf(s[hd][i], c, nbias));
+          l[hd] += pv[i];
+        }
+        const uint32_t pb0 = pack2<kBF16>(pv[0], pv[1]), pb1 = pack2<kBF16>(pv[2], pv[3]);
+        const uint32_t sv = st + hd * kHB + kS * kRowBytes;
+#pragma unroll
+        for (int j = 0; j < kJ; ++j) {
+          uint32_t a[4];
+          const uint32_t ch = 2 * j + ((lane >> 3) & 1);
+          ldsm_x4_t(a, sv + vr * kRowBytes + ((ch ^ (vr & 7)) << 4));
+          mma16816<kBF16>(acc[hd][j], a[0], a[1], a[2], a[3], pb0, pb1);
+        }
+      }
+      __syncwarp();
+    }
+#pragma unroll
+    for (int hd = 0; hd < 2; ++hd) {
+      float lh = l[hd];
+      lh += __shfl_xor_sync(0xffffffffu, lh, 1);
+      lh += __shfl_xor_sync(0xffffffffu, lh, 2);
+      float v0 = acc[hd][0][0], v1 = acc[hd][0][2];
+#pragma unroll
+      for (int j = 1; j < 4; ++j)
+        if (t == j) {
+          v0 = acc[hd][j][0];
+          v1 = acc[hd][j][2];
+        }
+      const int d0 = 16 * t + g;
+      float inv = lh > 0.f ? 1.f / lh : 0.f;
+      bool write_o = final_out;
+      if (!final_out) {
+        const size_t idx = (size_t)(2 * u0 + hd) * p.n_fine_rows + fi;
+        __stcg(p.part_acc + idx * kD + d0, v0);
+        __stcg(p.part_acc + idx * kD + d0 + 8, v1);
+        if (lane == 0) __stcg(p.part_ml + idx, make_float2(m[hd], lh));
+        if (p.concurrent) {
+          __threadfence();
+          __syncwarp();
+          int old = 0;
+          if (lane == 0) old = atomicAdd(p.part_flags + idx, 1);
+          old = __shfl_sync(0xffffffffu, old, 0);
+          if (old & 1) {
+            __threadfence();
+            const float2 mlc = __ldcg(p.part_c_ml + idx);
+            const float mt = fmaxf(m[hd], mlc.x);
+            const float mu = mt == -INFINITY ? 0.f : mt;
+            const float af = ex2((m[hd] - mu) * c), ac = ex2((mlc.x - mu) * c);
+            const float den = lh * af + mlc.y * ac;
+            inv = den > 0.f ? 1.f / den : 0.f;
+            v0 = v0 * af + __ldcg(p.part_c_acc + idx * kD + d0) * ac;
+            v1 = v1 * af + __ldcg(p.part_c_acc + idx * kD + d0 + 8) * ac;
+            write_o = true;
+          }
+        }
+      }
+      if (pad_row) {
+        write_o = final_out;
+        v0 = v1 = 0.f;
+      }
+      if (write_o) {
+        uint16_t* orow = p.o.data + bb * p.o.sb + (hh + hd) * p.o.sh + (int64_t)r * p.o.sl;
+        const uint32_t pk = pack2<kBF16>(v0 * inv, v1 * inv);
+        orow[d0] = (uint16_t)(pk & 0xffffu);
+        orow[d0 + 8] = (uint16_t)(pk >> 16);
+      }
+    }
+  }
+}
+
+cudaError_t launch_fine_tma2(const FineParams& p, const CUtensorMap& tmq2, const CUtensorMap& tmk2,
+                             const CUtensorMap& tmv2, bool bf16, int sms, cudaStream_t stream) {
+  const int64_t units = (int64_t)(p.BH / 2) * p.n_fine_rows;
+  if (units == 0) return cudaSuccess;
+  using K = void (*)(const CUtensorMap, const CUtensorMap, const CUtensorMap, const FineParams);
+  static const K table[4] = {fine_tma2_kernel<false, false>, fine_tma2_kernel<false, true>,
+                             fine_tma2_kernel<true, false>, fine_tma2_kernel<true, true>};
+  const K kern = table[(bf16 ? 2 : 0) + (p.valid_len ? 1 : 0)];
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytesT);
+  if (e != cudaSuccess) return e;
+  static std::mutex mu;
+  static std::map<std::pair<int, int>, int> per_sm;
+  const int vi = (bf16 ? 2 : 0) + (p.valid_len ? 1 : 0);
+  int dev = 0, n = 0;
+  if ((e = cudaGetDevice(&dev)) != cudaSuccess) return e;
+  {
+    std::lock_guard<std::mutex> lk(mu);
+    auto it = per_sm.find({dev, vi});
+    if (it == per_sm.end()) {
+      if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kern, kWarps * 32, kSmemBytesT)) != cudaSuccess)
+        return e;
+      it = per_sm.emplace(std::make_pair(dev, vi), std::max(n, 1)).first;
+    }
+    n = it->second;
+  }
+  const int64_t blocks = std::min<int64_t>((units + kWarps - 1) / kWarps, (int64_t)n * std::max(sms, 1));
+  kern<<<(unsigned)blocks, kWarps * 32, kSmemBytesT, stream>>>(tmq2, tmk2, tmv2, p);
+  return cudaGetLastError();
+}
+
 cudaError_t launch_fine_mma(const FineParams& p, bool bf16, int sms, cudaStream_t stream) {
   const int64_t warps = (int64_t)p.BH * p.n_fine_rows;
   if (warps == 0) return cudaSuccess;

@@ -72,6 +72,7 @@ struct FineParams {
   TensorView q, k, v, o;
   int32_t H, BH, n_fine_rows;   // (BH = row units per fine row: B*H, or H for a batched plan)
   int32_t d;                    // head dimension (64 or 128; the CUDA-core kernel takes 64 only)
+  longlong3 rq, rk, rv;         // TMA gather variant: row of (b, h, l) in the 2-D [rows, 64] views
   const int32_t* fine_sample;   // batched plan: sample of each fine row (else null)
   float scale_log2;
   int32_t concurrent;         // see CoarseParams::concurrent
@@ -122,6 +123,9 @@ int coarse_pp_ctas_per_sm(int d);
 cudaError_t launch_fine(const FineParams& p, bool bf16, cudaStream_t stream);
 // Warp-level tensor-core variant (mma.sync m16n8k16), the default; see fine_mma.cu.
 cudaError_t launch_fine_mma(const FineParams& p, bool bf16, int sms, cudaStream_t stream);
+// Two heads per warp with TMA tile::gather4 row gathers (d = 64, even head count, gather views).
+cudaError_t launch_fine_tma2(const FineParams& p, const CUtensorMap& tmq2, const CUtensorMap& tmk2,
+                             const CUtensorMap& tmv2, bool bf16, int sms, cudaStream_t stream);
 cudaError_t launch_selftest_umma(int mode, const void* A, const void* B, float* D, cudaStream_t stream);
 
 }  // namespace mg

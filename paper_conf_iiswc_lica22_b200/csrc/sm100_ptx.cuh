@@ -113,6 +113,23 @@ __device__ __forceinline__ void tma_load_4d(uint32_t dst, const CUtensorMap* m, 
       "l"(reinterpret_cast<uint64_t>(m)), "r"(c0), "r"(c1), "r"(c2), "r"(c3), "r"(bar), "l"(policy)
       : "memory");
 }
+// rows of the 2-D [rows, 64] view of a tensor: base + idx * step; idx < 0 -> -1 (out of bounds:
+// the TMA zero-fills the row)
+__device__ __forceinline__ int4 row_coords(int4 ix, int64_t base, int64_t step) {
+  auto f = [&](int i) { return i < 0 ? -1 : (int)(base + (int64_t)i * step); };
+  return make_int4(f(ix.x), f(ix.y), f(ix.z), f(ix.w));
+}
+// TMA row gather (tile::gather4): 4 rows of 64 16-bit elements into 4 consecutive 128-byte rows
+// of a SWIZZLE_128B tile at `dst` (the swizzle follows the shared address, as for tiled loads)
+__device__ __forceinline__ void gather4(uint32_t dst, const CUtensorMap* m, uint32_t bar, int4 rows,
+                                        uint64_t policy) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.tile::gather4.mbarrier::complete_tx::bytes.L2::cache_hint"
+      " [%0], [%1, {%2, %3, %4, %5, %6}], [%7], %8;" ::"r"(dst),
+      "l"(reinterpret_cast<uint64_t>(m)), "r"(0), "r"(rows.x), "r"(rows.y), "r"(rows.z), "r"(rows.w), "r"(bar),
+      "l"(policy)
+      : "memory");
+}
 // TMA store of a 4-D tensor tile from shared memory (bulk-group completion)
 __device__ __forceinline__ void tma_store_4d(const CUtensorMap* m, uint32_t src, int c0, int c1, int c2, int c3) {
   asm volatile("cp.async.bulk.tensor.4d.global.shared::cta.bulk_group [%0, {%2, %3, %4, %5}], [%1];" ::"l"(

@@ -328,3 +328,28 @@ def test_batched_plan_per_sample_positions(kw):
             check(gotp[b, h], dense_masked_attention(Qh, Kh, Vh, w, Gs[b], Es[b], valid_len=int(lens[b])))
     with pytest.raises(mg.MGError):                 # batch must match the plan's samples
         run_gpu(plan, q[:2], k[:2], v[:2])
+
+
+def test_fine_tma_gather_variant_subprocess():
+    """The TMA tile::gather4 variant of the two-head fine kernel (off by default, MG_FINE_TMA=1)
+    against the oracle, in a subprocess (the switch is read once per process)."""
+    import os
+    import subprocess
+    import sys
+    code = (
+        "import numpy as np, sys; sys.path.insert(0, 'tests');"
+        "import paper_conf_iiswc_lica22_b200 as mg;"
+        "from gpu_util import from_device, to_device, err_stats;"
+        "from oracle import dense_masked_attention, head_inputs_f64;"
+        "from workloads import make_qkv, random_residual;"
+        "L, H, W = 1024, 4, 128; G = np.array([0, 300], np.int32); E = random_residual(L, W, 9, seed=3);"
+        "q, k, v = make_qkv(2, H, L, 64, seed=5);"
+        "plan = mg.Plan(L, H, 64, W, G, E, strip_max_cols=-1);"
+        "got = from_device(mg.sparse_attention_fwd(plan, *(to_device(x) for x in (q, k, v))));"
+        "w = max(err_stats(got[b, h], dense_masked_attention(*head_inputs_f64(q, k, v, b, h), W, G, E))[0]"
+        "        for b in range(2) for h in range(H));"
+        "assert w <= 2e-2, w; print('ok', w)")
+    env = dict(os.environ, MG_FINE_TMA="1")
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, env=env, cwd=root, timeout=300)
+    assert r.returncode == 0 and "ok" in r.stdout, r.stderr[-2000:]
