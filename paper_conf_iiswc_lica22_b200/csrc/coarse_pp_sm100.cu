@@ -53,37 +53,16 @@ namespace {
 #ifndef MG_CSPLIT128
 #define MG_CSPLIT128 1
 #endif
-// Pipelines per CTA (d = 64 without column split): two independent pipelines (each its own work
-// items, shared-memory ring, barriers and 256 TMEM columns) in one 512-thread CTA per SM, instead
-// of two 256-thread CTAs per SM, so that the two pipelines' softmax warps on one SM sub-partition
-// can coordinate through shared memory (MG_PINGPONG below). MG_PIPES=1 restores two CTAs per SM.
-#ifndef MG_PIPES
-#define MG_PIPES 1
-#endif
-// Exponential-phase exclusion (two pipelines): a softmax warp waits, before its tile's
-// exponentials, until the other pipeline's warp on the same SM sub-partition (same TMEM lane
-// quarter) has left its own exponential phase, so the two warps take turns on the sub-partition's
-// MUFU instead of sharing it in lock step, and each warp's barrier / TMEM latency hides behind the
-// other's exponentials. (A flag per warp in shared memory; a race only costs an overlap.)
-#ifndef MG_PINGPONG
-#define MG_PINGPONG 1
-#endif
 template <int kD>
 struct WCfg {
   static constexpr bool kCS = kD == 64 ? (bool)MG_CSPLIT : (bool)MG_CSPLIT128;
-  static constexpr int kPipes = (kD == 64 && !kCS) ? MG_PIPES : 1;
-  static constexpr bool kPP = kPipes == 2 && MG_PINGPONG;
-  static constexpr int kSoftWarps = kCS ? 8 : 4;              // per pipeline
-  static constexpr int kThreads = 32 * kPipes * (kSoftWarps + 4);
-  // warps [0, kWCtl0): softmax (pipeline w / kSoftWarps); then per pipeline one control warpgroup:
-  // producer, MMA issuer, scheduler, idle (role = (w - kWCtl0) & 3, pipeline = (w - kWCtl0) >> 2)
-  static constexpr int kWCtl0 = kPipes * kSoftWarps;
-  static constexpr int kWProd = kWCtl0, kWMma = kWCtl0 + 1, kWSched = kWCtl0 + 2, kWIdle = kWCtl0 + 3;
+  static constexpr int kSoftWarps = kCS ? 8 : 4;
+  static constexpr int kThreads = 32 * (kSoftWarps + 4);
+  static constexpr int kWProd = kSoftWarps, kWMma = kSoftWarps + 1, kWSched = kSoftWarps + 2, kWIdle = kSoftWarps + 3;
   // setmaxnreg per warpgroup: (65536 / CTAs per SM / threads, rounded down to 8) per thread in the pool
   static constexpr int kRegsCtl = kCS ? (kD == 64 ? 48 : 88) : 64;
   static constexpr int kRegsSoftmax = kCS ? (kD == 64 ? 96 : 208) : 192;
 };
-static_assert(WCfg<64>::kPipes == 1 || 256 * 192 + 256 * 64 <= 65536, "register pool (two pipelines)");
 static_assert(256 * 96 + 128 * 48 <= (65536 / 2 / 384 & ~7) * 384, "register pool (column split, d = 64)");
 static_assert(256 * 208 + 128 * 88 <= (65536 / 1 / 384 & ~7) * 384, "register pool (column split, d = 128)");
 constexpr int kThreads = 256;
@@ -102,7 +81,7 @@ struct DCfg {
   static constexpr int kNSub = kD / 64;
   static constexpr uint32_t kTmemCols = kD == 64 ? 256 : 512;
   static constexpr uint32_t kTO = kD == 64 ? 192 : 256;
-  static constexpr int kMinBlocks = kD == 64 ? 2 / WCfg<64>::kPipes : 1;   // CTAs per SM
+  static constexpr int kMinBlocks = kD == 64 ? 2 : 1;
 };
 
 struct __align__(16) Slot {
@@ -120,23 +99,17 @@ struct __align__(16) Ctl {
   uint64_t k_full[kSt], k_empty[kSt], v_full[kSt], v_empty[kSt];
   uint64_t s_full, s_free, p_full, pv_done;
   uint64_t mk_full[kSt], mk_empty[kSt];       // late-P.V mode: tile descriptor / bitmask ring
-  uint32_t tmem_base;                         // (pipeline 0's: the CTA's allocation)
-  int32_t dense_last;
-  int32_t pp_busy[4];                         // MG_PINGPONG: this pipeline's warp q is in its exponentials                         // split dense item: this chunk finished its row group last
+  uint32_t tmem_base;
+  int32_t dense_last;                         // split dense item: this chunk finished its row group last
   float xmax[2][2][128];                      // column split: [tile parity][half][row] half-tile maxima
   float xsum[128];                            // column split: half 1's row sum for the epilogue
 };
 
-// one pipeline's shared memory: Q[2], K[kSt], V[kSt] tiles, kSt bitmasks, Ctl (1024-aligned stride)
-template <int kD>
-__host__ __device__ constexpr uint32_t pipe_bytes() {
-  return (uint32_t)((6 * DCfg<kD>::kTileBytes + kSt * kMaskBytes + sizeof(Ctl) + 1023) & ~(size_t)1023);
-}
 template <int kD>
 constexpr size_t smem_bytes() {
-  return 1024 + WCfg<kD>::kPipes * pipe_bytes<kD>();
+  return 1024 + 6 * DCfg<kD>::kTileBytes + kSt * kMaskBytes + sizeof(Ctl);
 }
-static_assert(smem_bytes<64>() <= (WCfg<64>::kPipes == 2 ? 227 : 113) * 1024, "d = 64 shared memory per CTA");
+static_assert(smem_bytes<64>() <= 113 * 1024, "two CTAs per SM at d = 64");
 static_assert(smem_bytes<128>() <= 227 * 1024, "one CTA per SM at d = 128");
 // setmaxnreg applies per warpgroup: warps 0-3 (softmax) grow, warps 4-7 (control) shrink. The
 // pool of one CTA is (65536 / CTAs per SM / kThreads) x kThreads registers.
@@ -317,28 +290,27 @@ __device__ __forceinline__ void chunk_exp_f32(uint32_t (&r)[32], float2 c2, floa
 // 8-10 softmax warps 1-3 P(n) stored, 11/12/13 epilogue start / O read / end (last tile of an
 // item), 14 MMA sees k_full(n), 15 SM id (tile 0 only). tools/timeline_pp.py reads it.
 constexpr int kTlTiles = 128;
-// (vc = virtual CTA = blockIdx.x * pipelines + pipeline, nv = their number)
-__device__ __forceinline__ void tl_rec(const CoarseParams& p, int vc, int nv, uint32_t n, int field) {
+__device__ __forceinline__ void tl_rec(const CoarseParams& p, uint32_t n, int field) {
 #ifdef MG_TIMELINE
   if (p.trace == nullptr || n >= (uint32_t)kTlTiles ||
-      (int64_t)p.trace_cap < 256 + (int64_t)8 * kTlTiles * (int64_t)nv)
+      (int64_t)p.trace_cap < 256 + (int64_t)8 * kTlTiles * (int64_t)gridDim.x)
     return;
   uint32_t v = (uint32_t)clock64();
   if (field == 15) asm("mov.u32 %0, %%smid;" : "=r"(v));
-  reinterpret_cast<uint32_t*>(p.trace + 256)[((size_t)vc * kTlTiles + n) * 16 + field] = v;
+  reinterpret_cast<uint32_t*>(p.trace + 256)[((size_t)blockIdx.x * kTlTiles + n) * 16 + field] = v;
 #endif
 }
 
 // Item-level events (MG_TIMELINE): [CTA][item < 32][8] uint32 after the tile records: 0 scheduler
 // slot free, 1 scheduler item published, 2 producer item seen, 3 producer Q issued, 4 producer tile
 // refs loaded, 5 softmax item seen, 6 MMA item seen, 7 MMA Q ready.
-__device__ __forceinline__ void tl_item(const CoarseParams& p, int vc, int nv, uint32_t it, int field) {
+__device__ __forceinline__ void tl_item(const CoarseParams& p, uint32_t it, int field) {
 #ifdef MG_TIMELINE
   if (p.trace == nullptr || it >= 32u ||
-      (int64_t)p.trace_cap < 256 + (int64_t)(8 * kTlTiles + 128) * (int64_t)nv)
+      (int64_t)p.trace_cap < 256 + (int64_t)(8 * kTlTiles + 128) * (int64_t)gridDim.x)
     return;
-  reinterpret_cast<uint32_t*>(p.trace + 256)[(size_t)nv * kTlTiles * 16 + ((size_t)vc * 32 + it) * 8 + field] =
-      (uint32_t)clock64();
+  reinterpret_cast<uint32_t*>(p.trace + 256)[(size_t)gridDim.x * kTlTiles * 16 + ((size_t)blockIdx.x * 32 + it) * 8 +
+                                             field] = (uint32_t)clock64();
 #endif
 }
 
@@ -381,9 +353,6 @@ struct TileCtx {
   uint32_t s_free, pv_done, p_full;
   float c, thresh;
   const CoarseParams* prm;   // diagnostics only (tl_rec, debug_flags)
-  int vc, nv;                // diagnostics only (tl_rec: virtual CTA, count)
-  volatile int32_t* pp_mine;         // MG_PINGPONG: this warp's busy flag, the other pipeline's (or null)
-  const volatile int32_t* pp_other;
 };
 
 // One tile of the online SpSoftmax for this thread's row (NQ x 32 columns): read S(n) from TMEM
@@ -428,43 +397,18 @@ __device__ __forceinline__ void softmax_tile(const TileCtx& x, float& m, float& 
   l *= alpha;
   const float mu = (m == -INFINITY) ? 0.f : m;
   const float2 c2 = make_float2(x.c, x.c);
+  const float2 nb2 = make_float2(-mu * x.c, -mu * x.c);
   float2 rs[2] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
-  float2 nb2 = make_float2(-mu * x.c, -mu * x.c);
-  if (x.pp_mine) {
-    // MG_PINGPONG: wait until the other pipeline's warp on this sub-partition has left its
-    // exponentials, then mark ours. The poll's result (always 0) is added to the exponent bias so
-    // that the compiler cannot hoist the exponentials above the wait.
-    uint32_t busy;
-    do {
-      asm volatile("ld.volatile.shared.u32 %0, [%1];" : "=r"(busy) : "r"(smem_u32((const void*)x.pp_other)) : "memory");
-      busy = __shfl_sync(0xffffffffu, busy, 0);
-    } while (busy);
-    if (lane == 0) *x.pp_mine = 1;
-    uint32_t zero;
-    asm volatile("mov.b32 %0, %1;" : "=r"(zero) : "r"(busy));   // opaque 0 (busy == 0 here)
-    nb2.x += __uint_as_float(zero);
-    nb2.y += __uint_as_float(zero);
-  }
   // the first kPre chunks' exponentials are computed before waiting for P.V(n-1) (they overlap its
   // issue and execution; their packed P waits in registers)
   constexpr int kPreN = kPre < NQ ? kPre : NQ;
   uint32_t pre[kPreN > 0 ? kPreN : 1][16];
 #pragma unroll
   for (int q = 0; q < kPreN; ++q) chunk_exp<kBF16>(r[q], c2, nb2, rs, pre[q]);
-  if (x.pp_mine) {
-    // end of this warp's exponential phase (the row sums depend on every exponential: the store
-    // cannot move above them)
-    __syncwarp();
-    if (lane == 0)
-      asm volatile("st.volatile.shared.u32 [%0], 0;" ::"r"(smem_u32((const void*)x.pp_mine)), "f"(rs[0].x),
-                   "f"(rs[0].y), "f"(rs[1].x), "f"(rs[1].y)
-                   : "memory");
-  }
-  const bool t0 = (threadIdx.x & 127) == 0;
   // P.V(n-1) has consumed P(n-1) and updated O: rescale O if the max moved, then store P(n)
-  // chunk by chunk as it is produced (the other pipeline on this SM keeps the pipes busy meanwhile)
+  // chunk by chunk as it is produced (the other CTA on this SM keeps the pipes busy meanwhile)
   if (x.n > 0) mbar_wait(x.pv_done, (x.n - 1) & 1);
-  if (t0) tl_rec(*x.prm, x.vc, x.nv, x.n, 1);
+  if (threadIdx.x == 0) tl_rec(*x.prm, x.n, 1);
   tc_fence_after();
   if (x.j > 0 && __any_sync(0xffffffffu, need && alpha != 1.f)) {
 #pragma unroll 1
@@ -491,7 +435,7 @@ __device__ __forceinline__ void softmax_tile(const TileCtx& x, float& m, float& 
   __syncwarp();
   if (lane == 0) {
     mbar_arrive(x.p_full);
-    tl_rec(*x.prm, x.vc, x.nv, x.n, t0 ? 2 : 7 + ((threadIdx.x >> 5) & 3));
+    tl_rec(*x.prm, x.n, threadIdx.x == 0 ? 2 : 7 + (threadIdx.x >> 5));
   }
 }
 
@@ -550,7 +494,7 @@ __device__ __forceinline__ void softmax_tile_cs(const TileCtx& x, float& m, floa
 #pragma unroll
   for (int q = 0; q < NH; ++q) chunk_exp<kBF16>(r[q], c2, nb2, rs, pre[q]);
   if (x.n > 0) mbar_wait(x.pv_done, (x.n - 1) & 1);
-  if (threadIdx.x == 0) tl_rec(*x.prm, x.vc, x.nv, x.n, 1);
+  if (threadIdx.x == 0) tl_rec(*x.prm, x.n, 1);
   tc_fence_after();
   if (x.j > 0 && __any_sync(0xffffffffu, need && alpha != 1.f)) {
 #pragma unroll 1
@@ -571,7 +515,7 @@ __device__ __forceinline__ void softmax_tile_cs(const TileCtx& x, float& m, floa
   __syncwarp();
   if (lane == 0) {
     mbar_arrive(x.p_full);
-    tl_rec(*x.prm, x.vc, x.nv, x.n, threadIdx.x == 0 ? 2 : 7 + ((threadIdx.x >> 5) & 3));
+    tl_rec(*x.prm, x.n, threadIdx.x == 0 ? 2 : 7 + ((threadIdx.x >> 5) & 3));
   }
 }
 
@@ -594,32 +538,18 @@ __global__ void __launch_bounds__(WCfg<kD>::kThreads, DCfg<kD>::kMinBlocks)
   constexpr bool kCS = W::kCS;
   constexpr int kSoftWarps = W::kSoftWarps;
   constexpr int kRegsCtl = W::kRegsCtl, kRegsSoftmax = W::kRegsSoftmax;
-  constexpr int kPipes = W::kPipes;
   extern __shared__ uint8_t smem_raw[];
-  const int warp = threadIdx.x >> 5;
-  const int lane = threadIdx.x & 31;
-  // this warp's pipeline (softmax warps [0, kWCtl0), then one control warpgroup per pipeline)
-  const int pipe = kPipes == 1 ? 0 : (warp < W::kWCtl0 ? warp / kSoftWarps : (warp - W::kWCtl0) >> 2);
-  const int cwarp = warp < W::kWCtl0 ? -1 : W::kWCtl0 + ((warp - W::kWCtl0) & 3);   // role as pipeline 0's
-  const int vc = blockIdx.x * kPipes + pipe, nv = gridDim.x * kPipes;   // (diagnostics: virtual CTA)
-  (void)vc;
-  (void)nv;
-  const uint32_t sbase0 = (smem_u32(smem_raw) + 1023u) & ~1023u;
-  auto ctl_of = [&](int pi) {
-    return reinterpret_cast<Ctl*>(smem_raw + (sbase0 + pi * pipe_bytes<kD>() + 6 * kTileBytes + kSt * kMaskBytes -
-                                              smem_u32(smem_raw)));
-  };
-  const uint32_t sQ = sbase0 + pipe * pipe_bytes<kD>();
+  const uint32_t sbase = (smem_u32(smem_raw) + 1023u) & ~1023u;
+  const uint32_t sQ = sbase;
   const uint32_t sK = sQ + 2 * kTileBytes;
   const uint32_t sV = sK + kSt * kTileBytes;
-  const uint32_t sMsk = sV + kSt * kTileBytes;            // [stage] tile bitmasks
-  Ctl* ctl = ctl_of(pipe);
+  const uint32_t sMsk = sV + kSt * kTileBytes;            // [V stage] tile bitmasks
+  Ctl* ctl = reinterpret_cast<Ctl*>(smem_raw + (sMsk + kSt * kMaskBytes - smem_u32(smem_raw)));
+  const int warp = threadIdx.x >> 5;
+  const int lane = threadIdx.x & 31;
   auto bar = [&](const uint64_t& b) { return smem_u32(&b); };
 
   if (threadIdx.x == 0) {
-    for (int pi = 0; pi < kPipes; ++pi) {
-    Ctl* ctl = ctl_of(pi);
-    for (int q = 0; q < 4; ++q) ctl->pp_busy[q] = 0;
     for (int b = 0; b < kItems; ++b) {
       mbar_init(bar(ctl->item_full[b]), 1);
       mbar_init(bar(ctl->item_empty[b]), 2 + kSoftWarps);   // producer + MMA thread + softmax warps
@@ -640,7 +570,6 @@ __global__ void __launch_bounds__(WCfg<kD>::kThreads, DCfg<kD>::kMinBlocks)
     mbar_init(bar(ctl->s_free), kSoftWarps);
     mbar_init(bar(ctl->p_full), kSoftWarps);
     mbar_init(bar(ctl->pv_done), 1);
-    }
     fence_barrier_init();
   }
   if (warp == W::kWProd && lane == 0) {
@@ -653,16 +582,16 @@ __global__ void __launch_bounds__(WCfg<kD>::kThreads, DCfg<kD>::kMinBlocks)
       prefetch_tmap(&tmv2);
     }
   }
-  if (warp == W::kWMma) {   // (pipeline 0's MMA warp allocates both pipelines' columns)
-    tmem_alloc(smem_u32(&ctl->tmem_base), kTmemCols * kPipes);
+  if (warp == W::kWMma) {
+    tmem_alloc(smem_u32(&ctl->tmem_base), kTmemCols);
     tmem_relinquish();
   }
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
-  const uint32_t tmem = ctl_of(0)->tmem_base + (uint32_t)pipe * kTmemCols;
+  const uint32_t tmem = ctl->tmem_base;
 
-  if (cwarp == W::kWProd) {
+  if (warp == W::kWProd) {
     // ============================================================ producer
     asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(kRegsCtl) : "memory");
     const uint64_t pol_kv = policy_evict_last();   // K/V tiles are re-read by neighbouring items
@@ -677,7 +606,7 @@ __global__ void __launch_bounds__(WCfg<kD>::kThreads, DCfg<kD>::kMinBlocks)
       __syncwarp();
       if (lane == 0) {
         mbar_arrive(bar(ctl->item_empty[slot]));
-        tl_item(p, vc, nv, it, 2);
+        tl_item(p, it, 2);
       }
       if (u >= p.total_units) break;
       const int bb = bh / p.H, hh = bh % p.H;
@@ -706,14 +635,14 @@ __global__ void __launch_bounds__(WCfg<kD>::kThreads, DCfg<kD>::kMinBlocks)
         __syncwarp();
         if (lane == 0) mbar_arrive(qf);
       }
-      if (lane == 0) tl_item(p, vc, nv, it, 3);
+      if (lane == 0) tl_item(p, it, 3);
       const int64_t krow0 = bb * p.rk.x + hh * p.rk.y, vrow0 = bb * p.rv.x + hh * p.rv.y;
       for (int j0 = 0; j0 < item.ntiles; j0 += 32) {
         // the item's tile references, 32 at a time (one per lane), broadcast per tile
         int4 mine = make_int4(0, 0, 0, -1);
         if (j0 + lane < item.ntiles) mine = __ldg(reinterpret_cast<const int4*>(p.trefs + item.tref_begin + j0 + lane));
         const int nj = min(32, item.ntiles - j0);
-        if (j0 == 0 && __shfl_sync(0xffffffffu, mine.z, 0) >= 0 && lane == 0) tl_item(p, vc, nv, it, 4);
+        if (j0 == 0 && __shfl_sync(0xffffffffu, mine.z, 0) >= 0 && lane == 0) tl_item(p, it, 4);
         for (int jj = 0; jj < nj; ++jj, ++g) {
           const int arg = __shfl_sync(0xffffffffu, mine.x, jj), kind = __shfl_sync(0xffffffffu, mine.y, jj);
           const int ncols = __shfl_sync(0xffffffffu, mine.z, jj), maskA = __shfl_sync(0xffffffffu, mine.w, jj);
@@ -726,7 +655,7 @@ __global__ void __launch_bounds__(WCfg<kD>::kThreads, DCfg<kD>::kMinBlocks)
           mbar_wait(bar(ctl->k_empty[st]), sph);
           if (lane == 0) {
             ctl->kcols[st] = ncols;   // published by the k_full arrive
-            tl_rec(p, vc, nv, g, 5);
+            tl_rec(p, g, 5);
           }
           if (kind == 0) {
             if (lane == 0) {
@@ -789,7 +718,7 @@ __global__ void __launch_bounds__(WCfg<kD>::kThreads, DCfg<kD>::kMinBlocks)
           }
           if (lane == 0) {
             ctl->vdesc[st] = make_int2(ncols, maskA);   // published by the v_full (mk_full) arrive
-            tl_rec(p, vc, nv, g, 6);
+            tl_rec(p, g, 6);
           }
           const uint32_t vmb = kLate ? 0u : mbytes;     // mask bytes completing on the V barrier
           if (kLate) {
@@ -830,7 +759,7 @@ __global__ void __launch_bounds__(WCfg<kD>::kThreads, DCfg<kD>::kMinBlocks)
         }
       }
     }
-  } else if (cwarp == W::kWSched) {
+  } else if (warp == W::kWSched) {
     // ============================================================ scheduler
     asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(kRegsCtl) : "memory");
     // Claims work items (dynamic counter) into a kItems-deep ring, i.e. up to kItems items ahead of
@@ -840,7 +769,7 @@ __global__ void __launch_bounds__(WCfg<kD>::kThreads, DCfg<kD>::kMinBlocks)
       int u = 0;
       if (lane == 0) {
         mbar_wait(bar(ctl->item_empty[slot]), ((it / kItems) & 1) ^ 1);
-        tl_item(p, vc, nv, it, 0);
+        tl_item(p, it, 0);
         u = atomicAdd(p.counter, 1);
         Slot sl;
         sl.u = u;
@@ -853,13 +782,13 @@ __global__ void __launch_bounds__(WCfg<kD>::kThreads, DCfg<kD>::kMinBlocks)
         }
         ctl->slot[slot] = sl;
         mbar_arrive(bar(ctl->item_full[slot]));
-        tl_item(p, vc, nv, it, 1);
+        tl_item(p, it, 1);
       }
       u = __shfl_sync(0xffffffffu, u, 0);
       if (u >= p.total_units) break;
       __syncwarp();
     }
-  } else if (cwarp == W::kWMma) {
+  } else if (warp == W::kWMma) {
     // ============================================================ MMA issuer (lane 0)
     asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(kRegsCtl) : "memory");
     if (lane == 0) {
@@ -880,7 +809,7 @@ __global__ void __launch_bounds__(WCfg<kD>::kThreads, DCfg<kD>::kMinBlocks)
       auto issue_pv = [&](const Pend& e) {
         mbar_wait(bar(ctl->v_full[e.st]), (e.n / kSt) & 1);
         mbar_wait(bar(ctl->p_full), e.n & 1);
-        tl_rec(p, vc, nv, e.n, 7);
+        tl_rec(p, e.n, 7);
         tc_fence_after();
         const uint32_t vA = sV + e.st * kTileBytes;
         // chunk c (16 keys): P at columns [kTP + 8c, kTP + 8c + 8) (packed pairs), V rows [16c, 16c + 16);
@@ -890,7 +819,7 @@ __global__ void __launch_bounds__(WCfg<kD>::kThreads, DCfg<kD>::kMinBlocks)
           for (int c = 0; c < (kDbgNoMma ? 0 : e.ncols >> 4); ++c)
             mma_ts(tmem + kTO + 64 * sb, tmem + kTP + c * 8, smem_desc_sw128(vA + sb * kSub + c * 2048, 8192, 1024),
                    idesc_pv, (e.first && c == 0) ? 0u : 1u);
-        tl_rec(p, vc, nv, e.n, 4);
+        tl_rec(p, e.n, 4);
         mma_commit(bar(ctl->pv_done));
         mma_commit(bar(ctl->v_empty[e.st]));
       };
@@ -904,7 +833,7 @@ __global__ void __launch_bounds__(WCfg<kD>::kThreads, DCfg<kD>::kMinBlocks)
         const int u = ctl->slot[slot].u;
         const int ntiles = ctl->slot[slot].item.ntiles;
         mbar_arrive(bar(ctl->item_empty[slot]));
-        tl_item(p, vc, nv, it, 6);
+        tl_item(p, it, 6);
         if (u >= p.total_units) break;
         const uint32_t qs = it & 1;
         // finish the previous item first unless this item's Q tile is already resident
@@ -915,13 +844,13 @@ __global__ void __launch_bounds__(WCfg<kD>::kThreads, DCfg<kD>::kMinBlocks)
           pend.valid = false;
         }
         mbar_wait(bar(ctl->q_full[qs]), (it >> 1) & 1);
-        tl_item(p, vc, nv, it, 7);
+        tl_item(p, it, 7);
         const uint32_t qa = sQ + qs * kTileBytes;
         for (int j = 0; j < ntiles; ++j, ++n) {
           const uint32_t st = n % kSt;
           mbar_wait(bar(ctl->k_full[st]), (n / kSt) & 1);
-          tl_rec(p, vc, nv, n, 14);
-          if (n == 0) tl_rec(p, vc, nv, 0, 15);
+          tl_rec(p, n, 14);
+          if (n == 0) tl_rec(p, 0, 15);
           const int ncols = ctl->kcols[st];
           if (n > 0) mbar_wait(bar(ctl->s_free), (n - 1) & 1);
           tc_fence_after();
@@ -936,7 +865,7 @@ __global__ void __launch_bounds__(WCfg<kD>::kThreads, DCfg<kD>::kMinBlocks)
           mma_commit(bar(ctl->s_full));
           mma_commit(bar(ctl->k_empty[st]));
           // (q_empty is arrived by the softmax epilogue: the Q buffer also stages the item's O tile)
-          tl_rec(p, vc, nv, n, 3);
+          tl_rec(p, n, 3);
           if (kLatePV) {
             // due now: P.V(k) for k <= n - 2, and P.V(n - 1) if it is its item's last tile
             int done = 0;
@@ -954,18 +883,14 @@ __global__ void __launch_bounds__(WCfg<kD>::kThreads, DCfg<kD>::kMinBlocks)
       if (pend.valid) issue_pv(pend);
     }
     __syncwarp();
-  } else if (cwarp == W::kWIdle) {
+  } else if (warp == W::kWIdle) {
     asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(kRegsCtl) : "memory");
   } else {
     // ============================================================ softmax + epilogue
     asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(kRegsSoftmax) : "memory");
     // row of the Q tile = TMEM lane (warp w owns lane quarter w % 4); column split: half h = w / 4
     const int hh_cs = kCS ? warp >> 2 : 0;
-    const int t = (warp & 3) * 32 + lane + 128 * hh_cs;   // (> 127: half-1 warp)
-    const bool st0 = threadIdx.x == (unsigned)(pipe * 32 * kSoftWarps);   // the pipeline's first softmax thread
-    // MG_PINGPONG: this warp's and the other pipeline's same-quarter warp's busy flags
-    volatile int32_t* pp_mine = W::kPP ? &ctl->pp_busy[warp & 3] : nullptr;
-    const volatile int32_t* pp_other = W::kPP ? &ctl_of(pipe ^ 1)->pp_busy[warp & 3] : nullptr;
+    const int t = kCS ? (warp & 3) * 32 + lane + 128 * hh_cs : warp * 32 + lane;   // (> 127: half-1 warp)
     const int row = (warp & 3) * 32 + lane;
     const uint32_t tl = tmem + ((uint32_t)((warp & 3) * 32) << 16);
     const float c = p.scale_log2;
@@ -981,7 +906,7 @@ __global__ void __launch_bounds__(WCfg<kD>::kThreads, DCfg<kD>::kMinBlocks)
       const int ubh = ctl->slot[slot].bh;
       __syncwarp();
       if (lane == 0) mbar_arrive(bar(ctl->item_empty[slot]));
-      if (st0) tl_item(p, vc, nv, it, 5);
+      if (threadIdx.x == 0) tl_item(p, it, 5);
       if (u >= p.total_units) break;
       // epilogue metadata, loaded now so its latency hides behind the item's tiles
       int r_out = -1, slot_f = -1;
@@ -996,7 +921,7 @@ __global__ void __launch_bounds__(WCfg<kD>::kThreads, DCfg<kD>::kMinBlocks)
       // (P.V computes garbage O rows that are never stored, and the next item's first P.V
       // overwrites O). It still takes part in the per-tile barriers, in order (s_free(n), then
       // p_full(n) only after P.V(n-1): a p_full arrival may not run ahead into the next phase).
-      const bool idle = kIdleQuarters && (warp & 3) * 32 >= item.nrowsA;
+      const bool idle = kIdleQuarters && warp * 32 >= item.nrowsA;
       for (int j = 0; j < item.ntiles; ++j, ++n) {
         if (idle) {
           mbar_wait(bar(ctl->s_full), n & 1);
@@ -1019,8 +944,8 @@ __global__ void __launch_bounds__(WCfg<kD>::kThreads, DCfg<kD>::kMinBlocks)
         const int2 desc = ctl->vdesc[st];                 // {ncols, maskA}
         const TileCtx tc{tl, sMsk + st * kMaskBytes + row * 16, desc.y >= 0, kPad ? ctl->cmask[st] : nullptr,
                          n, j, bar(ctl->s_free),
-                         bar(ctl->pv_done), bar(ctl->p_full), c, thresh, &p, vc, nv, pp_mine, pp_other};
-        if (st0) tl_rec(p, vc, nv, n, 0);
+                         bar(ctl->pv_done), bar(ctl->p_full), c, thresh, &p};
+        if (threadIdx.x == 0) tl_rec(p, n, 0);
         if constexpr (kCS) {
           // this warp's 32-column chunks of the tile: [2h, 2h + nh)
           const int nh = min(max((desc.x >> 5) - 2 * hh_cs, 0), 2);
@@ -1064,7 +989,7 @@ __global__ void __launch_bounds__(WCfg<kD>::kThreads, DCfg<kD>::kMinBlocks)
           lf = ml.y;
           accf = reinterpret_cast<const float4*>(p.part_acc + fidx * 64);
         }
-        if (st0) tl_rec(p, vc, nv, n - 1, 11);
+        if (threadIdx.x == 0) tl_rec(p, n - 1, 11);
         mbar_wait(bar(ctl->pv_done), (n - 1) & 1);          // the item's last P.V
         tc_fence_after();
         uint32_t o[2][32];
@@ -1072,7 +997,7 @@ __global__ void __launch_bounds__(WCfg<kD>::kThreads, DCfg<kD>::kMinBlocks)
         tmem_ld32(tl + kTO + 32, o[1]);
         tmem_wait_ld();
         tc_fence_before();
-        if (st0) tl_rec(p, vc, nv, n - 1, 12);
+        if (threadIdx.x == 0) tl_rec(p, n - 1, 12);
         bool skip = false;
         if (kSplit && item.kind == 1 && item.nrowsB > 1) {
           // split dense-row item: publish this chunk's (m, l, acc) per row; the chunk that finishes
@@ -1089,13 +1014,13 @@ __global__ void __launch_bounds__(WCfg<kD>::kThreads, DCfg<kD>::kMinBlocks)
             __stcg(reinterpret_cast<float2*>(part + 64), make_float2(m, l));
           }
           __threadfence();
-          named_bar_sync(1 + pipe, 128);
+          named_bar_sync(1, 128);
           // per-group chunk counter in [0, nrowsB): atomicInc wraps it back to 0 on the last chunk, so it
           // is ready for the next forward and never overflows
-          if (st0)
+          if (threadIdx.x == 0)
             ctl->dense_last = atomicInc(reinterpret_cast<unsigned*>(p.dense_ctr) + gidx, (unsigned)item.nrowsB - 1u) ==
                               (unsigned)item.nrowsB - 1u;
-          named_bar_sync(1 + pipe, 128);
+          named_bar_sync(1, 128);
           skip = !ctl->dense_last;
           if (!skip && t < item.nrowsA) {
             __threadfence();
@@ -1183,8 +1108,8 @@ __global__ void __launch_bounds__(WCfg<kD>::kThreads, DCfg<kD>::kMinBlocks)
             }
           }
           fence_proxy_async_smem();
-          named_bar_sync(1 + pipe, 128);
-          if (st0) {
+          named_bar_sync(1, 128);
+          if (threadIdx.x == 0) {
             tma_store_4d(&tmo, sO, 0, item.rowA, ubh % p.H, ubh / p.H);
             bulk_commit_group();
             bulk_wait_group_read0();   // the buffer is reloaded with a later item's Q after q_empty
@@ -1236,7 +1161,7 @@ __global__ void __launch_bounds__(WCfg<kD>::kThreads, DCfg<kD>::kMinBlocks)
           lf = ml.y;
           accf = reinterpret_cast<const float4*>(p.part_acc + fidx * kD);
         }
-        if (st0) tl_rec(p, vc, nv, n - 1, 11);
+        if (threadIdx.x == 0) tl_rec(p, n - 1, 11);
         mbar_wait(bar(ctl->pv_done), (n - 1) & 1);          // the item's last P.V
         tc_fence_after();
         uint32_t o[2][32];
@@ -1246,7 +1171,7 @@ __global__ void __launch_bounds__(WCfg<kD>::kThreads, DCfg<kD>::kMinBlocks)
           tmem_wait_ld();
         };
         if (kNSub == 1) load_o(0);
-        if (st0) tl_rec(p, vc, nv, n - 1, 12);
+        if (threadIdx.x == 0) tl_rec(p, n - 1, 12);
         bool skip = false;
         // split dense-row item whose chunk finishes its group last: O is merged from the chunk partials
         bool merge_chunks = false;
@@ -1273,13 +1198,13 @@ __global__ void __launch_bounds__(WCfg<kD>::kThreads, DCfg<kD>::kMinBlocks)
           }
           if (t < item.nrowsA) __stcg(reinterpret_cast<float2*>(part + kD), make_float2(m, l));
           __threadfence();
-          named_bar_sync(1 + pipe, 128);
+          named_bar_sync(1, 128);
           // per-group chunk counter in [0, nrowsB): atomicInc wraps it back to 0 on the last chunk, so it
           // is ready for the next forward and never overflows
-          if (st0)
+          if (threadIdx.x == 0)
             ctl->dense_last = atomicInc(reinterpret_cast<unsigned*>(p.dense_ctr) + gidx, (unsigned)item.nrowsB - 1u) ==
                               (unsigned)item.nrowsB - 1u;
-          named_bar_sync(1 + pipe, 128);
+          named_bar_sync(1, 128);
           skip = !ctl->dense_last;
           if (!skip && t < item.nrowsA) {
             __threadfence();
@@ -1428,8 +1353,8 @@ __global__ void __launch_bounds__(WCfg<kD>::kThreads, DCfg<kD>::kMinBlocks)
         }
         if (tma_out) {
           fence_proxy_async_smem();
-          named_bar_sync(1 + pipe, 128);
-          if (st0) {
+          named_bar_sync(1, 128);
+          if (threadIdx.x == 0) {
   #pragma unroll
             for (int sb = 0; sb < kNSub; ++sb) tma_store_4d(&tmo, sO + sb * kSub, 64 * sb, item.rowA, hh, bb);
             bulk_commit_group();
@@ -1440,16 +1365,16 @@ __global__ void __launch_bounds__(WCfg<kD>::kThreads, DCfg<kD>::kMinBlocks)
       }
       // the item's Q buffer is free (its last S MMA has completed: pv_done above; its O tile, if
       // staged there, has been read by the TMA store)
-      if (st0) {
+      if (threadIdx.x == 0) {
         mbar_arrive(bar(ctl->q_empty[it & 1]));
-        tl_rec(p, vc, nv, n - 1, 13);
+        tl_rec(p, n - 1, 13);
       }
     }
   }
 
   tc_fence_before();
   __syncthreads();
-  if (warp == W::kWMma) tmem_dealloc(ctl_of(0)->tmem_base, kTmemCols * kPipes);
+  if (warp == W::kWMma) tmem_dealloc(tmem, kTmemCols);
   // the last CTA to finish resets the work counter for the next launch (every CTA's scheduler has
   // claimed its final, out-of-range unit before its CTA gets here), so no memset precedes a launch
   if (threadIdx.x == 0) {

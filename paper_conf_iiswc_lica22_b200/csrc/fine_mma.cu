@@ -61,6 +61,15 @@ __device__ __forceinline__ uint32_t pack2(float lo, float hi) {
 __device__ __forceinline__ void cp_async16(uint32_t dst, const void* src) {
   asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dst), "l"(src) : "memory");
 }
+__device__ __forceinline__ void cp_async16a(uint32_t dst, uint64_t src) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dst), "l"(src) : "memory");
+}
+// base + a * b (64-bit result, one IMAD.WIDE.U32)
+__device__ __forceinline__ uint64_t mad_wide(uint32_t a, uint32_t b, uint64_t base) {
+  uint64_t r;
+  asm("mad.wide.u32 %0, %1, %2, %3;" : "=l"(r) : "r"(a), "r"(b), "l"(base));
+  return r;
+}
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
 template <int N>
 __device__ __forceinline__ void cp_async_wait() {
@@ -433,9 +442,10 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB2) fine_mma2_kernel(c
   const int64_t W = (int64_t)gridDim.x * kWarps;
   const int64_t w0 = (int64_t)blockIdx.x * kWarps + (threadIdx.x >> 5);
   const uint32_t ring = (uint32_t)__cvta_generic_to_shared(fsm) + (threadIdx.x >> 5) * (kStages * kStageBytes2);
-  const uint32_t ksl = (uint32_t)p.k.sl, vsl = (uint32_t)p.v.sl;
+  // row strides in bytes (fit 32 bits: (L - 1) * stride_l < 2^32, checked by the forward's validation)
+  const uint32_t kslb = 2u * (uint32_t)p.k.sl, vslb = 2u * (uint32_t)p.v.sl;
   // head strides fit 32 bits (checked by the launcher)
-  const uint32_t ksh = (uint32_t)p.k.sh, vsh = (uint32_t)p.v.sh, qsh = (uint32_t)p.q.sh;
+  const uint32_t qsh = (uint32_t)p.q.sh;
   constexpr int kIters = kS / kRPI;
   uint32_t doff[kIters];
 #pragma unroll
@@ -446,7 +456,10 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB2) fine_mma2_kernel(c
 
   int64_t gi = w0;
   int ibeg = 0, iend = 0, is = 0, icol = -1, icol_next = -1;
-  const uint16_t *iK = nullptr, *iV = nullptr, *iQ = nullptr;
+  // byte addresses of this lane's 16-byte chunk of row 0 of K / V of both heads of the issuing row: a
+  // gathered row's address is one mad.wide.u32 (column x row stride + base) per copy
+  uint64_t kb0 = 0, kb1 = 0, vb0 = 0, vb1 = 0;
+  const uint16_t* iQ = nullptr;
   auto open_issue_row = [&]() {
     if (gi < nrows) {
       int u0, fi;
@@ -455,8 +468,10 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB2) fine_mma2_kernel(c
       ibeg = __ldg(p.row_ptr + fi);
       iend = __ldg(p.row_ptr + fi + 1);
       const int bb = bh / p.H, hh = bh % p.H;
-      iK = p.k.data + bb * p.k.sb + hh * p.k.sh + (lane % kLPR) * 8;
-      iV = p.v.data + bb * p.v.sb + hh * p.v.sh + (lane % kLPR) * 8;
+      kb0 = reinterpret_cast<uint64_t>(p.k.data + bb * p.k.sb + hh * p.k.sh + (lane % kLPR) * 8);
+      vb0 = reinterpret_cast<uint64_t>(p.v.data + bb * p.v.sb + hh * p.v.sh + (lane % kLPR) * 8);
+      kb1 = kb0 + 2 * (uint64_t)p.k.sh;
+      vb1 = vb0 + 2 * (uint64_t)p.v.sh;
       const int rq = __ldg(p.fine_rows + fi) & 0x7fffffff;
       // lanes 0-7: q of the first head, lanes 8-15: q of the second
       iQ = p.q.data + bb * p.q.sb + hh * p.q.sh + (int64_t)rq * p.q.sl + (lane % kLPR) * 8 + ((lane >> 3) & 1) * qsh;
@@ -473,12 +488,10 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB2) fine_mma2_kernel(c
 #pragma unroll
       for (int i = 0; i < kIters; ++i) {
         const uint32_t cc = (uint32_t)max(__shfl_sync(0xffffffffu, icol, off + kRPI * i), 0);
-        const uint16_t* k0 = iK + cc * ksl;
-        const uint16_t* v0 = iV + cc * vsl;
-        cp_async16(st + doff[i], k0);
-        cp_async16(st + doff[i] + kS * kRowBytes, v0);
-        cp_async16(st + kHB + doff[i], k0 + ksh);
-        cp_async16(st + kHB + doff[i] + kS * kRowBytes, v0 + vsh);
+        cp_async16a(st + doff[i], mad_wide(cc, kslb, kb0));
+        cp_async16a(st + doff[i] + kS * kRowBytes, mad_wide(cc, vslb, vb0));
+        cp_async16a(st + kHB + doff[i], mad_wide(cc, kslb, kb1));
+        cp_async16a(st + kHB + doff[i] + kS * kRowBytes, mad_wide(cc, vslb, vb1));
       }
       if ((is & 1) == 1 && nb0 + kS < iend) icol_next = nb0 + kS + lane < iend ? __ldg(p.cols + nb0 + kS + lane) : -1;
       if (nb0 + kS < iend) {
@@ -506,7 +519,9 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB2) fine_mma2_kernel(c
     const int r = enc & 0x7fffffff;
     const bool final_out = enc < 0;
     const int bb = bh / p.H, hh = bh % p.H;
-    uint32_t qa[2][kJ], qb[2][kJ];
+    // q fragments as the SDDMM's A quads {q, q, q', q'} (rows g and g + 8 of the broadcast q: the
+    // rows g + 8 of the product are never read), kept for the whole row so no step re-packs them
+    uint32_t qq[2][kJ][4];
     const int beg = __ldg(p.row_ptr + fi), end = __ldg(p.row_ptr + fi + 1);
     const int nvalid = kPad ? max(__ldg(p.valid_len + bb), 0) : 0x7fffffff;
     const bool pad_row = kPad && r >= nvalid;
@@ -532,8 +547,10 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB2) fine_mma2_kernel(c
         for (int hd = 0; hd < 2; ++hd)
 #pragma unroll
           for (int j = 0; j < kJ; ++j) {
-            asm volatile("ld.shared.u32 %0, [%1];" : "=r"(qa[hd][j]) : "r"(st + kQOff2 + hd * 128 + 32 * j + 4 * t));
-            asm volatile("ld.shared.u32 %0, [%1];" : "=r"(qb[hd][j]) : "r"(st + kQOff2 + hd * 128 + 32 * j + 16 + 4 * t));
+            asm volatile("ld.shared.u32 %0, [%1];" : "=r"(qq[hd][j][0]) : "r"(st + kQOff2 + hd * 128 + 32 * j + 4 * t));
+            asm volatile("ld.shared.u32 %0, [%1];" : "=r"(qq[hd][j][2]) : "r"(st + kQOff2 + hd * 128 + 32 * j + 16 + 4 * t));
+            qq[hd][j][1] = qq[hd][j][0];
+            qq[hd][j][3] = qq[hd][j][2];
           }
       }
       const int rem = end - base - 2 * t;
@@ -541,23 +558,31 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB2) fine_mma2_kernel(c
 #pragma unroll
       for (int hd = 0; hd < 2; ++hd) {
         const uint32_t sk = st + hd * kHB;
-        float sa[2][4] = {{0.f, 0.f, 0.f, 0.f}, {0.f, 0.f, 0.f, 0.f}};
-        float sb[2][4] = {{0.f, 0.f, 0.f, 0.f}, {0.f, 0.f, 0.f, 0.f}};
+        // chunk A (nnz 0-7) and chunk B (nnz 8-15): one accumulator chain each over the 4 k16 steps
+        float sa[4] = {0.f, 0.f, 0.f, 0.f}, sb[4] = {0.f, 0.f, 0.f, 0.f};
 #pragma unroll
         for (int h = 0; h < 2; ++h) {
           uint32_t ka[4], kb[4];
           const uint32_t sw = ((uint32_t)(((lane >> 3) + 4 * h) ^ (lane & 7))) << 4;
           ldsm_x4(ka, sk + a_row + sw);
           ldsm_x4(kb, sk + b_row + sw);
-          mma16816<kBF16>(sa[h], qa[hd][2 * h], qa[hd][2 * h], qb[hd][2 * h], qb[hd][2 * h], ka[0], ka[1]);
-          mma16816<kBF16>(sb[h], qa[hd][2 * h], qa[hd][2 * h], qb[hd][2 * h], qb[hd][2 * h], kb[0], kb[1]);
-          mma16816<kBF16>(sa[h], qa[hd][2 * h + 1], qa[hd][2 * h + 1], qb[hd][2 * h + 1], qb[hd][2 * h + 1], ka[2], ka[3]);
-          mma16816<kBF16>(sb[h], qa[hd][2 * h + 1], qa[hd][2 * h + 1], qb[hd][2 * h + 1], qb[hd][2 * h + 1], kb[2], kb[3]);
+          const uint32_t(&q0)[4] = qq[hd][2 * h];
+          const uint32_t(&q1)[4] = qq[hd][2 * h + 1];
+          mma16816<kBF16>(sa, q0[0], q0[1], q0[2], q0[3], ka[0], ka[1]);
+          mma16816<kBF16>(sb, q0[0], q0[1], q0[2], q0[3], kb[0], kb[1]);
+          mma16816<kBF16>(sa, q1[0], q1[1], q1[2], q1[3], ka[2], ka[3]);
+          mma16816<kBF16>(sb, q1[0], q1[1], q1[2], q1[3], kb[2], kb[3]);
         }
-        s[hd][0] = rem > 0 ? sa[0][0] + sa[1][0] : -INFINITY;
-        s[hd][1] = rem > 1 ? sa[0][1] + sa[1][1] : -INFINITY;
-        s[hd][2] = rem > 8 ? sb[0][0] + sb[1][0] : -INFINITY;
-        s[hd][3] = rem > 9 ? sb[0][1] + sb[1][1] : -INFINITY;
+        s[hd][0] = sa[0];
+        s[hd][1] = sa[1];
+        s[hd][2] = sb[0];
+        s[hd][3] = sb[1];
+        if (end - base < kS) {   // the row's last, partial step (warp-uniform): entries past the row
+          s[hd][0] = rem > 0 ? s[hd][0] : -INFINITY;
+          s[hd][1] = rem > 1 ? s[hd][1] : -INFINITY;
+          s[hd][2] = rem > 8 ? s[hd][2] : -INFINITY;
+          s[hd][3] = rem > 9 ? s[hd][3] : -INFINITY;
+        }
       }
       if (kPad) {   // padding: mask the columns at or beyond n_b (same columns for both heads)
         const int o4[4] = {0, 1, 8, 9};
