@@ -284,20 +284,31 @@ __device__ __forceinline__ void chunk_exp_f32(uint32_t (&r)[32], float2 c2, floa
 }
 
 // Diagnostics (MG_TIMELINE builds only): per-tile event clocks (low 32 bits of clock64) of every
-// CTA for its first kTlTiles tiles, 16 fields per tile, after 256 uint64 header words of p.trace:
+// CTA for its first kTlTiles tiles, kTlF fields per tile (16 S in registers, 17 exponentials done,
+// 18 = 1 if S(n+1) was complete when P(n) was stored), after 256 uint64 header words of p.trace:
 // 0 softmax S(n)+V(n) ready, 1 softmax P.V(n-1) done, 2 softmax warp 0 P(n) stored, 3 MMA S(n)
 // issued, 4 MMA P.V(n) issued, 5 producer K(n) issued, 6 producer V(n) issued, 7 MMA sees p_full(n),
 // 8-10 softmax warps 1-3 P(n) stored, 11/12/13 epilogue start / O read / end (last tile of an
 // item), 14 MMA sees k_full(n), 15 SM id (tile 0 only). tools/timeline_pp.py reads it.
-constexpr int kTlTiles = 128;
+constexpr int kTlTiles = 128, kTlF = 24;   // tiles recorded per CTA, fields per tile
 __device__ __forceinline__ void tl_rec(const CoarseParams& p, uint32_t n, int field) {
 #ifdef MG_TIMELINE
   if (p.trace == nullptr || n >= (uint32_t)kTlTiles ||
-      (int64_t)p.trace_cap < 256 + (int64_t)8 * kTlTiles * (int64_t)gridDim.x)
+      (int64_t)p.trace_cap < 256 + (int64_t)(kTlF / 2) * kTlTiles * (int64_t)gridDim.x)
     return;
   uint32_t v = (uint32_t)clock64();
   if (field == 15) asm("mov.u32 %0, %%smid;" : "=r"(v));
-  reinterpret_cast<uint32_t*>(p.trace + 256)[((size_t)blockIdx.x * kTlTiles + n) * 16 + field] = v;
+  reinterpret_cast<uint32_t*>(p.trace + 256)[((size_t)blockIdx.x * kTlTiles + n) * kTlF + field] = v;
+#endif
+}
+
+// a value instead of a clock (field 18: S(n+1) already complete when P(n) is stored)
+__device__ __forceinline__ void tl_val(const CoarseParams& p, uint32_t n, int field, uint32_t v) {
+#ifdef MG_TIMELINE
+  if (p.trace == nullptr || n >= (uint32_t)kTlTiles ||
+      (int64_t)p.trace_cap < 256 + (int64_t)(kTlF / 2) * kTlTiles * (int64_t)gridDim.x)
+    return;
+  reinterpret_cast<uint32_t*>(p.trace + 256)[((size_t)blockIdx.x * kTlTiles + n) * kTlF + field] = v;
 #endif
 }
 
@@ -307,9 +318,9 @@ __device__ __forceinline__ void tl_rec(const CoarseParams& p, uint32_t n, int fi
 __device__ __forceinline__ void tl_item(const CoarseParams& p, uint32_t it, int field) {
 #ifdef MG_TIMELINE
   if (p.trace == nullptr || it >= 32u ||
-      (int64_t)p.trace_cap < 256 + (int64_t)(8 * kTlTiles + 128) * (int64_t)gridDim.x)
+      (int64_t)p.trace_cap < 256 + (int64_t)((kTlF / 2) * kTlTiles + 128) * (int64_t)gridDim.x)
     return;
-  reinterpret_cast<uint32_t*>(p.trace + 256)[(size_t)gridDim.x * kTlTiles * 16 + ((size_t)blockIdx.x * 32 + it) * 8 +
+  reinterpret_cast<uint32_t*>(p.trace + 256)[(size_t)gridDim.x * kTlTiles * kTlF + ((size_t)blockIdx.x * 32 + it) * 8 +
                                              field] = (uint32_t)clock64();
 #endif
 }
@@ -353,6 +364,7 @@ struct TileCtx {
   uint32_t s_free, pv_done, p_full;
   float c, thresh;
   const CoarseParams* prm;   // diagnostics only (tl_rec, debug_flags)
+  uint32_t s_full;           // diagnostics only (timeline field 18)
 };
 
 // One tile of the online SpSoftmax for this thread's row (NQ x 32 columns): read S(n) from TMEM
@@ -366,6 +378,7 @@ __device__ __forceinline__ void softmax_tile(const TileCtx& x, float& m, float& 
 #pragma unroll
   for (int q = 0; q < NQ; ++q) tmem_ld32(x.tl + kTS + q * 32, r[q]);
   tmem_wait_ld();
+  if (threadIdx.x == 0) tl_rec(*x.prm, x.n, 16);
   tc_fence_before();
   __syncwarp();
   if (lane == 0) mbar_arrive(x.s_free);                 // S may be overwritten by S(n+1)
@@ -405,6 +418,7 @@ __device__ __forceinline__ void softmax_tile(const TileCtx& x, float& m, float& 
   uint32_t pre[kPreN > 0 ? kPreN : 1][16];
 #pragma unroll
   for (int q = 0; q < kPreN; ++q) chunk_exp<kBF16>(r[q], c2, nb2, rs, pre[q]);
+  if (threadIdx.x == 0) tl_rec(*x.prm, x.n, 17);
   // P.V(n-1) has consumed P(n-1) and updated O: rescale O if the max moved, then store P(n)
   // chunk by chunk as it is produced (the other CTA on this SM keeps the pipes busy meanwhile)
   if (x.n > 0) mbar_wait(x.pv_done, (x.n - 1) & 1);
@@ -436,6 +450,9 @@ __device__ __forceinline__ void softmax_tile(const TileCtx& x, float& m, float& 
   if (lane == 0) {
     mbar_arrive(x.p_full);
     tl_rec(*x.prm, x.n, threadIdx.x == 0 ? 2 : 7 + (threadIdx.x >> 5));
+#ifdef MG_TIMELINE
+    if (threadIdx.x == 0) tl_val(*x.prm, x.n, 18, mbar_test_wait(x.s_full, (x.n + 1) & 1) ? 1u : 0u);
+#endif
   }
 }
 
@@ -944,7 +961,7 @@ __global__ void __launch_bounds__(WCfg<kD>::kThreads, DCfg<kD>::kMinBlocks)
         const int2 desc = ctl->vdesc[st];                 // {ncols, maskA}
         const TileCtx tc{tl, sMsk + st * kMaskBytes + row * 16, desc.y >= 0, kPad ? ctl->cmask[st] : nullptr,
                          n, j, bar(ctl->s_free),
-                         bar(ctl->pv_done), bar(ctl->p_full), c, thresh, &p};
+                         bar(ctl->pv_done), bar(ctl->p_full), c, thresh, &p, bar(ctl->s_full)};
         if (threadIdx.x == 0) tl_rec(p, n, 0);
         if constexpr (kCS) {
           // this warp's 32-column chunks of the tile: [2h, 2h + nh)

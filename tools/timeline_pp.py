@@ -18,6 +18,7 @@ import paper_conf_iiswc_lica22_b200 as mg  # noqa: E402
 from workloads import get_config, make_qkv  # noqa: E402
 
 T = 128
+F = 24   # fields per tile (coarse_pp_sm100.cu kTlF)
 
 
 def main():
@@ -31,14 +32,14 @@ def main():
     for _ in range(3):
         mg.sparse_attention_fwd(plan, Q, K, V)
     ncta = 2 * torch.cuda.get_device_properties(0).multi_processor_count
-    buf = torch.zeros(256 + (8 * T + 128) * ncta, dtype=torch.int64, device="cuda")
+    buf = torch.zeros(256 + (12 * T + 128) * ncta, dtype=torch.int64, device="cuda")
     plan.set_trace(buf)
     mg.sparse_attention_fwd(plan, Q, K, V)
     torch.cuda.synchronize()
     plan.set_trace(None)
     raw = buf.cpu().numpy()[256:].view(np.uint32).astype(np.int64)
-    rec = raw[:ncta * T * 16].reshape(ncta, T, 16)
-    itm = raw[ncta * T * 16:].reshape(ncta, 32, 8)
+    rec = raw[:ncta * T * F].reshape(ncta, T, F)
+    itm = raw[ncta * T * F:ncta * T * F + ncta * 256].reshape(ncta, 32, 8)
     smid = rec[:, 0, 15].copy()
     rec[:, 0, 15] = 0
     d = lambda a, b: (b - a + 2**31) % 2**32 - 2**31   # wrap-safe difference of 32-bit clocks
@@ -62,6 +63,10 @@ def main():
             add("MMA: S(n+1) issued -> softmax S(n+1) ready", d(f[3], f[0]))
             add("producer: K(n) issued -> MMA sees k_full(n)", d(e[5], e[14]))
             add("tile period (S ready n -> n+1)", d(e[0], f[0]))
+            add("softmax: S(n) ready -> S in registers", d(e[0], e[16]))
+            add("softmax: S in registers -> exps done", d(e[16], e[17]))
+            add("softmax: exps done -> P.V(n-1) done (wait)", d(e[17], e[1]))
+            add("softmax: S(n+1) complete when P(n) stored (fraction)", int(e[18]))
             if e[11]:
                 add("epilogue: start -> last P.V done + O read", d(e[11], e[12]))
                 add("epilogue: O read -> end", d(e[12], e[13]))
