@@ -56,8 +56,8 @@ def parse():
     ap.add_argument("--strip-max-cols", type=int, default=0)
     ap.add_argument("--ablation", action="store_true",
                     help="also time the staged paper-dataflow forward (mg_sparse_attention_fwd_staged)")
-    ap.add_argument("--concurrency", type=int, default=0, choices=[0, 1, 2],
-                    help="coarse vs CSR kernels: 0 = library default, 1 = serial, 2 = concurrent streams")
+    ap.add_argument("--concurrency", type=int, default=0, choices=[0, 1, 2, 3],
+                    help="coarse vs CSR kernels: 0 = library default, 1 = serial, 2 = concurrent streams, 3 = SM split")
     ap.add_argument("--tau", type=float, default=0.0, help="tile density threshold (0 = band rule)")
     ap.add_argument("--block", type=int, default=0, choices=[0, 64, 128], help="plan block size (0 = 128)")
     ap.add_argument("--head-dim", type=int, default=0, choices=[0, 64, 128],

@@ -118,7 +118,12 @@ typedef struct {
                              (mma.sync, default), 1 -> CUDA-core shuffle-reduction kernel (A/B) */
   int32_t concurrency;    /* coarse vs CUDA-core CSR kernels: 0 -> library default, 1 -> serial (fine
                              kernel, then coarse kernel merging its partials), 2 -> concurrent on two
-                             streams, rows merged by whichever side finishes second */
+                             streams, rows merged by whichever side finishes second,
+                             3 -> SM split: the coarse kernel first on a persistent grid of one CTA
+                             per SM on a share of the SMs proportional to its estimated work (env
+                             MG_SPLIT_CTAS overrides), the fine kernel beside it on a second stream
+                             over the whole device with dynamically claimed rows, merge as in 2
+                             (north_star item 5, "run concurrently in different SMs") */
   float tau;              /* tile rule: 0 -> every tile touched by the band of a non-global row is
                              coarse (default, A7); (0, 1] -> a tile is coarse iff its
                              non-global union elements number >= tau * block^2 (A17) */

@@ -23,7 +23,8 @@ class Plan:
     Args follow include/mg.h: L, heads, d, window, global_idx (int array), extra_idx (int [n, 2]).
     Options (test/ablation): block, force_all_fine, strip_max_cols, num_sms, fine_kernel
     (0 = warp-level tensor-core CSR kernel, 1 = CUDA-core CSR kernel), concurrency (0 = default,
-    1 = serial fine -> coarse, 2 = concurrent streams with last-finisher row merge), tau (tile
+    1 = serial fine -> coarse, 2 = concurrent streams with last-finisher row merge, 3 = SM split:
+    coarse kernel on a share of the SMs, fine kernel beside it with dynamic rows), tau (tile
     density threshold; 0 = band rule), dense_chunk (column tiles per dense-row item; 0 = default 8,
     -1 = no split).
     """

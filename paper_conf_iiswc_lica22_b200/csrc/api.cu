@@ -49,7 +49,7 @@ struct mg_plan_s {
   int num_sms = 0;
   int num_sms_override = 0;
   int fine_kernel = 0;   // 0: mma.sync kernel (fine_mma.cu), 1: CUDA-core kernel (fine_rows.cu)
-  int concurrency = 0;   // 0 default, 1 serial, 2 concurrent streams (see mg_plan_opts)
+  int concurrency = 0;   // 0 default, 1 serial, 2 concurrent streams, 3 SM split (see mg_plan_opts)
   cudaStream_t side = nullptr;              // second stream of the concurrent mode
   // host-buffer forward: copy streams and per-chunk events (H2D of chunk c+1 and D2H of chunk c-1
   // overlap the forward of chunk c)
@@ -206,7 +206,7 @@ mg_status create_impl(int64_t L, int32_t heads, int32_t d, int32_t window, const
     sms_override = opts->num_sms;
     if (opts->fine_kernel < 0 || opts->fine_kernel > 1) return fail(MG_ERR_INVALID_ARG, "fine_kernel must be 0 or 1");
     fine_kernel = opts->fine_kernel;
-    if (opts->concurrency < 0 || opts->concurrency > 2) return fail(MG_ERR_INVALID_ARG, "concurrency must be 0, 1 or 2");
+    if (opts->concurrency < 0 || opts->concurrency > 3) return fail(MG_ERR_INVALID_ARG, "concurrency must be 0, 1, 2 or 3");
     concurrency = opts->concurrency;
     if (!(opts->tau >= 0.f && opts->tau <= 1.f)) return fail(MG_ERR_INVALID_ARG, "tau must be in [0, 1]");
     po.tau = opts->tau;
@@ -360,6 +360,24 @@ mg::TensorView view(const mg_tensor* t) {
 // measured on B200: C4 serial vs concurrent
 constexpr bool kConcurrentDefault = false;
 
+// SM-split mode: coarse CTAs (one per SM) such that the coarse part takes about as long as the fine
+// kernel would alone, from measured costs (C4): ~5,800 cycles per 128 x 128 tile for
+// a coarse CTA sharing its SM with a fine block, ~6.4 cycles per CSR nnz and head per SM for the
+// fine kernel. The environment variable MG_SPLIT_CTAS overrides it (A/B).
+int coarse_split_ctas(const mg::HostPlan& h, int BH, int sms) {
+  static const int env = [] {
+    const char* e = std::getenv("MG_SPLIT_CTAS");
+    return e ? std::atoi(e) : 0;
+  }();
+  if (env > 0) return env;
+  int64_t tiles = 0;
+  for (const mg::Item& it : h.items) tiles += it.ntiles;
+  const double coarse_cta_cycles = (double)tiles * BH * 5800.0;
+  const double fine_cycles = (double)h.fine_col.size() * BH * 6.4 / std::max(sms, 1);
+  const int k = (int)std::ceil(coarse_cta_cycles / std::max(fine_cycles, 1.0));
+  return std::max(1, std::min(k, sms));
+}
+
 mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const mg_tensor* V, mg_tensor* O,
                    cudaStream_t stream, const int32_t* valid_len = nullptr) {
   mg_status s = upload(p);
@@ -378,7 +396,13 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
   // Concurrent coarse || fine (north_star item 5): chosen by measurement, only with
   // the tensor-core fine kernel and the paired-pipeline coarse kernel.
   const bool concurrent = nf > 0 && !h.items.empty() && p->fine_kernel == 0 &&
-                          (p->concurrency == 2 || (p->concurrency == 0 && kConcurrentDefault));
+                          (p->concurrency >= 2 || (p->concurrency == 0 && kConcurrentDefault));
+  // SM split (concurrency 3): the coarse kernel is launched first with a persistent grid of
+  // coarse_split_ctas() CTAs (one per SM, beside which one fine block still fits), then the fine
+  // kernel over the whole device with dynamically claimed rows, so its blocks that could not start
+  // next to a coarse CTA take the remaining rows once that CTA leaves; rows with both parts merge as in
+  // the concurrent mode
+  const bool sm_split = concurrent && p->concurrency == 3;
   // fp32 partials of the CUDA-core CSR rows (fine -> coarse; and coarse -> fine plus one counter
   // per row when concurrent). Layout by capacity: [fine acc d][fine ml 2][coarse acc d][coarse ml 2]
   // floats per slot, then one int32 counter per slot (zeroed at allocation; even between forwards).
@@ -480,8 +504,10 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
       mp.valid = true;
     }
   }
+  auto launch_fine_part = [&]() -> mg_status {
   if (nf > 0) {
     mg::FineParams fp{};
+    fp.row_ctr = sm_split ? p->d_counter + 2 : nullptr;
     fp.fine_rows = p->d_fine_rows;
     fp.row_ptr = p->d_fine_row_ptr;
     fp.cols = p->d_fine_col;
@@ -531,6 +557,9 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
       pc.fe = pc.cb = prof_rec(stream);
     }
   }
+  return MG_OK;
+  };
+  auto launch_coarse_part = [&]() -> mg_status {
   if (!h.items.empty()) {
     mg_plan_s::Maps& mp = p->maps;
     if (!mp.ok)
@@ -584,13 +613,20 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
       cp.rv = mp.rv;
       static const bool no_tma_store = std::getenv("MG_NO_TMA_STORE") != nullptr;   // A/B diagnostics
       cp.tma_store = !no_tma_store && mp.store_ok;
+      const int grid = sm_split ? coarse_split_ctas(h, BH, sms) : mg::coarse_pp_ctas_per_sm(D) * sms;
       if ((e = mg::launch_coarse_pp(cp, tq, tk, tv, mp.tq2, mp.tk2, mp.tv2, mp.to, bf16, use_split,
-                                    std::min(mg::coarse_pp_ctas_per_sm(D) * sms, cp.total_units),
-                                    stream)) != cudaSuccess)
+                                    std::min(grid, cp.total_units), stream)) != cudaSuccess)
         return cuda_fail(e, "coarse kernel launch");
     }
   }
   if (p->profiling && concurrent) pc.ce = prof_rec(stream);
+  return MG_OK;
+  };
+  if (sm_split) {
+    if ((s = launch_coarse_part()) != MG_OK || (s = launch_fine_part()) != MG_OK) return s;
+  } else {
+    if ((s = launch_fine_part()) != MG_OK || (s = launch_coarse_part()) != MG_OK) return s;
+  }
   if (concurrent) {
     if ((e = cudaEventRecord(p->join_ev, fstream)) != cudaSuccess ||
         (e = cudaStreamWaitEvent(stream, p->join_ev, 0)) != cudaSuccess)

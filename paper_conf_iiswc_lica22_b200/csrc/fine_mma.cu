@@ -428,8 +428,12 @@ constexpr int kStageBytes2 = kQOff2 + 2 * 128;
 constexpr int kSmemBytes2 = kWarps * kStages * kStageBytes2;
 }  // namespace
 
-template <bool kBF16, bool kPad>
+// kDyn (SM-split mode): the (head pair, CSR row) sequence of a warp comes from a global counter in
+// chunks of kChunk consecutive rows instead of the static stride; the issue side claims, the compute
+// side follows it one step behind (so it finds the chunk the issue side is in when it leaves its own).
+template <bool kBF16, bool kPad, bool kDyn>
 __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB2) fine_mma2_kernel(const FineParams p) {
+  constexpr int kChunk = 4;
   constexpr int kD = 64, kRowBytes = 128, kLPR = 8, kRPI = 4, kJ = 4;
   extern __shared__ __align__(128) uint8_t fsm[];
   const int lane = threadIdx.x & 31;
@@ -454,7 +458,31 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB2) fine_mma2_kernel(c
     doff[i] = R * kRowBytes + (((lane % kLPR) ^ (R & 7)) << 4);
   }
 
-  int64_t gi = w0;
+  // dynamic rows: claim a chunk (warp-uniform), -> its first row, or nrows when exhausted
+  auto claim = [&]() -> int64_t {
+    int c = 0;
+    if (lane == 0) c = atomicAdd(p.row_ctr, 1);
+    c = __shfl_sync(0xffffffffu, c, 0);
+    const int64_t g = (int64_t)c * kChunk;
+    return g < nrows ? g : nrows;
+  };
+  // Chunks claimed by the issue side for the compute side (the same warp, one step behind): the
+  // issue side is never more than the next chunk (plus the final exhausted claim) ahead, so two
+  // entries suffice.
+  int64_t fq0 = nrows, fq1 = nrows;
+  int fn = 0;
+  // the row after g in the issue side's sequence
+  auto next_row = [&](int64_t g) -> int64_t {
+    if (!kDyn) return g + W;
+    if ((g + 1) % kChunk != 0 && g + 1 < nrows) return g + 1;
+    const int64_t c = claim();
+    if (fn == 0) fq0 = c;
+    else fq1 = c;
+    ++fn;
+    return c;
+  };
+  int64_t gi = kDyn ? claim() : w0;
+  const int64_t g_first = gi;   // the compute side's first row (the prologue below may move gi on)
   int ibeg = 0, iend = 0, is = 0, icol = -1, icol_next = -1;
   // byte addresses of this lane's 16-byte chunk of row 0 of K / V of both heads of the issuing row: a
   // gathered row's address is one mad.wide.u32 (column x row stride + base) per copy
@@ -497,7 +525,7 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB2) fine_mma2_kernel(c
       if (nb0 + kS < iend) {
         ++is;
       } else {
-        gi += W;
+        gi = next_row(gi);
         open_issue_row();
       }
     }
@@ -511,7 +539,15 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB2) fine_mma2_kernel(c
   const uint32_t a_row = (lane & 7) * kRowBytes, b_row = a_row + 8 * kRowBytes;
   const uint32_t vr = (lane & 7) + 8 * (lane >> 4);
 
-  for (int64_t gw = w0; gw < nrows; gw += W) {
+  auto next_compute_row = [&](int64_t g) -> int64_t {
+    if (!kDyn) return g + W;
+    if ((g + 1) % kChunk != 0 && g + 1 < nrows) return g + 1;
+    const int64_t c = fn > 0 ? fq0 : nrows;
+    fq0 = fq1;
+    fn = fn > 0 ? fn - 1 : 0;
+    return c;
+  };
+  for (int64_t gw = g_first; gw < nrows; gw = next_compute_row(gw)) {
     int u0, fi;
     split_row(gw, p.n_fine_rows, r32, u0, fi);
     const int bh = (p.fine_sample ? __ldg(p.fine_sample + fi) * p.H : 0) + 2 * u0;
@@ -684,6 +720,17 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB2) fine_mma2_kernel(c
     }
   }
   cp_async_wait<0>();
+  if (kDyn) {
+    // the last block to finish resets the row counter for the next launch
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      __threadfence();
+      if (atomicAdd(p.row_ctr + 1, 1) == (int)gridDim.x - 1) {
+        atomicExch(p.row_ctr, 0);
+        atomicExch(p.row_ctr + 1, 0);
+      }
+    }
+  }
 }
 
 // ---------------------------------------------------------------------------------------------
@@ -999,10 +1046,13 @@ cudaError_t launch_fine_mma(const FineParams& p, bool bf16, int sms, cudaStream_
   }();
   const bool hp2 = !no_hp2 && p.d == 64 && (p.H % 2) == 0 && p.k.sh < (int64_t(1) << 31) &&
                    p.v.sh < (int64_t(1) << 31) && p.q.sh < (int64_t(1) << 31);
-  static const K table2[4] = {fine_mma2_kernel<false, false>, fine_mma2_kernel<false, true>,
-                              fine_mma2_kernel<true, false>, fine_mma2_kernel<true, true>};
+  static const K table2[8] = {fine_mma2_kernel<false, false, false>, fine_mma2_kernel<false, true, false>,
+                              fine_mma2_kernel<true, false, false>,  fine_mma2_kernel<true, true, false>,
+                              fine_mma2_kernel<false, false, true>,  fine_mma2_kernel<false, true, true>,
+                              fine_mma2_kernel<true, false, true>,   fine_mma2_kernel<true, true, true>};
   const int vi = hp2 ? 8 + (bf16 ? 2 : 0) + (p.valid_len ? 1 : 0) : (p.d == 128 ? 4 : 0) + (bf16 ? 2 : 0) + (p.valid_len ? 1 : 0);
-  const K kern = hp2 ? table2[vi - 8] : table[vi];
+  // dynamic rows (SM-split mode) exist in the two-head kernel only; the others keep the static order
+  const K kern = hp2 ? table2[vi - 8 + (p.row_ctr ? 4 : 0)] : table[vi];
   const int kSmemBytes = hp2 ? kSmemBytes2 : (p.d == 128 ? FCfg<128>::kSmemBytes : FCfg<64>::kSmemBytes);
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytes);
   if (e != cudaSuccess) return e;
@@ -1015,11 +1065,12 @@ cudaError_t launch_fine_mma(const FineParams& p, bool bf16, int sms, cudaStream_
   if ((e = cudaGetDevice(&dev)) != cudaSuccess) return e;
   {
     std::lock_guard<std::mutex> lk(mu);
-    auto it = per_sm.find({dev, vi});
+    const int key = vi + (hp2 && p.row_ctr ? 100 : 0);
+    auto it = per_sm.find({dev, key});
     if (it == per_sm.end()) {
       if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kern, kWarps * 32, kSmemBytes)) != cudaSuccess)
         return e;
-      it = per_sm.emplace(std::make_pair(dev, vi), std::max(n, 1)).first;
+      it = per_sm.emplace(std::make_pair(dev, key), std::max(n, 1)).first;
     }
     n = it->second;
   }

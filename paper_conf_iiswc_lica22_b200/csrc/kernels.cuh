@@ -80,6 +80,11 @@ struct FineParams {
   const float* part_c_acc;
   const float2* part_c_ml;
   int32_t* part_flags;
+  // SM-split mode (plan concurrency 3): rows are claimed dynamically in chunks of 4 from
+  // row_ctr[0] (row_ctr[1] counts finished blocks; the last one resets both), so blocks that start
+  // late, once the coarse kernel's CTAs leave their SMs, take the remaining rows. null: the static
+  // grid-stride row order.
+  int32_t* row_ctr;
 };
 
 // Staged (paper dataflow) kernels: S and P materialised in the plan's formats; see staged.cu.

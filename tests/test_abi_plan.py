@@ -137,6 +137,8 @@ def status_of(fn):
     (dict(L=64, heads=1, d=64, window=2, strip_max_cols=256), _lib.MG_ERR_INVALID_ARG),
     (dict(L=64, heads=1, d=64, window=2, tau=1.5), _lib.MG_ERR_INVALID_ARG),
     (dict(L=64, heads=1, d=64, window=2, tau=-0.1), _lib.MG_ERR_INVALID_ARG),
+    (dict(L=64, heads=1, d=64, window=2, concurrency=4), _lib.MG_ERR_INVALID_ARG),
+    (dict(L=64, heads=1, d=64, window=2, concurrency=-1), _lib.MG_ERR_INVALID_ARG),
 ])
 def test_plan_create_validation(kwargs, status):
     assert status_of(lambda: mg.Plan(**kwargs)) == status

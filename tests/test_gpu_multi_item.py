@@ -46,8 +46,8 @@ def check(got, ref):
 
 @pytest.mark.parametrize("num_sms", [1, 2, 3])
 @pytest.mark.parametrize("kw", [{}, dict(strip_max_cols=-1), dict(strip_max_cols=-1, concurrency=2),
-                                dict(dense_chunk=2), dict(force_all_fine=True)],
-                         ids=["strips", "csr_rows", "concurrent", "dense_split", "all_fine"])
+                                dict(strip_max_cols=-1, concurrency=3), dict(dense_chunk=2), dict(force_all_fine=True)],
+                         ids=["strips", "csr_rows", "concurrent", "sm_split", "dense_split", "all_fine"])
 def test_few_ctas_many_items(num_sms, kw):
     E = random_residual(L, W, 6, seed=3)
     q, k, v = make_qkv(B, H, L, 64, seed=5, dist="adversarial", global_idx=G)

@@ -67,7 +67,7 @@ def mixed_extra(L, seed=3, per_row=6):
     return random_residual(L, 128, per_row, seed=seed)
 
 
-@pytest.mark.parametrize("fine_kernel,concurrency", [(0, 1), (0, 2), (1, 1)])
+@pytest.mark.parametrize("fine_kernel,concurrency", [(0, 1), (0, 2), (0, 3), (1, 1)])
 @pytest.mark.parametrize("strip", [0, -1])
 @pytest.mark.parametrize("all_fine", [False, True])
 def test_mixed_pattern_all_parts(strip, all_fine, fine_kernel, concurrency):
@@ -86,7 +86,7 @@ def test_mixed_pattern_all_parts(strip, all_fine, fine_kernel, concurrency):
     check(got, ref)
 
 
-@pytest.mark.parametrize("fine_kernel,concurrency", [(0, 1), (0, 2), (1, 1)])
+@pytest.mark.parametrize("fine_kernel,concurrency", [(0, 1), (0, 2), (0, 3), (1, 1)])
 @pytest.mark.parametrize("dtype", ["bf16", "fp16"])
 @pytest.mark.parametrize("dist", ["normal", "peaky", "adversarial"])
 def test_fine_rows_all_lengths(fine_kernel, concurrency, dtype, dist):
@@ -246,7 +246,7 @@ def sample_rows(L, G, rng, n=48):
     return sorted(r for r in rows if 0 <= r < L)
 
 
-@pytest.mark.parametrize("cfg,fine_kernel,concurrency", [("C2", 0, 0), ("C3", 0, 0), ("C4", 0, 1), ("C4", 0, 2),
+@pytest.mark.parametrize("cfg,fine_kernel,concurrency", [("C2", 0, 0), ("C3", 0, 0), ("C4", 0, 1), ("C4", 0, 2), ("C4", 0, 3),
                                                           ("C4", 1, 1), ("QDS-LS", 0, 0), ("F9-LS", 0, 0),
                                                           ("F9-LSG", 0, 0), ("F9-LBR", 0, 0), ("F9-RBR", 0, 0),
                                                           ("F9-RBR", 0, 0.2)])
@@ -273,7 +273,7 @@ def test_full_size_sampled(cfg, fine_kernel, concurrency):
 
 
 # ------------------------------------------------------------------ padding (valid length, A18)
-@pytest.mark.parametrize("case", ["mixed", "c1", "fine_only", "dense_split", "concurrent"])
+@pytest.mark.parametrize("case", ["mixed", "c1", "fine_only", "dense_split", "concurrent", "sm_split"])
 def test_padded_batch(case):
     """mg_sparse_attention_fwd_padded: per-sample valid lengths (including 0, full, and cuts inside
     row blocks and strips); every part (tiles, strips, CSR rows, dense rows, split dense chunks,
@@ -287,7 +287,8 @@ def test_padded_batch(case):
         B, H, L, window, G = 4, m["H"], m["L"], m["window"], m["G"]
         E = mixed_extra(L, seed=12)
         kw = {"fine_only": dict(strip_max_cols=-1), "dense_split": dict(dense_chunk=2),
-              "concurrent": dict(strip_max_cols=-1, concurrency=2), "mixed": {}}[case]
+              "concurrent": dict(strip_max_cols=-1, concurrency=2),
+              "sm_split": dict(strip_max_cols=-1, concurrency=3), "mixed": {}}[case]
     q, k, v = make_qkv(B, H, L, 64, seed=41, dist="adversarial", global_idx=G)
     plan = mg.Plan(L, H, 64, window, G, E, **kw)
     lens = np.array([L, 0, L // 2 + 37, 129][:B], np.int32)
@@ -306,7 +307,7 @@ def test_padded_batch(case):
 
 # ------------------------------------------------------------------ batched plans (per-sample positions)
 @pytest.mark.parametrize("kw", [{}, dict(strip_max_cols=-1), dict(strip_max_cols=-1, concurrency=2),
-                                dict(fine_kernel=1, strip_max_cols=-1)])
+                                dict(strip_max_cols=-1, concurrency=3), dict(fine_kernel=1, strip_max_cols=-1)])
 def test_batched_plan_per_sample_positions(kw):
     """One launch over a batch whose samples have different global tokens and residuals (P:66,
     P:94), against the oracle per sample; padded too."""
