@@ -507,7 +507,18 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
   auto launch_fine_part = [&]() -> mg_status {
   if (nf > 0) {
     mg::FineParams fp{};
-    fp.row_ctr = sm_split ? p->d_counter + 2 : nullptr;
+    // Dynamic row chunks (two-head kernel): required by the SM split; otherwise when each warp of the
+    // persistent grid has many rows (>= 64 head-pair rows per warp: C4 fine kernel 1.885 -> 1.850 ms),
+    // while short row lists keep the static order (the start-up burst of claims on one counter costs
+    // more than the balance gains: F9-RBR 0.072 vs 0.094 ms). MG_FINE_DYN=0/1 forces it (A/B).
+    static const int fine_dyn_env = [] {
+      const char* ev = std::getenv("MG_FINE_DYN");
+      return ev ? std::atoi(ev) : -1;
+    }();
+    const int64_t rows2 = (int64_t)(BH / 2) * nf;
+    const int64_t grid_warps = 4 * 3 * (int64_t)std::max(p->num_sms, 1);   // (two-head kernel: 3 blocks x 4 warps per SM)
+    const bool dyn = sm_split || (fine_dyn_env < 0 ? rows2 >= 64 * grid_warps : fine_dyn_env == 1);
+    fp.row_ctr = dyn ? p->d_counter + 2 : nullptr;
     fp.fine_rows = p->d_fine_rows;
     fp.row_ptr = p->d_fine_row_ptr;
     fp.cols = p->d_fine_col;
