@@ -421,6 +421,11 @@ __global__ void __launch_bounds__(kWarps * 32, FCfg<kD>::kMinB) fine_mma_kernel(
 #ifndef MG_FINE_MINB2
 #define MG_FINE_MINB2 3
 #endif
+// SDDMM operand order of the two-head kernel: 1 = gathered K rows as the M operand (one 4-MMA chain
+// per 16 nnz), 0 = q broadcast as the M operand (two chains, twice the MMAs)
+#ifndef MG_FINE_SWAP
+#define MG_FINE_SWAP 1
+#endif
 namespace {
 constexpr int kHB = 2 * kS * 128;                 // K + V rows of one head in a stage
 constexpr int kQOff2 = 2 * kHB;
@@ -589,6 +594,76 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB2) fine_mma2_kernel(c
             qq[hd][j][3] = qq[hd][j][2];
           }
       }
+#if MG_FINE_SWAP
+      // SDDMM with the gathered K rows as the M operand: s = K_c q for the step's 16 nnz in one
+      // m16n8k16 chain over the 4 k16 steps (A = 16 K rows x 16 dims by ldmatrix, B = q broadcast to
+      // the 8 columns), half the MMAs of the q-broadcast form; lane (g, t) gets the scores of nnz g
+      // and g + 8 (the same in its 4 t-lanes).
+      const int remg = end - base - g;
+      float s[2][2];
+#pragma unroll
+      for (int hd = 0; hd < 2; ++hd) {
+        const uint32_t sk = st + hd * kHB;
+        float sd[4] = {0.f, 0.f, 0.f, 0.f};
+#pragma unroll
+        for (int j = 0; j < kJ; ++j) {
+          // matrices: rows 0-7 / 8-15 of chunk 2j, then of chunk 2j + 1 (lane -> row address)
+          uint32_t ka[4];
+          const uint32_t R = (lane & 7) + 8 * ((lane >> 3) & 1), ch = 2 * j + (lane >> 4);
+          ldsm_x4(ka, sk + R * kRowBytes + ((ch ^ (R & 7)) << 4));
+          mma16816<kBF16>(sd, ka[0], ka[1], ka[2], ka[3], qq[hd][j][0], qq[hd][j][2]);
+        }
+        s[hd][0] = sd[0];
+        s[hd][1] = sd[2];
+        if (end - base < kS) {   // the row's last, partial step (warp-uniform): entries past the row
+          s[hd][0] = remg > 0 ? s[hd][0] : -INFINITY;
+          s[hd][1] = remg > 8 ? s[hd][1] : -INFINITY;
+        }
+      }
+      if (kPad) {   // padding: mask the columns at or beyond n_b (same columns for both heads)
+        if (remg > 0 && __ldg(p.cols + base + g) >= nvalid) s[0][0] = s[1][0] = -INFINITY;
+        if (remg > 8 && __ldg(p.cols + base + g + 8) >= nvalid) s[0][1] = s[1][1] = -INFINITY;
+      }
+      float mx[2];
+#pragma unroll
+      for (int hd = 0; hd < 2; ++hd) mx[hd] = fmaxf(s[hd][0], s[hd][1]);
+#pragma unroll
+      for (int o = 4; o < 32; o <<= 1)
+#pragma unroll
+        for (int hd = 0; hd < 2; ++hd) mx[hd] = fmaxf(mx[hd], __shfl_xor_sync(0xffffffffu, mx[hd], o));
+#pragma unroll
+      for (int hd = 0; hd < 2; ++hd) {
+        if (mx[hd] > m[hd] + thresh) {
+          const float alpha = ex2((m[hd] - mx[hd]) * c);
+          l[hd] *= alpha;
+#pragma unroll
+          for (int j = 0; j < kJ; ++j)
+#pragma unroll
+            for (int e = 0; e < 4; ++e) acc[hd][j][e] *= alpha;
+          m[hd] = mx[hd];
+        }
+      }
+#pragma unroll
+      for (int hd = 0; hd < 2; ++hd) {
+        const float nbias = m[hd] == -INFINITY ? 0.f : -m[hd] * c;
+        const float p0 = ex2(fmaf(s[hd][0], c, nbias)), p1 = ex2(fmaf(s[hd][1], c, nbias));
+        l[hd] += p0 + p1;
+        // the SpMM's B fragment wants nnz 2t, 2t + 1 (b0) and 2t + 8, 2t + 9 (b1): from the lanes of
+        // groups 2t and 2t + 1, which hold (p_2t, p_2t+8) and (p_2t+1, p_2t+9)
+        const uint32_t pk = pack2<kBF16>(p0, p1);
+        const uint32_t x = __shfl_sync(0xffffffffu, pk, 8 * t), y = __shfl_sync(0xffffffffu, pk, 8 * t + 4);
+        const uint32_t pb0 = __byte_perm(x, y, 0x5410), pb1 = __byte_perm(x, y, 0x7632);
+        const uint32_t sv = st + hd * kHB + kS * kRowBytes;
+#pragma unroll
+        for (int j = 0; j < kJ; ++j) {
+          uint32_t a[4];
+          const uint32_t ch = 2 * j + ((lane >> 3) & 1);
+          ldsm_x4_t(a, sv + vr * kRowBytes + ((ch ^ (vr & 7)) << 4));
+          mma16816<kBF16>(acc[hd][j], a[0], a[1], a[2], a[3], pb0, pb1);
+        }
+      }
+      __syncwarp();
+#else
       const int rem = end - base - 2 * t;
       float s[2][4];
 #pragma unroll
@@ -665,13 +740,21 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB2) fine_mma2_kernel(c
         }
       }
       __syncwarp();
+#endif
     }
     // ---- row epilogue of both heads
 #pragma unroll
     for (int hd = 0; hd < 2; ++hd) {
       float lh = l[hd];
+#if MG_FINE_SWAP
+      // (each group g holds the sums of its own nnz, the same in its four t-lanes)
+      lh += __shfl_xor_sync(0xffffffffu, lh, 4);
+      lh += __shfl_xor_sync(0xffffffffu, lh, 8);
+      lh += __shfl_xor_sync(0xffffffffu, lh, 16);
+#else
       lh += __shfl_xor_sync(0xffffffffu, lh, 1);
       lh += __shfl_xor_sync(0xffffffffu, lh, 2);
+#endif
       float v0 = acc[hd][0][0], v1 = acc[hd][0][2];
 #pragma unroll
       for (int j = 1; j < 4; ++j)
