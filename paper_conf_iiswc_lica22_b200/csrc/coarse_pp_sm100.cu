@@ -1125,11 +1125,15 @@ __global__ void __launch_bounds__(WCfg<kD>::kThreads, DCfg<kD>::kMinBlocks)
             }
           }
           fence_proxy_async_smem();
+#ifndef MG_DIAG_NO_EPI_BAR
           named_bar_sync(1, 128);
+#endif
           if (threadIdx.x == 0) {
             tma_store_4d(&tmo, sO, 0, item.rowA, ubh % p.H, ubh / p.H);
             bulk_commit_group();
+#ifndef MG_DIAG_NO_STORE_WAIT
             bulk_wait_group_read0();   // the buffer is reloaded with a later item's Q after q_empty
+#endif
           }
         } else if (pad_row) {
           const int bb = ubh / p.H, hh = ubh % p.H;
@@ -1375,7 +1379,9 @@ __global__ void __launch_bounds__(WCfg<kD>::kThreads, DCfg<kD>::kMinBlocks)
   #pragma unroll
             for (int sb = 0; sb < kNSub; ++sb) tma_store_4d(&tmo, sO + sb * kSub, 64 * sb, item.rowA, hh, bb);
             bulk_commit_group();
+#ifndef MG_DIAG_NO_STORE_WAIT
             bulk_wait_group_read0();   // the buffer is reloaded with a later item's Q after q_empty
+#endif
           }
         }
         tc_fence_before();
