@@ -426,6 +426,10 @@ __global__ void __launch_bounds__(kWarps * 32, FCfg<kD>::kMinB) fine_mma_kernel(
 #ifndef MG_FINE_SWAP
 #define MG_FINE_SWAP 1
 #endif
+// lazy-rescale test by a warp vote before the max reduction (1) or after it (0)
+#ifndef MG_FINE_VOTE
+#define MG_FINE_VOTE 1
+#endif
 namespace {
 constexpr int kHB = 2 * kS * 128;                 // K + V rows of one head in a stage
 constexpr int kQOff2 = 2 * kHB;
@@ -624,16 +628,23 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB2) fine_mma2_kernel(c
         if (remg > 0 && __ldg(p.cols + base + g) >= nvalid) s[0][0] = s[1][0] = -INFINITY;
         if (remg > 8 && __ldg(p.cols + base + g + 8) >= nvalid) s[0][1] = s[1][1] = -INFINITY;
       }
+      // lazy rescale: the step's row max is only reduced across the warp when some lane's scores
+      // exceed the running max by the threshold (the same decision as comparing the full max, without
+      // the three dependent shuffles on the common path)
       float mx[2];
 #pragma unroll
       for (int hd = 0; hd < 2; ++hd) mx[hd] = fmaxf(s[hd][0], s[hd][1]);
 #pragma unroll
-      for (int o = 4; o < 32; o <<= 1)
-#pragma unroll
-        for (int hd = 0; hd < 2; ++hd) mx[hd] = fmaxf(mx[hd], __shfl_xor_sync(0xffffffffu, mx[hd], o));
-#pragma unroll
       for (int hd = 0; hd < 2; ++hd) {
+#if MG_FINE_VOTE
+        if (__any_sync(0xffffffffu, mx[hd] > m[hd] + thresh)) {
+#pragma unroll
+          for (int o = 4; o < 32; o <<= 1) mx[hd] = fmaxf(mx[hd], __shfl_xor_sync(0xffffffffu, mx[hd], o));
+#else
+#pragma unroll
+        for (int o = 4; o < 32; o <<= 1) mx[hd] = fmaxf(mx[hd], __shfl_xor_sync(0xffffffffu, mx[hd], o));
         if (mx[hd] > m[hd] + thresh) {
+#endif
           const float alpha = ex2((m[hd] - mx[hd]) * c);
           l[hd] *= alpha;
 #pragma unroll
