@@ -426,6 +426,10 @@ __global__ void __launch_bounds__(kWarps * 32, FCfg<kD>::kMinB) fine_mma_kernel(
 #ifndef MG_FINE_SWAP
 #define MG_FINE_SWAP 1
 #endif
+// p to the SpMM's B fragment by two movmatrix transposes (1) or two shuffles + byte permutes (0)
+#ifndef MG_FINE_MOVM
+#define MG_FINE_MOVM 1
+#endif
 // lazy-rescale test by a warp vote before the max reduction (1) or after it (0)
 #ifndef MG_FINE_VOTE
 #define MG_FINE_VOTE 1
@@ -661,9 +665,18 @@ __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB2) fine_mma2_kernel(c
         l[hd] += p0 + p1;
         // the SpMM's B fragment wants nnz 2t, 2t + 1 (b0) and 2t + 8, 2t + 9 (b1): from the lanes of
         // groups 2t and 2t + 1, which hold (p_2t, p_2t+8) and (p_2t+1, p_2t+9)
+#if MG_FINE_MOVM
+        // as 8 x 8 16-bit matrices M[g][c] = p_g (resp. p_g+8) for every column c, held one register
+        // per lane (row g, columns 2t, 2t + 1): their transposes put p_2t, p_2t+1 (resp. p_2t+8,
+        // p_2t+9) in lane (g, t), the SpMM's B fragment
+        uint32_t pb0, pb1;
+        asm("movmatrix.sync.aligned.m8n8.trans.b16 %0, %1;" : "=r"(pb0) : "r"(pack2<kBF16>(p0, p0)));
+        asm("movmatrix.sync.aligned.m8n8.trans.b16 %0, %1;" : "=r"(pb1) : "r"(pack2<kBF16>(p1, p1)));
+#else
         const uint32_t pk = pack2<kBF16>(p0, p1);
         const uint32_t x = __shfl_sync(0xffffffffu, pk, 8 * t), y = __shfl_sync(0xffffffffu, pk, 8 * t + 4);
         const uint32_t pb0 = __byte_perm(x, y, 0x5410), pb1 = __byte_perm(x, y, 0x7632);
+#endif
         const uint32_t sv = st + hd * kHB + kS * kRowBytes;
 #pragma unroll
         for (int j = 0; j < kJ; ++j) {
