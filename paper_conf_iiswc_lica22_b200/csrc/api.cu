@@ -624,6 +624,13 @@ mg_status fwd_impl(mg_plan_s* p, const mg_tensor* Q, const mg_tensor* K, const m
       cp.rv = mp.rv;
       static const bool no_tma_store = std::getenv("MG_NO_TMA_STORE") != nullptr;   // A/B diagnostics
       cp.tma_store = !no_tma_store && mp.store_ok;
+      // item-major band order in groups of at most 96 (b,h) units: C2's 96 heads' K/V windows stay in
+      // L2 (C2 0.1419 -> 0.1375 ms); one group over C5's 768 heads re-reads K/V from DRAM (+7%)
+      static const int group_env = [] {   // (A/B: MG_UNIT_GROUP=<heads per group>)
+        const char* e = std::getenv("MG_UNIT_GROUP");
+        return e ? std::atoi(e) : 0;
+      }();
+      cp.unit_group = mg::item_major_order() ? std::min(BH, group_env > 0 ? group_env : 96) : 0;
       const int grid = sm_split ? coarse_split_ctas(h, BH, sms) : mg::coarse_pp_ctas_per_sm(D) * sms;
       if ((e = mg::launch_coarse_pp(cp, tq, tk, tv, mp.tq2, mp.tk2, mp.tv2, mp.to, bf16, use_split,
                                     std::min(grid, cp.total_units), stream)) != cudaSuccess)

@@ -120,12 +120,20 @@ struct UnitInfo {
   int item, bh;
 };
 
-// dense units first (long items start early), then band units in (b,h)-major, row-block order
+// dense units first (long items start early), then band units: in groups of unit_group (b,h) units
+// (a group's K/V stays in L2), item-major within a group with the items sorted by decreasing tile
+// count on the host, so the short band-edge items come last; or (b,h)-major, row-block order
 __device__ __forceinline__ UnitInfo decode_unit(const CoarseParams& p, int u) {
   const int dense_units = p.n_dense_items * p.BH;
   if (u < dense_units) return {u % p.n_dense_items, u / p.n_dense_items};
   const int v = u - dense_units;
   const int nband = p.n_items - p.n_dense_items;
+  if (p.unit_group > 0) {   // groups of unit_group (b,h) units, item-major within a group
+    const int per_group = nband * p.unit_group;
+    const int hg = v / per_group, w = v - hg * per_group;
+    const int gsize = min(p.unit_group, p.BH - hg * p.unit_group);
+    return {p.n_dense_items + w / gsize, hg * p.unit_group + w % gsize};
+  }
   return {p.n_dense_items + v % nband, v / nband};
 }
 

@@ -58,6 +58,8 @@ struct CoarseParams {
   // band items whose rows are all theirs to write (Item::useA) store O by TMA from shared memory
   // (the item's Q buffer) instead of per-thread row stores
   int32_t tma_store;
+  int32_t unit_group;         // band units: 0 = (b,h)-major; G > 0 = groups of G (b,h) units, item-major
+                              // within a group (items by decreasing tile count)
   int32_t debug_flags;        // diagnostics (env MG_DEBUG_FLAGS): 1 = no softmax arithmetic, 2 = no MMA, 4 = no loads,
                               // 16 = no S loads from TMEM, 64 = MMA ignores P-ready/O-free (timing only)
 };

@@ -10,6 +10,7 @@
 #include "plan.hpp"
 
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 #include <iterator>
 
@@ -20,6 +21,23 @@ namespace {
 inline int popcount64(uint64_t x) { return __builtin_popcountll(x); }
 
 }  // namespace
+
+// Band items in decreasing tile count (stable), for the coarse kernel's item-major unit order
+// (CoarseParams::unit_order): the short band-edge items are claimed last, so the persistent CTAs'
+// finishing times differ by less than one short item. MG_UNIT_ORDER=0 keeps the build order (A/B).
+bool item_major_order() {
+  static const bool on = [] {
+    const char* e = std::getenv("MG_UNIT_ORDER");
+    return !(e && e[0] == '0');
+  }();
+  return on;
+}
+void sort_band_items(std::vector<Item>& items, int32_t n_dense) {
+  if (!item_major_order() || (int32_t)items.size() <= n_dense) return;
+  std::stable_sort(items.begin() + n_dense, items.end(),
+                   [](const Item& a, const Item& b) { return a.ntiles > b.ntiles; });
+}
+
 
 std::string build_plan(HostPlan& p, int64_t L, int32_t heads, int32_t d, int32_t window,
                        const int32_t* global_idx, int64_t n_global, const int32_t* extra_idx,
@@ -344,6 +362,8 @@ std::string build_plan(HostPlan& p, int64_t L, int32_t heads, int32_t d, int32_t
     p.fine_col.insert(p.fine_col.end(), p.csr_col.begin() + p.csr_row_ptr[r], p.csr_col.begin() + p.csr_row_ptr[r + 1]);
     p.fine_row_ptr.push_back((int32_t)p.fine_col.size());
   }
+  sort_band_items(p.items, p.n_dense_items);
+  sort_band_items(p.items_split, p.n_dense_items_split);
   return "";
 }
 
@@ -424,6 +444,7 @@ std::string build_batched_plan(HostPlan& out, int64_t L, int32_t heads, int32_t 
     }
     if (pass == 0) out.n_dense_items = (int32_t)out.items.size();
   }
+  sort_band_items(out.items, out.n_dense_items);
   out.items_split = out.items;
   out.n_dense_items_split = out.n_dense_items;
   out.dense_nsplit = 1;

@@ -10,6 +10,8 @@
 
 namespace mg {
 
+bool item_major_order();   // band units item-major with items by decreasing tile count (plan.cpp)
+
 struct PlanOptions {
   int block = 128;
   bool force_all_fine = false;
