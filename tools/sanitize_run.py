@@ -43,7 +43,8 @@ def main():
     q, k, v = make_qkv(1, H, L, 64, seed=5)
     for name, kw in [("mixed/strips", {}), ("mixed/csr", dict(strip_max_cols=-1)),
                      ("mixed/concurrent", dict(strip_max_cols=-1, concurrency=2)), ("mixed/dense-split", dict(dense_chunk=1)),
-                     ("mixed/b64", dict(block=64)), ("mixed/few-ctas", dict(num_sms=1, strip_max_cols=-1))]:
+                     ("mixed/b64", dict(block=64)), ("mixed/few-ctas", dict(num_sms=1, strip_max_cols=-1)),
+                     ("mixed/sm-split", dict(strip_max_cols=-1, concurrency=3))]:
         check(name, mg.Plan(L, H, 64, W, G, E, **kw), q, k, v, W, G, E)
     q2, k2, v2 = make_qkv(2, H, L, 64, seed=7)
     check("padded", mg.Plan(L, H, 64, W, G, E), q2, k2, v2, W, G, E, lens=np.array([L, 200], np.int32))
