@@ -67,7 +67,13 @@ static_assert(256 * 96 + 128 * 48 <= (65536 / 2 / 384 & ~7) * 384, "register poo
 static_assert(256 * 208 + 128 * 88 <= (65536 / 1 / 384 & ~7) * 384, "register pool (column split, d = 128)");
 constexpr int kThreads = 256;
 constexpr int kSt = 2;                       // K ring and V ring depth
-constexpr int kItems = 4;                    // work-item ring depth
+// work-item ring depth: a CTA's scheduler claims at most kItems - 1 items ahead of its softmax warps;
+// 2 measured best (C2 0.1393 vs 0.1410, C3 0.0734 vs 0.0754, C5 1.048 vs 1.068 ms at 4; 6 worse
+// still): items claimed ahead by a busy CTA are the end-of-kernel imbalance
+#ifndef MG_ITEMS
+#define MG_ITEMS 2
+#endif
+constexpr int kItems = MG_ITEMS;
 constexpr uint32_t kSub = 128 * 128;         // one SWIZZLE_128B sub-tile: 128 rows x 64 x 16-bit
 constexpr uint32_t kMaskBytes = 128 * 16;    // 128 rows x 128 validity bits
 constexpr uint32_t kTS = 0, kTP = 128;       // TMEM columns of S (fp32) and P (packed 16-bit pairs)
