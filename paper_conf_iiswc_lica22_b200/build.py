@@ -34,7 +34,7 @@ VARIANTS = {"base": [],   # (a plain build under another name: A/B against a sta
             "dbg1": ["-DMG_DBG=1"], "dbg2": ["-DMG_DBG=2"], "dbg3": ["-DMG_DBG=3"], "dbg7": ["-DMG_DBG=7"],
             "dbg8": ["-DMG_DBG=8"], "dbg16": ["-DMG_DBG=16"], "dbg24": ["-DMG_DBG=24"], "dbg25": ["-DMG_DBG=25"],
             "dbg31": ["-DMG_DBG=31"], "tl7": ["-DMG_TIMELINE", "-DMG_DBG=7"], "tl1": ["-DMG_TIMELINE", "-DMG_DBG=1"],
-            "iq1": ["-DMG_IDLE_QUARTERS=1"], "ia0": ["-DMG_FINE_IDX_AHEAD=0"], "late1": ["-DMG_PV_LATE=1"], "ring0": ["-DMG_MASK_RING=0"], "cs128off": ["-DMG_CSPLIT128=0"], "tlate": ["-DMG_TIMELINE"], "swap0": ["-DMG_FINE_SWAP=0"], "vote0": ["-DMG_FINE_VOTE=0"], "items4": ["-DMG_ITEMS=4"], "items3": ["-DMG_ITEMS=3"], "movm0": ["-DMG_FINE_MOVM=0"], "nsw": ["-DMG_DIAG_NO_STORE_WAIT"], "nswb": ["-DMG_DIAG_NO_STORE_WAIT", "-DMG_DIAG_NO_EPI_BAR"], "f2s3b2": ["-DMG_FINE_STAGES=3", "-DMG_FINE_MINB2=2"], "f2s2b2": ["-DMG_FINE_MINB2=2"], "f2s3b2w5": ["-DMG_FINE_STAGES=3", "-DMG_FINE_MINB2=2", "-DMG_FINE_WARPS=5"]}
+            "iq1": ["-DMG_IDLE_QUARTERS=1"], "ia0": ["-DMG_FINE_IDX_AHEAD=0"], "late1": ["-DMG_PV_LATE=1"], "ring0": ["-DMG_MASK_RING=0"], "cs128off": ["-DMG_CSPLIT128=0"], "tlate": ["-DMG_TIMELINE"], "swap0": ["-DMG_FINE_SWAP=0"], "vote0": ["-DMG_FINE_VOTE=0"], "items4": ["-DMG_ITEMS=4"], "fch4": ["-DMG_FINE_CHUNK=4"], "fch16": ["-DMG_FINE_CHUNK=16"], "fch64": ["-DMG_FINE_CHUNK=64"], "items3": ["-DMG_ITEMS=3"], "movm0": ["-DMG_FINE_MOVM=0"], "nsw": ["-DMG_DIAG_NO_STORE_WAIT"], "nswb": ["-DMG_DIAG_NO_STORE_WAIT", "-DMG_DIAG_NO_EPI_BAR"], "f2s3b2": ["-DMG_FINE_STAGES=3", "-DMG_FINE_MINB2=2"], "f2s2b2": ["-DMG_FINE_MINB2=2"], "f2s3b2w5": ["-DMG_FINE_STAGES=3", "-DMG_FINE_MINB2=2", "-DMG_FINE_WARPS=5"]}
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 
 SOURCES = ["plan.cpp", "api.cu", "coarse_pp_sm100.cu", "fine_rows.cu", "fine_mma.cu", "staged.cu", "selftest_umma.cu"]

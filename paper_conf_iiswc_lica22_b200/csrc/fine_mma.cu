@@ -430,6 +430,12 @@ __global__ void __launch_bounds__(kWarps * 32, FCfg<kD>::kMinB) fine_mma_kernel(
 #ifndef MG_FINE_MOVM
 #define MG_FINE_MOVM 1
 #endif
+// rows (head-pair rows) per dynamic claim of the two-head kernel: longer runs of one head pair's rows
+// per warp (K/V locality, fewer claims); measured on C4: 2 / 4 / 8 / 16 / 32 / 64 ->
+// 2.06 / 2.03 / 1.99 / 1.95 / 1.87 / 1.98 ms
+#ifndef MG_FINE_CHUNK
+#define MG_FINE_CHUNK 32
+#endif
 // lazy-rescale test by a warp vote before the max reduction (1) or after it (0)
 #ifndef MG_FINE_VOTE
 #define MG_FINE_VOTE 1
@@ -446,7 +452,7 @@ constexpr int kSmemBytes2 = kWarps * kStages * kStageBytes2;
 // side follows it one step behind (so it finds the chunk the issue side is in when it leaves its own).
 template <bool kBF16, bool kPad, bool kDyn>
 __global__ void __launch_bounds__(kWarps * 32, MG_FINE_MINB2) fine_mma2_kernel(const FineParams p) {
-  constexpr int kChunk = 4;
+  constexpr int kChunk = MG_FINE_CHUNK;   // rows per dynamic claim
   constexpr int kD = 64, kRowBytes = 128, kLPR = 8, kRPI = 4, kJ = 4;
   extern __shared__ __align__(128) uint8_t fsm[];
   const int lane = threadIdx.x & 31;
